@@ -1,0 +1,397 @@
+"""Benchmark: fused Q-criterion on a 1024^3 fp32 rectilinear mesh per GPU.
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--impl ours|reference]
+
+Workload (BASELINE.json metric / configs[3]): synthetic
+Rayleigh-Taylor-like velocity (synth/), non-uniform x/y/z coordinates, the
+Q-criterion program of Fig. 3C (completed per DESIGN.md
+G1-G3), fused strategy.  N > 1: weak scaling, every rank owns a 1024^3 z-slab
+of a 1024 x 1024 x (1024 N) mesh, one ghost plane per side exchanged with
+NCCL inside dfg_execute.  One step = one dfg_execute (halo + fused kernel)
+with inputs resident in HBM; value = cells/s of the whole job.
+
+Prints ONE JSON line on rank 0.  See DESIGN.md section 7 for every key.
+"""
+
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import subprocess
+import sys
+import threading
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+METRIC = "Q-criterion cells/sec & HBM GB/s (fused vs staged vs roundtrip), 1/2/4/8 B200"
+N1 = 1024                       # cells per axis per GPU
+ALGO_BYTES_PER_CELL = 16        # fused Q, fp32: u, v, w read once + q written once
+
+
+def _peak():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    try:
+        with open(p) as f:
+            return float(json.load(f)["hbm_gbs"]), "measured (MEASURED_PEAKS.json hbm_gbs)"
+    except Exception:
+        return 6650.0, "fallback (B200_PROFILING.md 6.65 TB/s)"
+
+
+class ClockSampler:
+    """nvidia-smi clocks + throttle reasons sampled during the timed region."""
+    Q = ("clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.hw_slowdown,"
+         "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
+         "clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, index: int):
+        self.index = index
+        self.rows = []
+        self._stop = threading.Event()
+        self._t = None
+
+    def _run(self):
+        while not self._stop.is_set():
+            try:
+                out = subprocess.run(["nvidia-smi", f"--id={self.index}", f"--query-gpu={self.Q}",
+                                      "--format=csv,noheader,nounits"], capture_output=True, text=True,
+                                     timeout=5).stdout.strip()
+                if out:
+                    self.rows.append([c.strip() for c in out.split(",")])
+            except Exception:
+                pass
+            self._stop.wait(0.05)
+
+    def __enter__(self):
+        self._t = threading.Thread(target=self._run, daemon=True)
+        self._t.start()
+        return self
+
+    def __exit__(self, *a):
+        self._stop.set()
+        self._t.join(timeout=10)
+
+    def summary(self):
+        if not self.rows:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["unsampled"], "samples": 0}
+        sm = [float(r[0]) for r in self.rows if r[0].replace(".", "").isdigit()]
+        mx = [float(r[1]) for r in self.rows if r[1].replace(".", "").isdigit()]
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        reasons = sorted({names[i] for r in self.rows for i in range(4) if len(r) > 3 + i and r[3 + i] == "Active"})
+        return {"sm_mhz": float(np.median(sm)) if sm else None, "sm_max_mhz": max(mx) if mx else None,
+                "reasons": reasons, "samples": len(self.rows)}
+
+
+# ------------------------------------------------------------------ oracle
+def _oracle_sample(nx_rows: int, planes: int):
+    """Inputs for an oracle sample: a 1024 x nx_rows x planes block of the
+    bench mesh (plus its one-cell halo), generated on the CPU."""
+    import torch
+
+    import synth
+    x, y, z = synth.rt_coords(N1, N1, N1, np.float32)
+    x64, y64, z64 = (a.astype(np.float64) for a in (x, y, z))
+    k0, k1 = 100, 100 + planes
+    j0, j1 = 200, 200 + nx_rows
+    win = (k0 - 1, k1 + 1, j0 - 1, j1 + 1, 0, N1)
+    f = {c: synth.rt_velocity(c, x64, y64, z64, win, torch.float32).numpy() for c in "uvw"}
+    return x, y, z, f, win
+
+
+def _oracle_time(x, y, z, f, win):
+    from oracle import evaluate as oev
+    from oracle.lang import QCRIT, build_dag
+    dag = build_dag(QCRIT, ("u", "v", "w"), "f32")
+    t0 = time.perf_counter()
+    res, valid = oev.evaluate(dag, f, oev.MeshWindow(x, y, z, i0=win[4], j0=win[2], k0=win[0]))
+    dt = time.perf_counter() - t0
+    cells = int(valid[1:-1, 1:-1, :].sum())
+    return cells, dt
+
+
+def cpu_baseline_leg(target_s: float = 12.0):
+    """The oracle as it stands (numpy, one thread for element-wise ops) on a
+    bounded sample of the bench workload."""
+    x, y, z, f, win = _oracle_sample(256, 4)
+    cells, dt = _oracle_time(x, y, z, f, win)                 # calibration run
+    planes = int(max(1, min(128, round(4 * target_s / max(dt, 1e-3)))))
+    x, y, z, f, win = _oracle_sample(256, planes)
+    cells, dt = _oracle_time(x, y, z, f, win)
+    return {"value": cells / dt, "unit": "cells/s", "cores": 1, "kind": "oracle",
+            "sample": f"Q-criterion on a 1024 x 256 x {planes} block (+1-cell halo) of the 1024^3 RT-like "
+                      f"fp32 workload, numpy oracle, {dt:.1f} s"}
+
+
+def run_reference(args):
+    """--impl reference: the oracle is this tier's reference arm (CPU only)."""
+    rank = int(os.environ.get("RANK", "0"))
+    if rank != 0:
+        return 0
+    K, W = args.steps, args.warmup
+    budget = 150.0
+    x, y, z, f, win = _oracle_sample(16, 4)
+    _, dt = _oracle_time(x, y, z, f, win)
+    per_step = budget / (K + W)
+    scale = 16 * per_step / max(dt, 1e-3)          # in rows of 1024 x 1 x 4 cells
+    rows = int(max(1, min(800, round(scale))))
+    planes = int(4 * max(1, min(100, round(scale / rows))))
+    x, y, z, f, win = _oracle_sample(rows, planes)
+    for _ in range(W):
+        _oracle_time(x, y, z, f, win)
+    tot_cells, tot_t = 0, 0.0
+    for _ in range(K):
+        c, dt = _oracle_time(x, y, z, f, win)
+        tot_cells += c
+        tot_t += dt
+    v = tot_cells / tot_t
+    sample = (f"each step: Q-criterion on a 1024 x {rows} x {planes} block (+1-cell halo) of the RT-like "
+              f"workload, numpy oracle")
+    line = {"impl": "reference", "metric": METRIC, "value": v, "unit": "cells/s", "n_gpus": args.gpus,
+            "steps": K, "warmup": W, "ms_per_step": 1e3 * tot_t / K, "higher_is_better": True,
+            "scaling": "weak", "vs_baseline": None, "dtype": "f32", "data": "synthetic",
+            "config": {"workload": "fused Q-criterion 1024^3 fp32 per GPU (oracle: bounded CPU sample)",
+                       "expression": "qcrit"},
+            "cpu_baseline": {"value": v, "unit": "cells/s", "cores": 1, "kind": "oracle", "sample": sample},
+            "e2e": {"value": v, "unit": "cells/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+    return 0
+
+
+# ---------------------------------------------------------------- our arm
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=300)
+    ap.add_argument("--warmup", type=int, default=5)
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--n", type=int, default=N1, help="cells per axis per GPU (default 1024)")
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-strategies", action="store_true")
+    args = ap.parse_args()
+    if args.impl == "reference":
+        return run_reference(args)
+
+    import torch
+    import torch.distributed as dist
+
+    import paper_conf_sc_harrisonnmjc12_b200 as dfg
+    import synth
+    from oracle.lang import QCRIT  # the program text only (a string constant)
+
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    torch.cuda.set_device(local)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    assert world == args.gpus or world == 1, "launch with torchrun --nproc-per-node N for --gpus N"
+    n = args.n
+    NZ = n * world
+    K, W = args.steps, args.warmup
+    assert W >= 3, "at least 3 warm-up steps"
+
+    # mesh + inputs (slab of rank r with one ghost plane per side when N > 1)
+    x, y, z = synth.rt_coords(n, n, NZ, np.float32)
+    x64, y64, z64 = (a.astype(np.float64) for a in (x, y, z))
+    k0, nzl = dfg.dfg_partition(NZ, world, rank)
+    g = 1 if world > 1 else 0
+    fields = {}
+    for c in "uvw":
+        buf = torch.zeros((nzl + 2 * g, n, n), dtype=torch.float32, device="cuda")
+        buf[g:g + nzl] = synth.rt_velocity(
+            c, x64, y64, z64, (k0, k0 + nzl, 0, n, 0, n), torch.float32, "cuda")
+        fields[c] = buf
+    mesh = dfg.Mesh(x, y, z, nz_local=nzl, z_offset=k0, ghost=g)
+    for c, b in fields.items():
+        mesh.bind(c, b)
+    if world > 1:
+        uid = [dfg.dfg_nccl_unique_id() if rank == 0 else None]
+        dist.broadcast_object_list(uid, src=0)
+        dfg.dfg_mesh_init_comm(mesh.handle, uid[0], rank, world)
+    plan = dfg.Plan(mesh, QCRIT, "fused")
+    out = torch.empty((nzl, n, n), dtype=torch.float32, device="cuda")
+    stream = torch.cuda.Stream()
+    cells_rank = nzl * n * n
+
+    def barrier():
+        if world > 1:
+            dist.barrier()
+
+    with torch.cuda.stream(stream):
+        for _ in range(W):
+            plan.execute(out, stream=stream)
+    stream.synchronize()
+    plan.reset_stats()
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    barrier()
+    torch.cuda.synchronize()
+    with ClockSampler(local) as clk:
+        e0.record(stream)
+        for _ in range(K):
+            plan.execute(out, stream=stream)
+        e1.record(stream)
+        e1.synchronize()
+    torch.cuda.synchronize()
+    barrier()
+    ms = e0.elapsed_time(e1)
+    st = plan.stats()
+    kern_ms = st["kernel_ms_sum"] / max(1, st["kernel_launches_timed"])
+    t = torch.tensor([ms, kern_ms], device="cuda", dtype=torch.float64)
+    if world > 1:
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+    ms, kern_ms = float(t[0]), float(t[1])
+    ms_step = ms / K
+    value = cells_rank * world / (ms_step * 1e-3)
+    info = plan.info()
+
+    # roofline of the dominant kernel (the only kernel of the step)
+    peak, peak_src = _peak()
+    achieved = ALGO_BYTES_PER_CELL * cells_rank / (kern_ms * 1e-3) / 1e9
+    traffic = None
+    tp = os.path.join(ROOT, "profiles", "traffic.json")
+    if os.path.exists(tp):
+        try:
+            tj = json.load(open(tp))
+            if tj.get("n") == n:
+                traffic = tj.get("dram_bytes_per_launch")
+        except Exception:
+            pass
+
+    # e2e through the C ABI with host buffers (N = 1: host-pointer binding,
+    # the library uploads inputs and downloads the result inside dfg_execute)
+    e2e = None
+    if world == 1:
+        hostf = {c: fields[c].cpu().pin_memory() for c in "uvw"}
+        hout = torch.empty((nzl, n, n), dtype=torch.float32).pin_memory()
+        hmesh = dfg.Mesh(x, y, z)
+        for c in "uvw":
+            hmesh.bind(c, hostf[c], on_device=False)
+        hplan = dfg.Plan(hmesh, QCRIT, "fused")
+        hplan.execute(hout, out_on_device=False)
+        reps = 3
+        t0 = time.perf_counter()
+        for _ in range(reps):
+            hplan.execute(hout, out_on_device=False)
+        te = (time.perf_counter() - t0) / reps
+        hs = hplan.stats()
+        ok = bool(torch.equal(hout, out.cpu()))
+        e2e = {"value": cells_rank / te, "unit": "cells/s",
+               "h2d_bytes_per_step": hs["h2d_bytes"] // hs["executes"],
+               "d2h_bytes_per_step": hs["d2h_bytes"] // hs["executes"],
+               "ms_per_step": te * 1e3, "matches_device_result": ok}
+        hplan.close()
+        hmesh.close()
+        del hostf, hout
+    else:
+        # multi-GPU: pinned host -> device copies + dfg_execute + result read-back per step
+        hostf = {c: fields[c].cpu().pin_memory() for c in "uvw"}
+        hout = torch.empty((nzl, n, n), dtype=torch.float32).pin_memory()
+        barrier()
+        torch.cuda.synchronize()
+        t0 = time.perf_counter()
+        reps = 3
+        for _ in range(reps):
+            with torch.cuda.stream(stream):
+                for c in "uvw":
+                    fields[c].copy_(hostf[c], non_blocking=True)
+                plan.execute(out, stream=stream)
+                hout.copy_(out, non_blocking=True)
+            stream.synchronize()
+        te = torch.tensor([(time.perf_counter() - t0) / reps], dtype=torch.float64, device="cuda")
+        dist.all_reduce(te, op=dist.ReduceOp.MAX)
+        te = float(te[0])
+        e2e = {"value": cells_rank * world / te, "unit": "cells/s",
+               "h2d_bytes_per_step": 3 * fields["u"].numel() * 4 * world,
+               "d2h_bytes_per_step": out.numel() * 4 * world, "ms_per_step": te * 1e3}
+
+    strategies = None
+    if rank == 0 and world == 1 and not args.no_strategies:
+        strategies = strategy_sweep(dfg, synth, torch)
+
+    cpu = None
+    if rank == 0 and world == 1 and not args.no_cpu_baseline:
+        cpu = cpu_baseline_leg()
+
+    if rank == 0:
+        line = {
+            "metric": METRIC, "value": value, "unit": "cells/s", "n_gpus": world, "steps": K, "warmup": W,
+            "ms_per_step": ms_step, "higher_is_better": True, "scaling": "weak", "vs_baseline": None,
+            "dtype": "f32", "data": "synthetic",
+            "config": {"workload": f"fused Q-criterion, {n}^3 fp32 rectilinear mesh per GPU "
+                                   f"(mesh {n}x{n}x{NZ}, z-slabs + 1-plane NCCL halo when N>1)",
+                       "expression": "qcrit (Fig. 3C completed)", "strategy": "fused",
+                       "cells_per_gpu": cells_rank, "fused_kernel": {1: "tma", 2: "general", 3: "pointwise"}.get(
+                           info["variant"]), "regs": info["regs"],
+                       "l2": f"inputs {3 * cells_rank * 4 / 1e9:.1f} GB per GPU >> 126 MB L2; no flush needed",
+                       "parallelism": f"zslab{world}"},
+            "hbm_gbs": ALGO_BYTES_PER_CELL * cells_rank * world / (ms_step * 1e-3) / 1e9 / world,
+            "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
+                         "frac": achieved / peak, "traffic": traffic, "peak_source": peak_src,
+                         "kernel": "dfg_fused_tma", "kernel_ms": kern_ms,
+                         "algorithmic_bytes_per_launch": ALGO_BYTES_PER_CELL * cells_rank},
+            "e2e": e2e,
+            "gpu_launches": st["kernel_count"],
+            "clocks": clk.summary(),
+            "strategies": strategies,
+            "cpu_baseline": cpu,
+        }
+        print(json.dumps(line), flush=True)
+    if world > 1:
+        dist.destroy_process_group()
+    return 0
+
+
+def strategy_sweep(dfg, synth, torch):
+    """Fused vs staged vs roundtrip on Q (config 2, 192^3) with device-resident
+    inputs: cells/s and algorithmic device GB/s per strategy."""
+    from oracle.lang import QCRIT
+    n = 192
+    x, y, z = synth.rt_coords(n, n, n, np.float32)
+    x64, y64, z64 = (a.astype(np.float64) for a in (x, y, z))
+    mesh = dfg.Mesh(x, y, z)
+    bufs = {c: synth.rt_velocity(c, x64, y64, z64, None, torch.float32, "cuda") for c in "uvw"}
+    for c, b in bufs.items():
+        mesh.bind(c, b)
+    flush = torch.empty(512 * 1024 * 1024 // 4, dtype=torch.float32, device="cuda")
+    res = {}
+    ref = None
+    for s in ("fused", "staged", "roundtrip"):
+        plan = dfg.Plan(mesh, QCRIT, s)
+        out = torch.empty((n, n, n), dtype=torch.float32, device="cuda")
+        for _ in range(2):
+            plan.execute(out)
+        torch.cuda.synchronize()
+        times = []
+        for _ in range(7):                  # the paper's protocol: 7 runs, drop min/max (L241)
+            flush.zero_()                   # L2 flush (working set < 4x L2)
+            torch.cuda.synchronize()
+            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            e0.record()
+            plan.execute(out)
+            e1.record()
+            e1.synchronize()
+            times.append(e0.elapsed_time(e1))
+        times = sorted(times)[1:-1]
+        ms = sum(times) / len(times)
+        st = plan.stats()
+        ex = st["executes"]
+        res[s] = {"cells_per_s": n ** 3 / (ms * 1e-3), "ms": ms,
+                  "device_gb_per_s": st["predicted_hbm_bytes"] / (ms * 1e-3) / 1e9,
+                  "predicted_device_bytes": st["predicted_hbm_bytes"],
+                  "pcie_bytes": (st["h2d_bytes"] + st["d2h_bytes"]) // ex,
+                  "kernels_per_execute": st["kernel_count"] // ex,
+                  "highwater_bytes": st["dev_highwater_bytes"]}
+        if ref is None:
+            ref = out.clone()
+        else:
+            res[s]["bit_identical_to_fused"] = bool(torch.equal(ref, out))
+        plan.close()
+    return {"workload": "Q-criterion 192^3 fp32, device-resident inputs, L2 flushed, mean of 5 of 7", **res}
+
+
+if __name__ == "__main__":
+    sys.exit(main())

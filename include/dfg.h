@@ -1,0 +1,229 @@
+/*
+ * dfg.h -- C ABI of the B200-native derived-field generator (libdfg.so).
+ *
+ * The method (Harrison et al., SC-companion 2012; /root/reference/PAPER.md,
+ * cited as L<n>): a host application hands the framework an expression
+ * written in a VisIt-style language plus its input arrays and gets the
+ * derived field back, in situ (L116-L118).  The expression is parsed into a
+ * dataflow network (L66-L76), initialised (topological order, reference
+ * counts, L85) and executed by one of three strategies built from one
+ * library of primitives (L86-L105): roundtrip, staged or fusion.  The
+ * network is built once and re-executed whenever the data change (L122).
+ *
+ * Conventions for every entry point:
+ *   - returns DFG_OK (0) or a negative dfg_status; dfg_last_error() gives a
+ *     thread-local message for the last failing call of this thread;
+ *   - no entry point falls back to the CPU: without a usable CUDA device the
+ *     device-touching calls return DFG_E_CUDA;
+ *   - sizes are int64 element counts unless the name says bytes;
+ *   - fields are cell-centred (L154, L223), x fastest:
+ *       value(i, j, k) = field[i + nx * (j + ny * k_local)]
+ *     scalar arrays are T[nz][ny][nx]; vector results (grad3d, compose) are
+ *     stored 4-wide, T[nz][ny][nx][4] (the OpenCL vector types of L104),
+ *     unused lanes 0;
+ *   - T is float (DFG_F32) or double (DFG_F64), fixed per mesh.
+ */
+#ifndef DFG_H
+#define DFG_H
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef struct dfg_mesh_s* dfg_mesh;
+typedef struct dfg_plan_s* dfg_plan;
+
+/* Execution strategies, L88-L105. */
+typedef enum {
+  DFG_ROUNDTRIP = 0, /* one kernel per primitive, every result to the host (L92) */
+  DFG_STAGED = 1,    /* one kernel per primitive, intermediates on the device (L96) */
+  DFG_FUSED = 2      /* one generated kernel, intermediates in registers (L97) */
+} dfg_strategy;
+
+typedef enum { DFG_F32 = 0, DFG_F64 = 1 } dfg_dtype;
+
+typedef enum {
+  DFG_OK = 0,
+  DFG_E_INVALID = -1,     /* bad argument (null handle, size, coordinates, name) */
+  DFG_E_PARSE = -2,       /* expression syntax; message carries line:col      */
+  DFG_E_UNDEFINED = -3,   /* unknown identifier or function                   */
+  DFG_E_TYPE = -4,        /* arity, scalar/vector mismatch, index out of range */
+  DFG_E_NOMEM = -5,       /* footprint above the cap, or device allocation failed (L309) */
+  DFG_E_NVRTC = -6,       /* fused-kernel compilation failed                  */
+  DFG_E_CUDA = -7,        /* CUDA runtime/driver error or no device            */
+  DFG_E_NCCL = -8,        /* NCCL unavailable or failed                        */
+  DFG_E_UNBOUND = -9,     /* an input the network reads has no bound buffer    */
+  DFG_E_UNSUPPORTED = -10,/* valid request this build does not implement       */
+  DFG_E_RANGE = -11       /* caller buffer too small (see *needed)             */
+} dfg_status;
+
+/* Device events and memory of a plan (Table II L271-L285 quantities and the
+ * Fig. 6 high-water mark, L245-L247).  Counters accumulate over executes
+ * until dfg_reset_stats(). */
+typedef struct {
+  int64_t executes;
+  int64_t h2d_count;            /* host->device transfers ("Dev-W")           */
+  int64_t d2h_count;            /* device->host transfers ("Dev-R")           */
+  int64_t kernel_count;         /* kernel executions ("K-Exe")                */
+  int64_t h2d_bytes;
+  int64_t d2h_bytes;
+  int64_t halo_bytes;           /* bytes received into ghost planes           */
+  int64_t dev_highwater_bytes;  /* max live problem-sized device arrays, incl.
+                                   bound device inputs and the output (Fig. 2) */
+  int64_t predicted_highwater_bytes; /* model of the last-executed mode        */
+  int64_t predicted_hbm_bytes;  /* algorithmic device bytes of one execute    */
+  int64_t predicted_pcie_bytes; /* algorithmic host<->device bytes of one execute */
+  double last_ms;               /* device time of the last execute (CUDA events);
+                                   waits for it to finish; -1 if none          */
+  double kernel_ms_sum;         /* device time of every fused-kernel launch since
+                                   the last reset (CUDA events around the launch
+                                   on the execute stream; no host sync inside
+                                   execute -- resolved when stats are read)      */
+  int64_t kernel_launches_timed;/* launches summed in kernel_ms_sum            */
+} dfg_stats;
+
+/* ---------------------------------------------------------------- version */
+int dfg_version(void);                 /* 100 * major + minor */
+const char* dfg_last_error(void);      /* never NULL; "" after success */
+
+/* ------------------------------------------------------------------- mesh
+ * Rectilinear mesh (L86, L165): nx x ny x nz cells; point coordinates
+ *   x[0..nx], y[0..ny], z[0..nz_global]  (host pointers, element type T,
+ *   strictly increasing, finite) -- copied, the caller keeps ownership.
+ * z-slab decomposition (ghost data, L255 / L315): this mesh object holds
+ *   the cells k in [z_offset, z_offset + nz_local) of a global mesh with
+ *   nz_global cells in z; ghost = 0 or 1 extra planes on both ends of every
+ *   bound field buffer (filled by the halo exchange of dfg_execute).
+ *   Single GPU: nz_local = nz_global, z_offset = 0, ghost = 0.
+ * The mesh is created on the CUDA device current at the call; it builds and
+ * uploads the per-axis spacing tables (R1).
+ * Errors: DFG_E_INVALID (sizes < 1, z range outside the global mesh,
+ * coordinates not strictly increasing or not finite, ghost not 0/1),
+ * DFG_E_CUDA (no device). */
+int dfg_create_mesh(dfg_dtype dtype, int64_t nx, int64_t ny, int64_t nz_local,
+                    const void* x, const void* y, const void* z,
+                    int64_t nz_global, int64_t z_offset, int ghost,
+                    dfg_mesh* out);
+/* Idempotent on NULL.  Plans keep what they need alive: destroying a mesh
+ * with live plans is allowed (the plans stay valid). */
+void dfg_destroy_mesh(dfg_mesh mesh);
+
+/* Even z-slab split used by the driver:
+ *   nz_r = nz_global / n + (rank < nz_global % n), z_offset = sum of the
+ *   preceding slabs.  DFG_E_INVALID unless 1 <= nranks <= nz_global. */
+int dfg_partition(int64_t nz_global, int nranks, int rank,
+                  int64_t* z_offset, int64_t* nz_local);
+
+/* Ghost-plane map of this slab, 16 int64:
+ *   rank, nranks, NZ, k0, k1, nz_r, has_lo, has_hi, peer_lo, peer_hi,
+ *   send_lo_local_plane, send_hi_local_plane, recv_lo_local_plane,
+ *   recv_hi_local_plane, plane_bytes, halo_width
+ * Local planes count the lower ghost plane as 0 (owned planes 1..nz_r);
+ * absent entries are -1.  rank/nranks are 0/1 until a communicator is set. */
+int dfg_halo_map(dfg_mesh mesh, int64_t out[16]);
+
+/* Multi-GPU halo transport, one process per GPU (NCCL point-to-point,
+ * L255 ghost exchange re-done over NVLink).  dfg_nccl_unique_id fills 128
+ * bytes on rank 0; the caller broadcasts them (torch.distributed) and every
+ * rank calls dfg_mesh_init_comm on the device that owns its mesh.
+ * NCCL is loaded at run time (libnccl.so.2); DFG_E_NCCL if unavailable. */
+int dfg_nccl_unique_id(void* out128);
+int dfg_mesh_init_comm(dfg_mesh mesh, const void* id128, int rank, int nranks);
+
+/* Single-process halo transport: slabs that live in one process (one or
+ * several devices) exchange ghost planes with device-to-device copies.
+ * `lo` must hold the slab directly below `hi` (lo.k1 == hi.k0). */
+int dfg_mesh_link_local(dfg_mesh lo, dfg_mesh hi);
+
+/* ----------------------------------------------------------------- fields
+ * Bind a cell-centred scalar input under `name` (an identifier; not a
+ * keyword, not dims/x/y/z, not f<digits>).  BORROWED: the buffer must stay
+ * valid and unchanged in shape until the executes that read it complete.
+ * Layout T[nz_local + 2*ghost][ny][nx] (ghost planes at both ends).
+ * on_device = 1: a CUDA pointer on the mesh's device (in situ mode);
+ * on_device = 0: a host pointer -- the paper's host interface (L118):
+ * the strategies upload it and count the transfers (Table II).  Host
+ * pointers are single-slab only (nranks = 1).  Rebinding replaces;
+ * ptr = NULL unbinds.  The fused kernel's TMA fast path additionally wants
+ * 16-byte aligned device pointers and nx*sizeof(T) % 16 == 0; other
+ * layouts run the general kernel with the same arithmetic. */
+int dfg_bind_field(dfg_mesh mesh, const char* name, void* ptr, int on_device);
+
+/* ------------------------------------------------------------------ plans
+ * Parse -> dataflow network -> plan (L64-L105).  Every identifier the
+ * program reads must be a field bound at this point, an earlier assignment
+ * target, or one of dims/x/y/z as grad3d arguments.
+ * dev_mem_cap: bytes of problem-sized device arrays the plan may hold at
+ * once (0 = unlimited); checked against the predicted footprint here
+ * (DFG_E_NOMEM) and against the live ledger during execute.
+ * Fused plans generate, NVRTC-compile (sm_100a) and load their kernel here.
+ * Errors: DFG_E_PARSE, DFG_E_UNDEFINED, DFG_E_TYPE, DFG_E_NOMEM,
+ * DFG_E_NVRTC, DFG_E_CUDA, DFG_E_UNSUPPORTED (staged/roundtrip on a
+ * multi-slab mesh). */
+int dfg_compile(dfg_mesh mesh, const char* expr, dfg_strategy strategy,
+                size_t dev_mem_cap, dfg_plan* out);
+void dfg_destroy_plan(dfg_plan plan);
+
+/* Execute on `cuda_stream` (cudaStream_t; NULL = legacy default stream).
+ * out: T[nz_local][ny][nx] (or [..][4] for a vector program), a device
+ * pointer if out_on_device else a host pointer.  Fused and staged enqueue
+ * asynchronously when everything is on the device; any host buffer makes
+ * the call synchronous (roundtrip always is).  Multi-slab meshes first
+ * exchange the ghost planes of the fields grad3d reads (this writes the
+ * ghost planes of the caller's buffers).
+ * Errors: DFG_E_UNBOUND, DFG_E_NOMEM (ledger cap or allocation failure:
+ * the paper's failed GPU cases, L309), DFG_E_CUDA, DFG_E_NCCL. */
+int dfg_execute(dfg_plan plan, void* out, int out_on_device, void* cuda_stream);
+
+int dfg_plan_stats(dfg_plan plan, dfg_stats* out);
+int dfg_reset_stats(dfg_plan plan);
+
+/* Plan description: out[0] = strategy, out[1] = result width (1 or 4),
+ * out[2] = number of filters, out[3] = fused kernel variant in use
+ * (0 none, 1 TMA pipeline, 2 general), out[4] = registers per thread of the
+ * fused kernel (0 if none), out[5] = spilled bytes, out[6] = predicted
+ * device footprint in bytes for device-resident inputs,
+ * out[7] = same for host inputs. */
+int dfg_plan_info(dfg_plan plan, int64_t out[8]);
+
+/* Canonical network text (R10) -- stands in for the paper's
+ * optional Python script of network-definition API calls (L84).
+ * Copies up to cap bytes incl. the NUL; *needed = full size incl. NUL;
+ * DFG_E_RANGE if cap is too small. */
+int dfg_dump_dag(dfg_plan plan, char* buf, size_t cap, size_t* needed);
+/* Generated CUDA source of a fused plan (the paper's dynamic kernel
+ * generator output, L97-L105); same buffer protocol. */
+int dfg_dump_kernel(dfg_plan plan, char* buf, size_t cap, size_t* needed);
+
+/* ------------------------------------------------------- host-only tools
+ * Need no GPU: the parser / network builder, the strategy model and the
+ * kernel generator on their own, for tests and tooling. */
+
+/* Parse + lower `expr` with the named scalar inputs; write the canonical
+ * text.  Same errors as dfg_compile's language errors. */
+int dfg_dag_dump(const char* expr, const char* const* inputs, int n_inputs,
+                 dfg_dtype dtype, char* buf, size_t cap, size_t* needed);
+
+/* Planner's predictions for one execute: out[0..2] = h2d, d2h, kernels;
+ * out[3] = footprint in problem-array units (scalar 1, vector 4).
+ * host_mode = 1: inputs and output in host memory (Table II, Fig. 2);
+ * 0: everything device resident. */
+int dfg_model(const char* expr, const char* const* inputs, int n_inputs,
+              dfg_strategy strategy, int host_mode, int64_t out[4]);
+
+/* Generate the fused kernel source for `expr` on an nx x ny x nz mesh and,
+ * if compile != 0, NVRTC-compile it for sm_100a (no device needed); on
+ * success *regs / *spill (may be NULL) get the ptxas figures of the TMA
+ * kernel.  Writes the source with the buffer protocol above. */
+int dfg_fused_source(const char* expr, const char* const* inputs, int n_inputs,
+                     dfg_dtype dtype, int64_t nx, int64_t ny, int64_t nz,
+                     int compile, char* buf, size_t cap, size_t* needed,
+                     int* regs, int* spill);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* DFG_H */

@@ -1,0 +1,237 @@
+"""ctypes binding of libdfg.so (include/dfg.h) -- argument marshalling only.
+
+Every function has the C name and C argument order; pointers may be given as
+ints, numpy arrays or torch tensors (their data pointer is passed).  A
+negative status raises ``DfgError`` with the library's message.  There is no
+Python or CPU implementation of anything behind these names: if the shared
+library is missing the import fails.
+"""
+
+from __future__ import annotations
+
+import ctypes as C
+import os
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(_HERE, "libdfg.so")
+
+if not os.path.exists(LIB_PATH):
+    raise ImportError(
+        f"{LIB_PATH} is missing: build it with `python -c 'import __graft_entry__ as g; g.build()'` "
+        "or `make -C paper_conf_sc_harrisonnmjc12_b200/csrc`; libdfg has no CPU fallback")
+
+_lib = C.CDLL(LIB_PATH, mode=C.RTLD_GLOBAL)
+
+DFG_ROUNDTRIP, DFG_STAGED, DFG_FUSED = 0, 1, 2
+DFG_F32, DFG_F64 = 0, 1
+STRATEGIES = {"roundtrip": DFG_ROUNDTRIP, "staged": DFG_STAGED, "fused": DFG_FUSED}
+STATUS = {0: "DFG_OK", -1: "DFG_E_INVALID", -2: "DFG_E_PARSE", -3: "DFG_E_UNDEFINED", -4: "DFG_E_TYPE",
+          -5: "DFG_E_NOMEM", -6: "DFG_E_NVRTC", -7: "DFG_E_CUDA", -8: "DFG_E_NCCL", -9: "DFG_E_UNBOUND",
+          -10: "DFG_E_UNSUPPORTED", -11: "DFG_E_RANGE"}
+
+
+class DfgError(RuntimeError):
+    def __init__(self, status: int, msg: str):
+        super().__init__(f"{STATUS.get(status, status)}: {msg}")
+        self.status = status
+        self.name = STATUS.get(status, str(status))
+        self.msg = msg
+
+
+class dfg_stats(C.Structure):
+    _fields_ = [(n, C.c_int64) for n in (
+        "executes", "h2d_count", "d2h_count", "kernel_count", "h2d_bytes", "d2h_bytes", "halo_bytes",
+        "dev_highwater_bytes", "predicted_highwater_bytes", "predicted_hbm_bytes", "predicted_pcie_bytes")] + [
+        ("last_ms", C.c_double), ("kernel_ms_sum", C.c_double), ("kernel_launches_timed", C.c_int64)]
+
+    def as_dict(self):
+        return {n: getattr(self, n) for n, _ in self._fields_}
+
+
+_P = C.c_void_p
+_I64 = C.c_int64
+_SIGS = {
+    "dfg_version": (C.c_int, []),
+    "dfg_last_error": (C.c_char_p, []),
+    "dfg_create_mesh": (C.c_int, [C.c_int, _I64, _I64, _I64, _P, _P, _P, _I64, _I64, C.c_int, C.POINTER(_P)]),
+    "dfg_destroy_mesh": (None, [_P]),
+    "dfg_partition": (C.c_int, [_I64, C.c_int, C.c_int, C.POINTER(_I64), C.POINTER(_I64)]),
+    "dfg_halo_map": (C.c_int, [_P, C.POINTER(_I64)]),
+    "dfg_nccl_unique_id": (C.c_int, [_P]),
+    "dfg_mesh_init_comm": (C.c_int, [_P, _P, C.c_int, C.c_int]),
+    "dfg_mesh_link_local": (C.c_int, [_P, _P]),
+    "dfg_bind_field": (C.c_int, [_P, C.c_char_p, _P, C.c_int]),
+    "dfg_compile": (C.c_int, [_P, C.c_char_p, C.c_int, C.c_size_t, C.POINTER(_P)]),
+    "dfg_destroy_plan": (None, [_P]),
+    "dfg_execute": (C.c_int, [_P, _P, C.c_int, _P]),
+    "dfg_plan_stats": (C.c_int, [_P, C.POINTER(dfg_stats)]),
+    "dfg_reset_stats": (C.c_int, [_P]),
+    "dfg_plan_info": (C.c_int, [_P, C.POINTER(_I64)]),
+    "dfg_dump_dag": (C.c_int, [_P, C.c_char_p, C.c_size_t, C.POINTER(C.c_size_t)]),
+    "dfg_dump_kernel": (C.c_int, [_P, C.c_char_p, C.c_size_t, C.POINTER(C.c_size_t)]),
+    "dfg_dag_dump": (C.c_int, [C.c_char_p, C.POINTER(C.c_char_p), C.c_int, C.c_int, C.c_char_p, C.c_size_t,
+                               C.POINTER(C.c_size_t)]),
+    "dfg_model": (C.c_int, [C.c_char_p, C.POINTER(C.c_char_p), C.c_int, C.c_int, C.c_int, C.POINTER(_I64)]),
+    "dfg_fused_source": (C.c_int, [C.c_char_p, C.POINTER(C.c_char_p), C.c_int, C.c_int, _I64, _I64, _I64, C.c_int,
+                                   C.c_char_p, C.c_size_t, C.POINTER(C.c_size_t), C.POINTER(C.c_int),
+                                   C.POINTER(C.c_int)]),
+}
+EXPORTS = tuple(_SIGS)
+for _name, (_res, _args) in _SIGS.items():
+    _f = getattr(_lib, _name)
+    _f.restype = _res
+    _f.argtypes = _args
+
+
+def _check(status: int):
+    if status != 0:
+        raise DfgError(status, _lib.dfg_last_error().decode())
+
+
+def _ptr(x):
+    """Data pointer of an int / numpy array / torch tensor / None."""
+    if x is None:
+        return None
+    if isinstance(x, int):
+        return x
+    if hasattr(x, "data_ptr"):
+        return x.data_ptr()
+    if hasattr(x, "ctypes"):
+        return x.ctypes.data
+    raise TypeError(type(x))
+
+
+def _names(inputs):
+    arr = (C.c_char_p * max(len(inputs), 1))(*[s.encode() for s in inputs])
+    return arr, len(inputs)
+
+
+def _text(fn, *args):
+    need = C.c_size_t(0)
+    st = fn(*args, None, 0, C.byref(need))
+    if st not in (0, -11):
+        _check(st)
+    buf = C.create_string_buffer(need.value)
+    _check(fn(*args, buf, need.value, C.byref(need)))
+    return buf.value.decode()
+
+
+# --------------------------------------------------------------- C names
+def dfg_version() -> int:
+    return _lib.dfg_version()
+
+
+def dfg_last_error() -> str:
+    return _lib.dfg_last_error().decode()
+
+
+def dfg_create_mesh(dtype, nx, ny, nz_local, x, y, z, nz_global=None, z_offset=0, ghost=0):
+    h = _P()
+    _check(_lib.dfg_create_mesh(dtype, nx, ny, nz_local, _ptr(x), _ptr(y), _ptr(z),
+                                nz_local if nz_global is None else nz_global, z_offset, ghost, C.byref(h)))
+    return h.value
+
+
+def dfg_destroy_mesh(mesh):
+    _lib.dfg_destroy_mesh(mesh)
+
+
+def dfg_partition(nz_global, nranks, rank):
+    off, n = _I64(), _I64()
+    _check(_lib.dfg_partition(nz_global, nranks, rank, C.byref(off), C.byref(n)))
+    return off.value, n.value
+
+
+def dfg_halo_map(mesh):
+    out = (_I64 * 16)()
+    _check(_lib.dfg_halo_map(mesh, out))
+    return list(out)
+
+
+def dfg_nccl_unique_id() -> bytes:
+    buf = C.create_string_buffer(128)
+    _check(_lib.dfg_nccl_unique_id(buf))
+    return buf.raw
+
+
+def dfg_mesh_init_comm(mesh, uid: bytes, rank, nranks):
+    buf = C.create_string_buffer(bytes(uid), 128)
+    _check(_lib.dfg_mesh_init_comm(mesh, buf, rank, nranks))
+
+
+def dfg_mesh_link_local(lo, hi):
+    _check(_lib.dfg_mesh_link_local(lo, hi))
+
+
+def dfg_bind_field(mesh, name, ptr, on_device):
+    _check(_lib.dfg_bind_field(mesh, name.encode(), _ptr(ptr), int(on_device)))
+
+
+def dfg_compile(mesh, expr, strategy, dev_mem_cap=0):
+    if isinstance(strategy, str):
+        strategy = STRATEGIES[strategy]
+    h = _P()
+    _check(_lib.dfg_compile(mesh, expr.encode(), strategy, dev_mem_cap, C.byref(h)))
+    return h.value
+
+
+def dfg_destroy_plan(plan):
+    _lib.dfg_destroy_plan(plan)
+
+
+def dfg_execute(plan, out, out_on_device, cuda_stream=None):
+    _check(_lib.dfg_execute(plan, _ptr(out), int(out_on_device), cuda_stream))
+
+
+def dfg_plan_stats(plan) -> dict:
+    st = dfg_stats()
+    _check(_lib.dfg_plan_stats(plan, C.byref(st)))
+    return st.as_dict()
+
+
+def dfg_reset_stats(plan):
+    _check(_lib.dfg_reset_stats(plan))
+
+
+def dfg_plan_info(plan) -> dict:
+    out = (_I64 * 8)()
+    _check(_lib.dfg_plan_info(plan, out))
+    keys = ("strategy", "width", "filters", "variant", "regs", "spill", "footprint_device", "footprint_host")
+    return dict(zip(keys, list(out)))
+
+
+def dfg_dump_dag(plan) -> str:
+    return _text(_lib.dfg_dump_dag, plan)
+
+
+def dfg_dump_kernel(plan) -> str:
+    return _text(_lib.dfg_dump_kernel, plan)
+
+
+def dfg_dag_dump(expr, inputs, dtype=DFG_F32) -> str:
+    arr, n = _names(inputs)
+    return _text(_lib.dfg_dag_dump, expr.encode(), arr, n, dtype)
+
+
+def dfg_model(expr, inputs, strategy, host_mode=True):
+    if isinstance(strategy, str):
+        strategy = STRATEGIES[strategy]
+    arr, n = _names(inputs)
+    out = (_I64 * 4)()
+    _check(_lib.dfg_model(expr.encode(), arr, n, strategy, int(host_mode), out))
+    return list(out)
+
+
+def dfg_fused_source(expr, inputs, dtype, nx, ny, nz, compile=False):
+    """Returns (source, regs, spill)."""
+    arr, n = _names(inputs)
+    regs, spill = C.c_int(-1), C.c_int(-1)
+    need = C.c_size_t(0)
+    st = _lib.dfg_fused_source(expr.encode(), arr, n, dtype, nx, ny, nz, int(compile), None, 0, C.byref(need),
+                               C.byref(regs), C.byref(spill))
+    if st not in (0, -11):
+        _check(st)
+    buf = C.create_string_buffer(need.value)
+    _check(_lib.dfg_fused_source(expr.encode(), arr, n, dtype, nx, ny, nz, 0, buf, need.value, C.byref(need),
+                                 None, None))
+    return buf.value.decode(), regs.value, spill.value

@@ -1,0 +1,282 @@
+// extern "C" entry points of libdfg.so (include/dfg.h).  Each one catches
+// every internal DfgError, records the message for dfg_last_error() and
+// returns the status; nothing throws across the ABI.
+#include <cuda_runtime.h>
+
+#include <cstring>
+#include <memory>
+#include <string>
+
+#include "dfg.h"
+#include "runtime.hpp"
+
+struct dfg_mesh_s {
+  std::shared_ptr<dfg::MeshImpl> m;
+};
+struct dfg_plan_s {
+  std::unique_ptr<dfg::PlanImpl> p;
+};
+
+namespace dfg {
+namespace {
+thread_local std::string t_err;
+}
+void set_last_error(const std::string& m) { t_err = m; }
+void clear_last_error() { t_err.clear(); }
+}  // namespace dfg
+
+namespace {
+
+template <typename F>
+int guard(F&& f) {
+  try {
+    dfg::clear_last_error();
+    f();
+    return DFG_OK;
+  } catch (const dfg::DfgError& e) {
+    dfg::set_last_error(e.what());
+    return e.status;
+  } catch (const std::bad_alloc&) {
+    dfg::set_last_error("host out of memory");
+    return DFG_E_NOMEM;
+  } catch (const std::exception& e) {
+    dfg::set_last_error(std::string("internal error: ") + e.what());
+    return DFG_E_INVALID;
+  }
+}
+
+int copy_out(const std::string& s, char* buf, size_t cap, size_t* needed) {
+  if (needed) *needed = s.size() + 1;
+  if (!buf || cap < s.size() + 1) {
+    if (buf && cap) {
+      std::memcpy(buf, s.data(), cap - 1);
+      buf[cap - 1] = '\0';
+    }
+    dfg::fail(DFG_E_RANGE, "buffer too small: need " + std::to_string(s.size() + 1) + " bytes");
+  }
+  std::memcpy(buf, s.c_str(), s.size() + 1);
+  return 0;
+}
+
+std::vector<std::string> names_of(const char* const* inputs, int n) {
+  if (n < 0 || (n > 0 && !inputs)) dfg::fail(DFG_E_INVALID, "bad input name list");
+  std::vector<std::string> v;
+  for (int i = 0; i < n; ++i) {
+    if (!inputs[i]) dfg::fail(DFG_E_INVALID, "null input name");
+    v.emplace_back(inputs[i]);
+  }
+  return v;
+}
+
+dfg::DType to_dtype(int d) {
+  if (d != DFG_F32 && d != DFG_F64) dfg::fail(DFG_E_INVALID, "bad dtype");
+  return d == DFG_F32 ? dfg::DType::F32 : dfg::DType::F64;
+}
+
+}  // namespace
+
+extern "C" {
+
+int dfg_version(void) { return 100; }
+
+const char* dfg_last_error(void) { return dfg::t_err.c_str(); }
+
+int dfg_create_mesh(dfg_dtype dtype, int64_t nx, int64_t ny, int64_t nz_local, const void* x, const void* y,
+                    const void* z, int64_t nz_global, int64_t z_offset, int ghost, dfg_mesh* out) {
+  return guard([&] {
+    if (!out) dfg::fail(DFG_E_INVALID, "null output handle");
+    *out = nullptr;
+    auto m = dfg::create_mesh(to_dtype(dtype), nx, ny, nz_local, x, y, z, nz_global, z_offset, ghost);
+    *out = new dfg_mesh_s{std::move(m)};
+  });
+}
+
+void dfg_destroy_mesh(dfg_mesh mesh) { delete mesh; }
+
+int dfg_partition(int64_t nz_global, int nranks, int rank, int64_t* z_offset, int64_t* nz_local) {
+  return guard([&] {
+    if (nranks < 1 || nz_global < nranks || rank < 0 || rank >= nranks || !z_offset || !nz_local)
+      dfg::fail(DFG_E_INVALID, "need 1 <= nranks <= nz_global and 0 <= rank < nranks");
+    int64_t q = nz_global / nranks, r = nz_global % nranks;
+    *nz_local = q + (rank < r ? 1 : 0);
+    *z_offset = int64_t(rank) * q + (rank < r ? rank : r);
+  });
+}
+
+int dfg_halo_map(dfg_mesh mesh, int64_t out[16]) {
+  return guard([&] {
+    if (!mesh || !out) dfg::fail(DFG_E_INVALID, "null argument");
+    const dfg::MeshImpl& m = *mesh->m;
+    const int64_t k1 = m.k0 + m.nzl;
+    const int64_t lo = m.k0 > 0, hi = k1 < m.NZ;
+    int64_t v[16] = {m.rank,          m.nranks,         m.NZ,          m.k0,
+                     k1,              m.nzl,            lo,            hi,
+                     lo ? m.rank - 1 : -1, hi ? m.rank + 1 : -1, lo ? 1 : -1, hi ? m.nzl : -1,
+                     lo ? 0 : -1,     hi ? m.nzl + 1 : -1, m.nx * m.ny * int64_t(dfg::dsize(m.dt)), m.ghost};
+    std::memcpy(out, v, sizeof(v));
+  });
+}
+
+int dfg_nccl_unique_id(void* out128) {
+  return guard([&] {
+    if (!out128) dfg::fail(DFG_E_INVALID, "null buffer");
+    dfg::nccl_unique_id(out128);
+  });
+}
+
+int dfg_mesh_init_comm(dfg_mesh mesh, const void* id128, int rank, int nranks) {
+  return guard([&] {
+    if (!mesh || (!id128 && nranks > 1)) dfg::fail(DFG_E_INVALID, "null argument");
+    dfg::mesh_init_comm(*mesh->m, id128, rank, nranks);
+  });
+}
+
+int dfg_mesh_link_local(dfg_mesh lo, dfg_mesh hi) {
+  return guard([&] {
+    if (!lo || !hi) dfg::fail(DFG_E_INVALID, "null mesh");
+    auto& a = *lo->m;
+    auto& b = *hi->m;
+    if (a.k0 + a.nzl != b.k0 || a.NZ != b.NZ || a.nx != b.nx || a.ny != b.ny || a.dt != b.dt)
+      dfg::fail(DFG_E_INVALID, "meshes are not adjacent z slabs of one mesh");
+    a.link_hi = hi->m;
+    b.link_lo = lo->m;
+  });
+}
+
+int dfg_bind_field(dfg_mesh mesh, const char* name, void* ptr, int on_device) {
+  return guard([&] {
+    if (!mesh || !name) dfg::fail(DFG_E_INVALID, "null argument");
+    std::string n(name);
+    if (!dfg::valid_input_name(n)) dfg::fail(DFG_E_INVALID, "invalid field name '" + n + "'");
+    if (!ptr) {
+      mesh->m->fields.erase(n);
+      return;
+    }
+    if (on_device) {
+      cudaPointerAttributes a{};
+      if (cudaPointerGetAttributes(&a, ptr) != cudaSuccess || a.type != cudaMemoryTypeDevice) {
+        cudaGetLastError();
+        if (a.type != cudaMemoryTypeManaged)
+          dfg::fail(DFG_E_INVALID, "field '" + n + "' is not a device pointer");
+      }
+    }
+    mesh->m->fields[n] = dfg::Binding{ptr, on_device != 0};
+  });
+}
+
+int dfg_compile(dfg_mesh mesh, const char* expr, dfg_strategy strategy, size_t cap, dfg_plan* out) {
+  return guard([&] {
+    if (!mesh || !expr || !out) dfg::fail(DFG_E_INVALID, "null argument");
+    *out = nullptr;
+    auto p = dfg::compile_plan(mesh->m, expr, strategy, cap);
+    *out = new dfg_plan_s{std::move(p)};
+  });
+}
+
+void dfg_destroy_plan(dfg_plan plan) { delete plan; }
+
+int dfg_execute(dfg_plan plan, void* out, int out_on_device, void* stream) {
+  return guard([&] {
+    if (!plan) dfg::fail(DFG_E_INVALID, "null plan");
+    plan->p->execute(out, out_on_device != 0, static_cast<cudaStream_t>(stream));
+  });
+}
+
+int dfg_plan_stats(dfg_plan plan, dfg_stats* out) {
+  return guard([&] {
+    if (!plan || !out) dfg::fail(DFG_E_INVALID, "null argument");
+    auto& p = *plan->p;
+    if (p.timed) {
+      DFG_CUDA(cudaEventSynchronize(p.ev1));
+      float ms = 0;
+      DFG_CUDA(cudaEventElapsedTime(&ms, p.ev0, p.ev1));
+      p.st.last_ms = ms;
+    }
+    p.resolve_kernel_times();
+    *out = p.st;
+  });
+}
+
+int dfg_reset_stats(dfg_plan plan) {
+  return guard([&] {
+    if (!plan) dfg::fail(DFG_E_INVALID, "null plan");
+    plan->p->resolve_kernel_times();
+    plan->p->st = dfg_stats{};
+    plan->p->st.last_ms = -1;
+    plan->p->timed = false;
+  });
+}
+
+int dfg_plan_info(dfg_plan plan, int64_t out[8]) {
+  return guard([&] {
+    if (!plan || !out) dfg::fail(DFG_E_INVALID, "null argument");
+    auto& p = *plan->p;
+    const auto& m = *p.mesh;
+    out[0] = p.strategy;
+    out[1] = p.dag.width(p.dag.result) == 1 ? 1 : 4;
+    out[2] = int64_t(p.dag.filters.size());
+    out[3] = p.last_variant;
+    out[4] = p.regs > 0 ? p.regs : 0;
+    out[5] = p.spill > 0 ? p.spill : 0;
+    const int64_t unit = m.cells() * int64_t(dfg::dsize(m.dt));
+    out[6] = dfg::model(p.dag, p.strategy, false).units * unit;
+    out[7] = dfg::model(p.dag, p.strategy, true).units * unit;
+  });
+}
+
+int dfg_dump_dag(dfg_plan plan, char* buf, size_t cap, size_t* needed) {
+  return guard([&] {
+    if (!plan) dfg::fail(DFG_E_INVALID, "null plan");
+    copy_out(plan->p->dag.dump(), buf, cap, needed);
+  });
+}
+
+int dfg_dump_kernel(dfg_plan plan, char* buf, size_t cap, size_t* needed) {
+  return guard([&] {
+    if (!plan) dfg::fail(DFG_E_INVALID, "null plan");
+    copy_out(plan->p->fsrc.source, buf, cap, needed);
+  });
+}
+
+int dfg_dag_dump(const char* expr, const char* const* inputs, int n_inputs, dfg_dtype dtype, char* buf, size_t cap,
+                 size_t* needed) {
+  return guard([&] {
+    if (!expr) dfg::fail(DFG_E_INVALID, "null expression");
+    dfg::Dag d = dfg::build_dag(expr, names_of(inputs, n_inputs), to_dtype(dtype));
+    copy_out(d.dump(), buf, cap, needed);
+  });
+}
+
+int dfg_model(const char* expr, const char* const* inputs, int n_inputs, dfg_strategy strategy, int host_mode,
+              int64_t out[4]) {
+  return guard([&] {
+    if (!expr || !out) dfg::fail(DFG_E_INVALID, "null argument");
+    if (strategy != DFG_ROUNDTRIP && strategy != DFG_STAGED && strategy != DFG_FUSED)
+      dfg::fail(DFG_E_INVALID, "bad strategy");
+    dfg::Dag d = dfg::build_dag(expr, names_of(inputs, n_inputs), dfg::DType::F32);
+    dfg::Model m = dfg::model(d, strategy, host_mode != 0);
+    out[0] = m.h2d;
+    out[1] = m.d2h;
+    out[2] = m.kernels;
+    out[3] = m.units;
+  });
+}
+
+int dfg_fused_source(const char* expr, const char* const* inputs, int n_inputs, dfg_dtype dtype, int64_t nx,
+                     int64_t ny, int64_t nz, int compile, char* buf, size_t cap, size_t* needed, int* regs,
+                     int* spill) {
+  return guard([&] {
+    if (!expr) dfg::fail(DFG_E_INVALID, "null expression");
+    if (nx < 1 || ny < 1 || nz < 1) dfg::fail(DFG_E_INVALID, "mesh sizes must be >= 1");
+    dfg::Dag d = dfg::build_dag(expr, names_of(inputs, n_inputs), to_dtype(dtype));
+    dfg::FusedSource fs = dfg::generate_fused(d, nx, ny, nz, dfg::FusedConfig{});
+    if (compile) {
+      const dfg::Cubin& c = dfg::nvrtc_compile(fs.source, "dfg_fused.cu");
+      if (regs) *regs = c.regs;
+      if (spill) *spill = c.spill;
+    }
+    copy_out(fs.source, buf, cap, needed);
+  });
+}
+
+}  // extern "C"

@@ -1,0 +1,44 @@
+// Dynamic kernel generator of the fusion strategy:
+// one CUDA kernel per network, built from the building blocks of
+// blocks.cuh -- per-element calls for simple primitives (L101), direct
+// memory access for the gradient (L102), constants inserted as source
+// literals (L103), vector results as per-lane registers (L104) and
+// decompose as a register selection (L105).
+#pragma once
+
+#include <cstdint>
+#include <string>
+#include <vector>
+
+#include "lang.hpp"
+
+namespace dfg {
+
+struct FusedLayout {
+  std::vector<int> stencil_inputs;  // input indices read by some grad3d (+ centre)
+  std::vector<int> point_inputs;    // input indices read only at the cell
+  int outw = 1;                     // 1 or 4
+  bool has_grad = false;
+};
+
+struct FusedConfig {
+  int div_mode = 1;    // 0 ieee, 1 exact (Markstein), 2 fast; see blocks.cuh
+  int ncw = 15;        // consumer warps per CTA (tile rows); +1 producer = 512 threads
+  int stages = 0;      // smem ring depth (0: choose)
+  bool has_tma = false;
+};
+
+struct FusedSource {
+  std::string source;
+  FusedLayout layout;
+  FusedConfig cfg;
+};
+
+FusedLayout fused_layout(const Dag& dag);
+// nx/ny/nz: global mesh dims (axis degeneracy n == 1 is baked in).
+FusedSource generate_fused(const Dag& dag, int64_t nx, int64_t ny, int64_t nz, FusedConfig cfg);
+
+// Dynamic shared memory the TMA kernel needs for a config (bytes).
+size_t fused_tma_smem_bytes(DType dt, int nsf, int ncw, int stages);
+
+}  // namespace dfg

@@ -1,0 +1,231 @@
+// Precompiled per-primitive kernels of the roundtrip and staged strategies
+// ("one kernel is executed for each derived field
+// primitive").  Every kernel applies one building block of blocks.cuh, so
+// staged / roundtrip / fused evaluate identical arithmetic (L86, L90).
+//
+// All element kernels are HBM-bound streams: grid-stride loops over 16-byte
+// vectors (float4 / double2), grids sized to a multiple of the SM count,
+// 64-bit indices (a 1024^3 vector array has 2^32 elements).
+#include <cuda_runtime.h>
+
+#include <cstdint>
+
+#include "blocks.cuh"
+#include "kernels.hpp"
+
+namespace dfg {
+namespace kern {
+
+namespace {
+
+template <typename T> struct V16;
+template <> struct V16<float> { using type = float4; };
+template <> struct V16<double> { using type = double2; };
+
+template <typename T> __device__ __forceinline__ void unpack(const typename V16<T>::type& v, T* d);
+template <> __device__ __forceinline__ void unpack<float>(const float4& v, float* d) {
+  d[0] = v.x; d[1] = v.y; d[2] = v.z; d[3] = v.w;
+}
+template <> __device__ __forceinline__ void unpack<double>(const double2& v, double* d) {
+  d[0] = v.x; d[1] = v.y;
+}
+template <typename T> __device__ __forceinline__ typename V16<T>::type pack(const T* s);
+template <> __device__ __forceinline__ float4 pack<float>(const float* s) { return make_float4(s[0], s[1], s[2], s[3]); }
+template <> __device__ __forceinline__ double2 pack<double>(const double* s) { return make_double2(s[0], s[1]); }
+
+int g_sms = 0;
+int sms() {
+  if (!g_sms) {
+    int dev = 0;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&g_sms, cudaDevAttrMultiProcessorCount, dev);
+    if (g_sms <= 0) g_sms = 148;
+  }
+  return g_sms;
+}
+
+unsigned grid_for(long long work, int block) {
+  long long g = (work + block - 1) / block;
+  long long cap = (long long)sms() * 8;
+  if (g > cap) g = cap;
+  if (g < 1) g = 1;
+  return (unsigned)g;
+}
+
+bool aligned16(const void* p) { return (reinterpret_cast<uintptr_t>(p) & 15) == 0; }
+
+// Element-wise kernel over up to three inputs; F is a block from blocks.cuh.
+template <typename T, typename F, int NIN>
+__global__ void __launch_bounds__(256) k_elementwise(const T* __restrict__ a, const T* __restrict__ b,
+                                                     const T* __restrict__ c, T* __restrict__ o, long long n,
+                                                     int vec_ok, F fn) {
+  constexpr int V = 16 / sizeof(T);
+  using VT = typename V16<T>::type;
+  const long long tid = (long long)blockIdx.x * blockDim.x + threadIdx.x;
+  const long long stride = (long long)gridDim.x * blockDim.x;
+  const long long nv = vec_ok ? n / V : 0;
+  for (long long v = tid; v < nv; v += stride) {
+    T x[V], y[V], z[V], r[V];
+    if (NIN > 0) unpack<T>(__ldcs(reinterpret_cast<const VT*>(a) + v), x);
+    if (NIN > 1) unpack<T>(__ldcs(reinterpret_cast<const VT*>(b) + v), y);
+    if (NIN > 2) unpack<T>(__ldcs(reinterpret_cast<const VT*>(c) + v), z);
+#pragma unroll
+    for (int e = 0; e < V; ++e) r[e] = fn(x[e], y[e], z[e]);
+    __stcs(reinterpret_cast<VT*>(o) + v, pack<T>(r));
+  }
+  for (long long e = nv * V + tid; e < n; e += stride) {
+    T x = NIN > 0 ? a[e] : T(0), y = NIN > 1 ? b[e] : T(0), z = NIN > 2 ? c[e] : T(0);
+    o[e] = fn(x, y, z);
+  }
+}
+
+#define DFG_FN2(NAME)                                                                    \
+  struct F_##NAME {                                                                      \
+    template <typename T> __device__ __forceinline__ T operator()(T a, T b, T) const {   \
+      return dfg_##NAME(a, b);                                                           \
+    }                                                                                    \
+  };
+DFG_FN2(add) DFG_FN2(sub) DFG_FN2(mult) DFG_FN2(div)
+DFG_FN2(gt) DFG_FN2(lt) DFG_FN2(ge) DFG_FN2(le) DFG_FN2(eq) DFG_FN2(ne)
+#undef DFG_FN2
+struct F_neg {
+  template <typename T> __device__ __forceinline__ T operator()(T a, T, T) const { return dfg_neg(a); }
+};
+struct F_sqrt {
+  template <typename T> __device__ __forceinline__ T operator()(T a, T, T) const { return dfg_sqrt(a); }
+};
+struct F_select {
+  template <typename T> __device__ __forceinline__ T operator()(T c, T a, T b) const { return dfg_select(c, a, b); }
+};
+template <typename T> struct F_fill {
+  T v;
+  __device__ __forceinline__ T operator()(T, T, T) const { return v; }
+};
+
+template <typename T, typename F, int NIN>
+void launch_ew(const void* a, const void* b, const void* c, void* o, long long n, F fn, cudaStream_t s) {
+  constexpr int V = 16 / sizeof(T);
+  int vec_ok = aligned16(o) && (NIN < 1 || aligned16(a)) && (NIN < 2 || aligned16(b)) && (NIN < 3 || aligned16(c));
+  k_elementwise<T, F, NIN><<<grid_for(vec_ok ? n / V + 1 : n, 256), 256, 0, s>>>(
+      (const T*)a, (const T*)b, (const T*)c, (T*)o, n, vec_ok, fn);
+}
+
+template <typename T>
+void binary_t(Op op, const void* a, const void* b, void* o, long long n, cudaStream_t s) {
+  switch (op) {
+    case Op::Add: return launch_ew<T, F_add, 2>(a, b, nullptr, o, n, F_add{}, s);
+    case Op::Sub: return launch_ew<T, F_sub, 2>(a, b, nullptr, o, n, F_sub{}, s);
+    case Op::Mult: return launch_ew<T, F_mult, 2>(a, b, nullptr, o, n, F_mult{}, s);
+    case Op::Div: return launch_ew<T, F_div, 2>(a, b, nullptr, o, n, F_div{}, s);
+    case Op::Gt: return launch_ew<T, F_gt, 2>(a, b, nullptr, o, n, F_gt{}, s);
+    case Op::Lt: return launch_ew<T, F_lt, 2>(a, b, nullptr, o, n, F_lt{}, s);
+    case Op::Ge: return launch_ew<T, F_ge, 2>(a, b, nullptr, o, n, F_ge{}, s);
+    case Op::Le: return launch_ew<T, F_le, 2>(a, b, nullptr, o, n, F_le{}, s);
+    case Op::Eq: return launch_ew<T, F_eq, 2>(a, b, nullptr, o, n, F_eq{}, s);
+    case Op::Ne: return launch_ew<T, F_ne, 2>(a, b, nullptr, o, n, F_ne{}, s);
+    default: break;
+  }
+}
+
+// AoS 4-wide vector (L104) -> scalar lane
+template <typename T>
+__global__ void __launch_bounds__(256) k_decompose(const T* __restrict__ v4, int lane, T* __restrict__ o, long long n) {
+  const long long stride = (long long)gridDim.x * blockDim.x;
+  for (long long e = (long long)blockIdx.x * blockDim.x + threadIdx.x; e < n; e += stride)
+    o[e] = __ldcs(v4 + 4 * e + lane);
+}
+
+template <typename T>
+__global__ void __launch_bounds__(256) k_compose(const T* __restrict__ a, const T* __restrict__ b,
+                                                 const T* __restrict__ c, const T* __restrict__ d, int w,
+                                                 T* __restrict__ o, long long n) {
+  const long long stride = (long long)gridDim.x * blockDim.x;
+  for (long long e = (long long)blockIdx.x * blockDim.x + threadIdx.x; e < n; e += stride) {
+    T r[4] = {a[e], b[e], w > 2 ? c[e] : T(0), w > 3 ? d[e] : T(0)};
+#pragma unroll
+    for (int l = 0; l < 4; ++l) o[4 * e + l] = r[l];
+  }
+}
+
+// grad3d of a cell-centred scalar (reading R1) -> AoS 4-wide (lane 3 = 0).
+// f points at local plane 0 of a T[nzl + 2*ghost][ny][nx] buffer.
+template <typename T>
+__global__ void __launch_bounds__(256) k_grad3d(const T* __restrict__ f, T* __restrict__ o, const T* __restrict__ tx,
+                                                const T* __restrict__ ty, const T* __restrict__ tz, long long nx,
+                                                long long ny, long long nzl, long long NZ, long long k0,
+                                                long long ghost) {
+  const long long plane = nx * ny;
+  const long long n = plane * nzl;
+  const long long stride = (long long)gridDim.x * blockDim.x;
+  for (long long c = (long long)blockIdx.x * blockDim.x + threadIdx.x; c < n; c += stride) {
+    const long long i = c % nx, t = c / nx, j = t % ny, kl = t / ny, kg = k0 + kl;
+    const long long base = (kl + ghost) * plane + j * nx + i;
+    T g[4];
+    g[0] = nx == 1 ? T(0) : dfg_grad1(f[base + (i < nx - 1 ? 1 : 0)], f[base - (i > 0 ? 1 : 0)], tx[i], tx[nx + i]);
+    g[1] = ny == 1 ? T(0) : dfg_grad1(f[base + (j < ny - 1 ? nx : 0)], f[base - (j > 0 ? nx : 0)], ty[j], ty[ny + j]);
+    g[2] = NZ == 1 ? T(0)
+                   : dfg_grad1(f[base + (kg < NZ - 1 ? plane : 0)], f[base - (kg > 0 ? plane : 0)], tz[kg], tz[NZ + kg]);
+    g[3] = T(0);
+    T* dst = o + 4 * c;
+#pragma unroll
+    for (int l = 0; l < 4; ++l) dst[l] = g[l];
+  }
+}
+
+}  // namespace
+
+void binary(Op op, DType dt, const void* a, const void* b, void* o, long long n, cudaStream_t s) {
+  if (dt == DType::F32) binary_t<float>(op, a, b, o, n, s);
+  else binary_t<double>(op, a, b, o, n, s);
+}
+
+void unary(Op op, DType dt, const void* a, void* o, long long n, cudaStream_t s) {
+  if (dt == DType::F32) {
+    if (op == Op::Neg) launch_ew<float, F_neg, 1>(a, nullptr, nullptr, o, n, F_neg{}, s);
+    else launch_ew<float, F_sqrt, 1>(a, nullptr, nullptr, o, n, F_sqrt{}, s);
+  } else {
+    if (op == Op::Neg) launch_ew<double, F_neg, 1>(a, nullptr, nullptr, o, n, F_neg{}, s);
+    else launch_ew<double, F_sqrt, 1>(a, nullptr, nullptr, o, n, F_sqrt{}, s);
+  }
+}
+
+void select(DType dt, const void* c, const void* a, const void* b, void* o, long long n, cudaStream_t s) {
+  if (dt == DType::F32) launch_ew<float, F_select, 3>(c, a, b, o, n, F_select{}, s);
+  else launch_ew<double, F_select, 3>(c, a, b, o, n, F_select{}, s);
+}
+
+void fill(DType dt, double v, void* o, long long n, cudaStream_t s) {
+  if (dt == DType::F32) launch_ew<float, F_fill<float>, 0>(nullptr, nullptr, nullptr, o, n, F_fill<float>{float(v)}, s);
+  else launch_ew<double, F_fill<double>, 0>(nullptr, nullptr, nullptr, o, n, F_fill<double>{v}, s);
+}
+
+void decompose(DType dt, const void* v4, int lane, void* o, long long n, cudaStream_t s) {
+  if (dt == DType::F32) k_decompose<float><<<grid_for(n, 256), 256, 0, s>>>((const float*)v4, lane, (float*)o, n);
+  else k_decompose<double><<<grid_for(n, 256), 256, 0, s>>>((const double*)v4, lane, (double*)o, n);
+}
+
+void compose(DType dt, const void* const* in, int w, void* o, long long n, cudaStream_t s) {
+  const void* c = w > 2 ? in[2] : in[0];
+  const void* d = w > 3 ? in[3] : in[0];
+  if (dt == DType::F32)
+    k_compose<float><<<grid_for(n, 256), 256, 0, s>>>((const float*)in[0], (const float*)in[1], (const float*)c,
+                                                      (const float*)d, w, (float*)o, n);
+  else
+    k_compose<double><<<grid_for(n, 256), 256, 0, s>>>((const double*)in[0], (const double*)in[1], (const double*)c,
+                                                       (const double*)d, w, (double*)o, n);
+}
+
+void grad3d(DType dt, const void* f, void* o4, const void* tx, const void* ty, const void* tz, long long nx,
+            long long ny, long long nzl, long long NZ, long long k0, long long ghost, cudaStream_t s) {
+  long long n = nx * ny * nzl;
+  if (dt == DType::F32)
+    k_grad3d<float><<<grid_for(n, 256), 256, 0, s>>>((const float*)f, (float*)o4, (const float*)tx,
+                                                     (const float*)ty, (const float*)tz, nx, ny, nzl, NZ, k0, ghost);
+  else
+    k_grad3d<double><<<grid_for(n, 256), 256, 0, s>>>((const double*)f, (double*)o4, (const double*)tx,
+                                                      (const double*)ty, (const double*)tz, nx, ny, nzl, NZ, k0,
+                                                      ghost);
+}
+
+}  // namespace kern
+}  // namespace dfg

@@ -1,0 +1,23 @@
+// Launchers of the per-primitive kernels (kernels.cu).  Sizes are element
+// counts; vector arrays are AoS 4-wide.  All launches are asynchronous on `s`.
+#pragma once
+
+#include <cuda_runtime.h>
+
+#include "lang.hpp"
+
+namespace dfg {
+namespace kern {
+
+void binary(Op op, DType dt, const void* a, const void* b, void* o, long long n, cudaStream_t s);
+void unary(Op op, DType dt, const void* a, void* o, long long n, cudaStream_t s);  // Neg, Sqrt
+void select(DType dt, const void* c, const void* a, const void* b, void* o, long long n, cudaStream_t s);
+void fill(DType dt, double v, void* o, long long n, cudaStream_t s);
+void decompose(DType dt, const void* v4, int lane, void* o, long long n, cudaStream_t s);
+void compose(DType dt, const void* const* in, int w, void* o4, long long n, cudaStream_t s);
+// f: local plane 0 of T[nzl + 2*ghost][ny][nx]; tables d[n] then r[n]; tz global.
+void grad3d(DType dt, const void* f, void* o4, const void* tx, const void* ty, const void* tz, long long nx,
+            long long ny, long long nzl, long long NZ, long long k0, long long ghost, cudaStream_t s);
+
+}  // namespace kern
+}  // namespace dfg

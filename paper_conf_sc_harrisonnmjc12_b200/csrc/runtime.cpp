@@ -1,0 +1,1120 @@
+// libdfg runtime.  See runtime.hpp; DESIGN.md sections 2, 5 and 6.
+#include "runtime.hpp"
+
+#include <dlfcn.h>
+#include <nccl.h>
+
+#include <algorithm>
+#include <cmath>
+#include <cstdlib>
+#include <cstring>
+#include <mutex>
+#include <set>
+
+#include "driver.hpp"
+#include "kernels.hpp"
+
+namespace dfg {
+
+// ====================================================================== mesh
+namespace {
+
+template <typename T>
+void build_axis(const T* p, int64_t n, std::vector<char>& tab, bool& safe) {
+  // Reading R1: centres c_i = (p_i + p_{i+1}) * 0.5 in T; for each cell the
+  // clamped neighbour-centre distance d_i = c[ip] - c[im] and r_i = RN(1/d_i).
+  for (int64_t i = 0; i <= n; ++i)
+    if (!std::isfinite(double(p[i]))) fail(DFG_E_INVALID, "coordinates must be finite");
+  for (int64_t i = 0; i < n; ++i)
+    if (!(p[i] < p[i + 1])) fail(DFG_E_INVALID, "coordinates must be strictly increasing");
+  std::vector<T> c(n);
+  for (int64_t i = 0; i < n; ++i) c[i] = (p[i] + p[i + 1]) * T(0.5);
+  tab.assign(size_t(2 * n) * sizeof(T), 0);
+  T* d = reinterpret_cast<T*>(tab.data());
+  T* r = d + n;
+  for (int64_t i = 0; i < n; ++i) {
+    if (n == 1) {  // derivative is 0 by definition; the kernels never read these
+      d[i] = T(1);
+      r[i] = T(1);
+      continue;
+    }
+    int64_t ip = std::min(i + 1, n - 1), im = std::max<int64_t>(i - 1, 0);
+    d[i] = c[ip] - c[im];
+    if (!(d[i] > T(0))) fail(DFG_E_INVALID, "cell centres coincide (coordinates too close for T)");
+    r[i] = T(1) / d[i];
+    // Markstein's exact-quotient argument needs d and r well inside the normal range.
+    double ad = double(d[i]);
+    if (!(ad > 0x1p-60 && ad < 0x1p60) || !std::isfinite(double(r[i]))) safe = false;
+  }
+}
+
+std::mutex g_pool_mu;
+std::map<int, cudaMemPool_t> g_pools;
+
+cudaMemPool_t pool_for(int dev) {
+  std::lock_guard<std::mutex> lk(g_pool_mu);
+  auto it = g_pools.find(dev);
+  if (it != g_pools.end()) return it->second;
+  cudaMemPoolProps props{};
+  props.allocType = cudaMemAllocationTypePinned;
+  props.location.type = cudaMemLocationTypeDevice;
+  props.location.id = dev;
+  cudaMemPool_t pool;
+  DFG_CUDA(cudaMemPoolCreate(&pool, &props));
+  uint64_t thr = UINT64_MAX;
+  DFG_CUDA(cudaMemPoolSetAttribute(pool, cudaMemPoolAttrReleaseThreshold, &thr));
+  g_pools[dev] = pool;
+  return pool;
+}
+
+int sm_count(int dev) {
+  static std::map<int, int> cache;
+  static std::mutex mu;
+  std::lock_guard<std::mutex> lk(mu);
+  auto it = cache.find(dev);
+  if (it != cache.end()) return it->second;
+  int n = 0;
+  DFG_CUDA(cudaDeviceGetAttribute(&n, cudaDevAttrMultiProcessorCount, dev));
+  cache[dev] = n;
+  return n;
+}
+
+}  // namespace
+
+MeshImpl::~MeshImpl() {
+  int cur = -1;
+  cudaGetDevice(&cur);
+  cudaSetDevice(device);
+  for (auto& p : dev_tab)
+    if (p) cudaFree(p);
+  if (nccl) {
+    using destroy_fn = ncclResult_t (*)(ncclComm_t);
+    void* h = dlopen("libnccl.so.2", RTLD_NOW | RTLD_NOLOAD);
+    if (h) {
+      auto f = reinterpret_cast<destroy_fn>(dlsym(h, "ncclCommDestroy"));
+      if (f) f(static_cast<ncclComm_t>(nccl));
+    }
+  }
+  if (cur >= 0) cudaSetDevice(cur);
+}
+
+std::shared_ptr<MeshImpl> create_mesh(DType dt, int64_t nx, int64_t ny, int64_t nzl, const void* x, const void* y,
+                                      const void* z, int64_t NZ, int64_t k0, int ghost) {
+  if (nx < 1 || ny < 1 || nzl < 1 || NZ < 1) fail(DFG_E_INVALID, "mesh sizes must be >= 1");
+  if (k0 < 0 || k0 + nzl > NZ) fail(DFG_E_INVALID, "z slab outside the global mesh");
+  if (ghost != 0 && ghost != 1) fail(DFG_E_INVALID, "ghost must be 0 or 1");
+  if (nzl != NZ && ghost != 1) fail(DFG_E_INVALID, "a z slab of a larger mesh needs ghost = 1");
+  if (!x || !y || !z) fail(DFG_E_INVALID, "null coordinate pointer");
+  auto m = std::make_shared<MeshImpl>();
+  m->dt = dt;
+  m->nx = nx;
+  m->ny = ny;
+  m->nzl = nzl;
+  m->NZ = NZ;
+  m->k0 = k0;
+  m->ghost = ghost;
+  const void* P[3] = {x, y, z};
+  int64_t N[3] = {nx, ny, NZ};
+  for (int a = 0; a < 3; ++a) {
+    if (dt == DType::F32) build_axis(static_cast<const float*>(P[a]), N[a], m->host_tab[a], m->markstein_safe);
+    else build_axis(static_cast<const double*>(P[a]), N[a], m->host_tab[a], m->markstein_safe);
+  }
+  int ndev = 0;
+  if (cudaGetDeviceCount(&ndev) != cudaSuccess || ndev < 1) {
+    cudaGetLastError();
+    fail(DFG_E_CUDA, "no CUDA device available (libdfg has no CPU fallback)");
+  }
+  DFG_CUDA(cudaGetDevice(&m->device));
+  for (int a = 0; a < 3; ++a) {
+    DFG_CUDA(cudaMalloc(&m->dev_tab[a], m->host_tab[a].size()));
+    DFG_CUDA(cudaMemcpy(m->dev_tab[a], m->host_tab[a].data(), m->host_tab[a].size(), cudaMemcpyHostToDevice));
+  }
+  return m;
+}
+
+// ===================================================================== NCCL
+namespace {
+struct NcclApi {
+  void* h = nullptr;
+  ncclResult_t (*GetUniqueId)(ncclUniqueId*) = nullptr;
+  ncclResult_t (*CommInitRank)(ncclComm_t*, int, ncclUniqueId, int) = nullptr;
+  ncclResult_t (*Send)(const void*, size_t, ncclDataType_t, int, ncclComm_t, cudaStream_t) = nullptr;
+  ncclResult_t (*Recv)(void*, size_t, ncclDataType_t, int, ncclComm_t, cudaStream_t) = nullptr;
+  ncclResult_t (*GroupStart)() = nullptr;
+  ncclResult_t (*GroupEnd)() = nullptr;
+  const char* (*GetErrorString)(ncclResult_t) = nullptr;
+};
+
+NcclApi& nccl() {
+  static NcclApi api;
+  static std::once_flag once;
+  std::call_once(once, [] {
+    // Prefer the NCCL the process already loaded (torch's), else the system one.
+    void* h = dlopen("libnccl.so.2", RTLD_NOW | RTLD_NOLOAD);
+    if (!h) h = dlopen("libnccl.so.2", RTLD_NOW | RTLD_GLOBAL);
+    if (!h) h = dlopen("libnccl.so", RTLD_NOW | RTLD_GLOBAL);
+    if (!h) return;
+    api.h = h;
+    api.GetUniqueId = reinterpret_cast<decltype(api.GetUniqueId)>(dlsym(h, "ncclGetUniqueId"));
+    api.CommInitRank = reinterpret_cast<decltype(api.CommInitRank)>(dlsym(h, "ncclCommInitRank"));
+    api.Send = reinterpret_cast<decltype(api.Send)>(dlsym(h, "ncclSend"));
+    api.Recv = reinterpret_cast<decltype(api.Recv)>(dlsym(h, "ncclRecv"));
+    api.GroupStart = reinterpret_cast<decltype(api.GroupStart)>(dlsym(h, "ncclGroupStart"));
+    api.GroupEnd = reinterpret_cast<decltype(api.GroupEnd)>(dlsym(h, "ncclGroupEnd"));
+    api.GetErrorString = reinterpret_cast<decltype(api.GetErrorString)>(dlsym(h, "ncclGetErrorString"));
+  });
+  if (!api.h || !api.GetUniqueId || !api.CommInitRank || !api.Send || !api.Recv || !api.GroupStart ||
+      !api.GroupEnd)
+    fail(DFG_E_NCCL, "NCCL (libnccl.so.2) could not be loaded");
+  return api;
+}
+
+void nccl_check(ncclResult_t r, const char* what) {
+  if (r != ncclSuccess) {
+    const char* s = nccl().GetErrorString ? nccl().GetErrorString(r) : "?";
+    fail(DFG_E_NCCL, std::string(what) + ": " + s);
+  }
+}
+}  // namespace
+
+void nccl_unique_id(void* out128) {
+  ncclUniqueId id;
+  nccl_check(nccl().GetUniqueId(&id), "ncclGetUniqueId");
+  static_assert(sizeof(id) == 128, "ncclUniqueId is 128 bytes");
+  std::memcpy(out128, &id, 128);
+}
+
+void mesh_init_comm(MeshImpl& m, const void* id128, int rank, int nranks) {
+  if (nranks < 1 || rank < 0 || rank >= nranks) fail(DFG_E_INVALID, "bad rank/nranks");
+  if (nranks == 1) {
+    m.rank = 0;
+    m.nranks = 1;
+    return;
+  }
+  ncclUniqueId id;
+  std::memcpy(&id, id128, 128);
+  DFG_CUDA(cudaSetDevice(m.device));
+  ncclComm_t comm;
+  nccl_check(nccl().CommInitRank(&comm, nranks, id, rank), "ncclCommInitRank");
+  m.nccl = comm;
+  m.rank = rank;
+  m.nranks = nranks;
+}
+
+// ==================================================================== model
+namespace {
+struct Sources {
+  std::vector<int> inputs;  // first-use order (+ bare result)
+  bool mesh = false;
+};
+Sources sources(const Dag& dag) {
+  Sources s;
+  auto note = [&](const Ref& r) {
+    if (r.kind == Ref::Mesh) s.mesh = true;
+    else if (r.kind == Ref::Input && std::find(s.inputs.begin(), s.inputs.end(), r.id) == s.inputs.end())
+      s.inputs.push_back(r.id);
+  };
+  for (auto& f : dag.filters)
+    for (auto& r : f.in) note(r);
+  if (dag.result.kind == Ref::Input) note(dag.result);
+  return s;
+}
+int64_t units(const Dag& dag, const Ref& r) { return dag.width(r) == 1 ? 1 : 4; }
+bool host_side(Op op) { return op == Op::Decompose || op == Op::Const; }  // roundtrip: no kernel
+}  // namespace
+
+Model model(const Dag& dag, dfg_strategy s, bool host) {
+  Model m;
+  Sources src = sources(dag);
+  const int64_t F = int64_t(dag.filters.size());
+  const bool bare = dag.result.kind != Ref::Filter;
+  const int64_t out_u = units(dag, dag.result);
+  int64_t in_u = 0;
+  for (int i : src.inputs) (void)i, in_u += 1;
+  // ---- counts (Table II rules, R11-R13)
+  if (s == DFG_FUSED) {
+    m.kernels = 1;
+    if (host) { m.h2d = int64_t(src.inputs.size()) + (src.mesh ? 4 : 0); m.d2h = 1; }
+  } else if (s == DFG_STAGED) {
+    m.kernels = F;
+    if (host) { m.h2d = int64_t(src.inputs.size()) + (src.mesh ? 4 : 0); m.d2h = 1; }
+  } else {
+    for (auto& f : dag.filters) {
+      if (host_side(f.op)) continue;
+      m.kernels += 1;
+      m.d2h += 1;
+      for (auto& r : f.in) {
+        if (host) m.h2d += 1;                    // every argument of every kernel
+        else if (r.kind == Ref::Filter) m.h2d += 1;  // only host-resident values
+      }
+    }
+    if (!host && !bare) m.h2d += 1;              // final result to the device output
+  }
+  // ---- footprint (Fig. 2 rules)
+  if (s == DFG_FUSED) {
+    m.units = in_u + out_u;
+  } else if (s == DFG_ROUNDTRIP) {
+    int64_t base = host ? 0 : in_u + out_u, high = base;
+    for (size_t k = 0; k < dag.filters.size(); ++k) {
+      const Filter& f = dag.filters[k];
+      if (host_side(f.op)) continue;
+      int64_t args = 0;
+      for (auto& r : f.in) {
+        if (r.kind == Ref::Mesh) continue;
+        if (!host && r.kind == Ref::Input) continue;
+        args += units(dag, r);
+      }
+      high = std::max(high, base + args + units(dag, Ref{Ref::Filter, int(k)}));
+    }
+    m.units = high;
+  } else {
+    std::map<std::pair<int, int>, int64_t> rc;
+    auto key = [](const Ref& r) { return std::make_pair(int(r.kind), r.id); };
+    for (auto& f : dag.filters)
+      for (auto& r : f.in)
+        if (r.kind != Ref::Mesh) rc[key(r)] += 1;
+    rc[key(dag.result)] += 1;
+    std::set<int> resident;
+    int64_t live = 0, high = 0;
+    if (!host) {
+      live = in_u + out_u;
+      for (int i : src.inputs) resident.insert(i);
+      high = live;
+    }
+    for (size_t k = 0; k < dag.filters.size(); ++k) {
+      const Filter& f = dag.filters[k];
+      for (auto& r : f.in)
+        if (r.kind == Ref::Input && !resident.count(r.id)) {
+          resident.insert(r.id);
+          live += 1;
+        }
+      bool into_out = !host && dag.result.kind == Ref::Filter && dag.result.id == int(k) && k + 1 == dag.filters.size();
+      if (!into_out) live += f.width == 1 ? 1 : 4;
+      high = std::max(high, live);
+      for (auto& r : f.in) {
+        if (r.kind == Ref::Mesh) continue;
+        if (--rc[key(r)] == 0 && (host || r.kind == Ref::Filter)) live -= units(dag, r);
+      }
+    }
+    if (dag.result.kind == Ref::Input && !resident.count(dag.result.id)) {
+      live += 1;
+      high = std::max(high, live);
+    }
+    m.units = high;
+  }
+  return m;
+}
+
+int64_t predicted_device_bytes(const Dag& dag, dfg_strategy s, int64_t cells, size_t ts) {
+  // Algorithmic device-memory bytes of one execute:
+  // fused reads every input once and writes the result once; staged and
+  // roundtrip read every kernel argument and write every kernel result.
+  Sources src = sources(dag);
+  int64_t u = 0;
+  if (s == DFG_FUSED) {
+    u = int64_t(src.inputs.size()) + units(dag, dag.result);
+  } else {
+    for (size_t k = 0; k < dag.filters.size(); ++k) {
+      const Filter& f = dag.filters[k];
+      if (s == DFG_ROUNDTRIP && host_side(f.op)) continue;
+      for (auto& r : f.in)
+        if (r.kind != Ref::Mesh) u += units(dag, r);
+      u += f.width == 1 ? 1 : 4;
+    }
+  }
+  return u * cells * int64_t(ts);
+}
+
+int64_t predicted_pcie_bytes(const Dag& dag, dfg_strategy s, int64_t cells, size_t ts, bool host) {
+  Sources src = sources(dag);
+  int64_t u = 0;
+  if (s != DFG_ROUNDTRIP) {
+    if (host) u = int64_t(src.inputs.size()) + units(dag, dag.result);
+  } else {
+    for (auto& f : dag.filters) {
+      if (host_side(f.op)) continue;
+      for (auto& r : f.in)
+        if (r.kind != Ref::Mesh && (host || r.kind == Ref::Filter)) u += units(dag, r);
+      u += f.width == 1 ? 1 : 4;
+    }
+  }
+  return u * cells * int64_t(ts);
+}
+
+// ==================================================================== plans
+namespace {
+
+struct Ledger {
+  size_t cap, live = 0, high = 0;
+  explicit Ledger(size_t c) : cap(c) {}
+  void add(size_t b) {
+    if (cap && live + b > cap)
+      fail(DFG_E_NOMEM, "device memory cap exceeded: " + std::to_string(live + b) + " > " + std::to_string(cap) +
+                            " bytes");
+    live += b;
+    high = std::max(high, live);
+  }
+  void sub(size_t b) { live -= std::min(live, b); }
+};
+
+struct DevBuf {
+  void* p = nullptr;
+  size_t bytes = 0;
+  bool owned = false;     // allocated by this execute
+  bool counted = false;   // problem-sized: tracked by the ledger
+};
+
+void* dev_alloc(size_t bytes, int dev, cudaStream_t s) {
+  void* p = nullptr;
+  cudaError_t e = cudaMallocFromPoolAsync(&p, bytes ? bytes : 16, pool_for(dev), s);
+  if (e != cudaSuccess) {
+    cudaGetLastError();
+    fail(e == cudaErrorMemoryAllocation ? DFG_E_NOMEM : DFG_E_CUDA,
+         std::string("device allocation of ") + std::to_string(bytes) + " bytes failed: " + cudaGetErrorString(e));
+  }
+  return p;
+}
+
+bool aligned16(const void* p) { return (reinterpret_cast<uintptr_t>(p) & 15) == 0; }
+
+struct HostPool {
+  std::multimap<size_t, void*> free_;
+  std::vector<void*> all;
+  void* get(size_t b) {
+    auto it = free_.lower_bound(b);
+    if (it != free_.end() && it->first < 2 * b + 4096) {
+      void* p = it->second;
+      free_.erase(it);
+      return p;
+    }
+    void* p = nullptr;
+    DFG_CUDA(cudaHostAlloc(&p, b ? b : 16, cudaHostAllocDefault));
+    all.push_back(p);
+    sizes[p] = b;
+    return p;
+  }
+  void put(void* p) { free_.emplace(sizes[p], p); }
+  std::map<void*, size_t> sizes;
+  ~HostPool() {
+    for (void* p : all) cudaFreeHost(p);
+  }
+};
+
+// one pool per plan would pin memory per plan; share per process instead
+HostPool& host_pool() {
+  static HostPool* pool = new HostPool();  // leaked on purpose: outlives plans at exit
+  return *pool;
+}
+std::mutex g_host_mu;
+
+}  // namespace
+
+PlanImpl::~PlanImpl() {
+  int cur = -1;
+  cudaGetDevice(&cur);
+  if (mesh) cudaSetDevice(mesh->device);
+  if (ev0) cudaEventDestroy(ev0);
+  if (ev1) cudaEventDestroy(ev1);
+  for (auto* v : {&kev_free, &kev_pending})
+    for (auto& e : *v) {
+      cudaEventDestroy(e.first);
+      cudaEventDestroy(e.second);
+    }
+  if (mod.mod) drv().ModuleUnload(mod.mod);
+  if (cur >= 0) cudaSetDevice(cur);
+}
+
+std::unique_ptr<PlanImpl> compile_plan(std::shared_ptr<MeshImpl> mesh, const std::string& expr, dfg_strategy s,
+                                       size_t cap) {
+  if (s != DFG_ROUNDTRIP && s != DFG_STAGED && s != DFG_FUSED) fail(DFG_E_INVALID, "bad strategy");
+  std::vector<std::string> names;
+  for (auto& kv : mesh->fields) names.push_back(kv.first);
+  auto plan = std::make_unique<PlanImpl>();
+  plan->mesh = mesh;
+  plan->strategy = s;
+  plan->cap = cap;
+  plan->dag = build_dag(expr, names, mesh->dt);
+  const Dag& dag = plan->dag;
+  const bool multi = mesh->nzl != mesh->NZ;
+  if (multi && s != DFG_FUSED)
+    fail(DFG_E_UNSUPPORTED, "staged/roundtrip run on a single slab; multi-slab meshes use the fused strategy");
+
+  // Footprint check against the cap for the binding modes at compile time
+  bool any_host = false;
+  for (int i : sources(dag).inputs)
+    if (!mesh->fields[dag.inputs[i]].on_device) any_host = true;
+  Model mdl = model(dag, s, any_host);
+  size_t need = size_t(mdl.units) * size_t(mesh->cells()) * dsize(mesh->dt);
+  if (cap && need > cap)
+    fail(DFG_E_NOMEM, "predicted device footprint " + std::to_string(need) + " bytes exceeds the cap " +
+                          std::to_string(cap));
+
+  DFG_CUDA(cudaSetDevice(mesh->device));
+  DFG_CUDA(cudaEventCreate(&plan->ev0));
+  DFG_CUDA(cudaEventCreate(&plan->ev1));
+  plan->st.last_ms = -1;
+
+  if (s == DFG_FUSED) {
+    FusedConfig cfg;
+    const char* var = std::getenv("DFG_FUSED_VARIANT");
+    if (var && !std::strcmp(var, "ieee")) cfg.div_mode = 0;
+    else if (var && !std::strcmp(var, "fast")) cfg.div_mode = 2;
+    if (!mesh->markstein_safe && cfg.div_mode == 1) cfg.div_mode = 0;  // keep results exact
+    const char* ncw = std::getenv("DFG_NCW");
+    if (ncw) cfg.ncw = std::max(1, std::min(30, std::atoi(ncw)));
+    const char* st = std::getenv("DFG_STAGES");
+    if (st) cfg.stages = std::max(2, std::min(16, std::atoi(st)));
+    plan->fsrc = generate_fused(dag, mesh->nx, mesh->ny, mesh->NZ, cfg);
+    const Cubin& cb = nvrtc_compile(plan->fsrc.source, "dfg_fused.cu");
+    plan->regs = cb.regs;
+    plan->spill = cb.spill;
+    // the runtime API owns the primary context; make it current for the driver API
+    DFG_CUDA(cudaFree(0));
+    plan->mod = load_module(cb);
+    if (plan->mod.tma) {
+      size_t smem = fused_tma_smem_bytes(mesh->dt, int(plan->fsrc.layout.stencil_inputs.size()), plan->fsrc.cfg.ncw,
+                                         plan->fsrc.cfg.stages);
+      DFG_CU(drv().FuncSetAttribute(plan->mod.tma, CU_FUNC_ATTRIBUTE_MAX_DYNAMIC_SHARED_SIZE_BYTES, int(smem)));
+    }
+  }
+  return plan;
+}
+
+std::pair<cudaEvent_t, cudaEvent_t> PlanImpl::kernel_events() {
+  std::pair<cudaEvent_t, cudaEvent_t> e;
+  if (!kev_free.empty()) {
+    e = kev_free.back();
+    kev_free.pop_back();
+  } else {
+    DFG_CUDA(cudaEventCreate(&e.first));
+    DFG_CUDA(cudaEventCreate(&e.second));
+  }
+  kev_pending.push_back(e);
+  return e;
+}
+
+void PlanImpl::resolve_kernel_times() {
+  for (auto& e : kev_pending) {
+    DFG_CUDA(cudaEventSynchronize(e.second));
+    float ms = 0;
+    DFG_CUDA(cudaEventElapsedTime(&ms, e.first, e.second));
+    st.kernel_ms_sum += ms;
+    st.kernel_launches_timed += 1;
+    kev_free.push_back(e);
+  }
+  kev_pending.clear();
+}
+
+// -------------------------------------------------------------- halo
+void PlanImpl::halo_exchange(const std::vector<int>& inputs, cudaStream_t s) {
+  MeshImpl& m = *mesh;
+  const bool has_lo = m.k0 > 0, has_hi = m.k0 + m.nzl < m.NZ;
+  if (!has_lo && !has_hi) return;
+  const size_t ts = dsize(m.dt);
+  const size_t pb = size_t(m.plane()) * ts;
+  auto lo = m.link_lo.lock(), hi = m.link_hi.lock();
+  if (m.nccl) {
+    auto& api = nccl();
+    ncclComm_t comm = static_cast<ncclComm_t>(m.nccl);
+    ncclDataType_t t = m.dt == DType::F32 ? ncclFloat32 : ncclFloat64;
+    nccl_check(api.GroupStart(), "ncclGroupStart");
+    for (int in : inputs) {
+      char* base = static_cast<char*>(m.fields[dag.inputs[in]].ptr);
+      if (has_lo) {
+        nccl_check(api.Send(base + 1 * pb, size_t(m.plane()), t, m.rank - 1, comm, s), "ncclSend");
+        nccl_check(api.Recv(base + 0 * pb, size_t(m.plane()), t, m.rank - 1, comm, s), "ncclRecv");
+      }
+      if (has_hi) {
+        nccl_check(api.Send(base + size_t(m.nzl) * pb, size_t(m.plane()), t, m.rank + 1, comm, s), "ncclSend");
+        nccl_check(api.Recv(base + size_t(m.nzl + 1) * pb, size_t(m.plane()), t, m.rank + 1, comm, s), "ncclRecv");
+      }
+    }
+    nccl_check(api.GroupEnd(), "ncclGroupEnd");
+  } else if (lo || hi || (has_lo && !lo) || (has_hi && !hi)) {
+    if ((has_lo && !lo) || (has_hi && !hi))
+      fail(DFG_E_INVALID, "slab has neighbours but no halo transport (dfg_mesh_init_comm / dfg_mesh_link_local)");
+    for (int in : inputs) {
+      const std::string& name = dag.inputs[in];
+      char* base = static_cast<char*>(m.fields[name].ptr);
+      if (has_lo) {
+        auto it = lo->fields.find(name);
+        if (it == lo->fields.end() || !it->second.ptr || !it->second.on_device)
+          fail(DFG_E_UNBOUND, "linked slab below has no device field '" + name + "'");
+        DFG_CUDA(cudaMemcpyPeerAsync(base, m.device, static_cast<char*>(it->second.ptr) + size_t(lo->nzl) * pb,
+                                     lo->device, pb, s));
+      }
+      if (has_hi) {
+        auto it = hi->fields.find(name);
+        if (it == hi->fields.end() || !it->second.ptr || !it->second.on_device)
+          fail(DFG_E_UNBOUND, "linked slab above has no device field '" + name + "'");
+        DFG_CUDA(cudaMemcpyPeerAsync(base + size_t(m.nzl + 1) * pb, m.device, static_cast<char*>(it->second.ptr) + pb,
+                                     hi->device, pb, s));
+      }
+    }
+  }
+  st.halo_bytes += int64_t(inputs.size()) * int64_t((has_lo ? 1 : 0) + (has_hi ? 1 : 0)) * int64_t(pb);
+}
+
+// -------------------------------------------------------------- execute
+void PlanImpl::execute(void* out, bool out_dev, cudaStream_t s) {
+  if (!out) fail(DFG_E_INVALID, "null output pointer");
+  MeshImpl& m = *mesh;
+  DFG_CUDA(cudaSetDevice(m.device));
+  for (int i : sources(dag).inputs) {
+    auto it = m.fields.find(dag.inputs[i]);
+    if (it == m.fields.end() || !it->second.ptr) fail(DFG_E_UNBOUND, "input '" + dag.inputs[i] + "' is not bound");
+  }
+  DFG_CUDA(cudaEventRecord(ev0, s));
+  switch (strategy) {
+    case DFG_FUSED: exec_fused(out, out_dev, s); break;
+    case DFG_STAGED: exec_staged(out, out_dev, s); break;
+    case DFG_ROUNDTRIP: exec_roundtrip(out, out_dev, s); break;
+  }
+  DFG_CUDA(cudaEventRecord(ev1, s));
+  DFG_CUDA(cudaGetLastError());
+  timed = true;
+  st.executes += 1;
+  bool any_host = !out_dev;
+  for (int i : sources(dag).inputs)
+    if (!m.fields[dag.inputs[i]].on_device) any_host = true;
+  st.predicted_highwater_bytes =
+      model(dag, strategy, any_host).units * m.cells() * int64_t(dsize(m.dt));
+  st.predicted_hbm_bytes = predicted_device_bytes(dag, strategy, m.cells(), dsize(m.dt));
+  st.predicted_pcie_bytes = predicted_pcie_bytes(dag, strategy, m.cells(), dsize(m.dt), any_host);
+}
+
+namespace {
+// CUtensorMap for one stencil field: dims {nx, ny, nzl + 2g}, box
+// {32*VEC + 2*VEC, NCW + 2, 1}, OOB fill zero (never read: clamped in smem).
+void encode_map(CUtensorMap* map, const MeshImpl& m, void* base, int ncw) {
+  const size_t ts = dsize(m.dt);
+  const int vec = int(16 / ts);
+  cuuint64_t gdim[3] = {cuuint64_t(m.nx), cuuint64_t(m.ny), cuuint64_t(m.nzl + 2 * m.ghost)};
+  cuuint64_t gstride[2] = {cuuint64_t(m.nx) * ts, cuuint64_t(m.nx * m.ny) * ts};
+  cuuint32_t box[3] = {cuuint32_t(32 * vec + 2 * vec), cuuint32_t(ncw + 2), 1};
+  cuuint32_t estr[3] = {1, 1, 1};
+  DFG_CU(drv().TensorMapEncodeTiled(map, m.dt == DType::F32 ? CU_TENSOR_MAP_DATA_TYPE_FLOAT32 : CU_TENSOR_MAP_DATA_TYPE_FLOAT64,
+                                3, base, gdim, gstride, box, estr, CU_TENSOR_MAP_INTERLEAVE_NONE,
+                                CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+                                CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE));
+}
+
+// Host mirror of DfgParams in skeleton.cuh (same field order and widths).
+std::vector<uint64_t> pack_params(const std::vector<const void*>& f, void* out, const void* tx, const void* ty,
+                                  const void* tz, const MeshImpl& m, int64_t kbeg, int64_t kend, int64_t items,
+                                  int tiles_x, int tiles_y, int kz, int vec_ok) {
+  std::vector<uint64_t> w;
+  for (auto p : f) w.push_back(reinterpret_cast<uint64_t>(p));
+  if (f.empty()) w.push_back(0);
+  w.push_back(reinterpret_cast<uint64_t>(out));
+  w.push_back(reinterpret_cast<uint64_t>(tx));
+  w.push_back(reinterpret_cast<uint64_t>(ty));
+  w.push_back(reinterpret_cast<uint64_t>(tz));
+  for (int64_t v : {m.nx, m.ny, m.nzl, m.NZ, m.k0, int64_t(m.ghost), kbeg, kend, items}) w.push_back(uint64_t(v));
+  w.push_back(uint64_t(uint32_t(tiles_x)) | (uint64_t(uint32_t(tiles_y)) << 32));
+  w.push_back(uint64_t(uint32_t(kz)) | (uint64_t(uint32_t(vec_ok)) << 32));
+  return w;
+}
+}  // namespace
+
+void PlanImpl::exec_fused(void* out, bool out_dev, cudaStream_t s) {
+  MeshImpl& m = *mesh;
+  const size_t ts = dsize(m.dt);
+  const FusedLayout& L = fsrc.layout;
+  const int64_t N = m.cells();
+  Ledger led(cap);
+  std::vector<void*> scratch;
+  struct Free {
+    std::vector<void*>& v;
+    cudaStream_t s;
+    ~Free() {
+      for (void* p : v) cudaFreeAsync(p, s);
+    }
+  } guard{scratch, s};
+
+  bool any_host = false;
+  for (int i : L.stencil_inputs) any_host |= !m.fields[dag.inputs[i]].on_device;
+  for (int i : L.point_inputs) any_host |= !m.fields[dag.inputs[i]].on_device;
+  if (any_host && m.nzl != m.NZ) fail(DFG_E_UNSUPPORTED, "host-pointer fields are single-slab only");
+
+  // inputs: resident (in situ) or uploaded once (host interface, Table II "Dev-W")
+  auto input_ptr = [&](int in) -> const void* {
+    Binding& b = m.fields[dag.inputs[in]];
+    size_t bytes = m.field_bytes();
+    led.add(bytes);
+    if (b.on_device) return b.ptr;
+    void* d = dev_alloc(bytes, m.device, s);
+    scratch.push_back(d);
+    DFG_CUDA(cudaMemcpyAsync(d, b.ptr, bytes, cudaMemcpyHostToDevice, s));
+    st.h2d_count += 1;
+    st.h2d_bytes += int64_t(bytes);
+    return d;
+  };
+  std::vector<const void*> fptr;
+  std::vector<int> order;  // first-use order for the upload sequence
+  for (int i : sources(dag).inputs) order.push_back(i);
+  std::map<int, const void*> got;
+  for (int i : order) got[i] = input_ptr(i);
+  for (int i : L.stencil_inputs) fptr.push_back(got[i]);
+  for (int i : L.point_inputs) fptr.push_back(got[i]);
+
+  if (!any_host && !L.stencil_inputs.empty()) halo_exchange(L.stencil_inputs, s);
+
+  // mesh arrays: resident, or uploaded like the paper's dims/x/y/z (L225)
+  const void* tab[3] = {m.dev_tab[0], m.dev_tab[1], m.dev_tab[2]};
+  if (L.has_grad && any_host) {
+    int64_t dims[4] = {m.nx, m.ny, m.NZ, m.k0};
+    void* dd = dev_alloc(sizeof(dims), m.device, s);
+    scratch.push_back(dd);
+    DFG_CUDA(cudaMemcpyAsync(dd, dims, sizeof(dims), cudaMemcpyHostToDevice, s));
+    st.h2d_count += 1;
+    st.h2d_bytes += sizeof(dims);
+    for (int a = 0; a < 3; ++a) {
+      void* d = dev_alloc(m.host_tab[a].size(), m.device, s);
+      scratch.push_back(d);
+      DFG_CUDA(cudaMemcpyAsync(d, m.host_tab[a].data(), m.host_tab[a].size(), cudaMemcpyHostToDevice, s));
+      st.h2d_count += 1;
+      st.h2d_bytes += int64_t(m.host_tab[a].size());
+      tab[a] = d;
+    }
+  }
+
+  const size_t out_bytes = size_t(N) * size_t(L.outw) * ts;
+  led.add(out_bytes);
+  void* dout = out;
+  if (!out_dev) {
+    dout = dev_alloc(out_bytes, m.device, s);
+    scratch.push_back(dout);
+  }
+
+  const int vec = int(16 / ts);
+  bool vec_ok = aligned16(dout) && (N % vec == 0);
+  for (auto p : fptr) vec_ok = vec_ok && aligned16(p);
+  const char* force = std::getenv("DFG_FUSED_KERNEL");
+  bool want_general = force && !std::strcmp(force, "general");
+  const int sms = sm_count(m.device);
+  const int64_t kbeg = m.k0, kend = m.k0 + m.nzl;
+
+  if (L.stencil_inputs.empty()) {
+    auto w = pack_params(fptr, dout, tab[0], tab[1], tab[2], m, kbeg, kend, 0, 0, 0, 0, vec_ok ? 1 : 0);
+    void* args[] = {w.data()};
+    long long work = vec_ok ? N / vec : N;
+    unsigned grid = unsigned(std::max<long long>(1, std::min<long long>((work + 255) / 256, sms * 8LL)));
+    auto ke = kernel_events();
+    DFG_CUDA(cudaEventRecord(ke.first, s));
+    DFG_CU(drv().LaunchKernel(mod.pointwise, grid, 1, 1, 256, 1, 1, 0, s, args, nullptr));
+    DFG_CUDA(cudaEventRecord(ke.second, s));
+    last_variant = 3;
+  } else if (mod.tma && !want_general && m.nx % vec == 0 && vec_ok) {
+    const int ncw = fsrc.cfg.ncw;
+    const int nsf = int(L.stencil_inputs.size());
+    const int tiles_x = int((m.nx + 32 * vec - 1) / (32 * vec));
+    const int tiles_y = int((m.ny + ncw - 1) / ncw);
+    const int64_t range = kend - kbeg;
+    size_t smem = fused_tma_smem_bytes(m.dt, nsf, ncw, fsrc.cfg.stages);
+    int occ = 1;
+    DFG_CU(drv().OccupancyMaxActiveBlocksPerMultiprocessor(&occ, mod.tma, (ncw + 1) * 32, smem));
+    occ = std::max(occ, 1);
+    const int64_t slots = int64_t(sms) * occ;
+    // z-chunk length: balance whole rounds of items over the persistent CTAs
+    // against the two extra (z-halo) planes each chunk loads.
+    int64_t best_kz = range, best_cost = INT64_MAX;
+    const char* kzenv = std::getenv("DFG_KZ");
+    if (kzenv) {
+      best_kz = std::max<int64_t>(1, std::min<int64_t>(range, std::atoll(kzenv)));
+    } else {
+      for (int64_t kz = 1; kz <= range; kz = kz < 8 ? kz + 1 : kz + std::max<int64_t>(1, kz / 8)) {
+        int64_t items = int64_t(tiles_x) * tiles_y * ((range + kz - 1) / kz);
+        int64_t rounds = (items + slots - 1) / slots;
+        int64_t cost = rounds * (std::min(kz, range) + 2 + 4);  // +4: pipeline fill per item
+        if (cost < best_cost) {
+          best_cost = cost;
+          best_kz = kz;
+        }
+      }
+    }
+    const int64_t items = int64_t(tiles_x) * tiles_y * ((range + best_kz - 1) / best_kz);
+    const unsigned grid = unsigned(std::min<int64_t>(items, slots));
+    // parameter blob: DfgTmap map[NSF_] (128 B each, 64-aligned) then DfgParams
+    auto w = pack_params(fptr, dout, tab[0], tab[1], tab[2], m, kbeg, kend, items, tiles_x, tiles_y, int(best_kz),
+                         vec_ok ? 1 : 0);
+    size_t pbytes = size_t(nsf) * 128 + w.size() * 8;
+    pbytes = (pbytes + 63) / 64 * 64;
+    alignas(64) unsigned char blob[8 * 128 + 512];
+    if (pbytes > sizeof(blob)) fail(DFG_E_UNSUPPORTED, "too many stencil fields for the TMA kernel");
+    std::memset(blob, 0, sizeof(blob));
+    for (int f = 0; f < nsf; ++f)
+      encode_map(reinterpret_cast<CUtensorMap*>(blob + 128 * f), m, const_cast<void*>(fptr[f]), ncw);
+    std::memcpy(blob + 128 * nsf, w.data(), w.size() * 8);
+    void* args[] = {blob};
+    auto ke = kernel_events();
+    DFG_CUDA(cudaEventRecord(ke.first, s));
+    DFG_CU(drv().LaunchKernel(mod.tma, grid, 1, 1, (ncw + 1) * 32, 1, 1, unsigned(smem), s, args, nullptr));
+    DFG_CUDA(cudaEventRecord(ke.second, s));
+    last_variant = 1;
+  } else {
+    auto w = pack_params(fptr, dout, tab[0], tab[1], tab[2], m, kbeg, kend, 0, 0, 0, 0, 0);
+    void* args[] = {w.data()};
+    unsigned grid = unsigned(std::max<long long>(1, std::min<long long>((N + 255) / 256, sms * 8LL)));
+    auto ke = kernel_events();
+    DFG_CUDA(cudaEventRecord(ke.first, s));
+    DFG_CU(drv().LaunchKernel(mod.general, grid, 1, 1, 256, 1, 1, 0, s, args, nullptr));
+    DFG_CUDA(cudaEventRecord(ke.second, s));
+    last_variant = 2;
+  }
+  st.kernel_count += 1;
+  if (!out_dev) {
+    DFG_CUDA(cudaMemcpyAsync(out, dout, out_bytes, cudaMemcpyDeviceToHost, s));
+    st.d2h_count += 1;
+    st.d2h_bytes += int64_t(out_bytes);
+    DFG_CUDA(cudaStreamSynchronize(s));
+  }
+  st.dev_highwater_bytes = std::max<int64_t>(st.dev_highwater_bytes, int64_t(led.high));
+}
+
+// ------------------------------------------------------------- staged
+void PlanImpl::exec_staged(void* out, bool out_dev, cudaStream_t s) {
+  MeshImpl& m = *mesh;
+  const size_t ts = dsize(m.dt);
+  const int64_t N = m.cells();
+  const size_t sb = size_t(N) * ts;  // one scalar problem array
+  const int64_t goff = int64_t(m.ghost) * m.plane();
+  Ledger led(cap);
+  std::vector<void*> to_free;
+  struct Free {
+    std::vector<void*>& v;
+    cudaStream_t s;
+    ~Free() {
+      for (void* p : v) cudaFreeAsync(p, s);
+    }
+  } guard{to_free, s};
+
+  Sources src = sources(dag);
+  bool host = !out_dev;
+  for (int i : src.inputs) host |= !m.fields[dag.inputs[i]].on_device;
+
+  // reference counts (L85): uses as an input, plus the sink
+  std::map<std::pair<int, int>, int64_t> rc;
+  auto key = [](const Ref& r) { return std::make_pair(int(r.kind), r.id); };
+  for (auto& f : dag.filters)
+    for (auto& r : f.in)
+      if (r.kind != Ref::Mesh) rc[key(r)] += 1;
+  rc[key(dag.result)] += 1;
+
+  std::map<int, void*> in_dev;   // input index -> device base (incl. ghost planes)
+  std::map<int, bool> in_owned;  // uploaded by us (freed at refcount 0)
+  std::vector<void*> fval(dag.filters.size(), nullptr);
+  if (!host) {
+    for (int i : src.inputs) {
+      in_dev[i] = m.fields[dag.inputs[i]].ptr;
+      in_owned[i] = false;
+      led.add(m.field_bytes());
+    }
+    led.add(sb * size_t(dag.width(dag.result) == 1 ? 1 : 4));  // the caller's output buffer
+  }
+  auto ensure_input = [&](int i) {
+    if (in_dev.count(i)) return;
+    Binding& b = m.fields[dag.inputs[i]];
+    if (b.on_device) {
+      in_dev[i] = b.ptr;
+      in_owned[i] = false;
+      led.add(m.field_bytes());
+      return;
+    }
+    size_t bytes = m.field_bytes();
+    led.add(bytes);
+    void* d = dev_alloc(bytes, m.device, s);
+    DFG_CUDA(cudaMemcpyAsync(d, b.ptr, bytes, cudaMemcpyHostToDevice, s));
+    st.h2d_count += 1;
+    st.h2d_bytes += int64_t(bytes);
+    in_dev[i] = d;
+    in_owned[i] = true;
+  };
+  const void* tab[3] = {m.dev_tab[0], m.dev_tab[1], m.dev_tab[2]};
+  bool mesh_up = false;
+  auto ensure_mesh = [&]() {
+    if (mesh_up || !host) return;
+    mesh_up = true;
+    int64_t dims[4] = {m.nx, m.ny, m.NZ, m.k0};
+    void* dd = dev_alloc(sizeof(dims), m.device, s);
+    to_free.push_back(dd);
+    DFG_CUDA(cudaMemcpyAsync(dd, dims, sizeof(dims), cudaMemcpyHostToDevice, s));
+    st.h2d_count += 1;
+    st.h2d_bytes += sizeof(dims);
+    for (int a = 0; a < 3; ++a) {
+      void* d = dev_alloc(m.host_tab[a].size(), m.device, s);
+      to_free.push_back(d);
+      DFG_CUDA(cudaMemcpyAsync(d, m.host_tab[a].data(), m.host_tab[a].size(), cudaMemcpyHostToDevice, s));
+      st.h2d_count += 1;
+      st.h2d_bytes += int64_t(m.host_tab[a].size());
+      tab[a] = d;
+    }
+  };
+  // value pointer of a ref over the owned cells (inputs skip the ghost plane)
+  auto val = [&](const Ref& r) -> const void* {
+    if (r.kind == Ref::Filter) return fval[r.id];
+    return static_cast<const char*>(in_dev[r.id]) + goff * int64_t(ts);
+  };
+  auto release = [&](const Ref& r) {
+    if (r.kind == Ref::Mesh) return;
+    if (--rc[key(r)] > 0) return;
+    if (r.kind == Ref::Filter) {
+      if (fval[r.id] && fval[r.id] != out) {
+        cudaFreeAsync(fval[r.id], s);
+        led.sub(sb * size_t(dag.filters[r.id].width == 1 ? 1 : 4));
+      }
+      fval[r.id] = nullptr;
+    } else if (in_owned[r.id]) {
+      cudaFreeAsync(in_dev[r.id], s);
+      led.sub(m.field_bytes());
+      in_dev.erase(r.id);
+    }
+  };
+
+  const size_t nf = dag.filters.size();
+  for (size_t k = 0; k < nf; ++k) {
+    const Filter& f = dag.filters[k];
+    for (auto& r : f.in) {
+      if (r.kind == Ref::Input) ensure_input(r.id);
+      if (r.kind == Ref::Mesh) ensure_mesh();
+    }
+    const size_t ob = sb * size_t(f.width == 1 ? 1 : 4);
+    const bool into_out = out_dev && dag.result.kind == Ref::Filter && dag.result.id == int(k) && k + 1 == nf;
+    void* o;
+    if (into_out) {
+      o = out;
+      if (host) led.add(ob);
+    } else {
+      led.add(ob);
+      o = dev_alloc(ob, m.device, s);
+    }
+    fval[k] = o;
+    switch (f.op) {
+      case Op::Const: kern::fill(m.dt, f.cval, o, N, s); break;
+      case Op::Add: case Op::Sub: case Op::Mult: case Op::Div:
+      case Op::Gt: case Op::Lt: case Op::Ge: case Op::Le: case Op::Eq: case Op::Ne:
+        kern::binary(f.op, m.dt, val(f.in[0]), val(f.in[1]), o, N, s);
+        break;
+      case Op::Neg: case Op::Sqrt: kern::unary(f.op, m.dt, val(f.in[0]), o, N, s); break;
+      case Op::Select: kern::select(m.dt, val(f.in[0]), val(f.in[1]), val(f.in[2]), o, N, s); break;
+      case Op::Decompose: kern::decompose(m.dt, val(f.in[0]), f.k, o, N, s); break;
+      case Op::Compose: {
+        const void* ins[4];
+        for (size_t l = 0; l < f.in.size(); ++l) ins[l] = val(f.in[l]);
+        kern::compose(m.dt, ins, int(f.in.size()), o, N, s);
+        break;
+      }
+      case Op::Grad3d: {
+        const Ref& a = f.in[0];
+        if (a.kind == Ref::Input)
+          kern::grad3d(m.dt, in_dev[a.id], o, tab[0], tab[1], tab[2], m.nx, m.ny, m.nzl, m.NZ, m.k0, m.ghost, s);
+        else
+          kern::grad3d(m.dt, fval[a.id], o, tab[0], tab[1], tab[2], m.nx, m.ny, m.nzl, m.NZ, m.k0, 0, s);
+        break;
+      }
+    }
+    DFG_CUDA(cudaGetLastError());
+    st.kernel_count += 1;
+    for (auto& r : f.in) release(r);
+  }
+  // the sink (L80): result -> caller's buffer
+  const Ref& res = dag.result;
+  const size_t rb = sb * size_t(dag.width(res) == 1 ? 1 : 4);
+  const void* rp;
+  if (res.kind == Ref::Input) {
+    ensure_input(res.id);
+    rp = val(res);
+  } else {
+    rp = fval[res.id];
+  }
+  if (rp != out) {
+    if (out_dev) {
+      DFG_CUDA(cudaMemcpyAsync(out, rp, rb, cudaMemcpyDeviceToDevice, s));
+    } else {
+      DFG_CUDA(cudaMemcpyAsync(out, rp, rb, cudaMemcpyDeviceToHost, s));
+      st.d2h_count += 1;
+      st.d2h_bytes += int64_t(rb);
+    }
+  }
+  release(res);
+  for (auto& kv : in_dev)
+    if (in_owned[kv.first]) to_free.push_back(kv.second);
+  if (!out_dev) DFG_CUDA(cudaStreamSynchronize(s));
+  st.dev_highwater_bytes = std::max<int64_t>(st.dev_highwater_bytes, int64_t(led.high));
+}
+
+// ---------------------------------------------------------- roundtrip
+void PlanImpl::exec_roundtrip(void* out, bool out_dev, cudaStream_t s) {
+  MeshImpl& m = *mesh;
+  const size_t ts = dsize(m.dt);
+  const int64_t N = m.cells();
+  const size_t sb = size_t(N) * ts;
+  const int64_t goff = int64_t(m.ghost) * m.plane();
+  Ledger led(cap);
+  std::lock_guard<std::mutex> lk(g_host_mu);
+  HostPool& hp = host_pool();
+
+  Sources src = sources(dag);
+  bool host = !out_dev;
+  for (int i : src.inputs) host |= !m.fields[dag.inputs[i]].on_device;
+  if (!host) {  // in situ: resident inputs and output are live throughout
+    for (size_t q = 0; q < src.inputs.size(); ++q) led.add(m.field_bytes());
+    led.add(sb * size_t(dag.width(dag.result) == 1 ? 1 : 4));
+  }
+
+  std::map<std::pair<int, int>, int64_t> rc;
+  auto key = [](const Ref& r) { return std::make_pair(int(r.kind), r.id); };
+  for (auto& f : dag.filters)
+    for (auto& r : f.in)
+      if (r.kind != Ref::Mesh) rc[key(r)] += 1;
+  rc[key(dag.result)] += 1;
+  std::vector<void*> hval(dag.filters.size(), nullptr);  // every result lives in host memory (L92)
+
+  auto host_const = [&](const Filter& f) -> void* {
+    void* h = hp.get(sb);
+    if (m.dt == DType::F32) std::fill_n(static_cast<float*>(h), N, float(f.cval));
+    else std::fill_n(static_cast<double*>(h), N, f.cval);
+    return h;
+  };
+  auto release = [&](const Ref& r) {
+    if (r.kind != Ref::Filter) return;
+    if (--rc[key(r)] > 0) return;
+    if (hval[r.id]) hp.put(hval[r.id]);
+    hval[r.id] = nullptr;
+  };
+
+  for (size_t k = 0; k < dag.filters.size(); ++k) {
+    const Filter& f = dag.filters[k];
+    if (f.op == Op::Const) {  // a host buffer, uploaded by every consumer (L307)
+      hval[k] = host_const(f);
+      continue;
+    }
+    if (f.op == Op::Decompose) {  // on the host, no transfer (L289)
+      const Ref& a = f.in[0];
+      void* h = hp.get(sb);
+      if (m.dt == DType::F32) {
+        const float* v = static_cast<const float*>(hval[a.id]);
+        float* o = static_cast<float*>(h);
+        for (int64_t e = 0; e < N; ++e) o[e] = v[4 * e + f.k];
+      } else {
+        const double* v = static_cast<const double*>(hval[a.id]);
+        double* o = static_cast<double*>(h);
+        for (int64_t e = 0; e < N; ++e) o[e] = v[4 * e + f.k];
+      }
+      hval[k] = h;
+      release(a);
+      continue;
+    }
+    // one kernel: upload every argument, run, download the result (L92)
+    std::vector<void*> dfree;
+    std::vector<size_t> dsz;
+    auto upload = [&](const void* h, size_t bytes) -> void* {
+      led.add(bytes);
+      void* d = dev_alloc(bytes, m.device, s);
+      DFG_CUDA(cudaMemcpyAsync(d, h, bytes, cudaMemcpyHostToDevice, s));
+      st.h2d_count += 1;
+      st.h2d_bytes += int64_t(bytes);
+      dfree.push_back(d);
+      dsz.push_back(bytes);
+      return d;
+    };
+    auto upload_small = [&](const void* h, size_t bytes) -> void* {
+      void* d = dev_alloc(bytes, m.device, s);
+      DFG_CUDA(cudaMemcpyAsync(d, h, bytes, cudaMemcpyHostToDevice, s));
+      st.h2d_count += 1;
+      st.h2d_bytes += int64_t(bytes);
+      dfree.push_back(d);
+      dsz.push_back(0);
+      return d;
+    };
+    std::vector<const void*> args;   // owned-cell value pointers
+    const void* grad_base = nullptr; // grad3d: base incl. ghost planes
+    int64_t grad_ghost = 0;
+    const void* tab[3] = {m.dev_tab[0], m.dev_tab[1], m.dev_tab[2]};
+    int mesh_i = 0;
+    for (auto& r : f.in) {
+      if (r.kind == Ref::Mesh) {
+        if (host) {
+          if (r.id == 0) {
+            int64_t dims[4] = {m.nx, m.ny, m.NZ, m.k0};
+            upload_small(dims, sizeof(dims));
+          } else {
+            tab[r.id - 1] = upload_small(m.host_tab[r.id - 1].data(), m.host_tab[r.id - 1].size());
+          }
+        }
+        ++mesh_i;
+        continue;
+      }
+      if (r.kind == Ref::Input) {
+        Binding& b = m.fields[dag.inputs[r.id]];
+        const void* base = b.on_device ? b.ptr : upload(b.ptr, m.field_bytes());
+        args.push_back(static_cast<const char*>(base) + goff * int64_t(ts));
+        if (f.op == Op::Grad3d) {
+          grad_base = base;
+          grad_ghost = m.ghost;
+        }
+      } else {
+        const Filter& g = dag.filters[r.id];
+        size_t bytes = sb * size_t(g.width == 1 ? 1 : 4);
+        const void* d = upload(hval[r.id], bytes);
+        args.push_back(d);
+        if (f.op == Op::Grad3d) {
+          grad_base = d;
+          grad_ghost = 0;
+        }
+      }
+    }
+    const size_t ob = sb * size_t(f.width == 1 ? 1 : 4);
+    led.add(ob);
+    void* o = dev_alloc(ob, m.device, s);
+    dfree.push_back(o);
+    dsz.push_back(ob);
+    switch (f.op) {
+      case Op::Add: case Op::Sub: case Op::Mult: case Op::Div:
+      case Op::Gt: case Op::Lt: case Op::Ge: case Op::Le: case Op::Eq: case Op::Ne:
+        kern::binary(f.op, m.dt, args[0], args[1], o, N, s);
+        break;
+      case Op::Neg: case Op::Sqrt: kern::unary(f.op, m.dt, args[0], o, N, s); break;
+      case Op::Select: kern::select(m.dt, args[0], args[1], args[2], o, N, s); break;
+      case Op::Compose: kern::compose(m.dt, args.data(), int(args.size()), o, N, s); break;
+      case Op::Grad3d:
+        kern::grad3d(m.dt, grad_base, o, tab[0], tab[1], tab[2], m.nx, m.ny, m.nzl, m.NZ, m.k0, grad_ghost, s);
+        break;
+      default: fail(DFG_E_INVALID, "internal: unexpected roundtrip op");
+    }
+    DFG_CUDA(cudaGetLastError());
+    st.kernel_count += 1;
+    void* h = hp.get(ob);
+    DFG_CUDA(cudaMemcpyAsync(h, o, ob, cudaMemcpyDeviceToHost, s));
+    st.d2h_count += 1;
+    st.d2h_bytes += int64_t(ob);
+    DFG_CUDA(cudaStreamSynchronize(s));
+    hval[k] = h;
+    for (size_t q = 0; q < dfree.size(); ++q) {
+      cudaFreeAsync(dfree[q], s);
+      led.sub(dsz[q]);
+    }
+    for (auto& r : f.in) release(r);
+  }
+  // the sink: host result -> caller's buffer
+  const Ref& res = dag.result;
+  const size_t rb = sb * size_t(dag.width(res) == 1 ? 1 : 4);
+  if (res.kind == Ref::Input) {
+    Binding& b = m.fields[dag.inputs[res.id]];
+    const char* srcp = static_cast<const char*>(b.ptr) + goff * int64_t(ts);
+    DFG_CUDA(cudaMemcpyAsync(out, srcp, rb, cudaMemcpyDefault, s));
+  } else if (out_dev) {
+    DFG_CUDA(cudaMemcpyAsync(out, hval[res.id], rb, cudaMemcpyHostToDevice, s));
+    st.h2d_count += 1;
+    st.h2d_bytes += int64_t(rb);
+  } else {
+    std::memcpy(out, hval[res.id], rb);
+  }
+  DFG_CUDA(cudaStreamSynchronize(s));
+  release(res);
+  for (auto& p : hval)
+    if (p) hp.put(p);
+  st.dev_highwater_bytes = std::max<int64_t>(st.dev_highwater_bytes, int64_t(led.high));
+}
+
+}  // namespace dfg

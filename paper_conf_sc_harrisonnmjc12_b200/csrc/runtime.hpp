@@ -1,0 +1,89 @@
+// libdfg runtime: meshes, plans, the three execution strategies, the device
+// memory ledger and the halo exchange.
+#pragma once
+
+#include <cuda.h>
+#include <cuda_runtime.h>
+
+#include <map>
+#include <memory>
+#include <string>
+#include <vector>
+
+#include "codegen.hpp"
+#include "jit.hpp"
+#include "lang.hpp"
+
+namespace dfg {
+
+struct Binding {
+  void* ptr = nullptr;
+  bool on_device = false;
+};
+
+struct MeshImpl {
+  DType dt = DType::F32;
+  int64_t nx = 0, ny = 0, nzl = 0, NZ = 0, k0 = 0;
+  int ghost = 0;
+  int device = 0;
+  bool markstein_safe = true;        // spacing tables inside the exact-division range
+  std::vector<char> host_tab[3];     // per axis: d[n] then r[n] (T), reading R1
+  void* dev_tab[3] = {nullptr, nullptr, nullptr};
+  std::map<std::string, Binding> fields;
+  // halo transport
+  int rank = 0, nranks = 1;
+  void* nccl = nullptr;              // ncclComm_t
+  std::weak_ptr<MeshImpl> link_lo, link_hi;
+  ~MeshImpl();
+  int64_t plane() const { return nx * ny; }
+  int64_t cells() const { return nx * ny * nzl; }
+  size_t field_bytes() const { return size_t(nx * ny * (nzl + 2 * ghost)) * dsize(dt); }
+};
+
+std::shared_ptr<MeshImpl> create_mesh(DType dt, int64_t nx, int64_t ny, int64_t nzl, const void* x, const void* y,
+                                      const void* z, int64_t NZ, int64_t k0, int ghost);
+
+// Host-side analysis of a network (no device): what each strategy will do.
+struct Model {
+  int64_t h2d = 0, d2h = 0, kernels = 0;
+  int64_t units = 0;  // footprint in problem-array units (scalar 1, vector 4)
+};
+Model model(const Dag& dag, dfg_strategy s, bool host_mode);
+int64_t predicted_device_bytes(const Dag& dag, dfg_strategy s, int64_t cells, size_t tsize);
+int64_t predicted_pcie_bytes(const Dag& dag, dfg_strategy s, int64_t cells, size_t tsize, bool host_mode);
+
+struct PlanImpl {
+  std::shared_ptr<MeshImpl> mesh;
+  Dag dag;
+  dfg_strategy strategy = DFG_FUSED;
+  size_t cap = 0;
+  FusedSource fsrc;
+  LoadedModule mod;
+  int regs = 0, spill = 0;
+  int last_variant = 0;  // 1 TMA, 2 general, 3 pointwise
+  dfg_stats st{};
+  cudaEvent_t ev0 = nullptr, ev1 = nullptr;
+  bool timed = false;
+  // fused-kernel launch timing: event pairs resolved lazily in stats()
+  std::vector<std::pair<cudaEvent_t, cudaEvent_t>> kev_free, kev_pending;
+  std::pair<cudaEvent_t, cudaEvent_t> kernel_events();
+  void resolve_kernel_times();
+  std::map<std::string, std::vector<char>> const_cache;  // roundtrip host constants
+  ~PlanImpl();
+  void execute(void* out, bool out_dev, cudaStream_t s);
+
+ private:
+  void exec_fused(void* out, bool out_dev, cudaStream_t s);
+  void exec_staged(void* out, bool out_dev, cudaStream_t s);
+  void exec_roundtrip(void* out, bool out_dev, cudaStream_t s);
+  void halo_exchange(const std::vector<int>& inputs, cudaStream_t s);
+};
+
+std::unique_ptr<PlanImpl> compile_plan(std::shared_ptr<MeshImpl> mesh, const std::string& expr, dfg_strategy s,
+                                       size_t cap);
+
+// NCCL (loaded with dlopen)
+void nccl_unique_id(void* out128);
+void mesh_init_comm(MeshImpl& m, const void* id128, int rank, int nranks);
+
+}  // namespace dfg

@@ -1,0 +1,308 @@
+"""GPU parity: libdfg (all strategies, both kernels) against the oracle,
+element by element on the same seeded inputs.  Exact-division mode (the
+default) must be bit-identical to the oracle."""
+
+import os
+
+import numpy as np
+import pytest
+import torch
+
+import synth
+from oracle import evaluate as oev
+from oracle import model as omodel
+from oracle.lang import PAPER_PROGRAMS, build_dag
+from tests.dfg_testutil import assert_parity, run_lib, run_oracle, tdtype
+
+pytestmark = pytest.mark.gpu
+
+PROGS = ["velmag", "vortmag", "qcrit", "intro"]
+NAMES = {"velmag": ("u", "v", "w"), "vortmag": ("u", "v", "w"), "qcrit": ("u", "v", "w"), "intro": ("b", "c")}
+
+
+def _inputs(shape, T, names=("u", "v", "w")):
+    x, y, z, f = synth.rt_inputs(*shape, dtype=T, names=names)
+    return x, y, z, {k: v.numpy() for k, v in f.items()}
+
+
+@pytest.fixture(autouse=True)
+def _cuda():
+    if not torch.cuda.is_available():
+        pytest.skip("no CUDA device")
+    import paper_conf_sc_harrisonnmjc12_b200  # noqa: F401  (fails loudly if the .so is missing)
+
+
+@pytest.mark.parametrize("prog", PROGS)
+@pytest.mark.parametrize("strategy", ["fused", "staged", "roundtrip"])
+@pytest.mark.parametrize("T", [np.float32, np.float64])
+@pytest.mark.parametrize("shape", [(32, 32, 32), (132, 40, 33), (67, 45, 37)])
+def test_parity_paper_programs(prog, strategy, T, shape):
+    """32^3 is config 1; 132 x 40 x 33 spans two x tiles, a ragged y tile and
+    odd z (TMA path); nx = 67 is not a multiple of 4 (general kernel)."""
+    x, y, z, f = _inputs(shape, T, NAMES[prog])
+    src = PAPER_PROGRAMS[prog][0]
+    want = run_oracle(src, f, x, y, z)
+    got = run_lib(src, f, x, y, z, strategy)
+    assert_parity(got, want)
+
+
+@pytest.mark.parametrize("T", [np.float32, np.float64])
+def test_tma_and_general_kernels_identical(T, monkeypatch):
+    x, y, z, f = _inputs((128, 48, 40), T)
+    src = PAPER_PROGRAMS["qcrit"][0]
+    a, plan, *_ = run_lib(src, f, x, y, z, return_plan=True)
+    assert plan.info()["variant"] == 1           # TMA pipeline ran
+    monkeypatch.setenv("DFG_FUSED_KERNEL", "general")
+    b, plan2, *_ = run_lib(src, f, x, y, z, return_plan=True)
+    assert plan2.info()["variant"] == 2
+    assert np.array_equal(a, b)
+
+
+@pytest.mark.parametrize("kz", ["1", "3", "7", "1000"])
+def test_tma_z_chunking(kz, monkeypatch):
+    """Every z-chunk length gives the same bits (halo planes at chunk ends)."""
+    x, y, z, f = _inputs((64, 31, 29), np.float32)
+    src = PAPER_PROGRAMS["qcrit"][0]
+    want = run_oracle(src, f, x, y, z)
+    monkeypatch.setenv("DFG_KZ", kz)
+    got, plan, *_ = run_lib(src, f, x, y, z, return_plan=True)
+    assert plan.info()["variant"] == 1
+    assert_parity(got, want)
+
+
+@pytest.mark.parametrize("shape", [(1, 5, 6), (4, 1, 3), (8, 6, 1), (2, 2, 2), (3, 3, 3), (4, 4, 2), (1, 1, 1)])
+@pytest.mark.parametrize("strategy", ["fused", "staged", "roundtrip"])
+def test_degenerate_shapes(shape, strategy):
+    x, y, z, f = _inputs(shape, np.float32)
+    for prog in ("qcrit", "vortmag"):
+        src = PAPER_PROGRAMS[prog][0]
+        assert_parity(run_lib(src, f, x, y, z, strategy), run_oracle(src, f, x, y, z))
+
+
+EDGE = [
+    ("g = grad(u)", ("u",)),
+    ("g = grad(u * u + 1)", ("u",)),
+    ("c = {u, v * 2, u - v}", ("u", "v")),
+    ("c = {u, v}", ("u", "v")),
+    ("a = u", ("u",)),
+    ("a = 2.5", ("u",)),
+    ("a = u / v\nb = -a * (a >= 0.5) + (v != u)", ("u", "v")),
+    ("a = if (grad(u)[0] > grad(v)[1]) then (sqrt(u * u)) else (v / u)", ("u", "v")),
+    ("d = grad({u, v}[1] - u)\ne = norm(d) + d[2]", ("u", "v")),
+]
+
+
+@pytest.mark.parametrize("src,names", EDGE)
+@pytest.mark.parametrize("strategy", ["fused", "staged", "roundtrip"])
+@pytest.mark.parametrize("T", [np.float32, np.float64])
+def test_edge_programs(src, names, strategy, T):
+    x, y, z, f = _inputs((20, 9, 7), T, names)
+    assert_parity(run_lib(src, f, x, y, z, strategy), run_oracle(src, f, x, y, z))
+
+
+@pytest.mark.parametrize("kind", ["rotation", "strain", "shear", "linear"])
+def test_closed_forms_on_gpu(kind):
+    T = np.float32
+    x, y, z = (synth.dyadic_coords(12, s, T, o) for s, o in ((5, 0.5), (6, -0.25), (7, 1.0)))
+    f = {k: v.astype(T) for k, v in synth.closed_form(kind, x, y, z).items()}
+    progs = ["g = grad(f)"] if kind == "linear" else [PAPER_PROGRAMS["vortmag"][0], PAPER_PROGRAMS["qcrit"][0]]
+    for src in progs:
+        for s in ("fused", "staged"):
+            assert_parity(run_lib(src, f, x, y, z, s), run_oracle(src, f, x, y, z))
+
+
+@pytest.mark.parametrize("prog", ["velmag", "vortmag", "qcrit"])
+@pytest.mark.parametrize("strategy", ["roundtrip", "staged", "fused"])
+def test_table2_counts_measured(prog, strategy):
+    """Host-interface mode reproduces Table II (L271-L285) physically."""
+    import json
+    gold = json.load(open(os.path.join(os.path.dirname(__file__), "golden", "table2.json")))
+    x, y, z, f = _inputs((16, 12, 8), np.float32)
+    src = PAPER_PROGRAMS[prog][0]
+    got, plan, *_ = run_lib(src, f, x, y, z, strategy, host=True, return_plan=True)
+    st = plan.stats()
+    assert [st["h2d_count"], st["d2h_count"], st["kernel_count"]] == gold[prog][strategy]
+    assert_parity(got, run_oracle(src, f, x, y, z))
+    # device-resident (in situ) counts follow the same model
+    got, plan, *_ = run_lib(src, f, x, y, z, strategy, host=False, return_plan=True)
+    st = plan.stats()
+    c = omodel.counts(build_dag(src, ("u", "v", "w")), strategy, "device")
+    assert [st["h2d_count"], st["d2h_count"], st["kernel_count"]] == [c.h2d, c.d2h, c.kernels]
+
+
+@pytest.mark.parametrize("strategy", ["roundtrip", "staged", "fused"])
+@pytest.mark.parametrize("host", [True, False])
+def test_memory_highwater_measured(strategy, host):
+    """Fig. 2 (L112) in host mode; the ledger's high-water equals the model."""
+    g = {"roundtrip": 3, "staged": 4, "fused": 5}
+    x, y, z, f = _inputs((16, 8, 8), np.float32, ("a", "b", "c", "d"))
+    f["d"] = f["a"] * 2
+    src = "r = (a + b) * (c + d)\n"
+    got, plan, *_ = run_lib(src, f, x, y, z, strategy, host=host, return_plan=True)
+    N = 16 * 8 * 8 * 4
+    units = omodel.footprint(build_dag(src, tuple(f)), strategy, "host" if host else "device")
+    if host:
+        assert units == g[strategy]
+    assert plan.stats()["dev_highwater_bytes"] == units * N
+    assert_parity(got, run_oracle(src, f, x, y, z))
+    for prog in ("vortmag", "qcrit"):
+        src = PAPER_PROGRAMS[prog][0]
+        x, y, z, f = _inputs((16, 8, 8), np.float32)
+        _, plan, *_ = run_lib(src, f, x, y, z, strategy, host=host, return_plan=True)
+        units = omodel.footprint(build_dag(src, tuple(f)), strategy, "host" if host else "device")
+        assert plan.stats()["dev_highwater_bytes"] == units * N
+
+
+def test_memory_cap():
+    """A cap below the predicted footprint fails at compile with
+    DFG_E_NOMEM (the paper's failed GPU cases, L309); fused fits."""
+    import paper_conf_sc_harrisonnmjc12_b200 as dfg
+    x, y, z, f = _inputs((32, 32, 32), np.float32)
+    src = PAPER_PROGRAMS["qcrit"][0]
+    N = 32 ** 3 * 4
+    staged_units = omodel.footprint(build_dag(src, ("u", "v", "w")), "staged", "device")
+    with pytest.raises(dfg.DfgError) as e:
+        run_lib(src, f, x, y, z, "staged", cap=(staged_units - 1) * N)
+    assert e.value.name == "DFG_E_NOMEM"
+    got = run_lib(src, f, x, y, z, "staged", cap=staged_units * N)
+    assert_parity(got, run_oracle(src, f, x, y, z))
+    got = run_lib(src, f, x, y, z, "fused", cap=4 * N)
+    assert_parity(got, run_oracle(src, f, x, y, z))
+
+
+@pytest.mark.parametrize("G", [2, 3, 5])
+@pytest.mark.parametrize("T", [np.float32, np.float64])
+def test_zslab_emulation_matches_single_gpu(G, T):
+    """G z-slabs with one ghost plane each, halo by device copies
+    (dfg_mesh_link_local): the concatenated result equals the one-slab
+    result bit for bit, and the halo maps equal the closed form."""
+    import paper_conf_sc_harrisonnmjc12_b200 as dfg
+    from oracle import halo as ohalo
+    shape = (64, 20, 23)
+    x, y, z, f = _inputs(shape, T)
+    src = PAPER_PROGRAMS["qcrit"][0]
+    whole = run_lib(src, f, x, y, z)
+    NZ = shape[2]
+    meshes, plans, outs, keep = [], [], [], []
+    for r in range(G):
+        k0, nzr = dfg.dfg_partition(NZ, G, r)
+        m = dfg.Mesh(x, y, z, nz_local=nzr, z_offset=k0, ghost=1)
+        for n, a in f.items():
+            buf = torch.zeros((nzr + 2,) + a.shape[1:], dtype=tdtype(T), device="cuda")
+            buf[1:nzr + 1] = torch.from_numpy(a[k0:k0 + nzr])
+            keep.append(buf)
+            m.bind(n, buf)
+        meshes.append(m)
+        want = ohalo.halo_map(NZ, k0, nzr, r, G, shape[0], shape[1], np.dtype(T).itemsize)
+        got = m.halo_map()
+        assert got[2:8] == want[2:8] and got[10:] == want[10:]
+    for r in range(G - 1):
+        dfg.dfg_mesh_link_local(meshes[r].handle, meshes[r + 1].handle)
+    for r, m in enumerate(meshes):
+        p = dfg.Plan(m, src, "fused")
+        o = torch.empty((m.nz, shape[1], shape[0]), dtype=tdtype(T), device="cuda")
+        p.execute(o)
+        plans.append(p)
+        outs.append(o)
+    torch.cuda.synchronize()
+    got = torch.cat(outs).cpu().numpy()
+    assert np.array_equal(got, whole)
+    st = plans[1].stats()
+    assert st["halo_bytes"] == 3 * 2 * shape[0] * shape[1] * np.dtype(T).itemsize
+
+
+def test_config2_192_all_strategies():
+    """Config 2: 192^3, VelMag + VortMag + Q, all three strategies."""
+    x, y, z, f = _inputs((192, 192, 192), np.float32)
+    for prog in ("velmag", "vortmag", "qcrit"):
+        src = PAPER_PROGRAMS[prog][0]
+        want = run_oracle(src, f, x, y, z)
+        for s in ("fused", "staged", "roundtrip"):
+            assert_parity(run_lib(src, f, x, y, z, s), want)
+
+
+def _windows(shape, rng, n_random=6, w=10):
+    nx, ny, nz = shape
+    wins = []
+    for cz in (0, nz - w):
+        for cy in (0, ny - w):
+            for cx in (0, nx - w):
+                wins.append((cz, cy, cx))
+    for _ in range(n_random):
+        wins.append((int(rng.integers(0, nz - w)), int(rng.integers(0, ny - w)), int(rng.integers(0, nx - w))))
+    return [(k, k + w, j, j + w, i, i + w) for k, j, i in wins]
+
+
+def _sampled_parity(src, names, shape, T, strategy="fused", seed=0):
+    """Full-size run on the GPU; oracle on sampled windows (8 corners + random
+    interior), each evaluated with global indices and global coordinates."""
+    import paper_conf_sc_harrisonnmjc12_b200 as dfg
+    nx, ny, nz = shape
+    x, y, z = synth.rt_coords(nx, ny, nz, T)
+    x64, y64, z64 = (a.astype(np.float64) for a in (x, y, z))
+    mesh = dfg.Mesh(x, y, z)
+    bufs = {}
+    for n, comp in zip(names, "uvw"):
+        bufs[n] = synth.rt_velocity(comp, x64, y64, z64, dtype=tdtype(T), device="cuda")
+        mesh.bind(n, bufs[n])
+    plan = dfg.Plan(mesh, src, strategy)
+    out = torch.empty((nz, ny, nx), dtype=tdtype(T), device="cuda")
+    plan.execute(out)
+    torch.cuda.synchronize()
+    dag = build_dag(src, names, "f32" if T == np.float32 else "f64")
+    rng = np.random.default_rng(seed)
+    for (k0, k1, j0, j1, i0, i1) in _windows(shape, rng):
+        e = lambda a, b, n: (max(a - 1, 0), min(b + 1, n))
+        K0, K1 = e(k0, k1, nz)
+        J0, J1 = e(j0, j1, ny)
+        I0, I1 = e(i0, i1, nx)
+        win = {n: bufs[n][K0:K1, J0:J1, I0:I1].cpu().numpy() for n in names}
+        res, valid = oev.evaluate(dag, win, oev.MeshWindow(x, y, z, i0=I0, j0=J0, k0=K0))
+        sl = (slice(k0 - K0, k1 - K0), slice(j0 - J0, j1 - J0), slice(i0 - I0, i1 - I0))
+        assert valid[sl].all()
+        got = out[k0:k1, j0:j1, i0:i1].cpu().numpy()
+        assert_parity(got, res[sl])
+    return plan
+
+
+def test_config4_1024_fused_q_sampled():
+    """Config 4 at 1 GPU (the bench workload): 1024^3 fused Q, fp32."""
+    plan = _sampled_parity(PAPER_PROGRAMS["qcrit"][0], ("u", "v", "w"), (1024, 1024, 1024), np.float32)
+    assert plan.info()["variant"] == 1
+
+
+@pytest.mark.parametrize("prog", PROGS)
+@pytest.mark.parametrize("T", [np.float32, np.float64])
+def test_config5_768_sweep_sampled(prog, T):
+    """Config 5: 768^3 complexity sweep, fp32 and fp64, fused."""
+    _sampled_parity(PAPER_PROGRAMS[prog][0], NAMES[prog], (768, 768, 768), T)
+
+
+def test_config3_512_staged_caps():
+    """Config 3: 512^3 Q, staged under device-memory caps vs fused."""
+    import paper_conf_sc_harrisonnmjc12_b200 as dfg
+    GiB = 1 << 30
+    n = 512
+    x, y, z = synth.rt_coords(n, n, n, np.float32)
+    x64, y64, z64 = (a.astype(np.float64) for a in (x, y, z))
+    mesh = dfg.Mesh(x, y, z)
+    bufs = {c: synth.rt_velocity(c, x64, y64, z64, dtype=torch.float32, device="cuda") for c in "uvw"}
+    for c, b in bufs.items():
+        mesh.bind(c, b)
+    src = PAPER_PROGRAMS["qcrit"][0]
+    fused = dfg.Plan(mesh, src, "fused", 4 * GiB)
+    o1 = torch.empty((n, n, n), device="cuda")
+    fused.execute(o1)
+    units = omodel.footprint(build_dag(src, ("u", "v", "w")), "staged", "device")
+    need = units * n ** 3 * 4
+    for cap in (8 * GiB, 4 * GiB):
+        assert need > cap
+        with pytest.raises(dfg.DfgError) as e:
+            dfg.Plan(mesh, src, "staged", cap)
+        assert e.value.name == "DFG_E_NOMEM"
+    staged = dfg.Plan(mesh, src, "staged", 16 * GiB)
+    o2 = torch.empty((n, n, n), device="cuda")
+    staged.execute(o2)
+    torch.cuda.synchronize()
+    assert torch.equal(o1, o2)
+    assert staged.stats()["dev_highwater_bytes"] == need

@@ -1,0 +1,226 @@
+"""Host-side checks of libdfg.so that need no GPU: the library loads and
+exports every symbol include/dfg.h declares; its parser / network builder
+and strategy model agree with the oracle (byte-equal canonical text, same
+error classes, same predicted counts and footprints); its fused-kernel
+generator compiles for sm_100a under NVRTC without spills."""
+
+import os
+import random
+import re
+
+import pytest
+
+from oracle import halo as ohalo
+from oracle import model as omodel
+from oracle.lang import DfgError, PAPER_PROGRAMS, build_dag
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+LIB = os.path.join(ROOT, "paper_conf_sc_harrisonnmjc12_b200", "libdfg.so")
+
+pytestmark = pytest.mark.skipif(not os.path.exists(LIB), reason="libdfg.so not built (run __graft_entry__.build())")
+
+
+@pytest.fixture(scope="module")
+def dfg():
+    import paper_conf_sc_harrisonnmjc12_b200 as d
+    return d
+
+
+def test_exports_every_declared_symbol(dfg):
+    import ctypes
+    hdr = open(os.path.join(ROOT, "include", "dfg.h")).read()
+    declared = sorted(set(re.findall(r"\b(dfg_[a-z_0-9]+)\s*\(", hdr)))
+    assert len(declared) >= 20
+    lib = ctypes.CDLL(LIB)
+    for name in declared:
+        assert hasattr(lib, name), name
+    assert set(declared) == set(dfg.EXPORTS)
+    assert dfg.dfg_version() == 100
+
+
+KIND = {"DFG_E_PARSE": "parse", "DFG_E_UNDEFINED": "undefined", "DFG_E_TYPE": "type"}
+
+
+def _lib_dump(dfg, src, inputs, dt):
+    try:
+        return dfg.dfg_dag_dump(src, inputs, 0 if dt == "f32" else 1)
+    except dfg.DfgError as e:
+        return ("error", KIND.get(e.name, e.name))
+
+
+def _oracle_dump(src, inputs, dt):
+    try:
+        return build_dag(src, inputs, dt).dump()
+    except DfgError as e:
+        return ("error", e.kind)
+
+
+@pytest.mark.parametrize("name", sorted(PAPER_PROGRAMS))
+@pytest.mark.parametrize("dt", ["f32", "f64"])
+def test_paper_programs_dump_equal(dfg, name, dt):
+    src, inputs = PAPER_PROGRAMS[name]
+    assert _lib_dump(dfg, src, inputs, dt) == _oracle_dump(src, inputs, dt)
+    with open(os.path.join(ROOT, "tests", "golden", f"dag_{name}_{dt}.txt")) as f:
+        assert _lib_dump(dfg, src, inputs, dt) == f.read()
+
+
+# ------------------------------------------------------- differential fuzz
+_CONSTS = ["0.5", ".5", "5e-1", "1", "10", "2.0", "3.25e+2", "0.1", "1e39", "007", "1.", "0.0"]
+
+
+def _rand_expr(rng, depth, vec_ok=False):
+    r = rng.random()
+    if depth <= 0 or r < 0.2:
+        return rng.choice(["u", "v", "w", "u", rng.choice(_CONSTS)])
+    kind = rng.choice(["bin", "bin", "bin", "neg", "sqrt", "paren", "dec", "norm", "if", "cmp", "comp_dec"])
+    if kind == "bin":
+        return f"{_rand_expr(rng, depth - 1)} {rng.choice('+-*/')} {_rand_expr(rng, depth - 1)}"
+    if kind == "neg":
+        return f"-{_rand_expr(rng, depth - 1)}"
+    if kind == "sqrt":
+        return f"sqrt({_rand_expr(rng, depth - 1)})"
+    if kind == "paren":
+        return f"({_rand_expr(rng, depth - 1)})"
+    if kind == "dec":
+        g = rng.choice(["grad(u)", "grad3d(v, dims, x, y, z)", "grad(u*w)", "grad(w - 1)"])
+        return f"{g}[{rng.randrange(3)}]"
+    if kind == "norm":
+        return rng.choice(["norm(grad(u))", "norm(grad(v + w))", "norm({u, v})"])
+    if kind == "if":
+        return (f"if ({_rand_expr(rng, depth - 1)} > {_rand_expr(rng, depth - 1)}) then "
+                f"({_rand_expr(rng, depth - 1)}) else ({_rand_expr(rng, depth - 1)})")
+    if kind == "cmp":
+        return f"({_rand_expr(rng, depth - 1)} {rng.choice(['<', '>=', '<=', '==', '!='])} {_rand_expr(rng, depth - 1)})"
+    return f"{{{_rand_expr(rng, depth - 1)}, {_rand_expr(rng, depth - 1)}, u}}[{rng.randrange(3)}]"
+
+
+def _rand_program(rng):
+    lines = []
+    names = []
+    for i in range(rng.randint(1, 5)):
+        e = _rand_expr(rng, rng.randint(0, 3))
+        if names and rng.random() < 0.4:
+            e = e.replace("u", rng.choice(names), 1)
+        n = rng.choice(["a", "b", "t1", "q_", "u"]) if rng.random() < 0.3 else f"n{i}"
+        lines.append(f"{n} = {e}")
+        names.append(n)
+    src = "\n".join(lines)
+    if rng.random() < 0.3:
+        src = src.replace(" + ", " +\n  ", 1)
+    return src + rng.choice(["", "\n", "\n\n# tail comment\n"])
+
+
+def _mutate(rng, src):
+    ops = ["delete", "insert", "swap"]
+    toks = re.findall(r"\s+|[A-Za-z_][A-Za-z0-9_]*|\d+\.?\d*(?:[eE][+-]?\d+)?|\.\d+|>=|<=|==|!=|.", src)
+    if not toks:
+        return src
+    i = rng.randrange(len(toks))
+    op = rng.choice(ops)
+    junk = rng.choice(["(", ")", "[", "]", "{", "}", ",", "=", "+", "*", "-", "1", "x", "if", "then", "else",
+                       "\n", "$", ".", "1.5.", "[7]", "grad3d(", "dims", "f0"])
+    if op == "delete":
+        del toks[i]
+    elif op == "insert":
+        toks.insert(i, junk)
+    else:
+        toks[i] = junk
+    return "".join(toks)
+
+
+@pytest.mark.parametrize("seed", range(6))
+def test_differential_fuzz_parser(dfg, seed):
+    """Random well-formed programs and random single-token corruptions:
+    library and oracle must produce byte-equal networks or the same error
+    class (SURVEY section 4 test plan)."""
+    rng = random.Random(seed)
+    n_ok = n_err = 0
+    for _ in range(250):
+        src = _rand_program(rng)
+        if rng.random() < 0.5:
+            src = _mutate(rng, src)
+        dt = rng.choice(["f32", "f64"])
+        a = _lib_dump(dfg, src, ("u", "v", "w"), dt)
+        b = _oracle_dump(src, ("u", "v", "w"), dt)
+        assert a == b, src
+        if isinstance(a, str):
+            n_ok += 1
+        else:
+            n_err += 1
+    assert n_ok > 50 and n_err > 20
+
+
+@pytest.mark.parametrize("name", sorted(PAPER_PROGRAMS) + ["fig2"])
+@pytest.mark.parametrize("strategy", ["roundtrip", "staged", "fused"])
+@pytest.mark.parametrize("host", [True, False])
+def test_model_matches_oracle(dfg, name, strategy, host):
+    if name == "fig2":
+        src, inputs = "r = (a + b) * (c + d)\n", ("a", "b", "c", "d")
+    else:
+        src, inputs = PAPER_PROGRAMS[name]
+    dag = build_dag(src, inputs)
+    mode = "host" if host else "device"
+    c = omodel.counts(dag, strategy, mode)
+    assert dfg.dfg_model(src, inputs, strategy, host) == [c.h2d, c.d2h, c.kernels,
+                                                           omodel.footprint(dag, strategy, mode)]
+
+
+@pytest.mark.parametrize("seed", range(3))
+def test_model_fuzz(dfg, seed):
+    rng = random.Random(100 + seed)
+    checked = 0
+    for _ in range(120):
+        src = _rand_program(rng)
+        try:
+            dag = build_dag(src, ("u", "v", "w"))
+        except DfgError:
+            continue
+        for s in ("roundtrip", "staged", "fused"):
+            for host in (True, False):
+                mode = "host" if host else "device"
+                c = omodel.counts(dag, s, mode)
+                assert dfg.dfg_model(src, ("u", "v", "w"), s, host) == [
+                    c.h2d, c.d2h, c.kernels, omodel.footprint(dag, s, mode)], (src, s, mode)
+        checked += 1
+    assert checked > 30
+
+
+@pytest.mark.parametrize("NZ,G", [(1024, 8), (10, 3), (7, 7), (1000, 6), (5, 1), (33, 4)])
+def test_partition_matches_closed_form(dfg, NZ, G):
+    covered = 0
+    for r in range(G):
+        k0, n = dfg.dfg_partition(NZ, G, r)
+        assert (k0, n) == ohalo.partition(NZ, G, r)
+        assert k0 == covered
+        covered += n
+    assert covered == NZ
+    with pytest.raises(dfg.DfgError):
+        dfg.dfg_partition(NZ, NZ + 1, 0)
+
+
+@pytest.mark.parametrize("name", ["velmag", "vortmag", "qcrit", "intro"])
+@pytest.mark.parametrize("dtype", [0, 1])
+def test_fused_kernel_compiles_without_spills(dfg, name, dtype):
+    src, inputs = PAPER_PROGRAMS[name]
+    code, regs, spill = dfg.dfg_fused_source(src, inputs, dtype, 64, 48, 40, compile=True)
+    assert "dfg_body" in code and "extern \"C\" __global__" in code
+    assert regs > 0
+    assert spill == 0, (regs, spill)
+
+
+def test_fused_kernel_compiles_edge_programs(dfg):
+    for src, inputs in [("g = grad(u * u + 1)", ("u",)), ("c = {u, v, u * v}", ("u", "v")),
+                        ("a = u", ("u",)), ("a = 3", ("u",)),
+                        ("a = if (grad(u)[0] > grad(v)[1]) then (sqrt(u)) else (v / u)", ("u", "v"))]:
+        for dt in (0, 1):
+            code, regs, spill = dfg.dfg_fused_source(src, inputs, dt, 8, 4, 1, compile=True)
+            assert regs > 0 and spill == 0, src
+
+
+def test_errors_have_messages(dfg):
+    with pytest.raises(dfg.DfgError) as e:
+        dfg.dfg_dag_dump("a = (u", ("u",))
+    assert e.value.name == "DFG_E_PARSE" and "1:" in e.value.msg
+    with pytest.raises(dfg.DfgError) as e:
+        dfg.dfg_dag_dump("a = 1", ("x",))
+    assert e.value.name == "DFG_E_INVALID"
