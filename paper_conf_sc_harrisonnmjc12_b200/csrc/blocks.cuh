@@ -60,8 +60,7 @@ DFG_DEVICE double dfg_select(double c, double a, double b) { return (c != 0.0) ?
 #ifndef DFG_DIV_MODE
 #define DFG_DIV_MODE 1
 #endif
-DFG_DEVICE float dfg_grad1(float fp, float fm, float d, float r) {
-  float num = __fsub_rn(fp, fm);
+DFG_DEVICE float dfg_grad1q(float num, float d, float r) {
 #if DFG_DIV_MODE == 0
   (void)r;
   return __fdiv_rn(num, d);
@@ -74,8 +73,7 @@ DFG_DEVICE float dfg_grad1(float fp, float fm, float d, float r) {
   return __fmul_rn(num, r);
 #endif
 }
-DFG_DEVICE double dfg_grad1(double fp, double fm, double d, double r) {
-  double num = __dsub_rn(fp, fm);
+DFG_DEVICE double dfg_grad1q(double num, double d, double r) {
 #if DFG_DIV_MODE == 0
   (void)r;
   return __ddiv_rn(num, d);
@@ -88,3 +86,77 @@ DFG_DEVICE double dfg_grad1(double fp, double fm, double d, double r) {
   return __dmul_rn(num, r);
 #endif
 }
+DFG_DEVICE float dfg_grad1(float fp, float fm, float d, float r) {
+  float num = __fsub_rn(fp, fm);
+  return dfg_grad1q(num, d, r);
+}
+DFG_DEVICE double dfg_grad1(double fp, double fm, double d, double r) {
+  double num = __dsub_rn(fp, fm);
+  return dfg_grad1q(num, d, r);
+}
+
+// --- paired blocks: two cells per instruction ------------------------------
+// sm_100 executes FADD2 / FMUL2 / FFMA2 on float2 register pairs.  The fused
+// kernels evaluate the network on pairs of cells (float2 for T = float; for
+// T = double a "pair" is one double and the blocks are the scalar ones).
+// Contraction guard: ptxas contracts f32x2 multiply -> add sequences into
+// FFMA2 even with .rn and --fmad=false, which would change the rounding.
+// Products are therefore formed as fma(a, b, Z) with Z = (-0, -0) passed in
+// at run time (opaque to the compiler): RN(a*b + -0) == RN(a*b) for every a,
+// b (including signed zeros, Inf and NaN), and an FFMA2 feeding an add can
+// not be contracted further.
+#if defined(DFG_PAIRS)
+#if DFG_PAIRS_F32
+typedef float2 dfg2;
+DFG_DEVICE dfg2 dfg2_splat(float a) { return make_float2(a, a); }
+DFG_DEVICE dfg2 dfg2_add(dfg2 a, dfg2 b, dfg2) { return __fadd2_rn(a, b); }
+DFG_DEVICE dfg2 dfg2_sub(dfg2 a, dfg2 b, dfg2) { return __ffma2_rn(b, make_float2(-1.0f, -1.0f), a); }
+DFG_DEVICE dfg2 dfg2_mult(dfg2 a, dfg2 b, dfg2 z) { return __ffma2_rn(a, b, z); }
+DFG_DEVICE dfg2 dfg2_neg(dfg2 a, dfg2 z) { return __ffma2_rn(a, make_float2(-1.0f, -1.0f), z); }
+#define DFG2_LANEWISE1(name, f) \
+  DFG_DEVICE dfg2 name(dfg2 a, dfg2) { return make_float2(f(a.x), f(a.y)); }
+#define DFG2_LANEWISE2(name, f) \
+  DFG_DEVICE dfg2 name(dfg2 a, dfg2 b, dfg2) { return make_float2(f(a.x, b.x), f(a.y, b.y)); }
+DFG2_LANEWISE1(dfg2_sqrt, dfg_sqrt)
+DFG2_LANEWISE2(dfg2_div, dfg_div)
+DFG2_LANEWISE2(dfg2_gt, dfg_gt)
+DFG2_LANEWISE2(dfg2_lt, dfg_lt)
+DFG2_LANEWISE2(dfg2_ge, dfg_ge)
+DFG2_LANEWISE2(dfg2_le, dfg_le)
+DFG2_LANEWISE2(dfg2_eq, dfg_eq)
+DFG2_LANEWISE2(dfg2_ne, dfg_ne)
+DFG_DEVICE dfg2 dfg2_select(dfg2 c, dfg2 a, dfg2 b, dfg2) {
+  return make_float2(dfg_select(c.x, a.x, b.x), dfg_select(c.y, a.y, b.y));
+}
+// grad3d quotient on a pair, num = f[ip] - f[im] already formed; nd = -d
+// (the tables carry the exact negation so the correction is one FFMA2)
+DFG_DEVICE dfg2 dfg2_gradq(dfg2 num, dfg2 nd, dfg2 r, dfg2 z) {
+#if DFG_DIV_MODE == 0
+  return make_float2(__fdiv_rn(num.x, -nd.x), __fdiv_rn(num.y, -nd.y));
+#elif DFG_DIV_MODE == 1
+  dfg2 q0 = __ffma2_rn(num, r, z);      // RN(num * r)
+  dfg2 rem = __ffma2_rn(q0, nd, num);   // num - q0*d, exact
+  return __ffma2_rn(rem, r, q0);        // RN(q0 + rem*r)
+#else
+  return __ffma2_rn(num, r, z);
+#endif
+}
+#else   // T = double: one cell per "pair", scalar blocks
+typedef double dfg2;
+DFG_DEVICE dfg2 dfg2_splat(double a) { return a; }
+DFG_DEVICE dfg2 dfg2_add(dfg2 a, dfg2 b, dfg2) { return dfg_add(a, b); }
+DFG_DEVICE dfg2 dfg2_sub(dfg2 a, dfg2 b, dfg2) { return dfg_sub(a, b); }
+DFG_DEVICE dfg2 dfg2_mult(dfg2 a, dfg2 b, dfg2) { return dfg_mult(a, b); }
+DFG_DEVICE dfg2 dfg2_neg(dfg2 a, dfg2) { return dfg_neg(a); }
+DFG_DEVICE dfg2 dfg2_sqrt(dfg2 a, dfg2) { return dfg_sqrt(a); }
+DFG_DEVICE dfg2 dfg2_div(dfg2 a, dfg2 b, dfg2) { return dfg_div(a, b); }
+DFG_DEVICE dfg2 dfg2_gt(dfg2 a, dfg2 b, dfg2) { return dfg_gt(a, b); }
+DFG_DEVICE dfg2 dfg2_lt(dfg2 a, dfg2 b, dfg2) { return dfg_lt(a, b); }
+DFG_DEVICE dfg2 dfg2_ge(dfg2 a, dfg2 b, dfg2) { return dfg_ge(a, b); }
+DFG_DEVICE dfg2 dfg2_le(dfg2 a, dfg2 b, dfg2) { return dfg_le(a, b); }
+DFG_DEVICE dfg2 dfg2_eq(dfg2 a, dfg2 b, dfg2) { return dfg_eq(a, b); }
+DFG_DEVICE dfg2 dfg2_ne(dfg2 a, dfg2 b, dfg2) { return dfg_ne(a, b); }
+DFG_DEVICE dfg2 dfg2_select(dfg2 c, dfg2 a, dfg2 b, dfg2) { return dfg_select(c, a, b); }
+DFG_DEVICE dfg2 dfg2_gradq(dfg2 num, dfg2 nd, dfg2 r, dfg2) { return dfg_grad1q(num, -nd, r); }
+#endif
+#endif  // DFG_PAIRS

@@ -1,0 +1,316 @@
+// dfg_fused_tma: the B200 fused-kernel skeleton (PAPER.md L97-L105 fusion,
+// re-designed for sm_100a).  Compiled by NVRTC after skeleton.cuh.
+//
+// Work decomposition: persistent CTAs (grid = #SM x occupancy) walk items
+// (x-tile of 32*VEC cells) x (y-tile of DFG_NCW rows) x (z-chunk of kz
+// planes), item = blockIdx.x + t*gridDim.x.  Warp DFG_NCW is the producer:
+// one lane streams, per z-plane, one halo'd x-y tile per stencil field
+// (box (32*VEC + 2*VEC) x (NCW + 2) x 1, cp.async.bulk.tensor.3d) into a
+// DFG_STAGES-deep ring of shared-memory stages guarded by full/empty
+// mbarriers (complete_tx byte counts; all consumer threads arrive on
+// "empty", so no divergent branch).  For every item the producer loads
+// kz + 2 planes: the pre-plane max(kb-1, 0), planes kb..ke-1 and the post-plane
+// min(ke, NZ-1).  At the global ends these duplicate the first / last plane,
+// which is exactly the clamped neighbour of reading R1, so the consumer loop
+// has no boundary branch.
+// Consumers: warp w owns tile row w, lane l owns VEC consecutive x cells;
+// the z-1 / z / z+1 centres live in a 3-entry register queue whose roles
+// rotate through a 3-way unrolled loop (no register copies); x/y neighbours
+// come from shared memory through per-thread clamped offsets; the network
+// body runs on pairs of cells (FADD2/FFMA2); results leave as 16-byte
+// streaming stores.
+
+#if DFG_NSF > 0 && DFG_HAS_TMA
+struct __align__(64) DfgTmap { unsigned long long v[16]; };  // CUtensorMap
+struct DfgTmaParams {
+  DfgTmap map[DFG_NSF_];
+  DfgParams p;
+};
+
+#define DFG_TX (32 * DFG_VEC)
+#define DFG_HX DFG_VEC
+#define DFG_ROWW (DFG_TX + 2 * DFG_HX)
+#define DFG_ROWS (DFG_NCW + 2)
+#define DFG_TILE_ELEMS (DFG_ROWW * DFG_ROWS)
+#define DFG_TILE_BYTES ((DFG_TILE_ELEMS * (int)sizeof(DFG_T) + 127) / 128 * 128)
+#define DFG_STAGE_BYTES (DFG_TILE_BYTES * DFG_NSF)
+
+__device__ __forceinline__ unsigned dfg_smem(const void* p) {
+  return (unsigned)__cvta_generic_to_shared(p);
+}
+__device__ __forceinline__ void dfg_mbar_init(unsigned bar, unsigned count) {
+  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(bar), "r"(count) : "memory");
+}
+__device__ __forceinline__ void dfg_mbar_expect_tx(unsigned bar, unsigned bytes) {
+  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(bar), "r"(bytes) : "memory");
+}
+__device__ __forceinline__ void dfg_mbar_arrive(unsigned bar) {
+  asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(bar) : "memory");
+}
+// try_wait with a suspend-time hint: the thread sleeps in hardware until the
+// phase completes (or the hint expires) instead of spinning on issue slots
+__device__ __forceinline__ bool dfg_mbar_try(unsigned bar, unsigned parity, unsigned hint_ns) {
+  unsigned done;
+  asm volatile(
+      "{\n\t.reg .pred p;\n\t"
+      "mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2, %3;\n\t"
+      "selp.u32 %0, 1, 0, p;\n\t}"
+      : "=r"(done)
+      : "r"(bar), "r"(parity), "r"(hint_ns)
+      : "memory");
+  return done != 0;
+}
+__device__ __forceinline__ void dfg_mbar_wait(unsigned bar, unsigned parity, unsigned hint_ns) {
+  while (!dfg_mbar_try(bar, parity, hint_ns)) {
+  }
+}
+__device__ __forceinline__ void dfg_tma_load3(unsigned dst, const DfgTmap* map, unsigned bar, int x, int y, int z) {
+  asm volatile(
+      "cp.async.bulk.tensor.3d.shared::cluster.global.mbarrier::complete_tx::bytes"
+      " [%0], [%1, {%3, %4, %5}], [%2];" ::"r"(dst),
+      "l"(reinterpret_cast<unsigned long long>(map)), "r"(bar), "r"(x), "r"(y), "r"(z)
+      : "memory");
+}
+__device__ __forceinline__ void dfg_lds16(DFG_T (&d)[DFG_VEC], unsigned addr) {
+#if DFG_VEC == 4
+  asm volatile("ld.shared.v4.f32 {%0, %1, %2, %3}, [%4];"
+               : "=f"(d[0]), "=f"(d[1]), "=f"(d[2]), "=f"(d[3])
+               : "r"(addr)
+               : "memory");
+#else
+  asm volatile("ld.shared.v2.f64 {%0, %1}, [%2];" : "=d"(d[0]), "=d"(d[1]) : "r"(addr) : "memory");
+#endif
+}
+__device__ __forceinline__ DFG_T dfg_lds1(unsigned addr) {
+  DFG_T v;
+#if DFG_VEC == 4
+  asm volatile("ld.shared.f32 %0, [%1];" : "=f"(v) : "r"(addr) : "memory");
+#else
+  asm volatile("ld.shared.f64 %0, [%1];" : "=d"(v) : "r"(addr) : "memory");
+#endif
+  return v;
+}
+
+// Ring cursor: shared-memory byte address of the current stage and of its
+// full / empty barriers, advanced without multiplies (same sequence as the
+// producer's).
+struct DfgRing {
+  unsigned tile;   // smem byte address of stage s, field 0
+  unsigned full;   // smem byte address of full[s]
+  unsigned phase;
+  int stage;
+  unsigned tile0, full0;
+  __device__ __forceinline__ void advance() {
+    ++stage;
+    tile += DFG_STAGE_BYTES;
+    full += 8;
+    if (stage == DFG_STAGES) {
+      stage = 0;
+      tile = tile0;
+      full = full0;
+      phase ^= 1u;
+    }
+  }
+};
+#define DFG_EMPTY(full_addr) ((full_addr) + 8 * DFG_STAGES)
+
+// per-item, per-thread constants of a consumer thread
+struct DfgCol {
+  unsigned off_c, off_xm, off_xp, off_ym, off_yp;  // byte offsets in a tile
+  dfg2 ndx[DFG_NPAIR], rx[DFG_NPAIR], ndy, ry, Z;  // -d and 1/d spacing entries
+  bool act;
+};
+
+// One z-plane.  `cur` = smem address of the plane's stage (tile, full bar);
+// the next plane's stage is always present (the producer loads a clamped
+// post-plane).  Queue roles are template parameters (no copies).
+template <int ZM, int ZC, int ZN>
+__device__ __forceinline__ void dfg_plane(const DfgCol& C, DfgRing& R, unsigned& cur_tile, unsigned& cur_full,
+                                          DFG_T (&zq)[3][DFG_NSF][DFG_VEC], DFG_T*& outp, const DFG_T* (&pin)[DFG_NPF_],
+                                          long long plane, const DFG_T*& tzp, long long NZ) {
+  dfg_mbar_wait(R.full, R.phase, 0x100000u);
+  const unsigned nxt_tile = R.tile, nxt_full = R.full;
+#pragma unroll
+  for (int f = 0; f < DFG_NSF; ++f) dfg_lds16(zq[ZN][f], nxt_tile + f * DFG_TILE_BYTES + C.off_c);
+  R.advance();
+  dfg2 s[DFG_NPAIR][DFG_NSF][7], gn[DFG_NPAIR][DFG_NSF][3];
+#pragma unroll
+  for (int f = 0; f < DFG_NSF; ++f) {
+    const unsigned t = cur_tile + f * DFG_TILE_BYTES;
+    const DFG_T xm = dfg_lds1(t + C.off_xm), xp = dfg_lds1(t + C.off_xp);
+    DFG_T ym[DFG_VEC], yp[DFG_VEC];
+    dfg_lds16(ym, t + C.off_ym);
+    dfg_lds16(yp, t + C.off_yp);
+    DFG_T lft[DFG_VEC], rgt[DFG_VEC];
+#pragma unroll
+    for (int c = 0; c < DFG_VEC; ++c) {
+      lft[c] = c == 0 ? xm : zq[ZC][f][c == 0 ? 0 : c - 1];
+      rgt[c] = c == DFG_VEC - 1 ? xp : zq[ZC][f][c == DFG_VEC - 1 ? c : c + 1];
+    }
+#pragma unroll
+    for (int h = 0; h < DFG_NPAIR; ++h) {
+      const int a = h * DFG_LANES, b = h * DFG_LANES + DFG_LANES - 1;
+      s[h][f][0] = dfg2_mk(zq[ZC][f][a], zq[ZC][f][b]);
+      s[h][f][1] = dfg2_mk(lft[a], lft[b]);
+      s[h][f][2] = dfg2_mk(rgt[a], rgt[b]);
+      s[h][f][3] = dfg2_mk(ym[a], ym[b]);
+      s[h][f][4] = dfg2_mk(yp[a], yp[b]);
+      s[h][f][5] = dfg2_mk(zq[ZM][f][a], zq[ZM][f][b]);
+      s[h][f][6] = dfg2_mk(zq[ZN][f][a], zq[ZN][f][b]);
+      // x numerators as scalar subtractions (no pair shuffles), y/z as pairs
+      gn[h][f][0] = dfg2_mk(dfg_sub(rgt[a], lft[a]), dfg_sub(rgt[b], lft[b]));
+      gn[h][f][1] = dfg2_sub(s[h][f][4], s[h][f][3], C.Z);
+      gn[h][f][2] = dfg2_sub(s[h][f][6], s[h][f][5], C.Z);
+    }
+  }
+  const dfg2 ndz = dfg2_splat(__ldg(tzp + 2 * NZ)), rz = dfg2_splat(__ldg(tzp + NZ));
+  ++tzp;
+  dfg2 p[DFG_NPAIR][DFG_NPF_];
+#pragma unroll
+  for (int f = 0; f < DFG_NPF; ++f) {
+    DFG_T pv[DFG_VEC];
+    if (C.act) {
+      dfg_ldg16(pv, pin[f]);
+    } else {
+#pragma unroll
+      for (int c = 0; c < DFG_VEC; ++c) pv[c] = DFG_T(0);
+    }
+    pin[f] += plane;
+#pragma unroll
+    for (int h = 0; h < DFG_NPAIR; ++h) p[h][f] = dfg2_mk(pv[h * DFG_LANES], pv[h * DFG_LANES + DFG_LANES - 1]);
+  }
+  dfg2 o[DFG_NPAIR][DFG_OUTW];
+#pragma unroll
+  for (int h = 0; h < DFG_NPAIR; ++h)
+    dfg_body(s[h], gn[h], p[h], C.ndx[h], C.rx[h], C.ndy, C.ry, ndz, rz, C.Z, o[h]);
+  if (C.act) dfg_store_cells(outp, o);
+  outp += plane * DFG_OUTW;
+  dfg_mbar_arrive(DFG_EMPTY(cur_full));  // every consumer thread (count NCW*32)
+  cur_tile = nxt_tile;
+  cur_full = nxt_full;
+}
+
+extern "C" __global__ void __launch_bounds__((DFG_NCW + 1) * 32, 1)
+    dfg_fused_tma(const __grid_constant__ DfgTmaParams TP) {
+  const DfgParams& P = TP.p;
+  // dynamic shared memory starts at the (1024-aligned) base of the CTA's
+  // window: no static __shared__ in this kernel
+  extern __shared__ __align__(1024) unsigned char dfg_smem_raw[];
+  const unsigned smem = dfg_smem(dfg_smem_raw);
+  const unsigned full0 = smem + DFG_STAGES * DFG_STAGE_BYTES;  // full[s] at full0 + 8s, empty[s] = full[s] + 8*STAGES
+  const int warp = threadIdx.x >> 5;
+  const int lane = threadIdx.x & 31;
+
+  if (threadIdx.x == 0) {
+    for (int s = 0; s < DFG_STAGES; ++s) {
+      dfg_mbar_init(full0 + 8 * s, 1);
+      dfg_mbar_init(DFG_EMPTY(full0 + 8 * s), DFG_NCW * 32);
+    }
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+  }
+  __syncthreads();
+
+  if (warp == DFG_NCW) {
+    // ---------------- producer: one lane issues all TMA loads
+    if (lane == 0) {
+      for (int f = 0; f < DFG_NSF; ++f)
+        asm volatile("prefetch.tensormap [%0];" ::"l"(reinterpret_cast<unsigned long long>(&TP.map[f]))
+                     : "memory");
+      DfgRing W{smem, full0, 0u, 0, smem, full0};
+      for (long long item = blockIdx.x; item < P.items; item += gridDim.x) {
+        const long long tx_ = item % P.tiles_x;
+        const long long rest = item / P.tiles_x;
+        const long long ty_ = rest % P.tiles_y;
+        const long long zc = rest / P.tiles_y;
+        const int x0 = (int)(tx_ * DFG_TX) - DFG_HX;
+        const int y0 = (int)(ty_ * DFG_NCW) - 1;
+        const long long kb = P.kbeg + zc * P.kz;
+        const long long ke = min(kb + (long long)P.kz, P.kend);
+        // pre-plane, kb..ke-1, post-plane; clamped to the global mesh (R1)
+        for (long long q = kb - 1; q <= ke; ++q) {
+          const long long pg = max(0LL, min(q, P.NZ - 1));
+          // wait until every consumer released this slot (the producer runs
+          // ahead; the suspend hint keeps it off the issue slots)
+          dfg_mbar_wait(DFG_EMPTY(W.full), W.phase ^ 1u, 0x100000u);
+          dfg_mbar_expect_tx(W.full, (unsigned)(DFG_NSF * DFG_TILE_ELEMS * sizeof(DFG_T)));
+          const int zl = (int)(pg - P.k0 + P.ghost);
+#pragma unroll
+          for (int f = 0; f < DFG_NSF; ++f) dfg_tma_load3(W.tile + f * DFG_TILE_BYTES, &TP.map[f], W.full, x0, y0, zl);
+          W.advance();
+        }
+      }
+    }
+    return;
+  }
+
+  // ------------------- consumers: warp w computes tile row w
+  DfgRing R{smem, full0, 0u, 0, smem, full0};
+  DfgCol C;
+  C.Z = dfg2_splat(P.nzero);
+  const long long plane = P.nx * P.ny;
+  const unsigned c0 = DFG_HX + DFG_VEC * lane;
+  const unsigned r = 1 + warp;
+  for (long long item = blockIdx.x; item < P.items; item += gridDim.x) {
+    const long long tx_ = item % P.tiles_x;
+    const long long rest = item / P.tiles_x;
+    const long long ty_ = rest % P.tiles_y;
+    const long long zc = rest / P.tiles_y;
+    const long long i = tx_ * DFG_TX + DFG_VEC * lane;
+    const long long j = ty_ * DFG_NCW + warp;
+    const long long kb = P.kbeg + zc * P.kz;
+    const long long ke = min(kb + (long long)P.kz, P.kend);
+    C.act = (i < P.nx) && (j < P.ny);
+    const long long ic = min(i, P.nx - DFG_VEC);
+    const long long jc = min(j, P.ny - 1);
+#pragma unroll
+    for (int h = 0; h < DFG_NPAIR; ++h) {
+      const long long a = ic + h * DFG_LANES, b = ic + h * DFG_LANES + DFG_LANES - 1;
+      C.ndx[h] = dfg2_mk(__ldg(P.tx + 2 * P.nx + a), __ldg(P.tx + 2 * P.nx + b));
+      C.rx[h] = dfg2_mk(__ldg(P.tx + P.nx + a), __ldg(P.tx + P.nx + b));
+    }
+    C.ndy = dfg2_splat(__ldg(P.ty + 2 * P.ny + jc));
+    C.ry = dfg2_splat(__ldg(P.ty + P.ny + jc));
+    const unsigned cxm = (i == 0) ? c0 : c0 - 1;
+    const unsigned cxp = (i + DFG_VEC >= P.nx) ? c0 + DFG_VEC - 1 : c0 + DFG_VEC;
+    const unsigned rm = (j == 0) ? r : r - 1;
+    const unsigned rp = (j >= P.ny - 1) ? r : r + 1;
+    const unsigned TS = (unsigned)sizeof(DFG_T);
+    C.off_c = (r * DFG_ROWW + c0) * TS;
+    C.off_xm = (r * DFG_ROWW + cxm) * TS;
+    C.off_xp = (r * DFG_ROWW + cxp) * TS;
+    C.off_ym = (rm * DFG_ROWW + c0) * TS;
+    C.off_yp = (rp * DFG_ROWW + c0) * TS;
+    const long long cell0 = (kb - P.k0) * plane + jc * P.nx + ic;
+    DFG_T* outp = P.out + cell0 * DFG_OUTW;
+    const DFG_T* pin[DFG_NPF_];
+#pragma unroll
+    for (int f = 0; f < DFG_NPF; ++f) pin[f] = P.f[DFG_NSF + f] + cell0 + P.ghost * plane;
+    const DFG_T* tzp = P.tz + kb;
+
+    DFG_T zq[3][DFG_NSF][DFG_VEC];
+    // pre-plane (clamped): its centre becomes z-1 of plane kb
+    dfg_mbar_wait(R.full, R.phase, 0x100000u);
+#pragma unroll
+    for (int f = 0; f < DFG_NSF; ++f) dfg_lds16(zq[0][f], R.tile + f * DFG_TILE_BYTES + C.off_c);
+    dfg_mbar_arrive(DFG_EMPTY(R.full));
+    R.advance();
+    dfg_mbar_wait(R.full, R.phase, 0x100000u);
+    unsigned cur_tile = R.tile, cur_full = R.full;
+#pragma unroll
+    for (int f = 0; f < DFG_NSF; ++f) dfg_lds16(zq[1][f], cur_tile + f * DFG_TILE_BYTES + C.off_c);
+    R.advance();
+    long long k = kb;
+    for (; k + 3 <= ke; k += 3) {
+      dfg_plane<0, 1, 2>(C, R, cur_tile, cur_full, zq, outp, pin, plane, tzp, P.NZ);
+      dfg_plane<1, 2, 0>(C, R, cur_tile, cur_full, zq, outp, pin, plane, tzp, P.NZ);
+      dfg_plane<2, 0, 1>(C, R, cur_tile, cur_full, zq, outp, pin, plane, tzp, P.NZ);
+    }
+    if (k < ke) {
+      dfg_plane<0, 1, 2>(C, R, cur_tile, cur_full, zq, outp, pin, plane, tzp, P.NZ);
+      if (k + 1 < ke) dfg_plane<1, 2, 0>(C, R, cur_tile, cur_full, zq, outp, pin, plane, tzp, P.NZ);
+    }
+    // the post-plane stage was read for its centre only
+    dfg_mbar_arrive(DFG_EMPTY(cur_full));
+  }
+}
+#endif

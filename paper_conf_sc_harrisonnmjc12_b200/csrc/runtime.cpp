@@ -29,19 +29,22 @@ void build_axis(const T* p, int64_t n, std::vector<char>& tab, bool& safe) {
     if (!(p[i] < p[i + 1])) fail(DFG_E_INVALID, "coordinates must be strictly increasing");
   std::vector<T> c(n);
   for (int64_t i = 0; i < n; ++i) c[i] = (p[i] + p[i + 1]) * T(0.5);
-  tab.assign(size_t(2 * n) * sizeof(T), 0);
+  tab.assign(size_t(3 * n) * sizeof(T), 0);
   T* d = reinterpret_cast<T*>(tab.data());
   T* r = d + n;
+  T* nd = r + n;  // exact negation: the fused kernels form num - q0*d with one FFMA2
   for (int64_t i = 0; i < n; ++i) {
     if (n == 1) {  // derivative is 0 by definition; the kernels never read these
       d[i] = T(1);
       r[i] = T(1);
+      nd[i] = T(-1);
       continue;
     }
     int64_t ip = std::min(i + 1, n - 1), im = std::max<int64_t>(i - 1, 0);
     d[i] = c[ip] - c[im];
     if (!(d[i] > T(0))) fail(DFG_E_INVALID, "cell centres coincide (coordinates too close for T)");
     r[i] = T(1) / d[i];
+    nd[i] = -d[i];
     // Markstein's exact-quotient argument needs d and r well inside the normal range.
     double ad = double(d[i]);
     if (!(ad > 0x1p-60 && ad < 0x1p60) || !std::isfinite(double(r[i]))) safe = false;
@@ -613,6 +616,8 @@ std::vector<uint64_t> pack_params(const std::vector<const void*>& f, void* out, 
   for (int64_t v : {m.nx, m.ny, m.nzl, m.NZ, m.k0, int64_t(m.ghost), kbeg, kend, items}) w.push_back(uint64_t(v));
   w.push_back(uint64_t(uint32_t(tiles_x)) | (uint64_t(uint32_t(tiles_y)) << 32));
   w.push_back(uint64_t(uint32_t(kz)) | (uint64_t(uint32_t(vec_ok)) << 32));
+  // nzero = -0.0 in T (the contraction guard of the paired blocks)
+  w.push_back(m.dt == DType::F32 ? uint64_t(0x80000000u) : uint64_t(0x8000000000000000ull));
   return w;
 }
 }  // namespace
