@@ -308,9 +308,11 @@ def main():
                "h2d_bytes_per_step": 3 * fields["u"].numel() * 4 * world,
                "d2h_bytes_per_step": out.numel() * 4 * world, "ms_per_step": te * 1e3}
 
-    strategies = None
+    strategies = variants = sweep = None
     if rank == 0 and world == 1 and not args.no_strategies:
+        variants = variant_leg(dfg, mesh, out, QCRIT, torch, n)
         strategies = strategy_sweep(dfg, synth, torch)
+        sweep = complexity_sweep(dfg, synth, torch)
 
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
@@ -336,7 +338,10 @@ def main():
             "e2e": e2e,
             "gpu_launches": st["kernel_count"],
             "clocks": clk.summary(),
+            "frac_of_spec_8tbs": achieved / 8000.0,
+            "variants": variants,
             "strategies": strategies,
+            "complexity_sweep_768": sweep,
             "cpu_baseline": cpu,
         }
         print(json.dumps(line), flush=True)
@@ -345,11 +350,103 @@ def main():
     return 0
 
 
+def _time_plan(plan, out, torch, iters):
+    for _ in range(3):
+        plan.execute(out)
+    torch.cuda.synchronize()
+    plan.reset_stats()
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    e0.record()
+    for _ in range(iters):
+        plan.execute(out)
+    e1.record()
+    e1.synchronize()
+    st = plan.stats()
+    return e0.elapsed_time(e1) / iters, st["kernel_ms_sum"] / max(1, st["kernel_launches_timed"])
+
+
+def variant_leg(dfg, mesh, out_exact, src, torch, n):
+    """The division variants of the fused kernel on the bench inputs (context:
+    the headline uses the exact variant).  'fast' = num * (1/d): one rounding
+    more per derivative, not bit-identical to the oracle."""
+    res = {}
+    for var in ("fast",):
+        os.environ["DFG_FUSED_VARIANT"] = var
+        try:
+            plan = dfg.Plan(mesh, src, "fused")
+        finally:
+            os.environ.pop("DFG_FUSED_VARIANT", None)
+        out = torch.empty_like(out_exact)
+        ms, kms = _time_plan(plan, out, torch, 50)
+        diff = (out - out_exact).abs().max().item() / out_exact.abs().max().item()
+        res[var] = {"kernel_ms": kms, "cells_per_s": n ** 3 / (kms * 1e-3),
+                    "algorithmic_gb_per_s": ALGO_BYTES_PER_CELL * n ** 3 / (kms * 1e-3) / 1e9,
+                    "normwise_diff_vs_exact": diff, "bit_identical": bool(torch.equal(out, out_exact))}
+        plan.close()
+        del out
+    return res
+
+
+def complexity_sweep(dfg, synth, torch):
+    """Config 5: the expression-complexity sweep (intro -> VelMag -> VortMag
+    -> Q) at 768^3, fp32 and fp64, fused strategy, device-resident inputs."""
+    from oracle.lang import PAPER_PROGRAMS
+    n = 768
+    res = {}
+    for dt, tt, npt in (("f32", torch.float32, np.float32), ("f64", torch.float64, np.float64)):
+        x, y, z = synth.rt_coords(n, n, n, npt)
+        x64, y64, z64 = (a.astype(np.float64) for a in (x, y, z))
+        fields = {c: synth.rt_velocity(c, x64, y64, z64, None, tt, "cuda") for c in "uvw"}
+        out = torch.empty((n, n, n), dtype=tt, device="cuda")
+        for name in ("intro", "velmag", "vortmag", "qcrit"):
+            src, names = PAPER_PROGRAMS[name]
+            mesh = dfg.Mesh(x, y, z)
+            for nm, c in zip(names, "uvw"):
+                mesh.bind(nm, fields[c])
+            plan = dfg.Plan(mesh, src, "fused")
+            ms, kms = _time_plan(plan, out, torch, 20)
+            nbytes = (len(names) + 1) * np.dtype(npt).itemsize
+            info = plan.info()
+            res[f"{name}_{dt}"] = {"filters": info["filters"], "kernel_ms": kms, "cells_per_s": n ** 3 / (kms * 1e-3),
+                                   "algorithmic_gb_per_s": nbytes * n ** 3 / (kms * 1e-3) / 1e9,
+                                   "bytes_per_cell": nbytes, "regs": info["regs"],
+                                   "kernel": {1: "tma", 2: "general", 3: "pointwise"}.get(info["variant"])}
+            plan.close()
+            mesh.close()
+        del fields, out
+        torch.cuda.empty_cache()
+    return res
+
+
 def strategy_sweep(dfg, synth, torch):
-    """Fused vs staged vs roundtrip on Q (config 2, 192^3) with device-resident
-    inputs: cells/s and algorithmic device GB/s per strategy."""
-    from oracle.lang import QCRIT
-    n = 192
+    """Config 2 (192^3: fused vs staged vs roundtrip, VelMag / VortMag / Q) and
+    config 3 (512^3 Q: staged under device-memory caps vs fused)."""
+    from oracle.lang import PAPER_PROGRAMS
+    out = {"config2_192": {}}
+    for name in ("velmag", "vortmag", "qcrit"):
+        out["config2_192"][name] = _strategies_at(dfg, synth, torch, 192, PAPER_PROGRAMS[name][0],
+                                                  ("fused", "staged", "roundtrip"), 7)
+    GiB = 1 << 30
+    c3 = _strategies_at(dfg, synth, torch, 512, PAPER_PROGRAMS["qcrit"][0], ("fused", "staged"), 3)
+    caps = {}
+    x, y, z = synth.rt_coords(512, 512, 512, np.float32)
+    mesh = dfg.Mesh(x, y, z)
+    dummy = torch.empty((512, 512, 512), device="cuda")
+    for c in "uvw":
+        mesh.bind(c, dummy)
+    for cap_gib in (16, 8, 4):
+        try:
+            p = dfg.Plan(mesh, PAPER_PROGRAMS["qcrit"][0], "staged", cap_gib * GiB)
+            caps[f"{cap_gib}GiB"] = "runs"
+            p.close()
+        except dfg.DfgError as e:
+            caps[f"{cap_gib}GiB"] = e.name
+    c3["staged_caps"] = caps
+    out["config3_512_qcrit"] = c3
+    return out
+
+
+def _strategies_at(dfg, synth, torch, n, src, strategies, runs):
     x, y, z = synth.rt_coords(n, n, n, np.float32)
     x64, y64, z64 = (a.astype(np.float64) for a in (x, y, z))
     mesh = dfg.Mesh(x, y, z)
@@ -359,14 +456,14 @@ def strategy_sweep(dfg, synth, torch):
     flush = torch.empty(512 * 1024 * 1024 // 4, dtype=torch.float32, device="cuda")
     res = {}
     ref = None
-    for s in ("fused", "staged", "roundtrip"):
-        plan = dfg.Plan(mesh, QCRIT, s)
+    for s in strategies:
+        plan = dfg.Plan(mesh, src, s)
         out = torch.empty((n, n, n), dtype=torch.float32, device="cuda")
         for _ in range(2):
             plan.execute(out)
         torch.cuda.synchronize()
         times = []
-        for _ in range(7):                  # the paper's protocol: 7 runs, drop min/max (L241)
+        for _ in range(runs):               # the paper's protocol: 7 runs, drop min/max (L241)
             flush.zero_()                   # L2 flush (working set < 4x L2)
             torch.cuda.synchronize()
             e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
@@ -390,7 +487,10 @@ def strategy_sweep(dfg, synth, torch):
         else:
             res[s]["bit_identical_to_fused"] = bool(torch.equal(ref, out))
         plan.close()
-    return {"workload": "Q-criterion 192^3 fp32, device-resident inputs, L2 flushed, mean of 5 of 7", **res}
+        del out
+    del bufs, flush
+    torch.cuda.empty_cache()
+    return {"workload": f"{n}^3 fp32, device-resident inputs, L2 flushed, trimmed mean of {runs} runs", **res}
 
 
 if __name__ == "__main__":
