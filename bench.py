@@ -345,7 +345,12 @@ def main():
             "cpu_baseline": cpu,
         }
         print(json.dumps(line), flush=True)
+    # release the library's NCCL communicator before torch tears its own down
+    torch.cuda.synchronize()
+    plan.close()
+    mesh.close()
     if world > 1:
+        dist.barrier()
         dist.destroy_process_group()
     return 0
 
