@@ -227,6 +227,9 @@ bool host_side(Op op) { return op == Op::Decompose || op == Op::Const; }  // rou
 }  // namespace
 
 Model model(const Dag& dag, dfg_strategy s, bool host) {
+  // the streamed strategy is fusion per z-chunk: its network-level numbers
+  // are fusion's (per-chunk transfers and the ring footprint are physical)
+  if (s == DFG_STREAMED) s = DFG_FUSED;
   Model m;
   Sources src = sources(dag);
   const int64_t F = int64_t(dag.filters.size());
@@ -314,7 +317,7 @@ int64_t predicted_device_bytes(const Dag& dag, dfg_strategy s, int64_t cells, si
   // roundtrip read every kernel argument and write every kernel result.
   Sources src = sources(dag);
   int64_t u = 0;
-  if (s == DFG_FUSED) {
+  if (s == DFG_FUSED || s == DFG_STREAMED) {
     u = int64_t(src.inputs.size()) + units(dag, dag.result);
   } else {
     for (size_t k = 0; k < dag.filters.size(); ++k) {
@@ -424,12 +427,16 @@ PlanImpl::~PlanImpl() {
       cudaEventDestroy(e.second);
     }
   if (mod.mod) drv().ModuleUnload(mod.mod);
+  release_stream_buffers();
+  if (sH2D) cudaStreamDestroy(sH2D);
+  if (sD2H) cudaStreamDestroy(sD2H);
   if (cur >= 0) cudaSetDevice(cur);
 }
 
 std::unique_ptr<PlanImpl> compile_plan(std::shared_ptr<MeshImpl> mesh, const std::string& expr, dfg_strategy s,
                                        size_t cap) {
-  if (s != DFG_ROUNDTRIP && s != DFG_STAGED && s != DFG_FUSED) fail(DFG_E_INVALID, "bad strategy");
+  if (s != DFG_ROUNDTRIP && s != DFG_STAGED && s != DFG_FUSED && s != DFG_STREAMED)
+    fail(DFG_E_INVALID, "bad strategy");
   std::vector<std::string> names;
   for (auto& kv : mesh->fields) names.push_back(kv.first);
   auto plan = std::make_unique<PlanImpl>();
@@ -440,15 +447,16 @@ std::unique_ptr<PlanImpl> compile_plan(std::shared_ptr<MeshImpl> mesh, const std
   const Dag& dag = plan->dag;
   const bool multi = mesh->nzl != mesh->NZ;
   if (multi && s != DFG_FUSED)
-    fail(DFG_E_UNSUPPORTED, "staged/roundtrip run on a single slab; multi-slab meshes use the fused strategy");
+    fail(DFG_E_UNSUPPORTED, "staged/roundtrip/streamed run on a single slab; multi-slab meshes use fusion");
 
   // Footprint check against the cap for the binding modes at compile time
+  // (the streamed ring is bounded by construction; its ledger checks at run time)
   bool any_host = false;
   for (int i : sources(dag).inputs)
     if (!mesh->fields[dag.inputs[i]].on_device) any_host = true;
   Model mdl = model(dag, s, any_host);
   size_t need = size_t(mdl.units) * size_t(mesh->cells()) * dsize(mesh->dt);
-  if (cap && need > cap)
+  if (cap && need > cap && s != DFG_STREAMED)
     fail(DFG_E_NOMEM, "predicted device footprint " + std::to_string(need) + " bytes exceeds the cap " +
                           std::to_string(cap));
 
@@ -457,7 +465,7 @@ std::unique_ptr<PlanImpl> compile_plan(std::shared_ptr<MeshImpl> mesh, const std
   DFG_CUDA(cudaEventCreate(&plan->ev1));
   plan->st.last_ms = -1;
 
-  if (s == DFG_FUSED) {
+  if (s == DFG_FUSED || s == DFG_STREAMED) {
     FusedConfig cfg;
     const char* var = std::getenv("DFG_FUSED_VARIANT");
     if (var && !std::strcmp(var, "ieee")) cfg.div_mode = 0;
@@ -570,6 +578,7 @@ void PlanImpl::execute(void* out, bool out_dev, cudaStream_t s) {
   DFG_CUDA(cudaEventRecord(ev0, s));
   switch (strategy) {
     case DFG_FUSED: exec_fused(out, out_dev, s); break;
+    case DFG_STREAMED: exec_streamed(out, out_dev, s); break;
     case DFG_STAGED: exec_staged(out, out_dev, s); break;
     case DFG_ROUNDTRIP: exec_roundtrip(out, out_dev, s); break;
   }
@@ -589,7 +598,7 @@ void PlanImpl::execute(void* out, bool out_dev, cudaStream_t s) {
 namespace {
 // CUtensorMap for one stencil field: dims {nx, ny, nzl + 2g}, box
 // {32*VEC + 2*VEC, NCW + 2, 1}, OOB fill zero (never read: clamped in smem).
-void encode_map(CUtensorMap* map, const MeshImpl& m, void* base, int ncw) {
+void encode_map(CUtensorMap* map, const SlabView& m, void* base, int ncw) {
   const size_t ts = dsize(m.dt);
   const int vec = int(16 / ts);
   cuuint64_t gdim[3] = {cuuint64_t(m.nx), cuuint64_t(m.ny), cuuint64_t(m.nzl + 2 * m.ghost)};
@@ -604,7 +613,7 @@ void encode_map(CUtensorMap* map, const MeshImpl& m, void* base, int ncw) {
 
 // Host mirror of DfgParams in skeleton.cuh (same field order and widths).
 std::vector<uint64_t> pack_params(const std::vector<const void*>& f, void* out, const void* tx, const void* ty,
-                                  const void* tz, const MeshImpl& m, int64_t kbeg, int64_t kend, int64_t items,
+                                  const void* tz, const SlabView& m, int64_t kbeg, int64_t kend, int64_t items,
                                   int tiles_x, int tiles_y, int kz, int vec_ok) {
   std::vector<uint64_t> w;
   for (auto p : f) w.push_back(reinterpret_cast<uint64_t>(p));
@@ -692,12 +701,29 @@ void PlanImpl::exec_fused(void* out, bool out_dev, cudaStream_t s) {
     scratch.push_back(dout);
   }
 
+  launch_fused(fptr, dout, tab, SlabView::of(m), s);
+  if (!out_dev) {
+    DFG_CUDA(cudaMemcpyAsync(out, dout, out_bytes, cudaMemcpyDeviceToHost, s));
+    st.d2h_count += 1;
+    st.d2h_bytes += int64_t(out_bytes);
+    DFG_CUDA(cudaStreamSynchronize(s));
+  }
+  st.dev_highwater_bytes = std::max<int64_t>(st.dev_highwater_bytes, int64_t(led.high));
+}
+
+// One launch of the generated kernel over the owned planes of a slab view
+// (the mesh itself, or one z-chunk of the streamed strategy).
+void PlanImpl::launch_fused(const std::vector<const void*>& fptr, void* dout, const void* const tab[3],
+                            const SlabView& m, cudaStream_t s) {
+  const size_t ts = dsize(m.dt);
+  const FusedLayout& L = fsrc.layout;
+  const int64_t N = m.nx * m.ny * m.nzl;
   const int vec = int(16 / ts);
   bool vec_ok = aligned16(dout) && (N % vec == 0);
   for (auto p : fptr) vec_ok = vec_ok && aligned16(p);
   const char* force = std::getenv("DFG_FUSED_KERNEL");
   bool want_general = force && !std::strcmp(force, "general");
-  const int sms = sm_count(m.device);
+  const int sms = sm_count(mesh->device);
   const int64_t kbeg = m.k0, kend = m.k0 + m.nzl;
 
   if (L.stencil_inputs.empty()) {
@@ -768,13 +794,146 @@ void PlanImpl::exec_fused(void* out, bool out_dev, cudaStream_t s) {
     last_variant = 2;
   }
   st.kernel_count += 1;
-  if (!out_dev) {
-    DFG_CUDA(cudaMemcpyAsync(out, dout, out_bytes, cudaMemcpyDeviceToHost, s));
-    st.d2h_count += 1;
-    st.d2h_bytes += int64_t(out_bytes);
-    DFG_CUDA(cudaStreamSynchronize(s));
+}
+
+// ----------------------------------------------------------- streamed
+// The paper's future-work streaming strategy (L344, L245): host-resident
+// fields flow through a ring of DFG_STREAM_SLOTS z-chunk slabs.  Chunk c
+// (planes [a, b)) is uploaded with one ghost plane on each side (the
+// neighbour planes inside the mesh), computed by the fused kernel exactly as
+// a z-slab with ghost = 1, and downloaded -- upload, compute and download of
+// different chunks overlap on three streams.  Device memory is bounded by the
+// ring, so meshes larger than HBM run too.
+void PlanImpl::exec_streamed(void* out, bool out_dev, cudaStream_t s) {
+  MeshImpl& m = *mesh;
+  const FusedLayout& L = fsrc.layout;
+  bool all_dev = out_dev;
+  for (int i : sources(dag).inputs) all_dev = all_dev && m.fields[dag.inputs[i]].on_device;
+  if (all_dev) return exec_fused(out, out_dev, s);  // nothing to stream: in situ
+  if (m.nzl != m.NZ) fail(DFG_E_UNSUPPORTED, "the streamed strategy runs on a single slab");
+  const size_t ts = dsize(m.dt);
+  const int64_t plane = m.plane();
+  const int64_t pb = plane * int64_t(ts);
+  const int nf = int(L.stencil_inputs.size() + L.point_inputs.size());
+  std::vector<int> fin;  // input index per kernel field slot
+  for (int i : L.stencil_inputs) fin.push_back(i);
+  for (int i : L.point_inputs) fin.push_back(i);
+
+  // chunk height: ~512 MiB of input per chunk, at least 4 planes (balances the
+  // pipeline fill / drain against per-chunk overheads)
+  int64_t C = std::max<int64_t>(4, (512ll << 20) / std::max<int64_t>(1, pb * std::max(nf, 1)));
+  if (const char* e = std::getenv("DFG_STREAM_PLANES")) C = std::max<int64_t>(1, std::atoll(e));
+  C = std::min<int64_t>(C, m.nzl);
+  const int64_t nchunks = (m.nzl + C - 1) / C;
+  const int R = int(std::min<int64_t>(kStreamSlots, nchunks));
+
+  // ring buffers (cached in the plan; the ledger counts them)
+  const size_t in_bytes = size_t(C + 2) * size_t(pb), out_bytes = size_t(C) * size_t(pb) * size_t(L.outw);
+  if (!stream_ready || stream_C != C || stream_R != R) {
+    release_stream_buffers();
+    for (int r = 0; r < R; ++r) {
+      for (int f = 0; f < nf; ++f) {
+        void* p = nullptr;
+        DFG_CUDA(cudaMalloc(&p, in_bytes));
+        stream_in.push_back(p);
+      }
+      void* p = nullptr;
+      DFG_CUDA(cudaMalloc(&p, out_bytes));
+      stream_out.push_back(p);
+    }
+    for (auto* x : {&sH2D, &sD2H})
+      if (!*x) DFG_CUDA(cudaStreamCreateWithFlags(x, cudaStreamNonBlocking));
+    stream_C = C;
+    stream_R = R;
+    stream_ready = true;
   }
+  Ledger led(cap);
+  led.add(size_t(R) * (size_t(nf) * in_bytes + out_bytes));
+
+  std::vector<cudaEvent_t> ev;
+  auto new_event = [&]() {
+    cudaEvent_t e;
+    DFG_CUDA(cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
+    ev.push_back(e);
+    return e;
+  };
+  struct Destroy {
+    std::vector<cudaEvent_t>& v;
+    ~Destroy() {
+      for (auto e : v) cudaEventDestroy(e);
+    }
+  } guard{ev};
+  cudaEvent_t start = new_event();
+  DFG_CUDA(cudaEventRecord(start, s));
+  DFG_CUDA(cudaStreamWaitEvent(sH2D, start, 0));
+  DFG_CUDA(cudaStreamWaitEvent(sD2H, start, 0));
+  std::vector<cudaEvent_t> computed(nchunks), downloaded(nchunks);
+  const void* tab[3] = {m.dev_tab[0], m.dev_tab[1], m.dev_tab[2]};
+  for (int64_t c = 0; c < nchunks; ++c) {
+    const int r = int(c % R);
+    const int64_t a = c * C, b = std::min(m.nzl, a + C);
+    const int64_t lo = std::max<int64_t>(a - 1, 0), hi = std::min<int64_t>(b + 1, m.NZ);
+    // slot r is free once chunk c-R was computed (inputs) and downloaded (output)
+    if (c >= R) {
+      DFG_CUDA(cudaStreamWaitEvent(sH2D, computed[c - R], 0));
+      DFG_CUDA(cudaStreamWaitEvent(s, downloaded[c - R], 0));
+    }
+    std::vector<const void*> fptr;
+    for (int f = 0; f < nf; ++f) {
+      char* dst = static_cast<char*>(stream_in[size_t(r) * nf + f]);
+      const Binding& bd = m.fields[dag.inputs[fin[f]]];
+      // local plane index of global plane g is g - a + 1 (ghost plane 0)
+      int64_t from = lo;
+      if (c > 0) {
+        // planes a-1 and a already sit in the previous slot (its local C, C+1)
+        const char* prev = static_cast<const char*>(stream_in[size_t((c - 1) % R) * nf + f]);
+        DFG_CUDA(cudaMemcpyAsync(dst, prev + C * pb, size_t(2 * pb), cudaMemcpyDeviceToDevice, sH2D));
+        from = a + 1;
+      }
+      if (hi > from) {
+        const char* src = static_cast<const char*>(bd.ptr) + (from + m.ghost) * pb;
+        DFG_CUDA(cudaMemcpyAsync(dst + (from - a + 1) * pb, src, size_t(hi - from) * size_t(pb),
+                                 bd.on_device ? cudaMemcpyDeviceToDevice : cudaMemcpyHostToDevice, sH2D));
+        if (!bd.on_device) {
+          st.h2d_count += 1;
+          st.h2d_bytes += (hi - from) * pb;
+        }
+      }
+      fptr.push_back(dst);
+    }
+    cudaEvent_t up = new_event();
+    DFG_CUDA(cudaEventRecord(up, sH2D));
+    DFG_CUDA(cudaStreamWaitEvent(s, up, 0));
+    SlabView v{m.dt, m.nx, m.ny, b - a, m.NZ, a, 1};
+    launch_fused(fptr, stream_out[r], tab, v, s);
+    computed[c] = new_event();
+    DFG_CUDA(cudaEventRecord(computed[c], s));
+    DFG_CUDA(cudaStreamWaitEvent(sD2H, computed[c], 0));
+    char* dsto = static_cast<char*>(out) + a * pb * int64_t(L.outw);
+    DFG_CUDA(cudaMemcpyAsync(dsto, stream_out[r], size_t(b - a) * size_t(pb) * size_t(L.outw),
+                             out_dev ? cudaMemcpyDeviceToDevice : cudaMemcpyDeviceToHost, sD2H));
+    if (!out_dev) {
+      st.d2h_count += 1;
+      st.d2h_bytes += (b - a) * pb * int64_t(L.outw);
+    }
+    downloaded[c] = new_event();
+    DFG_CUDA(cudaEventRecord(downloaded[c], sD2H));
+  }
+  // join: the caller's stream waits for the last download and upload
+  cudaEvent_t up_done = new_event();
+  DFG_CUDA(cudaEventRecord(up_done, sH2D));
+  DFG_CUDA(cudaStreamWaitEvent(s, up_done, 0));
+  DFG_CUDA(cudaStreamWaitEvent(s, downloaded[nchunks - 1], 0));
+  if (!out_dev) DFG_CUDA(cudaStreamSynchronize(s));
   st.dev_highwater_bytes = std::max<int64_t>(st.dev_highwater_bytes, int64_t(led.high));
+}
+
+void PlanImpl::release_stream_buffers() {
+  for (void* p : stream_in) cudaFree(p);
+  for (void* p : stream_out) cudaFree(p);
+  stream_in.clear();
+  stream_out.clear();
+  stream_ready = false;
 }
 
 // ------------------------------------------------------------- staged

@@ -40,6 +40,18 @@ struct MeshImpl {
   size_t field_bytes() const { return size_t(nx * ny * (nzl + 2 * ghost)) * dsize(dt); }
 };
 
+// The part of a mesh one fused launch covers: a whole mesh, a z-slab of a
+// multi-GPU mesh, or one z-chunk of the streamed strategy (ghost planes at
+// local 0 and nzl+1 when ghost = 1).
+struct SlabView {
+  DType dt;
+  int64_t nx, ny, nzl, NZ, k0;
+  int ghost;
+  static SlabView of(const MeshImpl& m) { return SlabView{m.dt, m.nx, m.ny, m.nzl, m.NZ, m.k0, m.ghost}; }
+};
+
+constexpr int kStreamSlots = 3;  // ring depth of the streamed strategy
+
 std::shared_ptr<MeshImpl> create_mesh(DType dt, int64_t nx, int64_t ny, int64_t nzl, const void* x, const void* y,
                                       const void* z, int64_t NZ, int64_t k0, int ghost);
 
@@ -69,10 +81,20 @@ struct PlanImpl {
   std::pair<cudaEvent_t, cudaEvent_t> kernel_events();
   void resolve_kernel_times();
   std::map<std::string, std::vector<char>> const_cache;  // roundtrip host constants
+  // streamed strategy: ring of chunk slabs and the two copy streams
+  std::vector<void*> stream_in, stream_out;
+  int64_t stream_C = 0;
+  int stream_R = 0;
+  bool stream_ready = false;
+  cudaStream_t sH2D = nullptr, sD2H = nullptr;
   ~PlanImpl();
   void execute(void* out, bool out_dev, cudaStream_t s);
 
  private:
+  void launch_fused(const std::vector<const void*>& fptr, void* dout, const void* const tab[3], const SlabView& v,
+                    cudaStream_t s);
+  void exec_streamed(void* out, bool out_dev, cudaStream_t s);
+  void release_stream_buffers();
   void exec_fused(void* out, bool out_dev, cudaStream_t s);
   void exec_staged(void* out, bool out_dev, cudaStream_t s);
   void exec_roundtrip(void* out, bool out_dev, cudaStream_t s);
