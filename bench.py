@@ -392,6 +392,16 @@ def variant_leg(dfg, mesh, out_exact, src, torch, n):
                     "normwise_diff_vs_exact": diff, "bit_identical": bool(torch.equal(out, out_exact))}
         plan.close()
         del out
+    # the hand-written reference kernel (L243; strategy "reference")
+    plan = dfg.Plan(mesh, "qcrit", "reference")
+    out = torch.empty_like(out_exact)
+    ms, kms = _time_plan(plan, out, torch, 50)
+    diff = (out - out_exact).abs().max().item() / out_exact.abs().max().item()
+    res["reference_kernel"] = {"kernel_ms": kms, "cells_per_s": n ** 3 / (kms * 1e-3),
+                               "algorithmic_gb_per_s": ALGO_BYTES_PER_CELL * n ** 3 / (kms * 1e-3) / 1e9,
+                               "normwise_diff_vs_exact": diff}
+    plan.close()
+    del out
     return res
 
 

@@ -41,7 +41,7 @@ typedef enum {
   DFG_ROUNDTRIP = 0, /* one kernel per primitive, every result to the host (L92) */
   DFG_STAGED = 1,    /* one kernel per primitive, intermediates on the device (L96) */
   DFG_FUSED = 2,     /* one generated kernel, intermediates in registers (L97) */
-  DFG_STREAMED = 3   /* fusion over z-chunks streamed through a 3-slot device ring with
+  DFG_STREAMED = 3,  /* fusion over z-chunks streamed through a 3-slot device ring with
                         overlapped upload / kernel / download (the paper's future-work
                         streaming strategy, L245 / L344); bounded device memory, so host
                         meshes larger than HBM work; single slab; with everything
@@ -49,6 +49,11 @@ typedef enum {
                         input per chunk (env DFG_STREAM_PLANES overrides); each field
                         plane crosses PCIe once (chunk halos are copied on the device).
                         Pinned host buffers are needed for the copies to overlap. */
+  DFG_REFERENCE = 4  /* the hand-written reference kernel of a quantity (L243): expr is
+                        "velmag", "vortmag" or "qcrit" (fields u, v, w must be bound);
+                        same I/O and TMA pipeline as fusion, fewer flops (derivative =
+                        numerator x reciprocal spacing, FMA, Q = -1/2 tr(J^2)); agrees
+                        with the network within floating-point tolerance, not bitwise */
 } dfg_strategy;
 
 typedef enum { DFG_F32 = 0, DFG_F64 = 1 } dfg_dtype;

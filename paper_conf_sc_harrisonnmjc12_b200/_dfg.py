@@ -22,9 +22,10 @@ if not os.path.exists(LIB_PATH):
 
 _lib = C.CDLL(LIB_PATH, mode=C.RTLD_GLOBAL)
 
-DFG_ROUNDTRIP, DFG_STAGED, DFG_FUSED, DFG_STREAMED = 0, 1, 2, 3
+DFG_ROUNDTRIP, DFG_STAGED, DFG_FUSED, DFG_STREAMED, DFG_REFERENCE = 0, 1, 2, 3, 4
 DFG_F32, DFG_F64 = 0, 1
-STRATEGIES = {"roundtrip": DFG_ROUNDTRIP, "staged": DFG_STAGED, "fused": DFG_FUSED, "streamed": DFG_STREAMED}
+STRATEGIES = {"roundtrip": DFG_ROUNDTRIP, "staged": DFG_STAGED, "fused": DFG_FUSED, "streamed": DFG_STREAMED,
+              "reference": DFG_REFERENCE}
 STATUS = {0: "DFG_OK", -1: "DFG_E_INVALID", -2: "DFG_E_PARSE", -3: "DFG_E_UNDEFINED", -4: "DFG_E_TYPE",
           -5: "DFG_E_NOMEM", -6: "DFG_E_NVRTC", -7: "DFG_E_CUDA", -8: "DFG_E_NCCL", -9: "DFG_E_UNBOUND",
           -10: "DFG_E_UNSUPPORTED", -11: "DFG_E_RANGE"}

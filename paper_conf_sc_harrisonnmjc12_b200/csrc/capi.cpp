@@ -251,9 +251,11 @@ int dfg_model(const char* expr, const char* const* inputs, int n_inputs, dfg_str
               int64_t out[4]) {
   return guard([&] {
     if (!expr || !out) dfg::fail(DFG_E_INVALID, "null argument");
-    if (strategy != DFG_ROUNDTRIP && strategy != DFG_STAGED && strategy != DFG_FUSED && strategy != DFG_STREAMED)
-      dfg::fail(DFG_E_INVALID, "bad strategy");
-    dfg::Dag d = dfg::build_dag(expr, names_of(inputs, n_inputs), dfg::DType::F32);
+    if (strategy < DFG_ROUNDTRIP || strategy > DFG_REFERENCE) dfg::fail(DFG_E_INVALID, "bad strategy");
+    int ref = 0;
+    const char* prog = strategy == DFG_REFERENCE ? dfg::reference_program(expr, &ref) : expr;
+    if (!prog) dfg::fail(DFG_E_INVALID, "reference kernels exist for velmag, vortmag and qcrit");
+    dfg::Dag d = dfg::build_dag(prog, names_of(inputs, n_inputs), dfg::DType::F32);
     dfg::Model m = dfg::model(d, strategy, host_mode != 0);
     out[0] = m.h2d;
     out[1] = m.d2h;

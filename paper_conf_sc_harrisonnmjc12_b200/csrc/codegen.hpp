@@ -36,7 +36,13 @@ struct FusedSource {
 
 FusedLayout fused_layout(const Dag& dag);
 // nx/ny/nz: global mesh dims (axis degeneracy n == 1 is baked in).
-FusedSource generate_fused(const Dag& dag, int64_t nx, int64_t ny, int64_t nz, FusedConfig cfg);
+// ref > 0: use the hand-written reference body `ref` (reference_bodies.cuh)
+// instead of generating one from the network.
+FusedSource generate_fused(const Dag& dag, int64_t nx, int64_t ny, int64_t nz, FusedConfig cfg, int ref = 0);
+
+// Reference kernels: the paper program of a quantity
+// ("velmag", "vortmag", "qcrit") and its body id, or nullptr / 0.
+const char* reference_program(const std::string& which, int* id);
 
 // Dynamic shared memory the TMA kernel needs for a config (bytes).
 size_t fused_tma_smem_bytes(DType dt, int nsf, int ncw, int stages);

@@ -228,8 +228,9 @@ bool host_side(Op op) { return op == Op::Decompose || op == Op::Const; }  // rou
 
 Model model(const Dag& dag, dfg_strategy s, bool host) {
   // the streamed strategy is fusion per z-chunk: its network-level numbers
-  // are fusion's (per-chunk transfers and the ring footprint are physical)
-  if (s == DFG_STREAMED) s = DFG_FUSED;
+  // are fusion's (per-chunk transfers and the ring footprint are physical);
+  // a reference kernel has fusion's I/O
+  if (s == DFG_STREAMED || s == DFG_REFERENCE) s = DFG_FUSED;
   Model m;
   Sources src = sources(dag);
   const int64_t F = int64_t(dag.filters.size());
@@ -317,7 +318,7 @@ int64_t predicted_device_bytes(const Dag& dag, dfg_strategy s, int64_t cells, si
   // roundtrip read every kernel argument and write every kernel result.
   Sources src = sources(dag);
   int64_t u = 0;
-  if (s == DFG_FUSED || s == DFG_STREAMED) {
+  if (s == DFG_FUSED || s == DFG_STREAMED || s == DFG_REFERENCE) {
     u = int64_t(src.inputs.size()) + units(dag, dag.result);
   } else {
     for (size_t k = 0; k < dag.filters.size(); ++k) {
@@ -435,7 +436,7 @@ PlanImpl::~PlanImpl() {
 
 std::unique_ptr<PlanImpl> compile_plan(std::shared_ptr<MeshImpl> mesh, const std::string& expr, dfg_strategy s,
                                        size_t cap) {
-  if (s != DFG_ROUNDTRIP && s != DFG_STAGED && s != DFG_FUSED && s != DFG_STREAMED)
+  if (s != DFG_ROUNDTRIP && s != DFG_STAGED && s != DFG_FUSED && s != DFG_STREAMED && s != DFG_REFERENCE)
     fail(DFG_E_INVALID, "bad strategy");
   std::vector<std::string> names;
   for (auto& kv : mesh->fields) names.push_back(kv.first);
@@ -443,10 +444,17 @@ std::unique_ptr<PlanImpl> compile_plan(std::shared_ptr<MeshImpl> mesh, const std
   plan->mesh = mesh;
   plan->strategy = s;
   plan->cap = cap;
-  plan->dag = build_dag(expr, names, mesh->dt);
+  int ref = 0;
+  if (s == DFG_REFERENCE) {
+    const char* prog = reference_program(expr, &ref);
+    if (!prog) fail(DFG_E_INVALID, "reference kernels exist for \"velmag\", \"vortmag\" and \"qcrit\"");
+    plan->dag = build_dag(prog, names, mesh->dt);
+  } else {
+    plan->dag = build_dag(expr, names, mesh->dt);
+  }
   const Dag& dag = plan->dag;
   const bool multi = mesh->nzl != mesh->NZ;
-  if (multi && s != DFG_FUSED)
+  if (multi && s != DFG_FUSED && s != DFG_REFERENCE)
     fail(DFG_E_UNSUPPORTED, "staged/roundtrip/streamed run on a single slab; multi-slab meshes use fusion");
 
   // Footprint check against the cap for the binding modes at compile time
@@ -465,7 +473,7 @@ std::unique_ptr<PlanImpl> compile_plan(std::shared_ptr<MeshImpl> mesh, const std
   DFG_CUDA(cudaEventCreate(&plan->ev1));
   plan->st.last_ms = -1;
 
-  if (s == DFG_FUSED || s == DFG_STREAMED) {
+  if (s == DFG_FUSED || s == DFG_STREAMED || s == DFG_REFERENCE) {
     FusedConfig cfg;
     const char* var = std::getenv("DFG_FUSED_VARIANT");
     if (var && !std::strcmp(var, "ieee")) cfg.div_mode = 0;
@@ -475,7 +483,7 @@ std::unique_ptr<PlanImpl> compile_plan(std::shared_ptr<MeshImpl> mesh, const std
     if (ncw) cfg.ncw = std::max(1, std::min(30, std::atoi(ncw)));
     const char* st = std::getenv("DFG_STAGES");
     if (st) cfg.stages = std::max(2, std::min(16, std::atoi(st)));
-    plan->fsrc = generate_fused(dag, mesh->nx, mesh->ny, mesh->NZ, cfg);
+    plan->fsrc = generate_fused(dag, mesh->nx, mesh->ny, mesh->NZ, cfg, ref);
     const Cubin& cb = nvrtc_compile(plan->fsrc.source, "dfg_fused.cu");
     plan->regs = cb.regs;
     plan->spill = cb.spill;
@@ -579,6 +587,7 @@ void PlanImpl::execute(void* out, bool out_dev, cudaStream_t s) {
   switch (strategy) {
     case DFG_FUSED: exec_fused(out, out_dev, s); break;
     case DFG_STREAMED: exec_streamed(out, out_dev, s); break;
+    case DFG_REFERENCE: exec_fused(out, out_dev, s); break;
     case DFG_STAGED: exec_staged(out, out_dev, s); break;
     case DFG_ROUNDTRIP: exec_roundtrip(out, out_dev, s); break;
   }

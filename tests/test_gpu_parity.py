@@ -354,3 +354,22 @@ def test_streamed_pinned_large(monkeypatch):
     assert torch.equal(o1.cpu(), o2)
     st = p2.stats()
     assert st["dev_highwater_bytes"] < 4 * n ** 3 * 4      # bounded ring, below fused's footprint
+
+
+@pytest.mark.parametrize("prog", ["velmag", "vortmag", "qcrit"])
+@pytest.mark.parametrize("T", [np.float32, np.float64])
+@pytest.mark.parametrize("shape", [(64, 40, 33), (67, 21, 9)])
+def test_reference_kernels(prog, T, shape):
+    """Hand-written reference kernels (L243): same I/O as fusion, fewer flops;
+    they agree with the oracle within the floating-point tolerance (R15),
+    not bit for bit (one rounding more per derivative, FMA, Q = -tr(J^2)/2)."""
+    x, y, z, f = _inputs(shape, T)
+    want = run_oracle(PAPER_PROGRAMS[prog][0], f, x, y, z)
+    got, plan, *_ = run_lib(prog, f, x, y, z, "reference", return_plan=True)
+    assert_parity(got, want, exact=False)
+    assert plan.stats()["kernel_count"] == 1
+    assert "dfg-dag v1" in plan.dag()
+    # unknown quantities are rejected
+    import paper_conf_sc_harrisonnmjc12_b200 as dfg
+    with pytest.raises(dfg.DfgError):
+        run_lib("intro", f, x, y, z, "reference")
