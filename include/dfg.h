@@ -202,6 +202,13 @@ int dfg_reset_stats(dfg_plan plan);
  * out[7] = same for host inputs. */
 int dfg_plan_info(dfg_plan plan, int64_t out[8]);
 
+/* Execution order of the plan's filters (ids of the canonical text).  Staged
+ * plans run the paper's list order unless a dev_mem_cap rejected it and the
+ * memory-aware order (greedy minimum live memory) fits --
+ * or DFG_STAGED_ORDER=greedy was set at compile.  Writes min(cap, n) ids;
+ * *n = number of filters. */
+int dfg_plan_schedule(dfg_plan plan, int32_t* order, size_t cap, size_t* n);
+
 /* Canonical network text (R10) -- stands in for the paper's
  * optional Python script of network-definition API calls (L84).
  * Copies up to cap bytes incl. the NUL; *needed = full size incl. NUL;

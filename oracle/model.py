@@ -117,8 +117,25 @@ def _refcounts(dag: Dag):
     return rc
 
 
-def footprint(dag: Dag, strategy: str, mode: str = "host") -> int:
-    """Device high-water in problem-array units (Fig. 2)."""
+def is_topological(dag: Dag, order) -> bool:
+    """Every filter exactly once, each after all the filters it reads."""
+    if sorted(order) != list(range(len(dag.filters))):
+        return False
+    pos = {k: i for i, k in enumerate(order)}
+    for k, f in enumerate(dag.filters):
+        for r in f.inputs:
+            j = dag.ref_filter(r)
+            if j is not None and pos[int(r[1:])] > pos[k]:
+                return False
+    return True
+
+
+def footprint(dag: Dag, strategy: str, mode: str = "host", order=None) -> int:
+    """Device high-water in problem-array units (Fig. 2).  ``order`` = the
+    execution order of the staged strategy (default: list order, L72/L85)."""
+    if order is not None and strategy == "staged":
+        assert is_topological(dag, order)
+        return _staged_footprint(dag, mode, order)
     srcs, _ = _sources(dag)
     out_units = _units(dag, dag.result)
     if strategy == "fused":
@@ -144,6 +161,16 @@ def footprint(dag: Dag, strategy: str, mode: str = "host") -> int:
             high = max(high, base + args + _units(dag, f"f{k}"))
         return high
     if strategy == "staged":
+        return _staged_footprint(dag, mode, range(len(dag.filters)))
+    raise ValueError(strategy)
+
+
+def _staged_footprint(dag: Dag, mode: str, order) -> int:
+    """Lazy upload, free at reference count zero, filters run in ``order``."""
+    srcs, _ = _sources(dag)
+    out_units = _units(dag, dag.result)
+    order = list(order)
+    if True:
         rc = _refcounts(dag)
         live = 0
         high = 0
@@ -152,8 +179,9 @@ def footprint(dag: Dag, strategy: str, mode: str = "host") -> int:
             live = sum(_units(dag, s) for s in srcs) + out_units
             resident = set(srcs)
             high = live
-        last = len(dag.filters) - 1
-        for k, f in enumerate(dag.filters):
+        last = order[-1] if order else -1
+        for k in order:
+            f = dag.filters[k]
             ref = f"f{k}"
             for r in f.inputs:
                 if r in MESH_NAMES or _is_filter(dag, r) or r in resident:
@@ -174,4 +202,3 @@ def footprint(dag: Dag, strategy: str, mode: str = "host") -> int:
             live += _units(dag, dag.result)       # bare input result: upload it
             high = max(high, live)
         return high
-    raise ValueError(strategy)

@@ -89,6 +89,10 @@ class Plan:
     def dag(self):
         return dfg_dump_dag(self.handle)
 
+    def schedule(self):
+        from ._dfg import dfg_plan_schedule
+        return dfg_plan_schedule(self.handle)
+
     def kernel_source(self):
         return dfg_dump_kernel(self.handle)
 

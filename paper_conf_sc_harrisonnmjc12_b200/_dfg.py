@@ -68,6 +68,7 @@ _SIGS = {
     "dfg_plan_stats": (C.c_int, [_P, C.POINTER(dfg_stats)]),
     "dfg_reset_stats": (C.c_int, [_P]),
     "dfg_plan_info": (C.c_int, [_P, C.POINTER(_I64)]),
+    "dfg_plan_schedule": (C.c_int, [_P, C.POINTER(C.c_int32), C.c_size_t, C.POINTER(C.c_size_t)]),
     "dfg_dump_dag": (C.c_int, [_P, C.c_char_p, C.c_size_t, C.POINTER(C.c_size_t)]),
     "dfg_dump_kernel": (C.c_int, [_P, C.c_char_p, C.c_size_t, C.POINTER(C.c_size_t)]),
     "dfg_dag_dump": (C.c_int, [C.c_char_p, C.POINTER(C.c_char_p), C.c_int, C.c_int, C.c_char_p, C.c_size_t,
@@ -199,6 +200,14 @@ def dfg_plan_info(plan) -> dict:
     _check(_lib.dfg_plan_info(plan, out))
     keys = ("strategy", "width", "filters", "variant", "regs", "spill", "footprint_device", "footprint_host")
     return dict(zip(keys, list(out)))
+
+
+def dfg_plan_schedule(plan) -> list:
+    n = C.c_size_t(0)
+    _check(_lib.dfg_plan_schedule(plan, None, 0, C.byref(n)))
+    arr = (C.c_int32 * max(n.value, 1))()
+    _check(_lib.dfg_plan_schedule(plan, arr, n.value, C.byref(n)))
+    return list(arr)[: n.value]
 
 
 def dfg_dump_dag(plan) -> str:

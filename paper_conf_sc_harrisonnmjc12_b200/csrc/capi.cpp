@@ -224,6 +224,15 @@ int dfg_plan_info(dfg_plan plan, int64_t out[8]) {
   });
 }
 
+int dfg_plan_schedule(dfg_plan plan, int32_t* order, size_t cap, size_t* n) {
+  return guard([&] {
+    if (!plan || !n) dfg::fail(DFG_E_INVALID, "null argument");
+    const auto& o = plan->p->order;
+    *n = o.size();
+    for (size_t i = 0; i < o.size() && i < cap && order; ++i) order[i] = o[i];
+  });
+}
+
 int dfg_dump_dag(dfg_plan plan, char* buf, size_t cap, size_t* needed) {
   return guard([&] {
     if (!plan) dfg::fail(DFG_E_INVALID, "null plan");

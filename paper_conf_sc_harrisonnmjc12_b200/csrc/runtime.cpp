@@ -275,41 +275,92 @@ Model model(const Dag& dag, dfg_strategy s, bool host) {
     }
     m.units = high;
   } else {
-    std::map<std::pair<int, int>, int64_t> rc;
-    auto key = [](const Ref& r) { return std::make_pair(int(r.kind), r.id); };
-    for (auto& f : dag.filters)
-      for (auto& r : f.in)
-        if (r.kind != Ref::Mesh) rc[key(r)] += 1;
-    rc[key(dag.result)] += 1;
-    std::set<int> resident;
-    int64_t live = 0, high = 0;
-    if (!host) {
-      live = in_u + out_u;
-      for (int i : src.inputs) resident.insert(i);
-      high = live;
-    }
-    for (size_t k = 0; k < dag.filters.size(); ++k) {
-      const Filter& f = dag.filters[k];
-      for (auto& r : f.in)
-        if (r.kind == Ref::Input && !resident.count(r.id)) {
-          resident.insert(r.id);
-          live += 1;
-        }
-      bool into_out = !host && dag.result.kind == Ref::Filter && dag.result.id == int(k) && k + 1 == dag.filters.size();
-      if (!into_out) live += f.width == 1 ? 1 : 4;
-      high = std::max(high, live);
-      for (auto& r : f.in) {
-        if (r.kind == Ref::Mesh) continue;
-        if (--rc[key(r)] == 0 && (host || r.kind == Ref::Filter)) live -= units(dag, r);
-      }
-    }
-    if (dag.result.kind == Ref::Input && !resident.count(dag.result.id)) {
-      live += 1;
-      high = std::max(high, live);
-    }
-    m.units = high;
+    std::vector<int> order(dag.filters.size());
+    for (size_t k = 0; k < order.size(); ++k) order[k] = int(k);
+    m.units = staged_units(dag, order, host);
   }
   return m;
+}
+
+// Staged footprint of a given execution order: lazy upload of host inputs,
+// free at reference count zero (L85), Fig. 2 accounting.
+int64_t staged_units(const Dag& dag, const std::vector<int>& order, bool host) {
+  Sources src = sources(dag);
+  std::map<std::pair<int, int>, int64_t> rc;
+  auto key = [](const Ref& r) { return std::make_pair(int(r.kind), r.id); };
+  for (auto& f : dag.filters)
+    for (auto& r : f.in)
+      if (r.kind != Ref::Mesh) rc[key(r)] += 1;
+  rc[key(dag.result)] += 1;
+  std::set<int> resident;
+  int64_t live = 0, high = 0;
+  if (!host) {
+    live = int64_t(src.inputs.size()) + units(dag, dag.result);
+    for (int i : src.inputs) resident.insert(i);
+    high = live;
+  }
+  for (size_t pos = 0; pos < order.size(); ++pos) {
+    const int k = order[pos];
+    const Filter& f = dag.filters[k];
+    for (auto& r : f.in)
+      if (r.kind == Ref::Input && !resident.count(r.id)) {
+        resident.insert(r.id);
+        live += 1;
+      }
+    bool into_out = !host && dag.result.kind == Ref::Filter && dag.result.id == k && pos + 1 == order.size();
+    if (!into_out) live += f.width == 1 ? 1 : 4;
+    high = std::max(high, live);
+    for (auto& r : f.in) {
+      if (r.kind == Ref::Mesh) continue;
+      if (--rc[key(r)] == 0 && (host || r.kind == Ref::Filter)) live -= units(dag, r);
+    }
+  }
+  if (dag.result.kind == Ref::Input && !resident.count(dag.result.id)) {
+    live += 1;
+    high = std::max(high, live);
+  }
+  return high;
+}
+
+// Memory-aware staged schedule: repeatedly run the ready
+// filter whose execution changes the live device memory the least
+// (allocation minus arrays it frees; ties to the lowest id).
+std::vector<int> greedy_staged_order(const Dag& dag) {
+  const size_t n = dag.filters.size();
+  std::map<int, int64_t> rc;  // remaining uses of each filter result
+  for (auto& f : dag.filters)
+    for (auto& r : f.in)
+      if (r.kind == Ref::Filter) rc[r.id] += 1;
+  if (dag.result.kind == Ref::Filter) rc[dag.result.id] += 1;
+  std::vector<char> done(n, 0);
+  std::vector<int> order;
+  while (order.size() < n) {
+    int best = -1;
+    int64_t best_delta = 0;
+    for (size_t k = 0; k < n; ++k) {
+      if (done[k]) continue;
+      const Filter& f = dag.filters[k];
+      bool ready = true;
+      for (auto& r : f.in)
+        if (r.kind == Ref::Filter && !done[r.id]) ready = false;
+      if (!ready) continue;
+      int64_t delta = f.width == 1 ? 1 : 4;
+      std::map<int, int64_t> uses;
+      for (auto& r : f.in)
+        if (r.kind == Ref::Filter) uses[r.id] += 1;
+      for (auto& u : uses)
+        if (rc[u.first] == u.second) delta -= dag.filters[u.first].width == 1 ? 1 : 4;
+      if (best < 0 || delta < best_delta) {
+        best = int(k);
+        best_delta = delta;
+      }
+    }
+    done[best] = 1;
+    order.push_back(best);
+    for (auto& r : dag.filters[best].in)
+      if (r.kind == Ref::Filter) rc[r.id] -= 1;
+  }
+  return order;
 }
 
 int64_t predicted_device_bytes(const Dag& dag, dfg_strategy s, int64_t cells, size_t ts) {
@@ -463,7 +514,24 @@ std::unique_ptr<PlanImpl> compile_plan(std::shared_ptr<MeshImpl> mesh, const std
   for (int i : sources(dag).inputs)
     if (!mesh->fields[dag.inputs[i]].on_device) any_host = true;
   Model mdl = model(dag, s, any_host);
-  size_t need = size_t(mdl.units) * size_t(mesh->cells()) * dsize(mesh->dt);
+  const size_t unit_bytes = size_t(mesh->cells()) * dsize(mesh->dt);
+  size_t need = size_t(mdl.units) * unit_bytes;
+  plan->order.resize(dag.filters.size());
+  for (size_t k = 0; k < plan->order.size(); ++k) plan->order[k] = int(k);
+  if (s == DFG_STAGED) {
+    // the paper's list order, unless a cap rejects it and the memory-aware
+    // order fits (or DFG_STAGED_ORDER=greedy asks for it)
+    const char* env = std::getenv("DFG_STAGED_ORDER");
+    const bool force = env && !std::strcmp(env, "greedy");
+    if (force || (cap && need > cap)) {
+      std::vector<int> g = greedy_staged_order(dag);
+      size_t gneed = size_t(staged_units(dag, g, any_host)) * unit_bytes;
+      if (force || gneed <= cap) {
+        plan->order = g;
+        need = gneed;
+      }
+    }
+  }
   if (cap && need > cap && s != DFG_STREAMED)
     fail(DFG_E_NOMEM, "predicted device footprint " + std::to_string(need) + " bytes exceeds the cap " +
                           std::to_string(cap));
@@ -598,8 +666,8 @@ void PlanImpl::execute(void* out, bool out_dev, cudaStream_t s) {
   bool any_host = !out_dev;
   for (int i : sources(dag).inputs)
     if (!m.fields[dag.inputs[i]].on_device) any_host = true;
-  st.predicted_highwater_bytes =
-      model(dag, strategy, any_host).units * m.cells() * int64_t(dsize(m.dt));
+  const int64_t units = strategy == DFG_STAGED ? staged_units(dag, order, any_host) : model(dag, strategy, any_host).units;
+  st.predicted_highwater_bytes = units * m.cells() * int64_t(dsize(m.dt));
   st.predicted_hbm_bytes = predicted_device_bytes(dag, strategy, m.cells(), dsize(m.dt));
   st.predicted_pcie_bytes = predicted_pcie_bytes(dag, strategy, m.cells(), dsize(m.dt), any_host);
 }
@@ -1045,14 +1113,15 @@ void PlanImpl::exec_staged(void* out, bool out_dev, cudaStream_t s) {
   };
 
   const size_t nf = dag.filters.size();
-  for (size_t k = 0; k < nf; ++k) {
+  for (size_t pos = 0; pos < nf; ++pos) {
+    const size_t k = size_t(order[pos]);  // list order, or the memory-aware order
     const Filter& f = dag.filters[k];
     for (auto& r : f.in) {
       if (r.kind == Ref::Input) ensure_input(r.id);
       if (r.kind == Ref::Mesh) ensure_mesh();
     }
     const size_t ob = sb * size_t(f.width == 1 ? 1 : 4);
-    const bool into_out = out_dev && dag.result.kind == Ref::Filter && dag.result.id == int(k) && k + 1 == nf;
+    const bool into_out = out_dev && dag.result.kind == Ref::Filter && dag.result.id == int(k) && pos + 1 == nf;
     void* o;
     if (into_out) {
       o = out;

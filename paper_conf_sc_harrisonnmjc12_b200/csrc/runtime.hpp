@@ -61,6 +61,8 @@ struct Model {
   int64_t units = 0;  // footprint in problem-array units (scalar 1, vector 4)
 };
 Model model(const Dag& dag, dfg_strategy s, bool host_mode);
+int64_t staged_units(const Dag& dag, const std::vector<int>& order, bool host_mode);
+std::vector<int> greedy_staged_order(const Dag& dag);
 int64_t predicted_device_bytes(const Dag& dag, dfg_strategy s, int64_t cells, size_t tsize);
 int64_t predicted_pcie_bytes(const Dag& dag, dfg_strategy s, int64_t cells, size_t tsize, bool host_mode);
 
@@ -81,6 +83,7 @@ struct PlanImpl {
   std::pair<cudaEvent_t, cudaEvent_t> kernel_events();
   void resolve_kernel_times();
   std::map<std::string, std::vector<char>> const_cache;  // roundtrip host constants
+  std::vector<int> order;  // staged execution order (list order unless a cap forced a reorder)
   // streamed strategy: ring of chunk slabs and the two copy streams
   std::vector<void*> stream_in, stream_out;
   int64_t stream_C = 0;

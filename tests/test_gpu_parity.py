@@ -153,6 +153,31 @@ def test_memory_highwater_measured(strategy, host):
         assert plan.stats()["dev_highwater_bytes"] == units * N
 
 
+@pytest.mark.parametrize("host", [True, False])
+@pytest.mark.parametrize("prog", ["qcrit", "vortmag"])
+def test_memory_aware_staged_order(host, prog):
+    """A cap below the list-order footprint but above the memory-aware one:
+    the planner reorders (a valid topological order), the ledger's
+    high-water equals the oracle's simulation of that order, results stay
+    bit-identical (SURVEY 8f NEXT #3)."""
+    src, names = PAPER_PROGRAMS[prog]
+    x, y, z, f = _inputs((24, 16, 12), np.float32, names)
+    dag = build_dag(src, names)
+    mode = "host" if host else "device"
+    N = 24 * 16 * 12 * 4
+    list_units = omodel.footprint(dag, "staged", mode)
+    got, plan, *_ = run_lib(src, f, x, y, z, "staged", host=host, cap=(list_units - 1) * N, return_plan=True)
+    order = plan.schedule()
+    assert omodel.is_topological(dag, order) and order != list(range(len(dag.filters)))
+    units = omodel.footprint(dag, "staged", mode, order=order)
+    assert units < list_units
+    assert plan.stats()["dev_highwater_bytes"] == units * N
+    assert_parity(got, run_oracle(src, f, x, y, z))
+    # without a cap the paper's list order runs
+    _, plan2, *_ = run_lib(src, f, x, y, z, "staged", host=host, return_plan=True)
+    assert plan2.schedule() == list(range(len(dag.filters)))
+
+
 def test_memory_cap():
     """A cap below the predicted footprint fails at compile with
     DFG_E_NOMEM (the paper's failed GPU cases, L309); fused fits."""
@@ -161,8 +186,11 @@ def test_memory_cap():
     src = PAPER_PROGRAMS["qcrit"][0]
     N = 32 ** 3 * 4
     staged_units = omodel.footprint(build_dag(src, ("u", "v", "w")), "staged", "device")
+    with pytest.raises(dfg.DfgError) as e:          # below any schedule's footprint
+        run_lib(src, f, x, y, z, "staged", cap=5 * N)
+    assert e.value.name == "DFG_E_NOMEM"
     with pytest.raises(dfg.DfgError) as e:
-        run_lib(src, f, x, y, z, "staged", cap=(staged_units - 1) * N)
+        run_lib(src, f, x, y, z, "fused", cap=4 * N - 1)
     assert e.value.name == "DFG_E_NOMEM"
     got = run_lib(src, f, x, y, z, "staged", cap=staged_units * N)
     assert_parity(got, run_oracle(src, f, x, y, z))
