@@ -23,7 +23,7 @@
 #if DFG_NSF > 0 && DFG_HAS_TMA
 struct __align__(64) DfgTmap { unsigned long long v[16]; };  // CUtensorMap
 struct DfgTmaParams {
-  DfgTmap map[DFG_NSF_];
+  DfgTmap map[DFG_NF_];  // stencil fields, then point-wise fields
   DfgParams p;
 };
 
@@ -33,7 +33,9 @@ struct DfgTmaParams {
 #define DFG_ROWS (DFG_NCW + 2)
 #define DFG_TILE_ELEMS (DFG_ROWW * DFG_ROWS)
 #define DFG_TILE_BYTES ((DFG_TILE_ELEMS * (int)sizeof(DFG_T) + 127) / 128 * 128)
-#define DFG_STAGE_BYTES (DFG_TILE_BYTES * DFG_NSF)
+// every field streams through the ring (point-wise fields: centre only)
+#define DFG_NTF (DFG_NSF + DFG_NPF)
+#define DFG_STAGE_BYTES (DFG_TILE_BYTES * DFG_NTF)
 
 __device__ __forceinline__ unsigned dfg_smem(const void* p) {
   return (unsigned)__cvta_generic_to_shared(p);
@@ -126,8 +128,19 @@ struct DfgCol {
 // post-plane).  Queue roles are template parameters (no copies).
 template <int ZM, int ZC, int ZN>
 __device__ __forceinline__ void dfg_plane(const DfgCol& C, DfgRing& R, unsigned& cur_tile, unsigned& cur_full,
-                                          DFG_T (&zq)[3][DFG_NSF][DFG_VEC], DFG_T*& outp, const DFG_T* (&pin)[DFG_NPF_],
+                                          DFG_T (&zq)[3][DFG_NSF][DFG_VEC], DFG_T*& outp,
                                           long long plane, const DFG_T*& tzp, long long NZ) {
+  // x/y neighbours of this plane first (its stage is already resident), then
+  // wait for the next plane's stage: the loads overlap the barrier wait
+  DFG_T xmv[DFG_NSF], xpv[DFG_NSF], ymv[DFG_NSF][DFG_VEC], ypv[DFG_NSF][DFG_VEC];
+#pragma unroll
+  for (int f = 0; f < DFG_NSF; ++f) {
+    const unsigned t = cur_tile + f * DFG_TILE_BYTES;
+    xmv[f] = dfg_lds1(t + C.off_xm);
+    xpv[f] = dfg_lds1(t + C.off_xp);
+    dfg_lds16(ymv[f], t + C.off_ym);
+    dfg_lds16(ypv[f], t + C.off_yp);
+  }
   dfg_mbar_wait(R.full, R.phase, 0x100000u);
   const unsigned nxt_tile = R.tile, nxt_full = R.full;
 #pragma unroll
@@ -136,11 +149,9 @@ __device__ __forceinline__ void dfg_plane(const DfgCol& C, DfgRing& R, unsigned&
   dfg2 s[DFG_NPAIR][DFG_NSF][7], gn[DFG_NPAIR][DFG_NSF][3];
 #pragma unroll
   for (int f = 0; f < DFG_NSF; ++f) {
-    const unsigned t = cur_tile + f * DFG_TILE_BYTES;
-    const DFG_T xm = dfg_lds1(t + C.off_xm), xp = dfg_lds1(t + C.off_xp);
-    DFG_T ym[DFG_VEC], yp[DFG_VEC];
-    dfg_lds16(ym, t + C.off_ym);
-    dfg_lds16(yp, t + C.off_yp);
+    const DFG_T xm = xmv[f], xp = xpv[f];
+    const DFG_T(&ym)[DFG_VEC] = ymv[f];
+    const DFG_T(&yp)[DFG_VEC] = ypv[f];
     DFG_T lft[DFG_VEC], rgt[DFG_VEC];
 #pragma unroll
     for (int c = 0; c < DFG_VEC; ++c) {
@@ -169,13 +180,7 @@ __device__ __forceinline__ void dfg_plane(const DfgCol& C, DfgRing& R, unsigned&
 #pragma unroll
   for (int f = 0; f < DFG_NPF; ++f) {
     DFG_T pv[DFG_VEC];
-    if (C.act) {
-      dfg_ldg16(pv, pin[f]);
-    } else {
-#pragma unroll
-      for (int c = 0; c < DFG_VEC; ++c) pv[c] = DFG_T(0);
-    }
-    pin[f] += plane;
+    dfg_lds16(pv, cur_tile + (DFG_NSF + f) * DFG_TILE_BYTES + C.off_c);
 #pragma unroll
     for (int h = 0; h < DFG_NPAIR; ++h) p[h][f] = dfg2_mk(pv[h * DFG_LANES], pv[h * DFG_LANES + DFG_LANES - 1]);
   }
@@ -213,7 +218,7 @@ extern "C" __global__ void __launch_bounds__((DFG_NCW + 1) * 32, 1)
   if (warp == DFG_NCW) {
     // ---------------- producer: one lane issues all TMA loads
     if (lane == 0) {
-      for (int f = 0; f < DFG_NSF; ++f)
+      for (int f = 0; f < DFG_NTF; ++f)
         asm volatile("prefetch.tensormap [%0];" ::"l"(reinterpret_cast<unsigned long long>(&TP.map[f]))
                      : "memory");
       DfgRing W{smem, full0, 0u, 0, smem, full0};
@@ -232,10 +237,10 @@ extern "C" __global__ void __launch_bounds__((DFG_NCW + 1) * 32, 1)
           // wait until every consumer released this slot (the producer runs
           // ahead; the suspend hint keeps it off the issue slots)
           dfg_mbar_wait(DFG_EMPTY(W.full), W.phase ^ 1u, 0x100000u);
-          dfg_mbar_expect_tx(W.full, (unsigned)(DFG_NSF * DFG_TILE_ELEMS * sizeof(DFG_T)));
+          dfg_mbar_expect_tx(W.full, (unsigned)(DFG_NTF * DFG_TILE_ELEMS * sizeof(DFG_T)));
           const int zl = (int)(pg - P.k0 + P.ghost);
 #pragma unroll
-          for (int f = 0; f < DFG_NSF; ++f) dfg_tma_load3(W.tile + f * DFG_TILE_BYTES, &TP.map[f], W.full, x0, y0, zl);
+          for (int f = 0; f < DFG_NTF; ++f) dfg_tma_load3(W.tile + f * DFG_TILE_BYTES, &TP.map[f], W.full, x0, y0, zl);
           W.advance();
         }
       }
@@ -282,9 +287,6 @@ extern "C" __global__ void __launch_bounds__((DFG_NCW + 1) * 32, 1)
     C.off_yp = (rp * DFG_ROWW + c0) * TS;
     const long long cell0 = (kb - P.k0) * plane + jc * P.nx + ic;
     DFG_T* outp = P.out + cell0 * DFG_OUTW;
-    const DFG_T* pin[DFG_NPF_];
-#pragma unroll
-    for (int f = 0; f < DFG_NPF; ++f) pin[f] = P.f[DFG_NSF + f] + cell0 + P.ghost * plane;
     const DFG_T* tzp = P.tz + kb;
 
     DFG_T zq[3][DFG_NSF][DFG_VEC];
@@ -301,13 +303,13 @@ extern "C" __global__ void __launch_bounds__((DFG_NCW + 1) * 32, 1)
     R.advance();
     long long k = kb;
     for (; k + 3 <= ke; k += 3) {
-      dfg_plane<0, 1, 2>(C, R, cur_tile, cur_full, zq, outp, pin, plane, tzp, P.NZ);
-      dfg_plane<1, 2, 0>(C, R, cur_tile, cur_full, zq, outp, pin, plane, tzp, P.NZ);
-      dfg_plane<2, 0, 1>(C, R, cur_tile, cur_full, zq, outp, pin, plane, tzp, P.NZ);
+      dfg_plane<0, 1, 2>(C, R, cur_tile, cur_full, zq, outp, plane, tzp, P.NZ);
+      dfg_plane<1, 2, 0>(C, R, cur_tile, cur_full, zq, outp, plane, tzp, P.NZ);
+      dfg_plane<2, 0, 1>(C, R, cur_tile, cur_full, zq, outp, plane, tzp, P.NZ);
     }
     if (k < ke) {
-      dfg_plane<0, 1, 2>(C, R, cur_tile, cur_full, zq, outp, pin, plane, tzp, P.NZ);
-      if (k + 1 < ke) dfg_plane<1, 2, 0>(C, R, cur_tile, cur_full, zq, outp, pin, plane, tzp, P.NZ);
+      dfg_plane<0, 1, 2>(C, R, cur_tile, cur_full, zq, outp, plane, tzp, P.NZ);
+      if (k + 1 < ke) dfg_plane<1, 2, 0>(C, R, cur_tile, cur_full, zq, outp, plane, tzp, P.NZ);
     }
     // the post-plane stage was read for its centre only
     dfg_mbar_arrive(DFG_EMPTY(cur_full));

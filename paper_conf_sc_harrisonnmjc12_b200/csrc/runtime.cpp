@@ -559,7 +559,7 @@ std::unique_ptr<PlanImpl> compile_plan(std::shared_ptr<MeshImpl> mesh, const std
     DFG_CUDA(cudaFree(0));
     plan->mod = load_module(cb);
     if (plan->mod.tma) {
-      size_t smem = fused_tma_smem_bytes(mesh->dt, int(plan->fsrc.layout.stencil_inputs.size()), plan->fsrc.cfg.ncw,
+      size_t smem = fused_tma_smem_bytes(mesh->dt, int(plan->fsrc.layout.stencil_inputs.size() + plan->fsrc.layout.point_inputs.size()), plan->fsrc.cfg.ncw,
                                          plan->fsrc.cfg.stages);
       DFG_CU(drv().FuncSetAttribute(plan->mod.tma, CU_FUNC_ATTRIBUTE_MAX_DYNAMIC_SHARED_SIZE_BYTES, int(smem)));
     }
@@ -815,7 +815,7 @@ void PlanImpl::launch_fused(const std::vector<const void*>& fptr, void* dout, co
     last_variant = 3;
   } else if (mod.tma && !want_general && m.nx % vec == 0 && vec_ok) {
     const int ncw = fsrc.cfg.ncw;
-    const int nsf = int(L.stencil_inputs.size());
+    const int nsf = int(L.stencil_inputs.size() + L.point_inputs.size());  // TMA tiles per stage
     const int tiles_x = int((m.nx + 32 * vec - 1) / (32 * vec));
     const int tiles_y = int((m.ny + ncw - 1) / ncw);
     const int64_t range = kend - kbeg;
