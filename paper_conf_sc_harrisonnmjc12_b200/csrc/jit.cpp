@@ -86,13 +86,16 @@ const Cubin& nvrtc_compile(const std::string& source, const std::string& name) {
   return ref;
 }
 
-LoadedModule load_module(const Cubin& c) {
+LoadedModule load_module(const Cubin& c, bool has_stencil, bool has_tma) {
   LoadedModule m;
   DFG_CU(drv().ModuleLoadData(&m.mod, c.image.data()));
-  CUfunction f;
-  if (drv().ModuleGetFunction(&f, m.mod, "dfg_fused_pointwise") == CUDA_SUCCESS) m.pointwise = f;
-  if (drv().ModuleGetFunction(&f, m.mod, "dfg_fused_general") == CUDA_SUCCESS) m.general = f;
-  if (drv().ModuleGetFunction(&f, m.mod, "dfg_fused_tma") == CUDA_SUCCESS) m.tma = f;
+  // look up exactly the kernels skeleton.cuh / fused_tma.cuh emit for this layout
+  if (!has_stencil) {
+    DFG_CU(drv().ModuleGetFunction(&m.pointwise, m.mod, "dfg_fused_pointwise"));
+  } else {
+    DFG_CU(drv().ModuleGetFunction(&m.general, m.mod, "dfg_fused_general"));
+    if (has_tma) DFG_CU(drv().ModuleGetFunction(&m.tma, m.mod, "dfg_fused_tma"));
+  }
   return m;
 }
 

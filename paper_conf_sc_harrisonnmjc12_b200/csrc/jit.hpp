@@ -26,6 +26,6 @@ struct LoadedModule {
 };
 
 // Load into the current context (requires a device).
-LoadedModule load_module(const Cubin& c);
+LoadedModule load_module(const Cubin& c, bool has_stencil, bool has_tma);
 
 }  // namespace dfg

@@ -557,7 +557,7 @@ std::unique_ptr<PlanImpl> compile_plan(std::shared_ptr<MeshImpl> mesh, const std
     plan->spill = cb.spill;
     // the runtime API owns the primary context; make it current for the driver API
     DFG_CUDA(cudaFree(0));
-    plan->mod = load_module(cb);
+    plan->mod = load_module(cb, !plan->fsrc.layout.stencil_inputs.empty(), plan->fsrc.cfg.has_tma);
     if (plan->mod.tma) {
       size_t smem = fused_tma_smem_bytes(mesh->dt, int(plan->fsrc.layout.stencil_inputs.size() + plan->fsrc.layout.point_inputs.size()), plan->fsrc.cfg.ncw,
                                          plan->fsrc.cfg.stages);
