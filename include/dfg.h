@@ -222,6 +222,16 @@ int dfg_dump_kernel(dfg_plan plan, char* buf, size_t cap, size_t* needed);
  * Need no GPU: the parser / network builder, the strategy model and the
  * kernel generator on their own, for tests and tooling. */
 
+/* Paper-layout compatibility (Table I): the
+ * paper's data carry point coordinates as full 3-D arrays x3, y3, z3 of shape
+ * [nz+1][ny+1][nx+1] (x fastest, type T).  Extracts the per-axis point arrays
+ * x[nx+1], y[ny+1], z[nz+1] for dfg_create_mesh and checks that the mesh is
+ * rectilinear (x3 depends on i only, y3 on j only, z3 on k only; bitwise):
+ * DFG_E_INVALID otherwise.  Host pointers; no device needed. */
+int dfg_points3d_to_axes(dfg_dtype dtype, int64_t nx, int64_t ny, int64_t nz,
+                         const void* x3, const void* y3, const void* z3,
+                         void* x, void* y, void* z);
+
 /* Parse + lower `expr` with the named scalar inputs; write the canonical
  * text.  Same errors as dfg_compile's language errors. */
 int dfg_dag_dump(const char* expr, const char* const* inputs, int n_inputs,

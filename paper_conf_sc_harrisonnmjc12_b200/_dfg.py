@@ -74,6 +74,7 @@ _SIGS = {
     "dfg_dag_dump": (C.c_int, [C.c_char_p, C.POINTER(C.c_char_p), C.c_int, C.c_int, C.c_char_p, C.c_size_t,
                                C.POINTER(C.c_size_t)]),
     "dfg_model": (C.c_int, [C.c_char_p, C.POINTER(C.c_char_p), C.c_int, C.c_int, C.c_int, C.POINTER(_I64)]),
+    "dfg_points3d_to_axes": (C.c_int, [C.c_int, _I64, _I64, _I64, _P, _P, _P, _P, _P, _P]),
     "dfg_fused_source": (C.c_int, [C.c_char_p, C.POINTER(C.c_char_p), C.c_int, C.c_int, _I64, _I64, _I64, C.c_int,
                                    C.c_char_p, C.c_size_t, C.POINTER(C.c_size_t), C.POINTER(C.c_int),
                                    C.POINTER(C.c_int)]),
@@ -230,6 +231,19 @@ def dfg_model(expr, inputs, strategy, host_mode=True):
     out = (_I64 * 4)()
     _check(_lib.dfg_model(expr.encode(), arr, n, strategy, int(host_mode), out))
     return list(out)
+
+
+def dfg_points3d_to_axes(x3, y3, z3):
+    """numpy [nz+1][ny+1][nx+1] point arrays -> (x, y, z) 1-D axes (T)."""
+    import numpy as np
+    x3, y3, z3 = (np.ascontiguousarray(a) for a in (x3, y3, z3))
+    assert x3.shape == y3.shape == z3.shape and x3.dtype == y3.dtype == z3.dtype
+    pz, py, px = x3.shape
+    x, y, z = np.empty(px, x3.dtype), np.empty(py, x3.dtype), np.empty(pz, x3.dtype)
+    dt = DFG_F32 if x3.dtype == np.float32 else DFG_F64
+    _check(_lib.dfg_points3d_to_axes(dt, px - 1, py - 1, pz - 1, _ptr(x3), _ptr(y3), _ptr(z3),
+                                     _ptr(x), _ptr(y), _ptr(z)))
+    return x, y, z
 
 
 def dfg_fused_source(expr, inputs, dtype, nx, ny, nz, compile=False):

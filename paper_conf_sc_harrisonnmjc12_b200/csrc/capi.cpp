@@ -247,6 +247,44 @@ int dfg_dump_kernel(dfg_plan plan, char* buf, size_t cap, size_t* needed) {
   });
 }
 
+}  // extern "C"
+
+namespace {
+template <typename T>
+void axes_from_points3d(int64_t nx, int64_t ny, int64_t nz, const T* x3, const T* y3, const T* z3, T* x, T* y, T* z) {
+  const int64_t px = nx + 1, py = ny + 1, pz = nz + 1;
+  for (int64_t i = 0; i < px; ++i) x[i] = x3[i];
+  for (int64_t j = 0; j < py; ++j) y[j] = y3[j * px];
+  for (int64_t k = 0; k < pz; ++k) z[k] = z3[k * px * py];
+  for (int64_t k = 0; k < pz; ++k)
+    for (int64_t j = 0; j < py; ++j)
+      for (int64_t i = 0; i < px; ++i) {
+        const int64_t e = (k * py + j) * px + i;
+        if (!(x3[e] == x[i] && y3[e] == y[j] && z3[e] == z[k]))
+          dfg::fail(DFG_E_INVALID, "point coordinates are not rectilinear at (" + std::to_string(i) + "," +
+                                       std::to_string(j) + "," + std::to_string(k) + ")");
+      }
+}
+}  // namespace
+
+extern "C" {
+
+int dfg_points3d_to_axes(dfg_dtype dtype, int64_t nx, int64_t ny, int64_t nz, const void* x3, const void* y3,
+                         const void* z3, void* x, void* y, void* z) {
+  return guard([&] {
+    if (nx < 1 || ny < 1 || nz < 1) dfg::fail(DFG_E_INVALID, "mesh sizes must be >= 1");
+    if (!x3 || !y3 || !z3 || !x || !y || !z) dfg::fail(DFG_E_INVALID, "null pointer");
+    if (to_dtype(dtype) == dfg::DType::F32)
+      axes_from_points3d(nx, ny, nz, static_cast<const float*>(x3), static_cast<const float*>(y3),
+                         static_cast<const float*>(z3), static_cast<float*>(x), static_cast<float*>(y),
+                         static_cast<float*>(z));
+    else
+      axes_from_points3d(nx, ny, nz, static_cast<const double*>(x3), static_cast<const double*>(y3),
+                         static_cast<const double*>(z3), static_cast<double*>(x), static_cast<double*>(y),
+                         static_cast<double*>(z));
+  });
+}
+
 int dfg_dag_dump(const char* expr, const char* const* inputs, int n_inputs, dfg_dtype dtype, char* buf, size_t cap,
                  size_t* needed) {
   return guard([&] {

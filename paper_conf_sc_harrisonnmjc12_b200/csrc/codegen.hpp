@@ -25,6 +25,7 @@ struct FusedConfig {
   int div_mode = 1;    // 0 ieee, 1 exact (Markstein), 2 fast; see blocks.cuh
   int ncw = 15;        // consumer warps per CTA (tile rows); +1 producer = 512 threads
   int stages = 0;      // smem ring depth (0: choose)
+  int ctas = 1;        // resident CTAs per SM the TMA kernel is sized for
   bool has_tma = false;
 };
 

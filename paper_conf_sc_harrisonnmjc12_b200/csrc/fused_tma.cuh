@@ -195,7 +195,7 @@ __device__ __forceinline__ void dfg_plane(const DfgCol& C, DfgRing& R, unsigned&
   cur_full = nxt_full;
 }
 
-extern "C" __global__ void __launch_bounds__((DFG_NCW + 1) * 32, 1)
+extern "C" __global__ void __launch_bounds__((DFG_NCW + 1) * 32, DFG_CTAS)
     dfg_fused_tma(const __grid_constant__ DfgTmaParams TP) {
   const DfgParams& P = TP.p;
   // dynamic shared memory starts at the (1024-aligned) base of the CTA's

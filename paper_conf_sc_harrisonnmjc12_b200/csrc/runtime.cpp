@@ -549,6 +549,8 @@ std::unique_ptr<PlanImpl> compile_plan(std::shared_ptr<MeshImpl> mesh, const std
     if (!mesh->markstein_safe && cfg.div_mode == 1) cfg.div_mode = 0;  // keep results exact
     const char* ncw = std::getenv("DFG_NCW");
     if (ncw) cfg.ncw = std::max(1, std::min(30, std::atoi(ncw)));
+    const char* ctas = std::getenv("DFG_CTAS");
+    if (ctas) cfg.ctas = std::max(1, std::min(4, std::atoi(ctas)));
     const char* st = std::getenv("DFG_STAGES");
     if (st) cfg.stages = std::max(2, std::min(16, std::atoi(st)));
     plan->fsrc = generate_fused(dag, mesh->nx, mesh->ny, mesh->NZ, cfg, ref);

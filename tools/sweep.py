@@ -66,7 +66,7 @@ def main():
             ["exact", "fast", "ieee"], [15, 7])]
     nbytes = (len(names) + 1) * np.dtype(T).itemsize
     for conf in confs:
-        for k in ("DFG_FUSED_VARIANT", "DFG_NCW", "DFG_STAGES", "DFG_KZ", "DFG_FUSED_KERNEL"):
+        for k in ("DFG_FUSED_VARIANT", "DFG_NCW", "DFG_STAGES", "DFG_KZ", "DFG_FUSED_KERNEL", "DFG_CTAS"):
             os.environ.pop(k, None)
         os.environ.update(conf)
         plan = dfg.Plan(mesh, src, "fused")
