@@ -116,13 +116,13 @@ def _oracle_time(x, y, z, f, win):
 def cpu_baseline_leg(target_s: float = 12.0):
     """The oracle as it stands (numpy, one thread for element-wise ops) on a
     bounded sample of the bench workload."""
-    x, y, z, f, win = _oracle_sample(256, 4)
+    x, y, z, f, win = _oracle_sample(512, 4)
     cells, dt = _oracle_time(x, y, z, f, win)                 # calibration run
     planes = int(max(1, min(128, round(4 * target_s / max(dt, 1e-3)))))
-    x, y, z, f, win = _oracle_sample(256, planes)
+    x, y, z, f, win = _oracle_sample(512, planes)
     cells, dt = _oracle_time(x, y, z, f, win)
     return {"value": cells / dt, "unit": "cells/s", "cores": 1, "kind": "oracle",
-            "sample": f"Q-criterion on a 1024 x 256 x {planes} block (+1-cell halo) of the 1024^3 RT-like "
+            "sample": f"Q-criterion on a 1024 x 512 x {planes} block (+1-cell halo) of the 1024^3 RT-like "
                       f"fp32 workload, numpy oracle, {dt:.1f} s"}
 
 
