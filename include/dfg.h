@@ -120,6 +120,23 @@ int dfg_create_mesh(dfg_dtype dtype, int64_t nx, int64_t ny, int64_t nz_local,
                     const void* x, const void* y, const void* z,
                     int64_t nz_global, int64_t z_offset, int ghost,
                     dfg_mesh* out);
+/* VisIt-style sub-grid (the paper's distributed run: 3072 sub-grids of
+ * 192 x 192 x 256 cells "plus the necessary ghost cells", L253-L255, L315;
+ * SURVEY 8f NEXT #4): local nx x ny x nz cells at offsets (i0, j0, k0) of a
+ * global NX x NY x NZ mesh whose point coordinates x[0..NX], y[0..NY],
+ * z[0..NZ] are given (host, T).  ghost = 1: every bound field buffer carries
+ * a one-cell ghost shell on all six faces, T[nz+2][ny+2][nx+2], filled by
+ * the CALLER (VisIt's ghost exchange) -- no halo transport is used; cells on
+ * the global mesh boundary ignore their ghost cells (one-sided differences,
+ * reading R1).  ghost = 0 only for the whole mesh.  Output: T[nz][ny][nx].
+ * Fusion (and reference) strategies only; the TMA fast path additionally
+ * needs (nx + 2*ghost) * sizeof(T) % 16 == 0, other widths use the general
+ * kernel.  Errors as dfg_create_mesh. */
+int dfg_create_block(dfg_dtype dtype, int64_t nx, int64_t ny, int64_t nz,
+                     const void* x, const void* y, const void* z,
+                     int64_t NX, int64_t NY, int64_t NZ,
+                     int64_t i0, int64_t j0, int64_t k0, int ghost, dfg_mesh* out);
+
 /* Idempotent on NULL.  Plans keep what they need alive: destroying a mesh
  * with live plans is allowed (the plans stay valid). */
 void dfg_destroy_mesh(dfg_mesh mesh);
@@ -197,7 +214,8 @@ int dfg_reset_stats(dfg_plan plan);
 /* Plan description: out[0] = strategy, out[1] = result width (1 or 4),
  * out[2] = number of filters, out[3] = fused kernel variant in use
  * (0 none, 1 TMA pipeline, 2 general), out[4] = registers per thread of the
- * fused kernel (0 if none), out[5] = spilled bytes, out[6] = predicted
+ * fused kernel (0 if none), out[5] = local memory per thread of that kernel
+ * (bytes; spills and stack), out[6] = predicted
  * device footprint in bytes for device-resident inputs,
  * out[7] = same for host inputs. */
 int dfg_plan_info(dfg_plan plan, int64_t out[8]);

@@ -42,6 +42,24 @@ class Mesh:
                                       self.nz_global, z_offset, ghost)
         self._bound = {}
 
+    @classmethod
+    def block(cls, x, y, z, nx, ny, nz, i0, j0, k0, ghost=1):
+        """VisIt-style sub-grid of the global mesh with points x, y, z:
+        local nx x ny x nz cells at (i0, j0, k0), one-cell ghost shell on all
+        six faces filled by the caller (dfg_create_block)."""
+        import numpy as np
+        from ._dfg import dfg_create_block
+        self = cls.__new__(cls)
+        x, y, z = (np.ascontiguousarray(a) for a in (x, y, z))
+        self.dtype = x.dtype
+        self.nx, self.ny, self.nz, self.nz_global = nx, ny, nz, len(z) - 1
+        self.ghost = ghost
+        self._coords = (x, y, z)
+        self._bound = {}
+        self.handle = dfg_create_block(_dtype_code(x.dtype), nx, ny, nz, x, y, z, len(x) - 1, len(y) - 1,
+                                       len(z) - 1, i0, j0, k0, ghost)
+        return self
+
     def bind(self, name, buf, on_device=None):
         if on_device is None:
             on_device = bool(getattr(buf, "is_cuda", False))

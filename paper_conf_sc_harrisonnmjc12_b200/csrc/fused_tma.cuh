@@ -227,8 +227,9 @@ extern "C" __global__ void __launch_bounds__((DFG_NCW + 1) * 32, DFG_CTAS)
         const long long rest = item / P.tiles_x;
         const long long ty_ = rest % P.tiles_y;
         const long long zc = rest / P.tiles_y;
-        const int x0 = (int)(tx_ * DFG_TX) - DFG_HX;
-        const int y0 = (int)(ty_ * DFG_NCW) - 1;
+        // input coordinates include the block's x/y ghost columns / rows
+        const int x0 = (int)(tx_ * DFG_TX) - DFG_HX + (int)((P.px - P.nx) >> 1);
+        const int y0 = (int)(ty_ * DFG_NCW) - 1 + (int)((P.py - P.ny) >> 1);
         const long long kb = P.kbeg + zc * P.kz;
         const long long ke = min(kb + (long long)P.kz, P.kend);
         // pre-plane, kb..ke-1, post-plane; clamped to the global mesh (R1)
@@ -269,16 +270,19 @@ extern "C" __global__ void __launch_bounds__((DFG_NCW + 1) * 32, DFG_CTAS)
     const long long jc = min(j, P.ny - 1);
 #pragma unroll
     for (int h = 0; h < DFG_NPAIR; ++h) {
-      const long long a = ic + h * DFG_LANES, b = ic + h * DFG_LANES + DFG_LANES - 1;
-      C.ndx[h] = dfg2_mk(__ldg(P.tx + 2 * P.nx + a), __ldg(P.tx + 2 * P.nx + b));
-      C.rx[h] = dfg2_mk(__ldg(P.tx + P.nx + a), __ldg(P.tx + P.nx + b));
+      // spacing tables are indexed globally (blocks: i0 / j0 offsets)
+      const long long a = P.i0 + ic + h * DFG_LANES, b = P.i0 + ic + h * DFG_LANES + DFG_LANES - 1;
+      C.ndx[h] = dfg2_mk(__ldg(P.tx + 2 * P.NX + a), __ldg(P.tx + 2 * P.NX + b));
+      C.rx[h] = dfg2_mk(__ldg(P.tx + P.NX + a), __ldg(P.tx + P.NX + b));
     }
-    C.ndy = dfg2_splat(__ldg(P.ty + 2 * P.ny + jc));
-    C.ry = dfg2_splat(__ldg(P.ty + P.ny + jc));
-    const unsigned cxm = (i == 0) ? c0 : c0 - 1;
-    const unsigned cxp = (i + DFG_VEC >= P.nx) ? c0 + DFG_VEC - 1 : c0 + DFG_VEC;
-    const unsigned rm = (j == 0) ? r : r - 1;
-    const unsigned rp = (j >= P.ny - 1) ? r : r + 1;
+    C.ndy = dfg2_splat(__ldg(P.ty + 2 * P.NY + P.j0 + jc));
+    C.ry = dfg2_splat(__ldg(P.ty + P.NY + P.j0 + jc));
+    // one-sided differences only at the GLOBAL mesh ends (reading R1)
+    const long long ig = P.i0 + i, jg = P.j0 + j;
+    const unsigned cxm = (ig == 0) ? c0 : c0 - 1;
+    const unsigned cxp = (ig + DFG_VEC >= P.NX) ? c0 + DFG_VEC - 1 : c0 + DFG_VEC;
+    const unsigned rm = (jg == 0) ? r : r - 1;
+    const unsigned rp = (jg >= P.NY - 1) ? r : r + 1;
     const unsigned TS = (unsigned)sizeof(DFG_T);
     C.off_c = (r * DFG_ROWW + c0) * TS;
     C.off_xm = (r * DFG_ROWW + cxm) * TS;

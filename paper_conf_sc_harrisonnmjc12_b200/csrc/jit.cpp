@@ -1,6 +1,7 @@
 // NVRTC -> sm_100a cubin -> CUmodule.  See jit.hpp.
 #include "jit.hpp"
 
+#include <dlfcn.h>
 #include <nvrtc.h>
 
 #include <cstdlib>
@@ -16,6 +17,54 @@
 namespace dfg {
 
 namespace {
+
+// NVRTC is loaded by absolute path with RTLD_LOCAL, not linked: a process
+// that already holds another libnvrtc.so.12 (torch ships its own) would
+// otherwise bind libdfg to that compiler and the generated kernels would
+// depend on import order.
+struct NvrtcApi {
+  void* h = nullptr;
+  nvrtcResult (*CreateProgram)(nvrtcProgram*, const char*, const char*, int, const char* const*,
+                               const char* const*) = nullptr;
+  nvrtcResult (*CompileProgram)(nvrtcProgram, int, const char* const*) = nullptr;
+  nvrtcResult (*GetProgramLogSize)(nvrtcProgram, size_t*) = nullptr;
+  nvrtcResult (*GetProgramLog)(nvrtcProgram, char*) = nullptr;
+  nvrtcResult (*GetCUBINSize)(nvrtcProgram, size_t*) = nullptr;
+  nvrtcResult (*GetCUBIN)(nvrtcProgram, char*) = nullptr;
+  nvrtcResult (*DestroyProgram)(nvrtcProgram*) = nullptr;
+  const char* (*GetErrorString)(nvrtcResult) = nullptr;
+  nvrtcResult (*Version)(int*, int*) = nullptr;
+};
+
+NvrtcApi& nvrtc() {
+  static NvrtcApi api;
+  static std::once_flag once;
+  std::call_once(once, [] {
+    const char* env = std::getenv("DFG_NVRTC_LIB");
+    const char* cands[] = {env, "/usr/local/cuda/lib64/libnvrtc.so.12", "/usr/local/cuda/lib64/libnvrtc.so",
+                           "libnvrtc.so.12"};
+    for (const char* c : cands) {
+      if (!c) continue;
+      api.h = dlopen(c, RTLD_NOW | RTLD_LOCAL);
+      if (api.h) break;
+    }
+    if (!api.h) return;
+#define DFG_SYM(field, name) api.field = reinterpret_cast<decltype(api.field)>(dlsym(api.h, name))
+    DFG_SYM(CreateProgram, "nvrtcCreateProgram");
+    DFG_SYM(CompileProgram, "nvrtcCompileProgram");
+    DFG_SYM(GetProgramLogSize, "nvrtcGetProgramLogSize");
+    DFG_SYM(GetProgramLog, "nvrtcGetProgramLog");
+    DFG_SYM(GetCUBINSize, "nvrtcGetCUBINSize");
+    DFG_SYM(GetCUBIN, "nvrtcGetCUBIN");
+    DFG_SYM(DestroyProgram, "nvrtcDestroyProgram");
+    DFG_SYM(GetErrorString, "nvrtcGetErrorString");
+    DFG_SYM(Version, "nvrtcVersion");
+#undef DFG_SYM
+  });
+  if (!api.h || !api.CreateProgram || !api.CompileProgram || !api.GetCUBIN || !api.GetCUBINSize)
+    fail(DFG_E_NVRTC, "NVRTC (libnvrtc.so.12) could not be loaded");
+  return api;
+}
 
 std::mutex g_mu;
 std::map<std::string, std::unique_ptr<Cubin>> g_cache;
@@ -53,32 +102,33 @@ const Cubin& nvrtc_compile(const std::string& source, const std::string& name) {
   auto it = g_cache.find(source);
   if (it != g_cache.end()) return *it->second;
 
+  NvrtcApi& api = nvrtc();
   nvrtcProgram prog;
-  if (nvrtcCreateProgram(&prog, source.c_str(), name.c_str(), 0, nullptr, nullptr) != NVRTC_SUCCESS)
+  if (api.CreateProgram(&prog, source.c_str(), name.c_str(), 0, nullptr, nullptr) != NVRTC_SUCCESS)
     fail(DFG_E_NVRTC, "nvrtcCreateProgram failed");
   // Reading R6: no contraction across blocks, IEEE division/sqrt, denormals kept.
   const char* opts[] = {"--gpu-architecture=sm_100a", "--std=c++17",        "--fmad=false",
                         "--ftz=false",                "--prec-div=true",    "--prec-sqrt=true",
                         "--device-as-default-execution-space", "--generate-line-info",
                         "--ptxas-options=-v",         "-DNDEBUG"};
-  nvrtcResult rc = nvrtcCompileProgram(prog, int(sizeof(opts) / sizeof(opts[0])), opts);
+  nvrtcResult rc = api.CompileProgram(prog, int(sizeof(opts) / sizeof(opts[0])), opts);
   size_t log_size = 0;
-  nvrtcGetProgramLogSize(prog, &log_size);
+  api.GetProgramLogSize(prog, &log_size);
   std::string log(log_size, '\0');
-  if (log_size) nvrtcGetProgramLog(prog, &log[0]);
+  if (log_size) api.GetProgramLog(prog, &log[0]);
   if (rc != NVRTC_SUCCESS) {
-    nvrtcDestroyProgram(&prog);
-    fail(DFG_E_NVRTC, std::string("NVRTC: ") + nvrtcGetErrorString(rc) + "\n" + log);
+    api.DestroyProgram(&prog);
+    fail(DFG_E_NVRTC, std::string("NVRTC: ") + api.GetErrorString(rc) + "\n" + log);
   }
   auto c = std::make_unique<Cubin>();
   size_t n = 0;
-  if (nvrtcGetCUBINSize(prog, &n) != NVRTC_SUCCESS || n == 0) {
-    nvrtcDestroyProgram(&prog);
+  if (api.GetCUBINSize(prog, &n) != NVRTC_SUCCESS || n == 0) {
+    api.DestroyProgram(&prog);
     fail(DFG_E_NVRTC, "NVRTC produced no cubin\n" + log);
   }
   c->image.resize(n);
-  nvrtcGetCUBIN(prog, c->image.data());
-  nvrtcDestroyProgram(&prog);
+  api.GetCUBIN(prog, c->image.data());
+  api.DestroyProgram(&prog);
   c->log = log;
   parse_ptxas(log, *c);
   const Cubin& ref = *c;

@@ -108,6 +108,27 @@ std::shared_ptr<MeshImpl> create_mesh(DType dt, int64_t nx, int64_t ny, int64_t 
   if (ghost != 0 && ghost != 1) fail(DFG_E_INVALID, "ghost must be 0 or 1");
   if (nzl != NZ && ghost != 1) fail(DFG_E_INVALID, "a z slab of a larger mesh needs ghost = 1");
   if (!x || !y || !z) fail(DFG_E_INVALID, "null coordinate pointer");
+  return create_block_impl(dt, nx, ny, nzl, x, y, z, nx, ny, NZ, 0, 0, k0, ghost, 0);
+}
+
+std::shared_ptr<MeshImpl> create_block(DType dt, int64_t nx, int64_t ny, int64_t nz, const void* x, const void* y,
+                                       const void* z, int64_t NX, int64_t NY, int64_t NZ, int64_t i0, int64_t j0,
+                                       int64_t k0, int ghost) {
+  if (nx < 1 || ny < 1 || nz < 1 || NX < 1 || NY < 1 || NZ < 1) fail(DFG_E_INVALID, "block sizes must be >= 1");
+  if (i0 < 0 || j0 < 0 || k0 < 0 || i0 + nx > NX || j0 + ny > NY || k0 + nz > NZ)
+    fail(DFG_E_INVALID, "block outside the global mesh");
+  if (ghost != 0 && ghost != 1) fail(DFG_E_INVALID, "ghost must be 0 or 1");
+  if (ghost == 0 && (nx != NX || ny != NY || nz != NZ))
+    fail(DFG_E_INVALID, "a block of a larger mesh needs its one-cell ghost shell");
+  if (!x || !y || !z) fail(DFG_E_INVALID, "null coordinate pointer");
+  auto m = create_block_impl(dt, nx, ny, nz, x, y, z, NX, NY, NZ, i0, j0, k0, ghost, ghost);
+  m->ghosts_supplied = ghost == 1;
+  return m;
+}
+
+std::shared_ptr<MeshImpl> create_block_impl(DType dt, int64_t nx, int64_t ny, int64_t nzl, const void* x,
+                                            const void* y, const void* z, int64_t NX, int64_t NY, int64_t NZ,
+                                            int64_t i0, int64_t j0, int64_t k0, int ghost, int gxy) {
   auto m = std::make_shared<MeshImpl>();
   m->dt = dt;
   m->nx = nx;
@@ -115,9 +136,14 @@ std::shared_ptr<MeshImpl> create_mesh(DType dt, int64_t nx, int64_t ny, int64_t 
   m->nzl = nzl;
   m->NZ = NZ;
   m->k0 = k0;
+  m->NX = NX;
+  m->NY = NY;
+  m->i0 = i0;
+  m->j0 = j0;
   m->ghost = ghost;
+  m->gxy = gxy;
   const void* P[3] = {x, y, z};
-  int64_t N[3] = {nx, ny, NZ};
+  int64_t N[3] = {NX, NY, NZ};
   for (int a = 0; a < 3; ++a) {
     if (dt == DType::F32) build_axis(static_cast<const float*>(P[a]), N[a], m->host_tab[a], m->markstein_safe);
     else build_axis(static_cast<const double*>(P[a]), N[a], m->host_tab[a], m->markstein_safe);
@@ -504,9 +530,9 @@ std::unique_ptr<PlanImpl> compile_plan(std::shared_ptr<MeshImpl> mesh, const std
     plan->dag = build_dag(expr, names, mesh->dt);
   }
   const Dag& dag = plan->dag;
-  const bool multi = mesh->nzl != mesh->NZ;
+  const bool multi = mesh->nzl != mesh->NZ || mesh->nx != mesh->NX || mesh->ny != mesh->NY || mesh->gxy;
   if (multi && s != DFG_FUSED && s != DFG_REFERENCE)
-    fail(DFG_E_UNSUPPORTED, "staged/roundtrip/streamed run on a single slab; multi-slab meshes use fusion");
+    fail(DFG_E_UNSUPPORTED, "staged/roundtrip/streamed run on a whole mesh; slabs and blocks use fusion");
 
   // Footprint check against the cap for the binding modes at compile time
   // (the streamed ring is bounded by construction; its ledger checks at run time)
@@ -553,13 +579,22 @@ std::unique_ptr<PlanImpl> compile_plan(std::shared_ptr<MeshImpl> mesh, const std
     if (ctas) cfg.ctas = std::max(1, std::min(4, std::atoi(ctas)));
     const char* st = std::getenv("DFG_STAGES");
     if (st) cfg.stages = std::max(2, std::min(16, std::atoi(st)));
-    plan->fsrc = generate_fused(dag, mesh->nx, mesh->ny, mesh->NZ, cfg, ref);
+    // axis degeneracy (n == 1) is a property of the GLOBAL mesh
+    plan->fsrc = generate_fused(dag, mesh->NX, mesh->NY, mesh->NZ, cfg, ref);
     const Cubin& cb = nvrtc_compile(plan->fsrc.source, "dfg_fused.cu");
     plan->regs = cb.regs;
     plan->spill = cb.spill;
     // the runtime API owns the primary context; make it current for the driver API
     DFG_CUDA(cudaFree(0));
     plan->mod = load_module(cb, !plan->fsrc.layout.stencil_inputs.empty(), plan->fsrc.cfg.has_tma);
+    // registers / local memory of the main kernel from the loaded module (the
+    // NVRTC log can be empty when the compile is served from a cache)
+    CUfunction main_fn = plan->mod.tma ? plan->mod.tma : plan->mod.general ? plan->mod.general : plan->mod.pointwise;
+    int nregs = 0, local = 0;
+    DFG_CU(drv().FuncGetAttribute(&nregs, CU_FUNC_ATTRIBUTE_NUM_REGS, main_fn));
+    DFG_CU(drv().FuncGetAttribute(&local, CU_FUNC_ATTRIBUTE_LOCAL_SIZE_BYTES, main_fn));
+    plan->regs = nregs;
+    plan->spill = local;
     if (plan->mod.tma) {
       size_t smem = fused_tma_smem_bytes(mesh->dt, int(plan->fsrc.layout.stencil_inputs.size() + plan->fsrc.layout.point_inputs.size()), plan->fsrc.cfg.ncw,
                                          plan->fsrc.cfg.stages);
@@ -598,7 +633,7 @@ void PlanImpl::resolve_kernel_times() {
 void PlanImpl::halo_exchange(const std::vector<int>& inputs, cudaStream_t s) {
   MeshImpl& m = *mesh;
   const bool has_lo = m.k0 > 0, has_hi = m.k0 + m.nzl < m.NZ;
-  if (!has_lo && !has_hi) return;
+  if ((!has_lo && !has_hi) || m.ghosts_supplied) return;  // blocks: the caller filled the ghosts
   const size_t ts = dsize(m.dt);
   const size_t pb = size_t(m.plane()) * ts;
   auto lo = m.link_lo.lock(), hi = m.link_hi.lock();
@@ -680,8 +715,8 @@ namespace {
 void encode_map(CUtensorMap* map, const SlabView& m, void* base, int ncw) {
   const size_t ts = dsize(m.dt);
   const int vec = int(16 / ts);
-  cuuint64_t gdim[3] = {cuuint64_t(m.nx), cuuint64_t(m.ny), cuuint64_t(m.nzl + 2 * m.ghost)};
-  cuuint64_t gstride[2] = {cuuint64_t(m.nx) * ts, cuuint64_t(m.nx * m.ny) * ts};
+  cuuint64_t gdim[3] = {cuuint64_t(m.px()), cuuint64_t(m.py()), cuuint64_t(m.nzl + 2 * m.ghost)};
+  cuuint64_t gstride[2] = {cuuint64_t(m.px()) * ts, cuuint64_t(m.px() * m.py()) * ts};
   cuuint32_t box[3] = {cuuint32_t(32 * vec + 2 * vec), cuuint32_t(ncw + 2), 1};
   cuuint32_t estr[3] = {1, 1, 1};
   DFG_CU(drv().TensorMapEncodeTiled(map, m.dt == DType::F32 ? CU_TENSOR_MAP_DATA_TYPE_FLOAT32 : CU_TENSOR_MAP_DATA_TYPE_FLOAT64,
@@ -701,7 +736,9 @@ std::vector<uint64_t> pack_params(const std::vector<const void*>& f, void* out, 
   w.push_back(reinterpret_cast<uint64_t>(tx));
   w.push_back(reinterpret_cast<uint64_t>(ty));
   w.push_back(reinterpret_cast<uint64_t>(tz));
-  for (int64_t v : {m.nx, m.ny, m.nzl, m.NZ, m.k0, int64_t(m.ghost), kbeg, kend, items}) w.push_back(uint64_t(v));
+  for (int64_t v : {m.nx, m.ny, m.nzl, m.NZ, m.k0, int64_t(m.ghost), kbeg, kend, items, m.NX, m.NY, m.i0, m.j0,
+                    m.px(), m.py()})
+    w.push_back(uint64_t(v));
   w.push_back(uint64_t(uint32_t(tiles_x)) | (uint64_t(uint32_t(tiles_y)) << 32));
   w.push_back(uint64_t(uint32_t(kz)) | (uint64_t(uint32_t(vec_ok)) << 32));
   // nzero = -0.0 in T (the contraction guard of the paired blocks)
@@ -728,7 +765,8 @@ void PlanImpl::exec_fused(void* out, bool out_dev, cudaStream_t s) {
   bool any_host = false;
   for (int i : L.stencil_inputs) any_host |= !m.fields[dag.inputs[i]].on_device;
   for (int i : L.point_inputs) any_host |= !m.fields[dag.inputs[i]].on_device;
-  if (any_host && m.nzl != m.NZ) fail(DFG_E_UNSUPPORTED, "host-pointer fields are single-slab only");
+  if (any_host && m.nzl != m.NZ && !m.ghosts_supplied)
+    fail(DFG_E_UNSUPPORTED, "host-pointer fields are single-slab only");
 
   // inputs: resident (in situ) or uploaded once (host interface, Table II "Dev-W")
   auto input_ptr = [&](int in) -> const void* {
@@ -798,7 +836,7 @@ void PlanImpl::launch_fused(const std::vector<const void*>& fptr, void* dout, co
   const FusedLayout& L = fsrc.layout;
   const int64_t N = m.nx * m.ny * m.nzl;
   const int vec = int(16 / ts);
-  bool vec_ok = aligned16(dout) && (N % vec == 0);
+  bool vec_ok = aligned16(dout) && (N % vec == 0) && m.gxy == 0;
   for (auto p : fptr) vec_ok = vec_ok && aligned16(p);
   const char* force = std::getenv("DFG_FUSED_KERNEL");
   bool want_general = force && !std::strcmp(force, "general");
@@ -815,7 +853,8 @@ void PlanImpl::launch_fused(const std::vector<const void*>& fptr, void* dout, co
     DFG_CU(drv().LaunchKernel(mod.pointwise, grid, 1, 1, 256, 1, 1, 0, s, args, nullptr));
     DFG_CUDA(cudaEventRecord(ke.second, s));
     last_variant = 3;
-  } else if (mod.tma && !want_general && m.nx % vec == 0 && vec_ok) {
+  } else if (mod.tma && !want_general && m.nx % vec == 0 && m.px() % vec == 0 && aligned16(dout) &&
+             std::all_of(fptr.begin(), fptr.end(), [](const void* p) { return aligned16(p); })) {
     const int ncw = fsrc.cfg.ncw;
     const int nsf = int(L.stencil_inputs.size() + L.point_inputs.size());  // TMA tiles per stage
     const int tiles_x = int((m.nx + 32 * vec - 1) / (32 * vec));
@@ -983,7 +1022,10 @@ void PlanImpl::exec_streamed(void* out, bool out_dev, cudaStream_t s) {
     cudaEvent_t up = new_event();
     DFG_CUDA(cudaEventRecord(up, sH2D));
     DFG_CUDA(cudaStreamWaitEvent(s, up, 0));
-    SlabView v{m.dt, m.nx, m.ny, b - a, m.NZ, a, 1};
+    SlabView v = SlabView::of(m);
+    v.nzl = b - a;
+    v.k0 = a;
+    v.ghost = 1;
     launch_fused(fptr, stream_out[r], tab, v, s);
     computed[c] = new_event();
     DFG_CUDA(cudaEventRecord(computed[c], s));

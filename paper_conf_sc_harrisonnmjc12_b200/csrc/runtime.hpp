@@ -23,11 +23,15 @@ struct Binding {
 
 struct MeshImpl {
   DType dt = DType::F32;
+  // local cells (nx, ny, nzl) of a global NX x NY x NZ mesh at offsets (i0, j0, k0)
   int64_t nx = 0, ny = 0, nzl = 0, NZ = 0, k0 = 0;
-  int ghost = 0;
+  int64_t NX = 0, NY = 0, i0 = 0, j0 = 0;
+  int ghost = 0;     // ghost planes in z (slabs, blocks)
+  int gxy = 0;       // ghost columns / rows in x and y (VisIt blocks, caller-filled)
+  bool ghosts_supplied = false;  // blocks: the caller fills every ghost cell (no exchange)
   int device = 0;
   bool markstein_safe = true;        // spacing tables inside the exact-division range
-  std::vector<char> host_tab[3];     // per axis: d[n] then r[n] (T), reading R1
+  std::vector<char> host_tab[3];     // per axis over the GLOBAL mesh: d | r | -d (T), reading R1
   void* dev_tab[3] = {nullptr, nullptr, nullptr};
   std::map<std::string, Binding> fields;
   // halo transport
@@ -35,25 +39,44 @@ struct MeshImpl {
   void* nccl = nullptr;              // ncclComm_t
   std::weak_ptr<MeshImpl> link_lo, link_hi;
   ~MeshImpl();
-  int64_t plane() const { return nx * ny; }
+  int64_t px() const { return nx + 2 * gxy; }        // input row pitch
+  int64_t py() const { return ny + 2 * gxy; }        // input rows per plane
+  int64_t plane() const { return nx * ny; }          // owned cells per plane (output)
+  int64_t in_plane() const { return px() * py(); }   // input plane incl. x/y ghosts
   int64_t cells() const { return nx * ny * nzl; }
-  size_t field_bytes() const { return size_t(nx * ny * (nzl + 2 * ghost)) * dsize(dt); }
+  size_t field_bytes() const { return size_t(in_plane() * (nzl + 2 * ghost)) * dsize(dt); }
 };
 
 // The part of a mesh one fused launch covers: a whole mesh, a z-slab of a
-// multi-GPU mesh, or one z-chunk of the streamed strategy (ghost planes at
-// local 0 and nzl+1 when ghost = 1).
+// multi-GPU mesh, a VisIt-style block, or one z-chunk of the streamed
+// strategy (ghost planes at local 0 and nzl+1 when ghost = 1; ghost columns /
+// rows at local 0 and n+1 when gxy = 1).
 struct SlabView {
   DType dt;
   int64_t nx, ny, nzl, NZ, k0;
   int ghost;
-  static SlabView of(const MeshImpl& m) { return SlabView{m.dt, m.nx, m.ny, m.nzl, m.NZ, m.k0, m.ghost}; }
+  int64_t NX, NY, i0, j0;
+  int gxy;
+  static SlabView of(const MeshImpl& m) {
+    return SlabView{m.dt, m.nx, m.ny, m.nzl, m.NZ, m.k0, m.ghost, m.NX, m.NY, m.i0, m.j0, m.gxy};
+  }
+  int64_t px() const { return nx + 2 * gxy; }
+  int64_t py() const { return ny + 2 * gxy; }
 };
 
 constexpr int kStreamSlots = 3;  // ring depth of the streamed strategy
 
 std::shared_ptr<MeshImpl> create_mesh(DType dt, int64_t nx, int64_t ny, int64_t nzl, const void* x, const void* y,
                                       const void* z, int64_t NZ, int64_t k0, int ghost);
+// VisIt-style block (NEXT #4): local nx x ny x nz cells at (i0, j0, k0) of a
+// global NX x NY x NZ mesh, global point coordinates, ghost = 0/1 cell shell
+// on all six faces filled by the caller.
+std::shared_ptr<MeshImpl> create_block(DType dt, int64_t nx, int64_t ny, int64_t nz, const void* x, const void* y,
+                                       const void* z, int64_t NX, int64_t NY, int64_t NZ, int64_t i0, int64_t j0,
+                                       int64_t k0, int ghost);
+std::shared_ptr<MeshImpl> create_block_impl(DType dt, int64_t nx, int64_t ny, int64_t nzl, const void* x,
+                                            const void* y, const void* z, int64_t NX, int64_t NY, int64_t NZ,
+                                            int64_t i0, int64_t j0, int64_t k0, int ghost, int gxy);
 
 // Host-side analysis of a network (no device): what each strategy will do.
 struct Model {

@@ -55,6 +55,8 @@ struct DfgParams {
   long long nx, ny, nzl, NZ, k0, ghost;
   long long kbeg, kend;     // global planes computed by this launch
   long long items;          // TMA: tiles_x * tiles_y * zchunks
+  long long NX, NY, i0, j0; // global x/y cells and this block's offsets (whole mesh: NX = nx, i0 = 0)
+  long long px, py;         // input row pitch and rows per plane (nx / ny + 2 x/y ghosts)
   int tiles_x, tiles_y, kz, vec_ok;
   DFG_T nzero;              // -0.0, opaque to the compiler (contraction guard)
 };
@@ -135,10 +137,22 @@ extern "C" __global__ void __launch_bounds__(256) dfg_fused_pointwise(const DfgP
     }
     dfg_store_cells(P.out + (out_off + v * DFG_VEC) * DFG_OUTW, o);
   }
+  const long long gx = (P.px - P.nx) >> 1, gy = (P.py - P.ny) >> 1;
+  const bool pitched = gx != 0 || gy != 0;
   for (long long c = nv * DFG_VEC + tid; c < n; c += stride) {
+    // pitched input index (blocks carry x/y ghost columns / rows); 32-bit
+    // divisions: nx, ny and the launch's row count stay below 2^32
+    long long idx = in_off + c;
+    if (pitched) {
+      const unsigned long long row = (unsigned long long)c / (unsigned)P.nx;
+      const unsigned il = (unsigned)(c - (long long)row * P.nx);
+      const unsigned jl = (unsigned)row % (unsigned)P.ny;
+      const long long kl = (long long)((unsigned)row / (unsigned)P.ny) + (P.kbeg - P.k0);
+      idx = ((kl + P.ghost) * P.py + jl + gy) * P.px + il + gx;
+    }
     dfg2 p[DFG_NPF_];
 #pragma unroll
-    for (int f = 0; f < DFG_NPF; ++f) p[f] = dfg2_splat(P.f[DFG_NSF + f][in_off + c]);
+    for (int f = 0; f < DFG_NPF; ++f) p[f] = dfg2_splat(P.f[DFG_NSF + f][idx]);
     dfg2 o[DFG_OUTW];
     dfg_body(sz, gz, p, z0, z0, z0, z0, z0, z0, Z, o);
 #pragma unroll
@@ -150,20 +164,23 @@ extern "C" __global__ void __launch_bounds__(256) dfg_fused_pointwise(const DfgP
 #if DFG_NSF > 0
 // ------------------------------------------------------------- general
 extern "C" __global__ void __launch_bounds__(256) dfg_fused_general(const DfgParams P) {
-  const long long plane = P.nx * P.ny;
+  const long long plane = P.nx * P.ny;          // output plane (owned cells)
+  const long long in_plane = P.px * P.py;       // input plane (with x/y ghosts)
+  const long long gx = (P.px - P.nx) >> 1, gy = (P.py - P.ny) >> 1;
   const long long total = plane * (P.kend - P.kbeg);
   const long long stride = (long long)gridDim.x * blockDim.x;
   const dfg2 Z = dfg2_splat(P.nzero);
   for (long long c = (long long)blockIdx.x * blockDim.x + threadIdx.x; c < total; c += stride) {
-    const long long i = c % P.nx;
+    const long long il = c % P.nx;
     const long long t = c / P.nx;
-    const long long j = t % P.ny;
+    const long long jl = t % P.ny;
     const long long kg = P.kbeg + t / P.ny;
     const long long kl = kg - P.k0;
-    const long long base = (kl + P.ghost) * plane + j * P.nx + i;
-    const long long oxm = i > 0 ? 1 : 0, oxp = i < P.nx - 1 ? 1 : 0;
-    const long long oym = j > 0 ? P.nx : 0, oyp = j < P.ny - 1 ? P.nx : 0;
-    const long long ozm = kg > 0 ? plane : 0, ozp = kg < P.NZ - 1 ? plane : 0;
+    const long long i = P.i0 + il, j = P.j0 + jl;  // global indices: clamp only at the mesh ends
+    const long long base = ((kl + P.ghost) * P.py + jl + gy) * P.px + il + gx;
+    const long long oxm = i > 0 ? 1 : 0, oxp = i < P.NX - 1 ? 1 : 0;
+    const long long oym = j > 0 ? P.px : 0, oyp = j < P.NY - 1 ? P.px : 0;
+    const long long ozm = kg > 0 ? in_plane : 0, ozp = kg < P.NZ - 1 ? in_plane : 0;
     dfg2 s[DFG_NSF_][7], gn[DFG_NSF_][3];
 #pragma unroll
     for (int f = 0; f < DFG_NSF; ++f) {
@@ -179,9 +196,9 @@ extern "C" __global__ void __launch_bounds__(256) dfg_fused_general(const DfgPar
 #pragma unroll
     for (int f = 0; f < DFG_NPF; ++f) p[f] = dfg2_splat(P.f[DFG_NSF + f][base]);
     dfg2 o[DFG_OUTW];
-    dfg_body(s, gn, p, dfg2_splat(P.tx[2 * P.nx + i]), dfg2_splat(P.tx[P.nx + i]), dfg2_splat(P.ty[2 * P.ny + j]),
-             dfg2_splat(P.ty[P.ny + j]), dfg2_splat(P.tz[2 * P.NZ + kg]), dfg2_splat(P.tz[P.NZ + kg]), Z, o);
-    const long long ob = (kl * plane + j * P.nx + i) * DFG_OUTW;
+    dfg_body(s, gn, p, dfg2_splat(P.tx[2 * P.NX + i]), dfg2_splat(P.tx[P.NX + i]), dfg2_splat(P.ty[2 * P.NY + j]),
+             dfg2_splat(P.ty[P.NY + j]), dfg2_splat(P.tz[2 * P.NZ + kg]), dfg2_splat(P.tz[P.NZ + kg]), Z, o);
+    const long long ob = (kl * plane + jl * P.nx + il) * DFG_OUTW;
 #pragma unroll
     for (int w = 0; w < DFG_OUTW; ++w) P.out[ob + w] = dfg2_get(o[w], 0);
   }

@@ -178,6 +178,48 @@ def test_memory_aware_staged_order(host, prog):
     assert plan2.schedule() == list(range(len(dag.filters)))
 
 
+@pytest.mark.parametrize("shape,split", [((62, 30, 20), (2, 2, 2)), ((61, 23, 17), (2, 3, 2)),
+                                         ((126, 14, 9), (1, 2, 3))])
+@pytest.mark.parametrize("prog", ["qcrit", "intro", "velmag"])
+@pytest.mark.parametrize("strategy", ["fused", "reference"])
+def test_visit_blocks_with_ghost_shells(shape, split, prog, strategy):
+    """VisIt-style multi-block (L253-L255, L315; NEXT #4): every block gets a
+    one-cell ghost shell on all six faces filled from the global field (what
+    VisIt's ghost exchange does); the stitched block interiors equal the
+    whole-mesh result bit for bit (and the oracle)."""
+    import paper_conf_sc_harrisonnmjc12_b200 as dfg
+    if strategy == "reference" and prog == "intro":
+        pytest.skip("no reference kernel for the intro expression")
+    names = NAMES[prog]
+    x, y, z, f = _inputs(shape, np.float32, names)
+    src = PAPER_PROGRAMS[prog][0] if strategy == "fused" else prog
+    whole = run_lib(src, f, x, y, z, strategy)
+    if strategy == "fused":
+        assert_parity(whole, run_oracle(src, f, x, y, z))
+    nx, ny, nz = shape
+    cuts = [np.linspace(0, n, s + 1).astype(int) for n, s in zip(shape, split)]
+    got = np.empty_like(whole)
+    pad = {n: np.pad(a, 1, mode="edge") for n, a in f.items()}   # ghosts at the global ends are ignored
+    for a in range(split[0]):
+        for b in range(split[1]):
+            for c in range(split[2]):
+                i0, i1 = cuts[0][a], cuts[0][a + 1]
+                j0, j1 = cuts[1][b], cuts[1][b + 1]
+                k0, k1 = cuts[2][c], cuts[2][c + 1]
+                m = dfg.Mesh.block(x, y, z, i1 - i0, j1 - j0, k1 - k0, i0, j0, k0, ghost=1)
+                keep = []
+                for n in names:
+                    t = torch.from_numpy(np.ascontiguousarray(pad[n][k0:k1 + 2, j0:j1 + 2, i0:i1 + 2])).cuda()
+                    keep.append(t)
+                    m.bind(n, t)
+                p = dfg.Plan(m, src, strategy)
+                o = torch.empty((k1 - k0, j1 - j0, i1 - i0), device="cuda")
+                p.execute(o)
+                torch.cuda.synchronize()
+                got[k0:k1, j0:j1, i0:i1] = o.cpu().numpy()
+    assert np.array_equal(got, whole)
+
+
 def test_memory_cap():
     """A cap below the predicted footprint fails at compile with
     DFG_E_NOMEM (the paper's failed GPU cases, L309); fused fits."""
