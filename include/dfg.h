@@ -217,8 +217,12 @@ int dfg_reset_stats(dfg_plan plan);
  * fused kernel (0 if none), out[5] = local memory per thread of that kernel
  * (bytes; spills and stack), out[6] = predicted
  * device footprint in bytes for device-resident inputs,
- * out[7] = same for host inputs. */
-int dfg_plan_info(dfg_plan plan, int64_t out[8]);
+ * out[7] = same for host inputs, out[8] = grad3d quotient form of the fused
+ * kernel, bit a set = axis a uses the two-operation exact quotient (fp32,
+ * every divisor of the axis verified at mesh creation),
+ * clear = the three-operation correction (or IEEE / fast division when
+ * DFG_FUSED_VARIANT selects them). */
+int dfg_plan_info(dfg_plan plan, int64_t out[9]);
 
 /* Execution order of the plan's filters (ids of the canonical text).  Staged
  * plans run the paper's list order unless a dev_mem_cap rejected it and the
@@ -265,7 +269,10 @@ int dfg_model(const char* expr, const char* const* inputs, int n_inputs,
 /* Generate the fused kernel source for `expr` on an nx x ny x nz mesh and,
  * if compile != 0, NVRTC-compile it for sm_100a (no device needed); on
  * success *regs / *spill (may be NULL) get the ptxas figures of the TMA
- * kernel.  Writes the source with the buffer protocol above. */
+ * kernel.  fp32 sources use the two-operation quotient on every axis (the
+ * kernel of a mesh whose divisors all verified) unless the environment sets
+ * DFG_FUSED_VARIANT=markstein.  Writes the source with the buffer protocol
+ * above. */
 int dfg_fused_source(const char* expr, const char* const* inputs, int n_inputs,
                      dfg_dtype dtype, int64_t nx, int64_t ny, int64_t nz,
                      int compile, char* buf, size_t cap, size_t* needed,

@@ -206,9 +206,10 @@ def dfg_reset_stats(plan):
 
 
 def dfg_plan_info(plan) -> dict:
-    out = (_I64 * 8)()
+    out = (_I64 * 9)()
     _check(_lib.dfg_plan_info(plan, out))
-    keys = ("strategy", "width", "filters", "variant", "regs", "spill", "footprint_device", "footprint_host")
+    keys = ("strategy", "width", "filters", "variant", "regs", "spill", "footprint_device", "footprint_host",
+            "div2_axes")
     return dict(zip(keys, list(out)))
 
 

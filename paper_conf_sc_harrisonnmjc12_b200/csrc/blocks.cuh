@@ -60,6 +60,21 @@ DFG_DEVICE double dfg_select(double c, double a, double b) { return (c != 0.0) ?
 #ifndef DFG_DIV_MODE
 #define DFG_DIV_MODE 1
 #endif
+// Spacing table of an axis: d[n] | r[n] | -d[n] | yl[n].  The fused kernels
+// pass segment DFG_NDSEG_<axis> as the first table operand of the quotient:
+// -d for the correction, yl for the two-operation form (DFG_DIV2_<axis>).
+#ifndef DFG_DIV2_X
+#define DFG_DIV2_X 0
+#endif
+#ifndef DFG_DIV2_Y
+#define DFG_DIV2_Y 0
+#endif
+#ifndef DFG_DIV2_Z
+#define DFG_DIV2_Z 0
+#endif
+#define DFG_NDSEG_X (DFG_DIV2_X ? 3 : 2)
+#define DFG_NDSEG_Y (DFG_DIV2_Y ? 3 : 2)
+#define DFG_NDSEG_Z (DFG_DIV2_Z ? 3 : 2)
 DFG_DEVICE float dfg_grad1q(float num, float d, float r) {
 #if DFG_DIV_MODE == 0
   (void)r;
@@ -113,6 +128,8 @@ DFG_DEVICE dfg2 dfg2_add(dfg2 a, dfg2 b, dfg2) { return __fadd2_rn(a, b); }
 DFG_DEVICE dfg2 dfg2_sub(dfg2 a, dfg2 b, dfg2) { return __ffma2_rn(b, make_float2(-1.0f, -1.0f), a); }
 DFG_DEVICE dfg2 dfg2_mult(dfg2 a, dfg2 b, dfg2 z) { return __ffma2_rn(a, b, z); }
 DFG_DEVICE dfg2 dfg2_neg(dfg2 a, dfg2 z) { return __ffma2_rn(a, make_float2(-1.0f, -1.0f), z); }
+// RN(b + c*a) for a power of two c (scale folding: c*a is exact, one rounding)
+DFG_DEVICE dfg2 dfg2_axpy(dfg2 a, float c, dfg2 b) { return __ffma2_rn(a, make_float2(c, c), b); }
 #define DFG2_LANEWISE1(name, f) \
   DFG_DEVICE dfg2 name(dfg2 a, dfg2) { return make_float2(f(a.x), f(a.y)); }
 #define DFG2_LANEWISE2(name, f) \
@@ -141,6 +158,16 @@ DFG_DEVICE dfg2 dfg2_gradq(dfg2 num, dfg2 nd, dfg2 r, dfg2 z) {
   return __ffma2_rn(num, r, z);
 #endif
 }
+// Two-operation exact quotient for a divisor known in advance (Brisebarre,
+// Muller and Raina's scheme): yh = r = RN(1/d), yl ~ 1/d - yh, and
+//   q = RN(num*yh + RN(num*yl)).
+// It is not RN(num/d) for every divisor, so the runtime checks each divisor
+// of an axis against IEEE division for all 2^23 significands (kern::
+// verify_div2) and emits this block only for axes that passed: there it is
+// RN(num/d) under the same normal-range conditions as the correction above.
+DFG_DEVICE dfg2 dfg2_gradq2(dfg2 num, dfg2 yl, dfg2 yh, dfg2 z) {
+  return __ffma2_rn(num, yh, __ffma2_rn(num, yl, z));
+}
 #else   // T = double: one cell per "pair", scalar blocks
 typedef double dfg2;
 DFG_DEVICE dfg2 dfg2_splat(double a) { return a; }
@@ -148,6 +175,7 @@ DFG_DEVICE dfg2 dfg2_add(dfg2 a, dfg2 b, dfg2) { return dfg_add(a, b); }
 DFG_DEVICE dfg2 dfg2_sub(dfg2 a, dfg2 b, dfg2) { return dfg_sub(a, b); }
 DFG_DEVICE dfg2 dfg2_mult(dfg2 a, dfg2 b, dfg2) { return dfg_mult(a, b); }
 DFG_DEVICE dfg2 dfg2_neg(dfg2 a, dfg2) { return dfg_neg(a); }
+DFG_DEVICE dfg2 dfg2_axpy(dfg2 a, double c, dfg2 b) { return __fma_rn(a, c, b); }
 DFG_DEVICE dfg2 dfg2_sqrt(dfg2 a, dfg2) { return dfg_sqrt(a); }
 DFG_DEVICE dfg2 dfg2_div(dfg2 a, dfg2 b, dfg2) { return dfg_div(a, b); }
 DFG_DEVICE dfg2 dfg2_gt(dfg2 a, dfg2 b, dfg2) { return dfg_gt(a, b); }

@@ -3,6 +3,7 @@
 // returns the status; nothing throws across the ABI.
 #include <cuda_runtime.h>
 
+#include <cstdlib>
 #include <cstring>
 #include <memory>
 #include <string>
@@ -218,7 +219,7 @@ int dfg_reset_stats(dfg_plan plan) {
   });
 }
 
-int dfg_plan_info(dfg_plan plan, int64_t out[8]) {
+int dfg_plan_info(dfg_plan plan, int64_t out[9]) {
   return guard([&] {
     if (!plan || !out) dfg::fail(DFG_E_INVALID, "null argument");
     auto& p = *plan->p;
@@ -232,6 +233,7 @@ int dfg_plan_info(dfg_plan plan, int64_t out[8]) {
     const int64_t unit = m.cells() * int64_t(dfg::dsize(m.dt));
     out[6] = dfg::model(p.dag, p.strategy, false).units * unit;
     out[7] = dfg::model(p.dag, p.strategy, true).units * unit;
+    out[8] = p.fsrc.cfg.div2;
   });
 }
 
@@ -329,9 +331,15 @@ int dfg_fused_source(const char* expr, const char* const* inputs, int n_inputs, 
     if (!expr) dfg::fail(DFG_E_INVALID, "null expression");
     if (nx < 1 || ny < 1 || nz < 1) dfg::fail(DFG_E_INVALID, "mesh sizes must be >= 1");
     dfg::Dag d = dfg::build_dag(expr, names_of(inputs, n_inputs), to_dtype(dtype));
-    dfg::FusedSource fs = dfg::generate_fused(d, nx, ny, nz, dfg::FusedConfig{});
+    // no mesh here: describe the kernel of a mesh whose divisors all verified
+    // (fp32 two-operation quotient), unless DFG_FUSED_VARIANT=markstein
+    dfg::FusedConfig cfg;
+    const char* var = std::getenv("DFG_FUSED_VARIANT");
+    if (!(var && !std::strcmp(var, "markstein"))) cfg.div2 = 7;
+    dfg::FusedSource fs = dfg::generate_fused(d, nx, ny, nz, cfg);
     if (compile) {
-      const dfg::Cubin& c = dfg::nvrtc_compile(fs.source, "dfg_fused.cu");
+      static const std::string kUnit = "dfg_fused.cu";
+      const dfg::Cubin& c = dfg::nvrtc_compile(fs.source, kUnit);
       if (regs) *regs = c.regs;
       if (spill) *spill = c.spill;
     }

@@ -23,6 +23,8 @@ struct FusedLayout {
 
 struct FusedConfig {
   int div_mode = 1;    // 0 ieee, 1 exact (Markstein), 2 fast; see blocks.cuh
+  int div2 = 0;        // div_mode 1, fp32: bit a = axis a uses the verified two-op quotient
+  bool fold = true;    // power-of-two scale folding in the body (off for div_mode 0, "ieee")
   int ncw = 15;        // consumer warps per CTA (tile rows); +1 producer = 512 threads
   int stages = 0;      // smem ring depth (0: choose)
   int ctas = 1;        // resident CTAs per SM the TMA kernel is sized for

@@ -174,7 +174,7 @@ __device__ __forceinline__ void dfg_plane(const DfgCol& C, DfgRing& R, unsigned&
       gn[h][f][2] = dfg2_sub(s[h][f][6], s[h][f][5], C.Z);
     }
   }
-  const dfg2 ndz = dfg2_splat(__ldg(tzp + 2 * NZ)), rz = dfg2_splat(__ldg(tzp + NZ));
+  const dfg2 ndz = dfg2_splat(__ldg(tzp + DFG_NDSEG_Z * NZ)), rz = dfg2_splat(__ldg(tzp + NZ));
   ++tzp;
   dfg2 p[DFG_NPAIR][DFG_NPF_];
 #pragma unroll
@@ -272,10 +272,10 @@ extern "C" __global__ void __launch_bounds__((DFG_NCW + 1) * 32, DFG_CTAS)
     for (int h = 0; h < DFG_NPAIR; ++h) {
       // spacing tables are indexed globally (blocks: i0 / j0 offsets)
       const long long a = P.i0 + ic + h * DFG_LANES, b = P.i0 + ic + h * DFG_LANES + DFG_LANES - 1;
-      C.ndx[h] = dfg2_mk(__ldg(P.tx + 2 * P.NX + a), __ldg(P.tx + 2 * P.NX + b));
+      C.ndx[h] = dfg2_mk(__ldg(P.tx + DFG_NDSEG_X * P.NX + a), __ldg(P.tx + DFG_NDSEG_X * P.NX + b));
       C.rx[h] = dfg2_mk(__ldg(P.tx + P.NX + a), __ldg(P.tx + P.NX + b));
     }
-    C.ndy = dfg2_splat(__ldg(P.ty + 2 * P.NY + P.j0 + jc));
+    C.ndy = dfg2_splat(__ldg(P.ty + DFG_NDSEG_Y * P.NY + P.j0 + jc));
     C.ry = dfg2_splat(__ldg(P.ty + P.NY + P.j0 + jc));
     // one-sided differences only at the GLOBAL mesh ends (reading R1)
     const long long ig = P.i0 + i, jg = P.j0 + j;

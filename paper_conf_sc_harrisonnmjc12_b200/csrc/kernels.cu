@@ -227,5 +227,31 @@ void grad3d(DType dt, const void* f, void* o4, const void* tx, const void* ty, c
                                                       ghost);
 }
 
+namespace {
+// One CTA row (blockIdx.y) per divisor; the x-dimension strides over the
+// 2^23 significands of a in [1, 2).  Every quantity scales exactly with a
+// power of two as long as a*yl and the quotient stay normal, so these 2^23
+// values decide the whole range.
+__global__ void __launch_bounds__(256) k_verify_div2(const float* __restrict__ d, const float* __restrict__ yh,
+                                                     const float* __restrict__ yl, int n, unsigned* __restrict__ bad) {
+  for (int k = blockIdx.y; k < n; k += gridDim.y) {
+    const float dk = d[k], hk = yh[k], lk = yl[k];
+    unsigned miss = 0;
+    for (unsigned m = blockIdx.x * blockDim.x + threadIdx.x; m < (1u << 23); m += gridDim.x * blockDim.x) {
+      const float a = __uint_as_float(0x3f800000u | m);
+      const float q = __fmaf_rn(a, hk, __fmul_rn(a, lk));
+      miss |= __float_as_uint(q) ^ __float_as_uint(__fdiv_rn(a, dk));
+    }
+    if (__any_sync(0xffffffffu, miss != 0) && (threadIdx.x & 31) == 0) atomicOr(bad + k, 1u);
+  }
+}
+}  // namespace
+
+void verify_div2(const float* d, const float* yh, const float* yl, int n, unsigned* bad, cudaStream_t s) {
+  if (n <= 0) return;
+  dim3 grid(64, unsigned(n < 32768 ? n : 32768));
+  k_verify_div2<<<grid, 256, 0, s>>>(d, yh, yl, n, bad);
+}
+
 }  // namespace kern
 }  // namespace dfg

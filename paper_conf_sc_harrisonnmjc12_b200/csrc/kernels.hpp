@@ -19,5 +19,11 @@ void compose(DType dt, const void* const* in, int w, void* o4, long long n, cuda
 void grad3d(DType dt, const void* f, void* o4, const void* tx, const void* ty, const void* tz, long long nx,
             long long ny, long long nzl, long long NZ, long long k0, long long ghost, cudaStream_t s);
 
+// Exhaustive check of the two-operation quotient for n fp32 divisors
+// (DESIGN.md section 5): bad[k] = 1 unless, for all 2^23 significands
+// a in [1, 2), RN(a*yh[k] + RN(a*yl[k])) == RN(a / d[k]).  Device pointers;
+// bad must be zeroed by the caller.
+void verify_div2(const float* d, const float* yh, const float* yl, int n, unsigned* bad, cudaStream_t s);
+
 }  // namespace kern
 }  // namespace dfg

@@ -29,10 +29,11 @@ void build_axis(const T* p, int64_t n, std::vector<char>& tab, bool& safe) {
     if (!(p[i] < p[i + 1])) fail(DFG_E_INVALID, "coordinates must be strictly increasing");
   std::vector<T> c(n);
   for (int64_t i = 0; i < n; ++i) c[i] = (p[i] + p[i + 1]) * T(0.5);
-  tab.assign(size_t(3 * n) * sizeof(T), 0);
+  tab.assign(size_t(4 * n) * sizeof(T), 0);
   T* d = reinterpret_cast<T*>(tab.data());
   T* r = d + n;
   T* nd = r + n;  // exact negation: the fused kernels form num - q0*d with one FFMA2
+  T* yl = nd + n; // low part of 1/d for the two-operation quotient (fp32 only)
   for (int64_t i = 0; i < n; ++i) {
     if (n == 1) {  // derivative is 0 by definition; the kernels never read these
       d[i] = T(1);
@@ -45,10 +46,67 @@ void build_axis(const T* p, int64_t n, std::vector<char>& tab, bool& safe) {
     if (!(d[i] > T(0))) fail(DFG_E_INVALID, "cell centres coincide (coordinates too close for T)");
     r[i] = T(1) / d[i];
     nd[i] = -d[i];
+    // yl = RN(1/d - r): 1/d in double is within 2^-53 of the real quotient and
+    // the subtraction is exact (Sterbenz); the kernels only use yl on axes whose
+    // every divisor passed the exhaustive check (verify_div2 below), so its last
+    // bit needs no argument.
+    if (sizeof(T) == 4) yl[i] = T(1.0 / double(d[i]) - double(r[i]));
     // Markstein's exact-quotient argument needs d and r well inside the normal range.
     double ad = double(d[i]);
     if (!(ad > 0x1p-60 && ad < 0x1p60) || !std::isfinite(double(r[i]))) safe = false;
   }
+}
+
+// Two-operation quotient: an fp32 axis uses
+// q = RN(num*r + RN(num*yl)) in the fused kernels only if every divisor of
+// its table passed the exhaustive device check.  Verdicts are cached per
+// (d, yl) bit pattern (r is a function of d).
+std::mutex g_div2_mu;
+std::map<uint64_t, bool> g_div2_ok;  // key: d bits << 32 | yl bits
+
+uint64_t div2_key(float d, float yl) {
+  uint32_t a, b;
+  std::memcpy(&a, &d, 4);
+  std::memcpy(&b, &yl, 4);
+  return uint64_t(a) << 32 | b;
+}
+
+bool axis_div2(const std::vector<char>& tab, int64_t n) {
+  const float* d = reinterpret_cast<const float*>(tab.data());
+  const float* r = d + n;
+  const float* yl = d + 3 * n;
+  if (n == 1) return true;  // no division on a degenerate axis
+  std::lock_guard<std::mutex> lk(g_div2_mu);
+  std::vector<float> qd, qr, ql;
+  std::set<uint64_t> seen;
+  for (int64_t i = 0; i < n; ++i) {
+    const uint64_t b = div2_key(d[i], yl[i]);
+    if (g_div2_ok.count(b) || !seen.insert(b).second) continue;
+    qd.push_back(d[i]);
+    qr.push_back(r[i]);
+    ql.push_back(yl[i]);
+  }
+  if (!qd.empty()) {
+    const int m = int(qd.size());
+    float* buf = nullptr;
+    unsigned* bad = nullptr;
+    DFG_CUDA(cudaMalloc(&buf, 3 * size_t(m) * sizeof(float)));
+    DFG_CUDA(cudaMalloc(&bad, size_t(m) * sizeof(unsigned)));
+    DFG_CUDA(cudaMemcpy(buf, qd.data(), m * sizeof(float), cudaMemcpyHostToDevice));
+    DFG_CUDA(cudaMemcpy(buf + m, qr.data(), m * sizeof(float), cudaMemcpyHostToDevice));
+    DFG_CUDA(cudaMemcpy(buf + 2 * m, ql.data(), m * sizeof(float), cudaMemcpyHostToDevice));
+    DFG_CUDA(cudaMemset(bad, 0, size_t(m) * sizeof(unsigned)));
+    kern::verify_div2(buf, buf + m, buf + 2 * m, m, bad, nullptr);
+    std::vector<unsigned> hb(m);
+    cudaError_t e = cudaMemcpy(hb.data(), bad, m * sizeof(unsigned), cudaMemcpyDeviceToHost);
+    cudaFree(buf);
+    cudaFree(bad);
+    DFG_CUDA(e);
+    for (int k = 0; k < m; ++k) g_div2_ok[div2_key(qd[k], ql[k])] = hb[k] == 0;
+  }
+  for (int64_t i = 0; i < n; ++i)
+    if (!g_div2_ok[div2_key(d[i], yl[i])]) return false;
+  return true;
 }
 
 std::mutex g_pool_mu;
@@ -154,10 +212,21 @@ std::shared_ptr<MeshImpl> create_block_impl(DType dt, int64_t nx, int64_t ny, in
     fail(DFG_E_CUDA, "no CUDA device available (libdfg has no CPU fallback)");
   }
   DFG_CUDA(cudaGetDevice(&m->device));
+  // DFG_DIV2=0: never use the two-operation quotient; DFG_DIV2=test-1op (tests
+  // only): yl = 0, i.e. the one-operation RN(num*r), which the check must reject
+  // unless every divisor is a power of two
+  const char* d2 = std::getenv("DFG_DIV2");
+  const bool div2_off = d2 && !std::strcmp(d2, "0");
+  if (dt == DType::F32 && d2 && !std::strcmp(d2, "test-1op"))
+    for (int a = 0; a < 3; ++a)
+      std::fill_n(reinterpret_cast<float*>(m->host_tab[a].data()) + 3 * N[a], N[a], 0.0f);
   for (int a = 0; a < 3; ++a) {
     DFG_CUDA(cudaMalloc(&m->dev_tab[a], m->host_tab[a].size()));
     DFG_CUDA(cudaMemcpy(m->dev_tab[a], m->host_tab[a].data(), m->host_tab[a].size(), cudaMemcpyHostToDevice));
   }
+  if (dt == DType::F32 && m->markstein_safe && !div2_off)
+    for (int a = 0; a < 3; ++a)
+      if (axis_div2(m->host_tab[a], N[a])) m->div2_mask |= 1 << a;
   return m;
 }
 
@@ -573,6 +642,13 @@ std::unique_ptr<PlanImpl> compile_plan(std::shared_ptr<MeshImpl> mesh, const std
     if (var && !std::strcmp(var, "ieee")) cfg.div_mode = 0;
     else if (var && !std::strcmp(var, "fast")) cfg.div_mode = 2;
     if (!mesh->markstein_safe && cfg.div_mode == 1) cfg.div_mode = 0;  // keep results exact
+    // exact quotient with two operations on the axes whose divisors all verified;
+    // DFG_FUSED_VARIANT=markstein keeps the three-operation correction everywhere
+    const bool markstein_only = var && !std::strcmp(var, "markstein");
+    if (cfg.div_mode == 1 && mesh->dt == DType::F32 && !markstein_only) cfg.div2 = mesh->div2_mask;
+    // scale folding is exact in the normal range only; "ieee" keeps every op
+    const char* fold = std::getenv("DFG_SCALE_FOLD");
+    cfg.fold = cfg.div_mode != 0 && !(fold && !std::strcmp(fold, "0"));
     const char* ncw = std::getenv("DFG_NCW");
     if (ncw) cfg.ncw = std::max(1, std::min(30, std::atoi(ncw)));
     const char* ctas = std::getenv("DFG_CTAS");
@@ -581,7 +657,8 @@ std::unique_ptr<PlanImpl> compile_plan(std::shared_ptr<MeshImpl> mesh, const std
     if (st) cfg.stages = std::max(2, std::min(16, std::atoi(st)));
     // axis degeneracy (n == 1) is a property of the GLOBAL mesh
     plan->fsrc = generate_fused(dag, mesh->NX, mesh->NY, mesh->NZ, cfg, ref);
-    const Cubin& cb = nvrtc_compile(plan->fsrc.source, "dfg_fused.cu");
+    static const std::string kUnit = "dfg_fused.cu";
+    const Cubin& cb = nvrtc_compile(plan->fsrc.source, kUnit);  // cached for the process lifetime
     plan->regs = cb.regs;
     plan->spill = cb.spill;
     // the runtime API owns the primary context; make it current for the driver API

@@ -49,9 +49,9 @@ __device__ __forceinline__ DFG_T dfg2_get(dfg2 v, int) { return v; }
 struct DfgParams {
   const DFG_T* f[DFG_NF_];  // fields: base of T[nzl + 2*ghost][ny][nx]
   DFG_T* out;               // T[nzl][ny][nx][DFG_OUTW]
-  const DFG_T* tx;          // x table: d[nx] | r[nx] | -d[nx]
-  const DFG_T* ty;          // y table: d[ny] | r[ny] | -d[ny]
-  const DFG_T* tz;          // z table over the GLOBAL mesh: d[NZ] | r[NZ] | -d[NZ]
+  const DFG_T* tx;          // x table: d[nx] | r[nx] | -d[nx] | yl[nx]
+  const DFG_T* ty;          // y table: d[ny] | r[ny] | -d[ny] | yl[ny]
+  const DFG_T* tz;          // z table over the GLOBAL mesh: d[NZ] | r[NZ] | -d[NZ] | yl[NZ]
   long long nx, ny, nzl, NZ, k0, ghost;
   long long kbeg, kend;     // global planes computed by this launch
   long long items;          // TMA: tiles_x * tiles_y * zchunks
@@ -196,8 +196,8 @@ extern "C" __global__ void __launch_bounds__(256) dfg_fused_general(const DfgPar
 #pragma unroll
     for (int f = 0; f < DFG_NPF; ++f) p[f] = dfg2_splat(P.f[DFG_NSF + f][base]);
     dfg2 o[DFG_OUTW];
-    dfg_body(s, gn, p, dfg2_splat(P.tx[2 * P.NX + i]), dfg2_splat(P.tx[P.NX + i]), dfg2_splat(P.ty[2 * P.NY + j]),
-             dfg2_splat(P.ty[P.NY + j]), dfg2_splat(P.tz[2 * P.NZ + kg]), dfg2_splat(P.tz[P.NZ + kg]), Z, o);
+    dfg_body(s, gn, p, dfg2_splat(P.tx[DFG_NDSEG_X * P.NX + i]), dfg2_splat(P.tx[P.NX + i]), dfg2_splat(P.ty[DFG_NDSEG_Y * P.NY + j]),
+             dfg2_splat(P.ty[P.NY + j]), dfg2_splat(P.tz[DFG_NDSEG_Z * P.NZ + kg]), dfg2_splat(P.tz[P.NZ + kg]), Z, o);
     const long long ob = (kl * plane + jl * P.nx + il) * DFG_OUTW;
 #pragma unroll
     for (int w = 0; w < DFG_OUTW; ++w) P.out[ob + w] = dfg2_get(o[w], 0);

@@ -58,6 +58,52 @@ def test_tma_and_general_kernels_identical(T, monkeypatch):
     assert np.array_equal(a, b)
 
 
+@pytest.mark.parametrize("shape", [(132, 40, 33), (67, 45, 37)])
+def test_two_operation_quotient(shape, monkeypatch):
+    """on fp32 axes whose every divisor passed the
+    exhaustive check the fused kernels form d f/d axis as
+    RN(num*r + RN(num*yl)); the bits equal the oracle's IEEE division and the
+    three-operation correction's (TMA and general kernels)."""
+    x, y, z, f = _inputs(shape, np.float32)
+    src = PAPER_PROGRAMS["qcrit"][0]
+    want = run_oracle(src, f, x, y, z)
+    a, plan, *_ = run_lib(src, f, x, y, z, return_plan=True)
+    assert plan.info()["div2_axes"] == 7
+    assert_parity(a, want)
+    monkeypatch.setenv("DFG_FUSED_VARIANT", "markstein")
+    b, plan2, *_ = run_lib(src, f, x, y, z, return_plan=True)
+    assert plan2.info()["div2_axes"] == 0
+    assert np.array_equal(a.view(np.uint32), b.view(np.uint32))
+    monkeypatch.delenv("DFG_FUSED_VARIANT")
+    monkeypatch.setenv("DFG_DIV2", "0")
+    c, plan3, *_ = run_lib(src, f, x, y, z, return_plan=True)
+    assert plan3.info()["div2_axes"] == 0
+    assert np.array_equal(a.view(np.uint32), c.view(np.uint32))
+
+
+def test_two_operation_check_rejects_one_operation(monkeypatch):
+    """The device check is not vacuous: with yl = 0 (the one-operation
+    RN(num*r), not correctly rounded for most divisors) it rejects every axis
+    of the RT mesh, while on a uniform mesh with power-of-two spacing, where
+    r = 1/d exactly and RN(num*r) = RN(num/d), it accepts all three."""
+    monkeypatch.setenv("DFG_DIV2", "test-1op")
+    src = PAPER_PROGRAMS["vortmag"][0]
+    x, y, z, f = _inputs((64, 24, 20), np.float32)
+    got, plan, *_ = run_lib(src, f, x, y, z, return_plan=True)
+    assert plan.info()["div2_axes"] == 0
+    assert_parity(got, run_oracle(src, f, x, y, z))
+    x, y, z = (synth.uniform_coords(n, dtype=np.float32) for n in (64, 24, 20))
+    got, plan, *_ = run_lib(src, f, x, y, z, return_plan=True)
+    assert plan.info()["div2_axes"] == 7
+    assert_parity(got, run_oracle(src, f, x, y, z))
+
+
+def test_two_operation_quotient_fp32_only():
+    x, y, z, f = _inputs((40, 24, 20), np.float64)
+    _, plan, *_ = run_lib(PAPER_PROGRAMS["qcrit"][0], f, x, y, z, return_plan=True)
+    assert plan.info()["div2_axes"] == 0
+
+
 @pytest.mark.parametrize("kz", ["1", "3", "7", "1000"])
 def test_tma_z_chunking(kz, monkeypatch):
     """Every z-chunk length gives the same bits (halo planes at chunk ends)."""
@@ -89,6 +135,15 @@ EDGE = [
     ("a = u / v\nb = -a * (a >= 0.5) + (v != u)", ("u", "v")),
     ("a = if (grad(u)[0] > grad(v)[1]) then (sqrt(u * u)) else (v / u)", ("u", "v")),
     ("d = grad({u, v}[1] - u)\ne = norm(d) + d[2]", ("u", "v")),
+    # power-of-two scale folding: free scalings, FMA adds
+    # of unequal scales, sqrt of even / odd scales, compare / select / vector /
+    # result materialisation, the exponent cap, constant x constant
+    ("a = 0.5 * (u - v)\nb = a * a + 0.25 * u * (2 * v) - 4 * a / (0.125 * v)\nc = sqrt(0.25 * u * u) + b * 0.5",
+     ("u", "v")),
+    ("a = (u * 0.5) * (v * 0.25)\nb = if (a > 0.0625 * u) then (a / 2) else (-a * 8)\nc = {a * 2, b, sqrt(a * 4)}",
+     ("u", "v")),
+    ("a = u * 256 * 256 * 256 * 256 * 0.5 + v * (0.5 * 0.5)\nb = a / 256 / 256 / 256 - grad(u * 0.5)[0] * 0.25",
+     ("u", "v")),
 ]
 
 

@@ -200,10 +200,17 @@ def test_partition_matches_closed_form(dfg, NZ, G):
 
 @pytest.mark.parametrize("name", ["velmag", "vortmag", "qcrit", "intro"])
 @pytest.mark.parametrize("dtype", [0, 1])
-def test_fused_kernel_compiles_without_spills(dfg, name, dtype):
+@pytest.mark.parametrize("variant", ["", "markstein"])
+def test_fused_kernel_compiles_without_spills(dfg, name, dtype, variant, monkeypatch):
+    """Both grad3d quotient forms (two-operation on verified axes, the
+    three-operation correction otherwise)."""
+    if variant:
+        monkeypatch.setenv("DFG_FUSED_VARIANT", variant)
     src, inputs = PAPER_PROGRAMS[name]
     code, regs, spill = dfg.dfg_fused_source(src, inputs, dtype, 64, 48, 40, compile=True)
     assert "dfg_body" in code and "extern \"C\" __global__" in code
+    two_op = dtype == 0 and not variant and name != "velmag"
+    assert ("dfg2_gradq2(gn" in code) == two_op
     assert regs > 0
     assert spill == 0, (regs, spill)
 
