@@ -239,7 +239,10 @@ def main():
     barrier()
     ms = e0.elapsed_time(e1)
     st = plan.stats()
-    kern_ms = st["kernel_ms_sum"] / max(1, st["kernel_launches_timed"])
+    # fused-kernel time per step: one launch at N=1; at N>1 the interior launch
+    # plus the one or two boundary-plane launches that follow the halo exchange
+    launches_per_step = st["kernel_count"] / max(1, K)
+    kern_ms = st["kernel_ms_sum"] / max(1, st["kernel_launches_timed"]) * launches_per_step
     t = torch.tensor([ms, kern_ms], device="cuda", dtype=torch.float64)
     if world > 1:
         dist.all_reduce(t, op=dist.ReduceOp.MAX)

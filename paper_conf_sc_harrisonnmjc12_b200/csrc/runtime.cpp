@@ -577,6 +577,9 @@ PlanImpl::~PlanImpl() {
   release_stream_buffers();
   if (sH2D) cudaStreamDestroy(sH2D);
   if (sD2H) cudaStreamDestroy(sD2H);
+  if (sHalo) cudaStreamDestroy(sHalo);
+  if (evHaloIn) cudaEventDestroy(evHaloIn);
+  if (evHaloOut) cudaEventDestroy(evHaloOut);
   if (cur >= 0) cudaSetDevice(cur);
 }
 
@@ -866,7 +869,23 @@ void PlanImpl::exec_fused(void* out, bool out_dev, cudaStream_t s) {
   for (int i : L.stencil_inputs) fptr.push_back(got[i]);
   for (int i : L.point_inputs) fptr.push_back(got[i]);
 
-  if (!any_host && !L.stencil_inputs.empty()) halo_exchange(L.stencil_inputs, s);
+  // z-slab of a multi-GPU mesh: the ghost planes arrive while the interior
+  // planes (which read only owned planes) compute; the one or two planes next
+  // to a ghost plane run after the exchange.  DFG_HALO_OVERLAP=0: serial.
+  const bool need_lo = m.k0 > 0, need_hi = m.k0 + m.nzl < m.NZ;
+  const bool halo = !any_host && !L.stencil_inputs.empty() && (need_lo || need_hi) && !m.ghosts_supplied;
+  const char* ov = std::getenv("DFG_HALO_OVERLAP");
+  const bool overlap = halo && m.nzl >= 3 && !(ov && !std::strcmp(ov, "0"));
+  if (halo && !overlap) halo_exchange(L.stencil_inputs, s);
+  if (overlap) {
+    if (!sHalo) DFG_CUDA(cudaStreamCreateWithFlags(&sHalo, cudaStreamNonBlocking));
+    if (!evHaloIn) DFG_CUDA(cudaEventCreateWithFlags(&evHaloIn, cudaEventDisableTiming));
+    if (!evHaloOut) DFG_CUDA(cudaEventCreateWithFlags(&evHaloOut, cudaEventDisableTiming));
+    DFG_CUDA(cudaEventRecord(evHaloIn, s));
+    DFG_CUDA(cudaStreamWaitEvent(sHalo, evHaloIn, 0));
+    halo_exchange(L.stencil_inputs, sHalo);
+    DFG_CUDA(cudaEventRecord(evHaloOut, sHalo));
+  }
 
   // mesh arrays: resident, or uploaded like the paper's dims/x/y/z (L225)
   const void* tab[3] = {m.dev_tab[0], m.dev_tab[1], m.dev_tab[2]};
@@ -895,7 +914,15 @@ void PlanImpl::exec_fused(void* out, bool out_dev, cudaStream_t s) {
     scratch.push_back(dout);
   }
 
-  launch_fused(fptr, dout, tab, SlabView::of(m), s);
+  if (overlap) {
+    const int64_t a = m.k0 + (need_lo ? 1 : 0), b = m.k0 + m.nzl - (need_hi ? 1 : 0);
+    launch_fused(fptr, dout, tab, SlabView::of(m), s, a, b);
+    DFG_CUDA(cudaStreamWaitEvent(s, evHaloOut, 0));
+    if (need_lo) launch_fused(fptr, dout, tab, SlabView::of(m), s, m.k0, m.k0 + 1);
+    if (need_hi) launch_fused(fptr, dout, tab, SlabView::of(m), s, b, b + 1);
+  } else {
+    launch_fused(fptr, dout, tab, SlabView::of(m), s);
+  }
   if (!out_dev) {
     DFG_CUDA(cudaMemcpyAsync(out, dout, out_bytes, cudaMemcpyDeviceToHost, s));
     st.d2h_count += 1;
@@ -908,17 +935,17 @@ void PlanImpl::exec_fused(void* out, bool out_dev, cudaStream_t s) {
 // One launch of the generated kernel over the owned planes of a slab view
 // (the mesh itself, or one z-chunk of the streamed strategy).
 void PlanImpl::launch_fused(const std::vector<const void*>& fptr, void* dout, const void* const tab[3],
-                            const SlabView& m, cudaStream_t s) {
+                            const SlabView& m, cudaStream_t s, int64_t kb, int64_t ke) {
   const size_t ts = dsize(m.dt);
   const FusedLayout& L = fsrc.layout;
-  const int64_t N = m.nx * m.ny * m.nzl;
+  const int64_t kbeg = kb < 0 ? m.k0 : kb, kend = ke < 0 ? m.k0 + m.nzl : ke;
+  const int64_t N = m.nx * m.ny * (kend - kbeg);
   const int vec = int(16 / ts);
   bool vec_ok = aligned16(dout) && (N % vec == 0) && m.gxy == 0;
   for (auto p : fptr) vec_ok = vec_ok && aligned16(p);
   const char* force = std::getenv("DFG_FUSED_KERNEL");
   bool want_general = force && !std::strcmp(force, "general");
   const int sms = sm_count(mesh->device);
-  const int64_t kbeg = m.k0, kend = m.k0 + m.nzl;
 
   if (L.stencil_inputs.empty()) {
     auto w = pack_params(fptr, dout, tab[0], tab[1], tab[2], m, kbeg, kend, 0, 0, 0, 0, vec_ok ? 1 : 0);

@@ -114,12 +114,17 @@ struct PlanImpl {
   int stream_R = 0;
   bool stream_ready = false;
   cudaStream_t sH2D = nullptr, sD2H = nullptr;
+  // multi-slab fused execute: halo exchange on its own stream, overlapped
+  // with the interior planes
+  cudaStream_t sHalo = nullptr;
+  cudaEvent_t evHaloIn = nullptr, evHaloOut = nullptr;
   ~PlanImpl();
   void execute(void* out, bool out_dev, cudaStream_t s);
 
  private:
+  // kb / ke: global plane range of this launch (default: all owned planes of v)
   void launch_fused(const std::vector<const void*>& fptr, void* dout, const void* const tab[3], const SlabView& v,
-                    cudaStream_t s);
+                    cudaStream_t s, int64_t kb = -1, int64_t ke = -1);
   void exec_streamed(void* out, bool out_dev, cudaStream_t s);
   void release_stream_buffers();
   void exec_fused(void* out, bool out_dev, cudaStream_t s);

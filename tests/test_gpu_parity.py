@@ -295,14 +295,18 @@ def test_memory_cap():
     assert_parity(got, run_oracle(src, f, x, y, z))
 
 
-@pytest.mark.parametrize("G", [2, 3, 5])
+@pytest.mark.parametrize("G", [2, 3, 5, 12])
 @pytest.mark.parametrize("T", [np.float32, np.float64])
-def test_zslab_emulation_matches_single_gpu(G, T):
+@pytest.mark.parametrize("overlap", ["1", "0"])
+def test_zslab_emulation_matches_single_gpu(G, T, overlap, monkeypatch):
     """G z-slabs with one ghost plane each, halo by device copies
     (dfg_mesh_link_local): the concatenated result equals the one-slab
-    result bit for bit, and the halo maps equal the closed form."""
+    result bit for bit, and the halo maps equal the closed form.  With the
+    overlap the exchange runs on a side stream during the
+    interior planes and each slab launches 1 + (number of halo sides) kernels."""
     import paper_conf_sc_harrisonnmjc12_b200 as dfg
     from oracle import halo as ohalo
+    monkeypatch.setenv("DFG_HALO_OVERLAP", overlap)
     shape = (64, 20, 23)
     x, y, z, f = _inputs(shape, T)
     src = PAPER_PROGRAMS["qcrit"][0]
@@ -334,7 +338,9 @@ def test_zslab_emulation_matches_single_gpu(G, T):
     assert np.array_equal(got, whole)
     for r, p in enumerate(plans):
         sides = (r > 0) + (r < G - 1)
-        assert p.stats()["halo_bytes"] == 3 * sides * shape[0] * shape[1] * np.dtype(T).itemsize
+        st = p.stats()
+        assert st["halo_bytes"] == 3 * sides * shape[0] * shape[1] * np.dtype(T).itemsize
+        assert st["kernel_count"] == (1 + sides if overlap == "1" and meshes[r].nz >= 3 else 1)
 
 
 def test_config2_192_all_strategies():
