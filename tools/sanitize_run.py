@@ -32,6 +32,31 @@ def main():
         os.environ["DFG_KZ"] = "2"
         dfg.Plan(mesh, PAPER_PROGRAMS["qcrit"][0], "fused").execute(out)
         os.environ.pop("DFG_KZ")
+        # streamed strategy from host fields (3-slot chunk ring, three streams)
+        host = dfg.Mesh(x, y, z)
+        for k, v in f.items():
+            host.bind(k, v.numpy(), on_device=False)
+        os.environ["DFG_STREAM_PLANES"] = "4"
+        hout = np.empty((shape[2], shape[1], shape[0]), dtype=T)
+        dfg.Plan(host, PAPER_PROGRAMS["qcrit"][0], "streamed").execute(hout, out_on_device=False)
+        os.environ.pop("DFG_STREAM_PLANES")
+        # three z-slabs linked in one process: halo exchange on the side stream
+        # overlapped with the interior planes, then the boundary-plane launches
+        slabs, keep = [], []
+        for r in range(3):
+            k0, nzr = dfg.dfg_partition(shape[2], 3, r)
+            m = dfg.Mesh(x, y, z, nz_local=nzr, z_offset=k0, ghost=1)
+            for k, v in f.items():
+                buf = torch.zeros((nzr + 2,) + tuple(v.shape[1:]), dtype=tt, device="cuda")
+                buf[1:nzr + 1] = v[k0:k0 + nzr].cuda()
+                keep.append(buf)
+                m.bind(k, buf)
+            slabs.append(m)
+        for r in range(2):
+            dfg.dfg_mesh_link_local(slabs[r].handle, slabs[r + 1].handle)
+        for m in slabs:
+            o = torch.empty((m.nz, shape[1], shape[0]), dtype=tt, device="cuda")
+            dfg.Plan(m, PAPER_PROGRAMS["qcrit"][0], "fused").execute(o)
         torch.cuda.synchronize()
     print("sanitize run done")
 
