@@ -202,3 +202,160 @@ def _staged_footprint(dag: Dag, mode: str, order) -> int:
             live += _units(dag, dag.result)       # bare input result: upload it
             high = max(high, live)
         return high
+
+
+# ---------------------------------------------------------------- hybrid
+# Staged execution under a device-memory cap with spill-to-host (SURVEY 8f
+# NEXT #3, the Fig. 2 argument L107-L114 that staged execution can run where
+# memory is short, carried one step further).  The policy is stated in
+# DESIGN.md section 5b ("Hybrid"); this is a plain restatement of it, written
+# independently of libdfg's C++ planner.
+
+@dataclass
+class Hybrid:
+    events: list      # (kind, ref) in execution order
+    counts: Counts    # h2d / d2h transfers and kernels of one execution
+    high: int         # device high-water in units
+    h2d_units: int    # problem-array units moved host -> device
+    d2h_units: int    # problem-array units moved device -> host
+
+
+class HybridInfeasible(Exception):
+    """The cap is below the working set of some filter."""
+
+
+def hybrid(dag: Dag, mode: str, cap: int, order=None) -> Hybrid:
+    """Run the filters in ``order`` (default list order) holding at most
+    ``cap`` units on the device.
+
+    * device mode: the bound inputs and the output buffer stay resident and
+      count against the cap throughout; host mode: inputs are uploaded when a
+      filter needs them.
+    * Before a filter runs, each operand that is not resident is brought in
+      (an input: upload from the caller's host array; an intermediate: reload
+      from its pinned host copy), then its result array is allocated (unless,
+      in device mode, it is the result computed last, which goes straight into
+      the output buffer).  Whenever the next array does not fit, the resident
+      array with the furthest next use is evicted (ties: the larger, then
+      filters before inputs, then the higher id), never an operand of the
+      current filter: an intermediate without a host copy is spilled
+      (device -> host, once: values never change; later evictions just discard
+      the device copy), an input is dropped.
+    * After the filter, every operand whose reference count reaches zero is
+      freed (device and host copies).
+    * The sink: the result goes to the caller (host mode: device -> host if it
+      is resident, else from its host copy without a transfer; device mode:
+      nothing if computed into the output buffer, a device copy if resident,
+      else host -> device from its host copy).
+    """
+    if order is None:
+        order = list(range(len(dag.filters)))
+    order = list(order)
+    assert is_topological(dag, order)
+    srcs, mesh = _sources(dag)
+    n = len(order)
+    uses: dict = {}
+    for p, k in enumerate(order):
+        for r in dag.filters[k].inputs:
+            if r not in MESH_NAMES:
+                uses.setdefault(r, []).append(p)
+    uses.setdefault(dag.result, []).append(n)          # the sink reads the result
+
+    def next_use(ref, pos):
+        later = [p for p in uses.get(ref, []) if p >= pos]
+        return min(later) if later else n + 1
+
+    def tie_key(ref):
+        kind = 1 if _is_filter(dag, ref) else 0
+        ident = int(ref[1:]) if kind else list(dag.inputs).index(ref)
+        return (kind, ident)
+
+    rc = _refcounts(dag)
+    events: list = []
+    resident: dict = {}                 # evictable device arrays -> units
+    host_copy: set = set()
+    base = 0
+    if mode == "device":
+        base = sum(_units(dag, s) for s in srcs) + _units(dag, dag.result)
+    high = base
+    h2d = d2h = h2du = d2hu = 0
+    mesh_up = False
+
+    def live():
+        return base + sum(resident.values())
+
+    def make_room(units, protect, pos):
+        nonlocal d2h, d2hu
+        while live() + units > cap:
+            cands = [r for r in resident if r not in protect]
+            if not cands:
+                raise HybridInfeasible(f"cap {cap} below the working set at position {pos}")
+            victim = max(cands, key=lambda r: (next_use(r, pos), resident[r]) + tie_key(r))
+            if _is_filter(dag, victim):
+                if victim not in host_copy:
+                    events.append(("spill", victim))
+                    host_copy.add(victim)
+                    d2h += 1
+                    d2hu += resident[victim]
+                else:
+                    events.append(("discard", victim))      # host copy still valid
+            else:
+                events.append(("drop", victim))
+            del resident[victim]
+
+    def bring(ref, protect, pos):
+        nonlocal h2d, h2du
+        if ref in resident or (mode == "device" and not _is_filter(dag, ref)):
+            return
+        u = _units(dag, ref)
+        make_room(u, protect, pos)
+        if _is_filter(dag, ref):
+            assert ref in host_copy
+            events.append(("reload", ref))
+        else:
+            events.append(("upload", ref))
+        h2d += 1
+        h2du += u
+        resident[ref] = u
+
+    for pos, k in enumerate(order):
+        f = dag.filters[k]
+        ref = f"f{k}"
+        need = [r for r in f.inputs if r not in MESH_NAMES]
+        if mode == "host" and not mesh_up and any(r in MESH_NAMES for r in f.inputs):
+            mesh_up = True
+            h2d += 4                                        # dims, x, y, z (R13)
+        for r in dict.fromkeys(need):
+            bring(r, set(need), pos)
+        writes_out = mode == "device" and ref == dag.result and pos == n - 1
+        if not writes_out:
+            make_room(_units(dag, ref), set(need), pos)
+            resident[ref] = _units(dag, ref)
+        high = max(high, live())
+        events.append(("run", ref))
+        for r in need:
+            rc[r] -= 1
+            if rc[r] == 0:
+                resident.pop(r, None)
+                host_copy.discard(r)
+
+    res = dag.result
+    if mode == "host":
+        if res in resident:
+            events.append(("sink_d2h", res))
+            d2h += 1
+            d2hu += _units(dag, res)
+        elif res in host_copy:
+            events.append(("sink_host", res))
+        else:                                               # bare input result
+            bring(res, {res}, n)
+            high = max(high, live())
+            events.append(("sink_d2h", res))
+            d2h += 1
+            d2hu += _units(dag, res)
+    else:
+        if _is_filter(dag, res) and res not in resident and not (order and f"f{order[-1]}" == res):
+            events.append(("sink_h2d", res))
+            h2d += 1
+            h2du += _units(dag, res)
+    return Hybrid(events, Counts(h2d, d2h, len(order)), high, h2du, d2hu)
