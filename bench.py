@@ -474,9 +474,27 @@ def strategy_sweep(dfg, synth, torch):
             p.close()
         except dfg.DfgError as e:
             caps[f"{cap_gib}GiB"] = {"runs": False, "error": e.name}
+    # hybrid (NEXT #3 spill-to-host): the caps staged cannot meet, intermediates
+    # spill to pinned host memory (device-resident inputs and output)
+    hyb = {}
+    for cap_gib in (8, 6, 4):
+        try:
+            p = dfg.Plan(mesh, q, "hybrid", cap_gib * GiB)
+            ms, _ = _time_plan(p, o, torch, 2)
+            st = p.stats()
+            ex = max(1, st["executes"])
+            hyb[f"{cap_gib}GiB"] = {"runs": True, "ms": ms, "highwater_gib": st["dev_highwater_bytes"] / GiB,
+                                    "spills_per_execute": st["d2h_count"] // ex,
+                                    "reloads_per_execute": st["h2d_count"] // ex,
+                                    "pcie_gib_per_execute": (st["h2d_bytes"] + st["d2h_bytes"]) / ex / GiB,
+                                    "bit_identical_to_fused": bool(torch.equal(o, ref))}
+            p.close()
+        except dfg.DfgError as e:
+            hyb[f"{cap_gib}GiB"] = {"runs": False, "error": e.name}
     del flds, ref, o
     torch.cuda.empty_cache()
     c3["staged_caps"] = caps
+    c3["hybrid_caps"] = hyb
     out["config3_512_qcrit"] = c3
     return out
 

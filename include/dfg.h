@@ -49,11 +49,25 @@ typedef enum {
                         input per chunk (env DFG_STREAM_PLANES overrides); each field
                         plane crosses PCIe once (chunk halos are copied on the device).
                         Pinned host buffers are needed for the copies to overlap. */
-  DFG_REFERENCE = 4  /* the hand-written reference kernel of a quantity (L243): expr is
+  DFG_REFERENCE = 4, /* the hand-written reference kernel of a quantity (L243): expr is
                         "velmag", "vortmag" or "qcrit" (fields u, v, w must be bound);
                         same I/O and TMA pipeline as fusion, fewer flops (derivative =
                         numerator x reciprocal spacing, FMA, Q = -1/2 tr(J^2)); agrees
                         with the network within floating-point tolerance, not bitwise */
+  DFG_HYBRID = 5     /* staged execution (the same kernels and results) that fits a
+                        dev_mem_cap below the staged footprint by spilling
+                        intermediates to pinned host memory (SURVEY 8f NEXT #3,
+                        the Fig. 2 argument L107-L114): list
+                        order if it fits the cap, else the memory-aware order, and
+                        if that does not fit either, before each array that does
+                        not fit the resident array with the furthest next use is
+                        evicted (an intermediate is copied to the host once, an
+                        uploaded input is dropped) and brought back when needed.
+                        All inputs and the output either in host memory (the
+                        paper's host interface) or all on the device; whole mesh
+                        only.  DFG_E_NOMEM at compile if the cap is below some
+                        filter's working set (its operands plus its result, plus
+                        the resident inputs and output in device mode). */
 } dfg_strategy;
 
 typedef enum { DFG_F32 = 0, DFG_F64 = 1 } dfg_dtype;
@@ -231,6 +245,17 @@ int dfg_plan_info(dfg_plan plan, int64_t out[9]);
  * *n = number of filters. */
 int dfg_plan_schedule(dfg_plan plan, int32_t* order, size_t cap, size_t* n);
 
+/* Transfer schedule of a DFG_HYBRID plan for the binding mode of its last
+ * execute (or, before the first, of the bindings at compile): n events, each
+ * two int32 (kind, ref), kinds: 0 upload input, 1 reload intermediate from
+ * its host copy, 2 spill intermediate to the host, 3 discard a device copy
+ * whose host copy is valid, 4 drop an uploaded input, 5 run filter, 6 sink
+ * device -> host, 7 sink from the host copy (no transfer), 8 sink host copy
+ * -> device output.  ref = filter id, or -1 - (input index) for a bound
+ * input.  Writes min(cap, n) events (2 int32 each); *n = number of events.
+ * DFG_E_INVALID for other strategies. */
+int dfg_plan_transfers(dfg_plan plan, int32_t* events, size_t cap, size_t* n);
+
 /* Canonical network text (R10) -- stands in for the paper's
  * optional Python script of network-definition API calls (L84).
  * Copies up to cap bytes incl. the NUL; *needed = full size incl. NUL;
@@ -265,6 +290,17 @@ int dfg_dag_dump(const char* expr, const char* const* inputs, int n_inputs,
  * 0: everything device resident. */
 int dfg_model(const char* expr, const char* const* inputs, int n_inputs,
               dfg_strategy strategy, int host_mode, int64_t out[4]);
+
+/* The DFG_HYBRID planner on its own: schedule of
+ * `expr` in host (host_mode = 1) or device mode under cap_units problem
+ * arrays, filters in `order` (n_order ids, a topological order; NULL = list
+ * order).  Events as dfg_plan_transfers (min(cap, n) written, *n = count);
+ * out[0..4] = high-water units, h2d transfers, d2h transfers, h2d units,
+ * d2h units.  DFG_E_NOMEM if the cap is below a filter's working set,
+ * DFG_E_INVALID if `order` is not a topological order. */
+int dfg_hybrid_model(const char* expr, const char* const* inputs, int n_inputs,
+                     int host_mode, int64_t cap_units, const int32_t* order, size_t n_order,
+                     int32_t* events, size_t cap, size_t* n, int64_t out[5]);
 
 /* Generate the fused kernel source for `expr` on an nx x ny x nz mesh and,
  * if compile != 0, NVRTC-compile it for sm_100a (no device needed); on

@@ -111,6 +111,10 @@ class Plan:
         from ._dfg import dfg_plan_schedule
         return dfg_plan_schedule(self.handle)
 
+    def transfers(self):
+        from ._dfg import dfg_plan_transfers
+        return dfg_plan_transfers(self.handle)
+
     def kernel_source(self):
         return dfg_dump_kernel(self.handle)
 

@@ -22,10 +22,11 @@ if not os.path.exists(LIB_PATH):
 
 _lib = C.CDLL(LIB_PATH, mode=C.RTLD_GLOBAL)
 
-DFG_ROUNDTRIP, DFG_STAGED, DFG_FUSED, DFG_STREAMED, DFG_REFERENCE = 0, 1, 2, 3, 4
+DFG_ROUNDTRIP, DFG_STAGED, DFG_FUSED, DFG_STREAMED, DFG_REFERENCE, DFG_HYBRID = 0, 1, 2, 3, 4, 5
 DFG_F32, DFG_F64 = 0, 1
 STRATEGIES = {"roundtrip": DFG_ROUNDTRIP, "staged": DFG_STAGED, "fused": DFG_FUSED, "streamed": DFG_STREAMED,
-              "reference": DFG_REFERENCE}
+              "reference": DFG_REFERENCE, "hybrid": DFG_HYBRID}
+TRANSFER_KINDS = ("upload", "reload", "spill", "discard", "drop", "run", "sink_d2h", "sink_host", "sink_h2d")
 STATUS = {0: "DFG_OK", -1: "DFG_E_INVALID", -2: "DFG_E_PARSE", -3: "DFG_E_UNDEFINED", -4: "DFG_E_TYPE",
           -5: "DFG_E_NOMEM", -6: "DFG_E_NVRTC", -7: "DFG_E_CUDA", -8: "DFG_E_NCCL", -9: "DFG_E_UNBOUND",
           -10: "DFG_E_UNSUPPORTED", -11: "DFG_E_RANGE"}
@@ -71,6 +72,10 @@ _SIGS = {
     "dfg_reset_stats": (C.c_int, [_P]),
     "dfg_plan_info": (C.c_int, [_P, C.POINTER(_I64)]),
     "dfg_plan_schedule": (C.c_int, [_P, C.POINTER(C.c_int32), C.c_size_t, C.POINTER(C.c_size_t)]),
+    "dfg_plan_transfers": (C.c_int, [_P, C.POINTER(C.c_int32), C.c_size_t, C.POINTER(C.c_size_t)]),
+    "dfg_hybrid_model": (C.c_int, [C.c_char_p, C.POINTER(C.c_char_p), C.c_int, C.c_int, C.c_int64,
+                                   C.POINTER(C.c_int32), C.c_size_t, C.POINTER(C.c_int32), C.c_size_t,
+                                   C.POINTER(C.c_size_t), C.POINTER(_I64)]),
     "dfg_dump_dag": (C.c_int, [_P, C.c_char_p, C.c_size_t, C.POINTER(C.c_size_t)]),
     "dfg_dump_kernel": (C.c_int, [_P, C.c_char_p, C.c_size_t, C.POINTER(C.c_size_t)]),
     "dfg_dag_dump": (C.c_int, [C.c_char_p, C.POINTER(C.c_char_p), C.c_int, C.c_int, C.c_char_p, C.c_size_t,
@@ -211,6 +216,34 @@ def dfg_plan_info(plan) -> dict:
     keys = ("strategy", "width", "filters", "variant", "regs", "spill", "footprint_device", "footprint_host",
             "div2_axes")
     return dict(zip(keys, list(out)))
+
+
+def dfg_plan_transfers(plan) -> list:
+    """DFG_HYBRID transfer schedule: [(kind name, ref)], ref = filter id or
+    -1 - input index."""
+    n = C.c_size_t(0)
+    _check(_lib.dfg_plan_transfers(plan, None, 0, C.byref(n)))
+    arr = (C.c_int32 * max(2 * n.value, 1))()
+    _check(_lib.dfg_plan_transfers(plan, arr, n.value, C.byref(n)))
+    return [(TRANSFER_KINDS[arr[2 * i]], int(arr[2 * i + 1])) for i in range(n.value)]
+
+
+def dfg_hybrid_model(expr, inputs, host_mode, cap_units, order=None):
+    """(events, high, h2d, d2h, h2d_units, d2h_units) of the hybrid planner."""
+    arr, n_in = _names(inputs)
+    ordp, n_ord = None, 0
+    if order is not None:
+        ordp = (C.c_int32 * max(len(order), 1))(*order)
+        n_ord = len(order)
+    n = C.c_size_t(0)
+    out = (_I64 * 5)()
+    _check(_lib.dfg_hybrid_model(expr.encode(), arr, n_in, int(host_mode), cap_units, ordp, n_ord, None, 0,
+                                 C.byref(n), out))
+    ev = (C.c_int32 * max(2 * n.value, 1))()
+    _check(_lib.dfg_hybrid_model(expr.encode(), arr, n_in, int(host_mode), cap_units, ordp, n_ord, ev, n.value,
+                                 C.byref(n), out))
+    events = [(TRANSFER_KINDS[ev[2 * i]], int(ev[2 * i + 1])) for i in range(n.value)]
+    return (events,) + tuple(int(v) for v in out)
 
 
 def dfg_plan_schedule(plan) -> list:

@@ -246,6 +246,20 @@ int dfg_plan_schedule(dfg_plan plan, int32_t* order, size_t cap, size_t* n) {
   });
 }
 
+int dfg_plan_transfers(dfg_plan plan, int32_t* events, size_t cap, size_t* n) {
+  return guard([&] {
+    if (!plan || !n) dfg::fail(DFG_E_INVALID, "null argument");
+    const auto& p = *plan->p;
+    if (p.strategy != DFG_HYBRID) dfg::fail(DFG_E_INVALID, "not a hybrid plan");
+    const auto& ev = p.hyb.ev;
+    *n = ev.size();
+    for (size_t i = 0; i < ev.size() && i < cap && events; ++i) {
+      events[2 * i] = int32_t(ev[i].kind);
+      events[2 * i + 1] = ev[i].ref.kind == dfg::Ref::Input ? -1 - ev[i].ref.id : ev[i].ref.id;
+    }
+  });
+}
+
 int dfg_dump_dag(dfg_plan plan, char* buf, size_t cap, size_t* needed) {
   return guard([&] {
     if (!plan) dfg::fail(DFG_E_INVALID, "null plan");
@@ -311,7 +325,7 @@ int dfg_model(const char* expr, const char* const* inputs, int n_inputs, dfg_str
               int64_t out[4]) {
   return guard([&] {
     if (!expr || !out) dfg::fail(DFG_E_INVALID, "null argument");
-    if (strategy < DFG_ROUNDTRIP || strategy > DFG_REFERENCE) dfg::fail(DFG_E_INVALID, "bad strategy");
+    if (strategy < DFG_ROUNDTRIP || strategy > DFG_HYBRID) dfg::fail(DFG_E_INVALID, "bad strategy");
     int ref = 0;
     const char* prog = strategy == DFG_REFERENCE ? dfg::reference_program(expr, &ref) : expr;
     if (!prog) dfg::fail(DFG_E_INVALID, "reference kernels exist for velmag, vortmag and qcrit");
@@ -321,6 +335,41 @@ int dfg_model(const char* expr, const char* const* inputs, int n_inputs, dfg_str
     out[1] = m.d2h;
     out[2] = m.kernels;
     out[3] = m.units;
+  });
+}
+
+int dfg_hybrid_model(const char* expr, const char* const* inputs, int n_inputs, int host_mode, int64_t cap_units,
+                     const int32_t* order, size_t n_order, int32_t* events, size_t cap, size_t* n, int64_t out[5]) {
+  return guard([&] {
+    if (!expr || !n || !out) dfg::fail(DFG_E_INVALID, "null argument");
+    dfg::Dag d = dfg::build_dag(expr, names_of(inputs, n_inputs), dfg::DType::F32);
+    const size_t nf = d.filters.size();
+    std::vector<int> o(nf);
+    for (size_t k = 0; k < nf; ++k) o[k] = int(k);
+    if (order) {
+      if (n_order != nf) dfg::fail(DFG_E_INVALID, "order must list every filter once");
+      std::vector<int> pos(nf, -1);
+      for (size_t i = 0; i < nf; ++i) {
+        const int k = order[i];
+        if (k < 0 || size_t(k) >= nf || pos[size_t(k)] >= 0) dfg::fail(DFG_E_INVALID, "order must list every filter once");
+        pos[size_t(k)] = int(i);
+        o[i] = k;
+      }
+      for (size_t k = 0; k < nf; ++k)
+        for (auto& r : d.filters[k].in)
+          if (r.kind == dfg::Ref::Filter && pos[size_t(r.id)] > pos[k]) dfg::fail(DFG_E_INVALID, "order is not topological");
+    }
+    dfg::HybridPlan hp = dfg::plan_hybrid(d, o, cap_units, host_mode != 0);
+    *n = hp.ev.size();
+    for (size_t i = 0; i < hp.ev.size() && i < cap && events; ++i) {
+      events[2 * i] = int32_t(hp.ev[i].kind);
+      events[2 * i + 1] = hp.ev[i].ref.kind == dfg::Ref::Input ? -1 - hp.ev[i].ref.id : hp.ev[i].ref.id;
+    }
+    out[0] = hp.high;
+    out[1] = hp.h2d;
+    out[2] = hp.d2h;
+    out[3] = hp.h2d_units;
+    out[4] = hp.d2h_units;
   });
 }
 

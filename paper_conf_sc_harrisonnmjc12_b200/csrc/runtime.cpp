@@ -324,8 +324,9 @@ bool host_side(Op op) { return op == Op::Decompose || op == Op::Const; }  // rou
 Model model(const Dag& dag, dfg_strategy s, bool host) {
   // the streamed strategy is fusion per z-chunk: its network-level numbers
   // are fusion's (per-chunk transfers and the ring footprint are physical);
-  // a reference kernel has fusion's I/O
+  // a reference kernel has fusion's I/O; without a cap hybrid is staged
   if (s == DFG_STREAMED || s == DFG_REFERENCE) s = DFG_FUSED;
+  if (s == DFG_HYBRID) s = DFG_STAGED;
   Model m;
   Sources src = sources(dag);
   const int64_t F = int64_t(dag.filters.size());
@@ -458,6 +459,140 @@ std::vector<int> greedy_staged_order(const Dag& dag) {
   return order;
 }
 
+// Staged execution holding at most cap units on the device:
+// before each array that does not fit, evict the resident array read
+// furthest in the future (ties: larger, filter before input, higher id),
+// never an operand of the running filter; an intermediate is copied to the
+// host the first time it is evicted, an uploaded input is dropped.
+HybridPlan plan_hybrid(const Dag& dag, const std::vector<int>& order, int64_t cap, bool host) {
+  using Key = std::pair<int, int>;  // (kind, id): Ref::Filter = 0, Ref::Input = 1
+  auto key = [](const Ref& r) { return Key(int(r.kind), r.id); };
+  auto ref_of = [](const Key& k) { return Ref{Ref::Kind(k.first), k.second}; };
+  HybridPlan hp;
+  const int n = int(order.size());
+  Sources src = sources(dag);
+  std::map<Key, std::vector<int>> uses;  // positions reading each value; the sink reads the result at n
+  std::map<Key, int64_t> rc;
+  for (int p = 0; p < n; ++p)
+    for (auto& r : dag.filters[size_t(order[p])].in)
+      if (r.kind != Ref::Mesh) {
+        uses[key(r)].push_back(p);
+        rc[key(r)] += 1;
+      }
+  uses[key(dag.result)].push_back(n);
+  rc[key(dag.result)] += 1;
+  auto next_use = [&](const Key& k, int pos) {
+    for (int p : uses[k])
+      if (p >= pos) return p;
+    return n + 1;
+  };
+  std::map<Key, int64_t> resident;  // evictable device arrays -> units
+  std::set<Key> host_copy;
+  const int64_t base = host ? 0 : int64_t(src.inputs.size()) + units(dag, dag.result);
+  auto live = [&] {
+    int64_t l = base;
+    for (auto& kv : resident) l += kv.second;
+    return l;
+  };
+  auto note = [&](HybridEvent::Kind k, const Key& v) { hp.ev.push_back(HybridEvent{k, ref_of(v)}); };
+  auto make_room = [&](int64_t u, const std::set<Key>& protect, int pos) {
+    while (live() + u > cap) {
+      const Key* victim = nullptr;
+      std::tuple<int, int64_t, int, int> best{};
+      for (auto& kv : resident) {
+        if (protect.count(kv.first)) continue;
+        std::tuple<int, int64_t, int, int> t{next_use(kv.first, pos), kv.second,
+                                             kv.first.first == int(Ref::Filter) ? 1 : 0, kv.first.second};
+        if (!victim || t > best) {
+          victim = &kv.first;
+          best = t;
+        }
+      }
+      if (!victim)
+        fail(DFG_E_NOMEM, "dev_mem_cap of " + std::to_string(cap) + " problem arrays is below the working set of " +
+                              "the filter at position " + std::to_string(pos));
+      const Key v = *victim;
+      if (v.first == int(Ref::Filter)) {
+        if (!host_copy.count(v)) {
+          note(HybridEvent::Spill, v);
+          host_copy.insert(v);
+          hp.d2h += 1;
+          hp.d2h_units += resident[v];
+        } else {
+          note(HybridEvent::Discard, v);
+        }
+      } else {
+        note(HybridEvent::Drop, v);
+      }
+      resident.erase(v);
+    }
+  };
+  auto bring = [&](const Ref& r, const std::set<Key>& protect, int pos) {
+    const Key k = key(r);
+    if (resident.count(k) || (!host && r.kind == Ref::Input)) return;
+    const int64_t u = units(dag, r);
+    make_room(u, protect, pos);
+    note(r.kind == Ref::Filter ? HybridEvent::Reload : HybridEvent::Upload, k);
+    hp.h2d += 1;
+    hp.h2d_units += u;
+    resident[k] = u;
+  };
+  int64_t high = base;
+  bool mesh_up = false;
+  for (int pos = 0; pos < n; ++pos) {
+    const int k = order[size_t(pos)];
+    const Filter& f = dag.filters[size_t(k)];
+    std::vector<Ref> need;
+    std::set<Key> protect;
+    for (auto& r : f.in) {
+      if (r.kind == Ref::Mesh) {
+        if (host && !mesh_up) mesh_up = true, hp.h2d += 4;  // dims, x, y, z (R13)
+        continue;
+      }
+      if (protect.insert(key(r)).second) need.push_back(r);
+    }
+    for (auto& r : need) bring(r, protect, pos);
+    const Ref out{Ref::Filter, k};
+    const bool writes_out = !host && dag.result == out && pos == n - 1;
+    if (!writes_out) {
+      make_room(units(dag, out), protect, pos);
+      resident[key(out)] = units(dag, out);
+    }
+    high = std::max(high, live());
+    note(HybridEvent::Run, key(out));
+    for (auto& r : f.in) {
+      if (r.kind == Ref::Mesh) continue;
+      if (--rc[key(r)] == 0) {
+        resident.erase(key(r));
+        host_copy.erase(key(r));
+      }
+    }
+  }
+  const Ref& res = dag.result;
+  const Key rk = key(res);
+  if (host) {
+    if (resident.count(rk)) {
+      note(HybridEvent::SinkD2H, rk);
+    } else if (host_copy.count(rk)) {
+      note(HybridEvent::SinkHost, rk);
+    } else {  // a bare input result
+      bring(res, {rk}, n);
+      high = std::max(high, live());
+      note(HybridEvent::SinkD2H, rk);
+    }
+    if (hp.ev.back().kind == HybridEvent::SinkD2H) {
+      hp.d2h += 1;
+      hp.d2h_units += units(dag, res);
+    }
+  } else if (res.kind == Ref::Filter && !resident.count(rk) && !(n > 0 && order[size_t(n - 1)] == res.id)) {
+    note(HybridEvent::SinkH2D, rk);
+    hp.h2d += 1;
+    hp.h2d_units += units(dag, res);
+  }
+  hp.high = high;
+  return hp;
+}
+
 int64_t predicted_device_bytes(const Dag& dag, dfg_strategy s, int64_t cells, size_t ts) {
   // Algorithmic device-memory bytes of one execute:
   // fused reads every input once and writes the result once; staged and
@@ -585,7 +720,8 @@ PlanImpl::~PlanImpl() {
 
 std::unique_ptr<PlanImpl> compile_plan(std::shared_ptr<MeshImpl> mesh, const std::string& expr, dfg_strategy s,
                                        size_t cap) {
-  if (s != DFG_ROUNDTRIP && s != DFG_STAGED && s != DFG_FUSED && s != DFG_STREAMED && s != DFG_REFERENCE)
+  if (s != DFG_ROUNDTRIP && s != DFG_STAGED && s != DFG_FUSED && s != DFG_STREAMED && s != DFG_REFERENCE &&
+      s != DFG_HYBRID)
     fail(DFG_E_INVALID, "bad strategy");
   std::vector<std::string> names;
   for (auto& kv : mesh->fields) names.push_back(kv.first);
@@ -604,7 +740,7 @@ std::unique_ptr<PlanImpl> compile_plan(std::shared_ptr<MeshImpl> mesh, const std
   const Dag& dag = plan->dag;
   const bool multi = mesh->nzl != mesh->NZ || mesh->nx != mesh->NX || mesh->ny != mesh->NY || mesh->gxy;
   if (multi && s != DFG_FUSED && s != DFG_REFERENCE)
-    fail(DFG_E_UNSUPPORTED, "staged/roundtrip/streamed run on a whole mesh; slabs and blocks use fusion");
+    fail(DFG_E_UNSUPPORTED, "staged/hybrid/roundtrip/streamed run on a whole mesh; slabs and blocks use fusion");
 
   // Footprint check against the cap for the binding modes at compile time
   // (the streamed ring is bounded by construction; its ledger checks at run time)
@@ -616,21 +752,23 @@ std::unique_ptr<PlanImpl> compile_plan(std::shared_ptr<MeshImpl> mesh, const std
   size_t need = size_t(mdl.units) * unit_bytes;
   plan->order.resize(dag.filters.size());
   for (size_t k = 0; k < plan->order.size(); ++k) plan->order[k] = int(k);
-  if (s == DFG_STAGED) {
+  if (s == DFG_STAGED || s == DFG_HYBRID) {
     // the paper's list order, unless a cap rejects it and the memory-aware
-    // order fits (or DFG_STAGED_ORDER=greedy asks for it)
+    // order fits (or DFG_STAGED_ORDER=greedy asks for it); hybrid plans take
+    // the memory-aware order whenever the list order does not fit
     const char* env = std::getenv("DFG_STAGED_ORDER");
     const bool force = env && !std::strcmp(env, "greedy");
     if (force || (cap && need > cap)) {
       std::vector<int> g = greedy_staged_order(dag);
       size_t gneed = size_t(staged_units(dag, g, any_host)) * unit_bytes;
-      if (force || gneed <= cap) {
+      if (force || gneed <= cap || s == DFG_HYBRID) {
         plan->order = g;
         need = gneed;
       }
     }
   }
-  if (cap && need > cap && s != DFG_STREAMED)
+  if (s == DFG_HYBRID) plan->plan_hybrid_for(any_host);  // DFG_E_NOMEM below a filter's working set
+  if (cap && need > cap && s != DFG_STREAMED && s != DFG_HYBRID)
     fail(DFG_E_NOMEM, "predicted device footprint " + std::to_string(need) + " bytes exceeds the cap " +
                           std::to_string(cap));
 
@@ -774,6 +912,7 @@ void PlanImpl::execute(void* out, bool out_dev, cudaStream_t s) {
     case DFG_STREAMED: exec_streamed(out, out_dev, s); break;
     case DFG_REFERENCE: exec_fused(out, out_dev, s); break;
     case DFG_STAGED: exec_staged(out, out_dev, s); break;
+    case DFG_HYBRID: exec_hybrid(out, out_dev, s); break;
     case DFG_ROUNDTRIP: exec_roundtrip(out, out_dev, s); break;
   }
   DFG_CUDA(cudaEventRecord(ev1, s));
@@ -783,10 +922,14 @@ void PlanImpl::execute(void* out, bool out_dev, cudaStream_t s) {
   bool any_host = !out_dev;
   for (int i : sources(dag).inputs)
     if (!m.fields[dag.inputs[i]].on_device) any_host = true;
-  const int64_t units = strategy == DFG_STAGED ? staged_units(dag, order, any_host) : model(dag, strategy, any_host).units;
-  st.predicted_highwater_bytes = units * m.cells() * int64_t(dsize(m.dt));
+  const int64_t unit_b = m.cells() * int64_t(dsize(m.dt));
+  const int64_t units = strategy == DFG_HYBRID   ? hyb.high
+                        : strategy == DFG_STAGED ? staged_units(dag, order, any_host)
+                                                 : model(dag, strategy, any_host).units;
+  st.predicted_highwater_bytes = units * unit_b;
   st.predicted_hbm_bytes = predicted_device_bytes(dag, strategy, m.cells(), dsize(m.dt));
-  st.predicted_pcie_bytes = predicted_pcie_bytes(dag, strategy, m.cells(), dsize(m.dt), any_host);
+  st.predicted_pcie_bytes = strategy == DFG_HYBRID ? (hyb.h2d_units + hyb.d2h_units) * unit_b
+                                                   : predicted_pcie_bytes(dag, strategy, m.cells(), dsize(m.dt), any_host);
 }
 
 namespace {
@@ -1162,6 +1305,213 @@ void PlanImpl::release_stream_buffers() {
 }
 
 // ------------------------------------------------------------- staged
+namespace {
+// One primitive kernel over the owned cells of a whole mesh: o = f(args)
+// (args: operand values, mesh references skipped); grad3d reads `gsrc`, its
+// field's buffer from local plane 0, which has `gghost` ghost planes.
+void launch_primitive(const MeshImpl& m, const Filter& f, void* o, const std::vector<const void*>& a,
+                      const void* gsrc, int64_t gghost, const void* const tab[3], cudaStream_t s) {
+  const int64_t N = m.cells();
+  switch (f.op) {
+    case Op::Const: kern::fill(m.dt, f.cval, o, N, s); break;
+    case Op::Add: case Op::Sub: case Op::Mult: case Op::Div:
+    case Op::Gt: case Op::Lt: case Op::Ge: case Op::Le: case Op::Eq: case Op::Ne:
+      kern::binary(f.op, m.dt, a[0], a[1], o, N, s);
+      break;
+    case Op::Neg: case Op::Sqrt: kern::unary(f.op, m.dt, a[0], o, N, s); break;
+    case Op::Select: kern::select(m.dt, a[0], a[1], a[2], o, N, s); break;
+    case Op::Decompose: kern::decompose(m.dt, a[0], f.k, o, N, s); break;
+    case Op::Compose: kern::compose(m.dt, a.data(), int(a.size()), o, N, s); break;
+    case Op::Grad3d:
+      kern::grad3d(m.dt, gsrc, o, tab[0], tab[1], tab[2], m.nx, m.ny, m.nzl, m.NZ, m.k0, gghost, s);
+      break;
+  }
+}
+}  // namespace
+
+void PlanImpl::plan_hybrid_for(bool host) {
+  const int64_t unit_b = mesh->cells() * int64_t(dsize(mesh->dt));
+  const int64_t cap_units = cap ? int64_t(cap) / unit_b : (int64_t(1) << 40);
+  hyb = plan_hybrid(dag, order, cap_units, host);
+  hyb_host = host ? 1 : 0;
+}
+
+// ------------------------------------------------------------- hybrid
+// Replays the compile-time transfer schedule (plan_hybrid): the same
+// primitive kernels as staged, plus spills of intermediates to pinned host
+// buffers and their reloads.  One stream orders everything; host copies live
+// until the end of the execute.
+void PlanImpl::exec_hybrid(void* out, bool out_dev, cudaStream_t s) {
+  MeshImpl& m = *mesh;
+  const size_t ts = dsize(m.dt);
+  const size_t sb = size_t(m.cells()) * ts;
+  Sources src = sources(dag);
+  bool all_host = !out_dev, all_dev = out_dev;
+  for (int i : src.inputs) {
+    const bool d = m.fields[dag.inputs[i]].on_device;
+    all_host = all_host && !d;
+    all_dev = all_dev && d;
+  }
+  if (!all_host && !all_dev)
+    fail(DFG_E_UNSUPPORTED, "hybrid: inputs and output must all be in host memory or all on the device");
+  const bool host = all_host;
+  if (hyb_host != (host ? 1 : 0)) plan_hybrid_for(host);
+
+  Ledger led(cap);
+  std::lock_guard<std::mutex> lk(g_host_mu);
+  HostPool& hp = host_pool();
+  using Key = std::pair<int, int>;
+  auto key = [](const Ref& r) { return Key(int(r.kind), r.id); };
+  auto bytes_of = [&](const Ref& r) { return sb * size_t(units(dag, r)); };
+  std::map<Key, void*> dev, hcopy;
+  std::vector<void*> host_bufs;
+  struct Cleanup {
+    std::map<Key, void*>& dev;
+    cudaStream_t s;
+    ~Cleanup() {
+      for (auto& kv : dev) cudaFreeAsync(kv.second, s);
+    }
+  } cleanup{dev, s};
+  if (!host) {
+    for (size_t i = 0; i < src.inputs.size(); ++i) led.add(m.field_bytes());
+    led.add(bytes_of(dag.result));  // the caller's output buffer
+  }
+  std::map<Key, int64_t> rc;
+  for (auto& f : dag.filters)
+    for (auto& r : f.in)
+      if (r.kind != Ref::Mesh) rc[key(r)] += 1;
+  rc[key(dag.result)] += 1;
+
+  const void* tab[3] = {m.dev_tab[0], m.dev_tab[1], m.dev_tab[2]};
+  std::vector<void*> mesh_bufs;
+  auto ensure_mesh = [&] {
+    if (!host || !mesh_bufs.empty()) return;
+    int64_t dims[4] = {m.nx, m.ny, m.NZ, m.k0};
+    void* dd = dev_alloc(sizeof(dims), m.device, s);
+    mesh_bufs.push_back(dd);
+    DFG_CUDA(cudaMemcpyAsync(dd, dims, sizeof(dims), cudaMemcpyHostToDevice, s));
+    st.h2d_count += 1;
+    st.h2d_bytes += sizeof(dims);
+    for (int a = 0; a < 3; ++a) {
+      void* d = dev_alloc(m.host_tab[a].size(), m.device, s);
+      mesh_bufs.push_back(d);
+      DFG_CUDA(cudaMemcpyAsync(d, m.host_tab[a].data(), m.host_tab[a].size(), cudaMemcpyHostToDevice, s));
+      st.h2d_count += 1;
+      st.h2d_bytes += int64_t(m.host_tab[a].size());
+      tab[a] = d;
+    }
+  };
+  // buffer of a value (inputs: from local plane 0, ghost planes included)
+  auto base_of = [&](const Ref& r) -> void* {
+    if (!host && r.kind == Ref::Input) return m.fields[dag.inputs[r.id]].ptr;
+    auto it = dev.find(key(r));
+    if (it == dev.end()) fail(DFG_E_CUDA, "hybrid schedule: operand not resident");
+    return it->second;
+  };
+  const int64_t goff = int64_t(m.ghost) * m.plane() * int64_t(ts);
+  auto val = [&](const Ref& r) -> void* {
+    return static_cast<char*>(base_of(r)) + (r.kind == Ref::Input ? goff : 0);
+  };
+  auto drop_dev = [&](const Key& k, size_t b) {
+    cudaFreeAsync(dev[k], s);
+    dev.erase(k);
+    led.sub(b);
+  };
+  const Ref res = dag.result;
+  const size_t nf = order.size();
+  size_t pos = 0;
+  for (const HybridEvent& e : hyb.ev) {
+    const Key k = key(e.ref);
+    const size_t b = e.ref.kind == Ref::Input ? m.field_bytes() : bytes_of(e.ref);
+    switch (e.kind) {
+      case HybridEvent::Upload: {
+        led.add(b);
+        void* d = dev_alloc(b, m.device, s);
+        dev[k] = d;
+        DFG_CUDA(cudaMemcpyAsync(d, m.fields[dag.inputs[e.ref.id]].ptr, b, cudaMemcpyHostToDevice, s));
+        st.h2d_count += 1;
+        st.h2d_bytes += int64_t(b);
+        break;
+      }
+      case HybridEvent::Reload: {
+        led.add(b);
+        void* d = dev_alloc(b, m.device, s);
+        dev[k] = d;
+        DFG_CUDA(cudaMemcpyAsync(d, hcopy.at(k), b, cudaMemcpyHostToDevice, s));
+        st.h2d_count += 1;
+        st.h2d_bytes += int64_t(b);
+        break;
+      }
+      case HybridEvent::Spill: {
+        void* h = hp.get(b);
+        host_bufs.push_back(h);
+        hcopy[k] = h;
+        DFG_CUDA(cudaMemcpyAsync(h, dev.at(k), b, cudaMemcpyDeviceToHost, s));
+        st.d2h_count += 1;
+        st.d2h_bytes += int64_t(b);
+        drop_dev(k, b);
+        break;
+      }
+      case HybridEvent::Discard: case HybridEvent::Drop: drop_dev(k, b); break;
+      case HybridEvent::Run: {
+        const Filter& f = dag.filters[size_t(e.ref.id)];
+        std::vector<const void*> args;
+        for (auto& r : f.in) {
+          if (r.kind == Ref::Mesh) ensure_mesh();
+          else args.push_back(val(r));
+        }
+        const bool writes_out = !host && res == e.ref && pos + 1 == nf;
+        void* o = out;
+        if (!writes_out) {
+          led.add(b);
+          o = dev_alloc(b, m.device, s);
+          dev[k] = o;
+        }
+        const void* gsrc = nullptr;
+        int64_t gghost = 0;
+        if (f.op == Op::Grad3d) {
+          gsrc = base_of(f.in[0]);
+          gghost = f.in[0].kind == Ref::Input ? m.ghost : 0;
+        }
+        launch_primitive(m, f, o, args, gsrc, gghost, tab, s);
+        DFG_CUDA(cudaGetLastError());
+        st.kernel_count += 1;
+        ++pos;
+        for (auto& r : f.in) {
+          if (r.kind == Ref::Mesh || --rc[key(r)] > 0) continue;
+          if (dev.count(key(r))) drop_dev(key(r), r.kind == Ref::Input ? m.field_bytes() : bytes_of(r));
+          hcopy.erase(key(r));
+        }
+        break;
+      }
+      case HybridEvent::SinkD2H:
+        DFG_CUDA(cudaMemcpyAsync(out, val(res), bytes_of(res), cudaMemcpyDeviceToHost, s));
+        st.d2h_count += 1;
+        st.d2h_bytes += int64_t(bytes_of(res));
+        break;
+      case HybridEvent::SinkHost:
+        DFG_CUDA(cudaMemcpyAsync(out, hcopy.at(k), bytes_of(res), cudaMemcpyHostToHost, s));
+        break;
+      case HybridEvent::SinkH2D:
+        DFG_CUDA(cudaMemcpyAsync(out, hcopy.at(k), bytes_of(res), cudaMemcpyHostToDevice, s));
+        st.h2d_count += 1;
+        st.h2d_bytes += int64_t(bytes_of(res));
+        break;
+    }
+  }
+  // device mode: a result still resident (not computed into the output) or a bare input
+  if (!host) {
+    auto it = dev.find(key(res));
+    const void* rp = it != dev.end() ? it->second : nullptr;
+    if (res.kind == Ref::Input) rp = val(res);
+    if (rp && rp != out) DFG_CUDA(cudaMemcpyAsync(out, rp, bytes_of(res), cudaMemcpyDeviceToDevice, s));
+  }
+  for (void* p : mesh_bufs) cudaFreeAsync(p, s);
+  if (!host_bufs.empty() || host) DFG_CUDA(cudaStreamSynchronize(s));  // host copies / output complete
+  for (void* h : host_bufs) hp.put(h);
+  st.dev_highwater_bytes = std::max<int64_t>(st.dev_highwater_bytes, int64_t(led.high));
+}
+
 void PlanImpl::exec_staged(void* out, bool out_dev, cudaStream_t s) {
   MeshImpl& m = *mesh;
   const size_t ts = dsize(m.dt);
@@ -1279,30 +1629,17 @@ void PlanImpl::exec_staged(void* out, bool out_dev, cudaStream_t s) {
       o = dev_alloc(ob, m.device, s);
     }
     fval[k] = o;
-    switch (f.op) {
-      case Op::Const: kern::fill(m.dt, f.cval, o, N, s); break;
-      case Op::Add: case Op::Sub: case Op::Mult: case Op::Div:
-      case Op::Gt: case Op::Lt: case Op::Ge: case Op::Le: case Op::Eq: case Op::Ne:
-        kern::binary(f.op, m.dt, val(f.in[0]), val(f.in[1]), o, N, s);
-        break;
-      case Op::Neg: case Op::Sqrt: kern::unary(f.op, m.dt, val(f.in[0]), o, N, s); break;
-      case Op::Select: kern::select(m.dt, val(f.in[0]), val(f.in[1]), val(f.in[2]), o, N, s); break;
-      case Op::Decompose: kern::decompose(m.dt, val(f.in[0]), f.k, o, N, s); break;
-      case Op::Compose: {
-        const void* ins[4];
-        for (size_t l = 0; l < f.in.size(); ++l) ins[l] = val(f.in[l]);
-        kern::compose(m.dt, ins, int(f.in.size()), o, N, s);
-        break;
-      }
-      case Op::Grad3d: {
-        const Ref& a = f.in[0];
-        if (a.kind == Ref::Input)
-          kern::grad3d(m.dt, in_dev[a.id], o, tab[0], tab[1], tab[2], m.nx, m.ny, m.nzl, m.NZ, m.k0, m.ghost, s);
-        else
-          kern::grad3d(m.dt, fval[a.id], o, tab[0], tab[1], tab[2], m.nx, m.ny, m.nzl, m.NZ, m.k0, 0, s);
-        break;
-      }
+    std::vector<const void*> args;
+    for (auto& r : f.in)
+      if (r.kind != Ref::Mesh) args.push_back(val(r));
+    const void* gsrc = nullptr;
+    int64_t gghost = 0;
+    if (f.op == Op::Grad3d) {
+      const Ref& a0 = f.in[0];
+      gsrc = a0.kind == Ref::Input ? in_dev[a0.id] : fval[a0.id];
+      gghost = a0.kind == Ref::Input ? m.ghost : 0;
     }
+    launch_primitive(m, f, o, args, gsrc, gghost, tab, s);
     DFG_CUDA(cudaGetLastError());
     st.kernel_count += 1;
     for (auto& r : f.in) release(r);

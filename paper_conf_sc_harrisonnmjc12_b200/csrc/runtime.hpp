@@ -90,6 +90,23 @@ std::vector<int> greedy_staged_order(const Dag& dag);
 int64_t predicted_device_bytes(const Dag& dag, dfg_strategy s, int64_t cells, size_t tsize);
 int64_t predicted_pcie_bytes(const Dag& dag, dfg_strategy s, int64_t cells, size_t tsize, bool host_mode);
 
+// DFG_HYBRID: staged execution under a device-memory cap with spill-to-host
+// (policy in DESIGN.md section 5b).  Planned on the host
+// at compile, replayed by exec_hybrid.
+struct HybridEvent {
+  enum Kind : int { Upload = 0, Reload, Spill, Discard, Drop, Run, SinkD2H, SinkHost, SinkH2D };
+  Kind kind;
+  Ref ref;
+};
+struct HybridPlan {
+  std::vector<HybridEvent> ev;
+  int64_t high = 0;                  // device high-water, units
+  int64_t h2d = 0, d2h = 0;          // transfers (host mode: + 4 mesh arrays)
+  int64_t h2d_units = 0, d2h_units = 0;
+};
+// Throws DFG_E_NOMEM if cap_units is below some filter's working set.
+HybridPlan plan_hybrid(const Dag& dag, const std::vector<int>& order, int64_t cap_units, bool host);
+
 struct PlanImpl {
   std::shared_ptr<MeshImpl> mesh;
   Dag dag;
@@ -108,6 +125,9 @@ struct PlanImpl {
   void resolve_kernel_times();
   std::map<std::string, std::vector<char>> const_cache;  // roundtrip host constants
   std::vector<int> order;  // staged execution order (list order unless a cap forced a reorder)
+  HybridPlan hyb;          // DFG_HYBRID schedule for hyb_host (0 device, 1 host binding mode)
+  int hyb_host = -1;
+  void plan_hybrid_for(bool host);
   // streamed strategy: ring of chunk slabs and the two copy streams
   std::vector<void*> stream_in, stream_out;
   int64_t stream_C = 0;
@@ -129,6 +149,7 @@ struct PlanImpl {
   void release_stream_buffers();
   void exec_fused(void* out, bool out_dev, cudaStream_t s);
   void exec_staged(void* out, bool out_dev, cudaStream_t s);
+  void exec_hybrid(void* out, bool out_dev, cudaStream_t s);
   void exec_roundtrip(void* out, bool out_dev, cudaStream_t s);
   void halo_exchange(const std::vector<int>& inputs, cudaStream_t s);
 };

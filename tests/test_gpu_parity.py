@@ -233,6 +233,77 @@ def test_memory_aware_staged_order(host, prog):
     assert plan2.schedule() == list(range(len(dag.filters)))
 
 
+@pytest.mark.parametrize("prog", ["qcrit", "intro", "vortmag"])
+@pytest.mark.parametrize("host", [True, False])
+@pytest.mark.parametrize("where", ["min", "mid", "below_greedy"])
+def test_hybrid_spill_to_host(prog, host, where, monkeypatch):
+    """DFG_HYBRID: under a cap below even the
+    memory-aware staged footprint, intermediates spill to pinned host memory
+    and come back when needed.  Results bit-identical to the oracle; the
+    transfer events, counts, bytes and device high-water equal the oracle's
+    schedule (oracle/model.py hybrid) for the memory-aware order."""
+    src, names = PAPER_PROGRAMS[prog]
+    shape = (40, 12, 10)
+    x, y, z, f = _inputs(shape, np.float32, names)
+    dag = build_dag(src, names)
+    mode = "host" if host else "device"
+    N = shape[0] * shape[1] * shape[2] * 4
+    monkeypatch.setenv("DFG_STAGED_ORDER", "greedy")
+    _, sp, *_ = run_lib(src, f, x, y, z, "staged", host=host, return_plan=True)
+    greedy = sp.schedule()
+    monkeypatch.delenv("DFG_STAGED_ORDER")
+    fpg = omodel.footprint(dag, "staged", mode, order=greedy)
+    lo = None
+    for c in range(1, fpg + 1):
+        try:
+            omodel.hybrid(dag, mode, c, greedy)
+            lo = c
+            break
+        except omodel.HybridInfeasible:
+            pass
+    hi = min(fpg, omodel.footprint(dag, "staged", mode)) - 1   # below both orders' footprints
+    cap = {"min": lo, "mid": (lo + hi) // 2, "below_greedy": hi}[where]
+    got, plan, *_ = run_lib(src, f, x, y, z, "hybrid", host=host, cap=cap * N, return_plan=True)
+    assert_parity(got, run_oracle(src, f, x, y, z))
+    assert plan.schedule() == greedy
+    want = omodel.hybrid(dag, mode, cap, greedy)
+    assert any(k in ("spill", "drop") for k, _ in want.events)   # the cap forces evictions
+    code = lambda r: int(r[1:]) if dag.ref_filter(r) is not None else -1 - list(names).index(r)  # noqa: E731
+    assert plan.transfers() == [(k, code(r)) for k, r in want.events]
+    st = plan.stats()
+    assert (st["h2d_count"], st["d2h_count"], st["kernel_count"]) == (want.counts.h2d, want.counts.d2h,
+                                                                      want.counts.kernels)
+    assert st["d2h_bytes"] == want.d2h_units * N
+    assert st["dev_highwater_bytes"] == want.high * N <= cap * N
+    assert st["predicted_highwater_bytes"] == want.high * N
+
+
+def test_hybrid_edges():
+    """No cap: hybrid is staged (same counts, same bits).  A cap below a
+    filter's working set is DFG_E_NOMEM at compile; mixed host / device
+    bindings are DFG_E_UNSUPPORTED."""
+    import paper_conf_sc_harrisonnmjc12_b200 as dfg
+    src, names = PAPER_PROGRAMS["qcrit"]
+    x, y, z, f = _inputs((24, 10, 8), np.float32)
+    a, p1, *_ = run_lib(src, f, x, y, z, "hybrid", host=True, return_plan=True)
+    b, p2, *_ = run_lib(src, f, x, y, z, "staged", host=True, return_plan=True)
+    assert np.array_equal(a, b)
+    for k in ("h2d_count", "d2h_count", "kernel_count", "h2d_bytes", "d2h_bytes", "dev_highwater_bytes"):
+        assert p1.stats()[k] == p2.stats()[k], k
+    with pytest.raises(dfg.DfgError) as e:
+        run_lib(src, f, x, y, z, "hybrid", host=True, cap=4 * 24 * 10 * 8 * 4)
+    assert e.value.name == "DFG_E_NOMEM"
+    mesh = dfg.Mesh(x, y, z)
+    keep = [torch.from_numpy(f["u"]).cuda(), f["v"], f["w"]]
+    mesh.bind("u", keep[0])
+    mesh.bind("v", keep[1], on_device=False)
+    mesh.bind("w", keep[2], on_device=False)
+    plan = dfg.Plan(mesh, src, "hybrid", 12 * 24 * 10 * 8 * 4)
+    with pytest.raises(dfg.DfgError) as e:
+        plan.execute(np.empty((8, 10, 24), np.float32), out_on_device=False)
+    assert e.value.name == "DFG_E_UNSUPPORTED"
+
+
 @pytest.mark.parametrize("shape,split", [((62, 30, 20), (2, 2, 2)), ((61, 23, 17), (2, 3, 2)),
                                          ((126, 14, 9), (1, 2, 3))])
 @pytest.mark.parametrize("prog", ["qcrit", "intro", "velmag"])

@@ -231,3 +231,50 @@ def test_errors_have_messages(dfg):
     with pytest.raises(dfg.DfgError) as e:
         dfg.dfg_dag_dump("a = 1", ("x",))
     assert e.value.name == "DFG_E_INVALID"
+
+
+def _random_topo(dag, rng):
+    done, order = set(), []
+    n = len(dag.filters)
+    while len(order) < n:
+        ready = [k for k in range(n) if k not in done
+                 and all(dag.ref_filter(r) is None or int(r[1:]) in done for r in dag.filters[k].inputs)]
+        k = rng.choice(ready)
+        done.add(k)
+        order.append(k)
+    return order
+
+
+@pytest.mark.parametrize("prog", ["velmag", "vortmag", "qcrit", "intro", "fig2", "edge"])
+@pytest.mark.parametrize("mode", ["host", "device"])
+def test_hybrid_planner_matches_oracle(dfg, prog, mode):
+    """DFG_HYBRID's planner (C++) and the oracle's restatement of the policy
+    (oracle/model.py hybrid, pinned in test_oracle_hybrid.py) give the same
+    event list, counts and high-water for every cap from infeasible to the
+    staged footprint, in list order and in random topological orders."""
+    from oracle import model as M
+    progs = dict(PAPER_PROGRAMS)
+    progs["fig2"] = ("r = (a + b) * (c + d)\n", ("a", "b", "c", "d"))
+    progs["edge"] = ("g = grad(u * v)\nc = {g[0] * v, u - v, g[2]}\nd = c[1] * c[0] + g[1] / v\n", ("u", "v"))
+    src, names = progs[prog]
+    dag = build_dag(src, names)
+    rng = random.Random(7)
+    orders = [None] + [_random_topo(dag, rng) for _ in range(3)]
+    fp = M.footprint(dag, "staged", mode)
+    compared = 0
+    for order in orders:
+        for cap in range(1, fp + 2):
+            try:
+                want = M.hybrid(dag, mode, cap, order)
+            except M.HybridInfeasible:
+                with pytest.raises(dfg.DfgError) as e:
+                    dfg.dfg_hybrid_model(src, names, mode == "host", cap, order)
+                assert e.value.name == "DFG_E_NOMEM"
+                continue
+            ev, high, h2d, d2h, h2du, d2hu = dfg.dfg_hybrid_model(src, names, mode == "host", cap, order)
+            code = lambda r: int(r[1:]) if dag.ref_filter(r) is not None else -1 - names.index(r)  # noqa: E731
+            assert ev == [(k, code(r)) for k, r in want.events], (cap, order)
+            assert (high, h2d, d2h, h2du, d2hu) == (want.high, want.counts.h2d, want.counts.d2h,
+                                                    want.h2d_units, want.d2h_units)
+            compared += 1
+    assert compared >= 4
