@@ -54,7 +54,32 @@ class ClockSampler:
         self._stop = threading.Event()
         self._t = None
 
+    # NVML clocks-event reason bits (nvml.h): sw power cap, hw slowdown,
+    # sw thermal slowdown, hw thermal slowdown
+    BITS = ((0x8, 3), (0x40, 4), (0x20, 5), (0x4, 6))
+
     def _run(self):
+        try:  # NVML: a query takes microseconds, so ~100 samples per second
+            import pynvml
+            pynvml.nvmlInit()
+            h = pynvml.nvmlDeviceGetHandleByIndex(self.index)
+            mx = pynvml.nvmlDeviceGetMaxClockInfo(h, pynvml.NVML_CLOCK_SM)
+            get_reasons = getattr(pynvml, "nvmlDeviceGetCurrentClocksEventReasons", None) or \
+                pynvml.nvmlDeviceGetCurrentClocksThrottleReasons
+            while not self._stop.is_set():
+                sm = pynvml.nvmlDeviceGetClockInfo(h, pynvml.NVML_CLOCK_SM)
+                pw = pynvml.nvmlDeviceGetPowerUsage(h) / 1000.0
+                bits = get_reasons(h)
+                row = [str(sm), str(mx), f"{pw:.1f}", "", "", "", ""]
+                for bit, col in self.BITS:
+                    row[col] = "Active" if bits & bit else "Not Active"
+                self.rows.append(row)
+                self._stop.wait(0.01)
+            self.source = "nvml"
+            return
+        except Exception:
+            pass
+        self.source = "nvidia-smi"
         while not self._stop.is_set():
             try:
                 out = subprocess.run(["nvidia-smi", f"--id={self.index}", f"--query-gpu={self.Q}",
@@ -83,7 +108,7 @@ class ClockSampler:
         names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
         reasons = sorted({names[i] for r in self.rows for i in range(4) if len(r) > 3 + i and r[3 + i] == "Active"})
         return {"sm_mhz": float(np.median(sm)) if sm else None, "sm_max_mhz": max(mx) if mx else None,
-                "reasons": reasons, "samples": len(self.rows)}
+                "reasons": reasons, "samples": len(self.rows), "source": getattr(self, "source", None)}
 
 
 # ------------------------------------------------------------------ oracle
