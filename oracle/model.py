@@ -277,6 +277,8 @@ def hybrid(dag: Dag, mode: str, cap: int, order=None) -> Hybrid:
     base = 0
     if mode == "device":
         base = sum(_units(dag, s) for s in srcs) + _units(dag, dag.result)
+    if base > cap:
+        raise HybridInfeasible(f"cap {cap} below the resident inputs and output ({base})")
     high = base
     h2d = d2h = h2du = d2hu = 0
     mesh_up = False

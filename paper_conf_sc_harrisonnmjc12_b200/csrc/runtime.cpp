@@ -489,6 +489,9 @@ HybridPlan plan_hybrid(const Dag& dag, const std::vector<int>& order, int64_t ca
   std::map<Key, int64_t> resident;  // evictable device arrays -> units
   std::set<Key> host_copy;
   const int64_t base = host ? 0 : int64_t(src.inputs.size()) + units(dag, dag.result);
+  if (base > cap)
+    fail(DFG_E_NOMEM, "dev_mem_cap of " + std::to_string(cap) + " problem arrays is below the resident inputs and " +
+                          "output (" + std::to_string(base) + ")");
   auto live = [&] {
     int64_t l = base;
     for (auto& kv : resident) l += kv.second;

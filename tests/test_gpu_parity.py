@@ -278,6 +278,35 @@ def test_hybrid_spill_to_host(prog, host, where, monkeypatch):
     assert st["predicted_highwater_bytes"] == want.high * N
 
 
+@pytest.mark.parametrize("src,names", EDGE)
+@pytest.mark.parametrize("T", [np.float32, np.float64])
+@pytest.mark.parametrize("host", [True, False])
+def test_hybrid_edge_programs(src, names, T, host):
+    """Every EDGE program (vector results, bare-input and constant results,
+    select, compose) under the tightest feasible cap: bit-identical results
+    and the oracle's transfer events."""
+    x, y, z, f = _inputs((20, 9, 7), T, names)
+    dag = build_dag(src, names)
+    mode = "host" if host else "device"
+    N = 20 * 9 * 7 * np.dtype(T).itemsize
+    fp = omodel.footprint(dag, "staged", mode)
+    cap = next(c for c in range(1, fp + 2) if _feasible(dag, mode, c))
+    got, plan, *_ = run_lib(src, f, x, y, z, "hybrid", host=host, cap=cap * N, return_plan=True)
+    assert_parity(got, run_oracle(src, f, x, y, z))
+    want = omodel.hybrid(dag, mode, cap, plan.schedule())
+    code = lambda r: int(r[1:]) if dag.ref_filter(r) is not None else -1 - list(names).index(r)  # noqa: E731
+    assert plan.transfers() == [(k, code(r)) for k, r in want.events]
+    assert plan.stats()["dev_highwater_bytes"] == want.high * N
+
+
+def _feasible(dag, mode, cap):
+    try:
+        omodel.hybrid(dag, mode, cap)
+        return True
+    except omodel.HybridInfeasible:
+        return False
+
+
 def test_hybrid_edges():
     """No cap: hybrid is staged (same counts, same bits).  A cap below a
     filter's working set is DFG_E_NOMEM at compile; mixed host / device

@@ -40,6 +40,17 @@ def test_fig2_worked_example():
         M.hybrid(dag, "host", 2)          # f0 alone needs a, b and its result
 
 
+def test_device_mode_needs_room_for_resident_arrays():
+    """Device mode keeps the bound inputs and the output on the device: a
+    cap below them is infeasible even for a network with no filter."""
+    dag = build_dag("a = u\n", ("u",))
+    with pytest.raises(M.HybridInfeasible):
+        M.hybrid(dag, "device", 1)
+    assert M.hybrid(dag, "device", 2).high == 2
+    h = M.hybrid(dag, "host", 1)                # host mode: upload u, copy it back
+    assert h.events == [("upload", "u"), ("sink_d2h", "u")] and h.counts == M.Counts(1, 1, 0)
+
+
 @pytest.mark.parametrize("prog", ["velmag", "vortmag", "qcrit", "intro"])
 @pytest.mark.parametrize("mode", ["host", "device"])
 def test_reduces_to_staged_when_the_cap_suffices(prog, mode):
