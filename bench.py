@@ -323,21 +323,39 @@ def main():
         hout = torch.empty((nzl, n, n), dtype=torch.float32).pin_memory()
         barrier()
         torch.cuda.synchronize()
-        t0 = time.perf_counter()
         reps = 3
+        h0, h1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        h0.record(stream)
         for _ in range(reps):
             with torch.cuda.stream(stream):
                 for c in "uvw":
-                    fields[c].copy_(hostf[c], non_blocking=True)
+                    fields[c][g:g + nzl].copy_(hostf[c][g:g + nzl], non_blocking=True)
                 plan.execute(out, stream=stream)
                 hout.copy_(out, non_blocking=True)
-            stream.synchronize()
-        te = torch.tensor([(time.perf_counter() - t0) / reps], dtype=torch.float64, device="cuda")
-        dist.all_reduce(te, op=dist.ReduceOp.MAX)
+        h1.record(stream)
+        h1.synchronize()
+        te = torch.tensor([h0.elapsed_time(h1) * 1e-3 / reps], dtype=torch.float64, device="cuda")
+        dist.all_reduce(te, op=dist.ReduceOp.MAX)        # device time, max over ranks
         te = float(te[0])
         e2e = {"value": cells_rank * world / te, "unit": "cells/s",
-               "h2d_bytes_per_step": 3 * fields["u"].numel() * 4 * world,
-               "d2h_bytes_per_step": out.numel() * 4 * world, "ms_per_step": te * 1e3}
+               "h2d_bytes_per_step": 3 * nzl * n * n * 4 * world,
+               "d2h_bytes_per_step": out.numel() * 4 * world, "ms_per_step": te * 1e3,
+               "timing": "CUDA events on the step stream, max over ranks"}
+
+    multi = None
+    if world > 1:
+        # per-rank halo bytes, kernel time and step time; max over ranks
+        per = torch.tensor([st["halo_bytes"] / max(1, K), kern_ms, ms_step, launches_per_step],
+                           dtype=torch.float64, device="cuda")
+        allr = [torch.zeros_like(per) for _ in range(world)]
+        dist.all_gather(allr, per)
+        rows = [r.tolist() for r in allr]
+        multi = {"halo_bytes_per_step": [int(r[0]) for r in rows],
+                 "kernel_ms_per_step": [r[1] for r in rows],
+                 "step_ms": [r[2] for r in rows],
+                 "launches_per_step": [r[3] for r in rows],
+                 "halo": "NCCL send/recv of the first/last owned plane of u, v, w on a side stream, "
+                         "overlapped with the interior planes; boundary planes launched after it"}
 
     strategies = variants = sweep = None
     if rank == 0 and world == 1 and not args.no_strategies:
@@ -367,6 +385,7 @@ def main():
                          "kernel": "dfg_fused_tma", "kernel_ms": kern_ms,
                          "algorithmic_bytes_per_launch": ALGO_BYTES_PER_CELL * cells_rank},
             "e2e": e2e,
+            "multi_gpu": multi,
             "gpu_launches": st["kernel_count"],
             "clocks": clk.summary(),
             "frac_of_spec_8tbs": achieved / 8000.0,
