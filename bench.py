@@ -193,7 +193,7 @@ def main():
     ap.add_argument("--steps", type=int, default=300)
     ap.add_argument("--warmup", type=int, default=5)
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
-    ap.add_argument("--n", type=int, default=N1, help="cells per axis per GPU (default 1024)")
+    ap.add_argument("--size", type=int, default=N1, help="cells per axis per GPU (default 1024)")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-strategies", action="store_true")
     args = ap.parse_args()
@@ -210,11 +210,19 @@ def main():
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
     local = int(os.environ.get("LOCAL_RANK", "0"))
+    # Test hook, not a measurement: DFG_BENCH_ONE_GPU=1 puts every rank on cuda:0
+    # with its own NCCL_HOSTID (NCCL then uses its socket transport), so the
+    # N > 1 path runs end to end on a one-GPU box; its timings mean nothing.
+    one_gpu = world > 1 and os.environ.get("DFG_BENCH_ONE_GPU") == "1"
+    if one_gpu:
+        os.environ.update({"NCCL_HOSTID": f"dfg-bench-{rank}", "NCCL_SOCKET_IFNAME": "lo", "NCCL_IB_DISABLE": "1",
+                           "NCCL_P2P_DISABLE": "1", "NCCL_SHM_DISABLE": "1"})
+        local = 0
     torch.cuda.set_device(local)
     if world > 1:
         dist.init_process_group("nccl", device_id=torch.device("cuda", local))
     assert world == args.gpus or world == 1, "launch with torchrun --nproc-per-node N for --gpus N"
-    n = args.n
+    n = args.size
     NZ = n * world
     K, W = args.steps, args.warmup
     assert W >= 3, "at least 3 warm-up steps"
@@ -378,7 +386,8 @@ def main():
                        "cells_per_gpu": cells_rank, "fused_kernel": {1: "tma", 2: "general", 3: "pointwise"}.get(
                            info["variant"]), "regs": info["regs"],
                        "l2": f"inputs {3 * cells_rank * 4 / 1e9:.1f} GB per GPU >> 126 MB L2; no flush needed",
-                       "parallelism": f"zslab{world}"},
+                       "parallelism": f"zslab{world}",
+                       **({"one_gpu_functional_test": True} if one_gpu else {})},
             "hbm_gbs": ALGO_BYTES_PER_CELL * cells_rank * world / (ms_step * 1e-3) / 1e9 / world,
             "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
                          "frac": achieved / peak, "traffic": traffic, "peak_source": peak_src,
