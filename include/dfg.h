@@ -143,13 +143,22 @@ int dfg_create_mesh(dfg_dtype dtype, int64_t nx, int64_t ny, int64_t nz_local,
  * the CALLER (VisIt's ghost exchange) -- no halo transport is used; cells on
  * the global mesh boundary ignore their ghost cells (one-sided differences,
  * reading R1).  ghost = 0 only for the whole mesh.  Output: T[nz][ny][nx].
- * Fusion (and reference) strategies only; the TMA fast path additionally
- * needs (nx + 2*ghost) * sizeof(T) % 16 == 0, other widths use the general
- * kernel.  Errors as dfg_create_mesh. */
+ * Row layout (like cudaMallocPitch): a buffer is T[nz+2][ny+2][row_pitch];
+ * in each row the owned cells sit at columns x_offset .. x_offset+nx-1, the
+ * ghost columns at x_offset-1 and x_offset+nx, anything else is padding that
+ * is never read.  x_offset = 0 means ghost, row_pitch = 0 means
+ * x_offset + nx + ghost (the packed shell).  Fusion (and reference)
+ * strategies only; the TMA fast path needs nx, x_offset and row_pitch times
+ * sizeof(T) to be multiples of 16 bytes (TMA box coordinates along a row
+ * must be 16-byte aligned) -- e.g. for the paper's 192-wide fp32 blocks
+ * x_offset 4, row_pitch 200; other layouts use the general kernel.
+ * Errors as dfg_create_mesh; DFG_E_INVALID unless ghost <= x_offset and
+ * x_offset + nx + ghost <= row_pitch. */
 int dfg_create_block(dfg_dtype dtype, int64_t nx, int64_t ny, int64_t nz,
                      const void* x, const void* y, const void* z,
                      int64_t NX, int64_t NY, int64_t NZ,
-                     int64_t i0, int64_t j0, int64_t k0, int ghost, dfg_mesh* out);
+                     int64_t i0, int64_t j0, int64_t k0, int ghost,
+                     int64_t row_pitch, int64_t x_offset, dfg_mesh* out);
 
 /* Idempotent on NULL.  Plans keep what they need alive: destroying a mesh
  * with live plans is allowed (the plans stay valid). */

@@ -43,10 +43,12 @@ class Mesh:
         self._bound = {}
 
     @classmethod
-    def block(cls, x, y, z, nx, ny, nz, i0, j0, k0, ghost=1):
+    def block(cls, x, y, z, nx, ny, nz, i0, j0, k0, ghost=1, row_pitch=0, x_offset=0):
         """VisIt-style sub-grid of the global mesh with points x, y, z:
         local nx x ny x nz cells at (i0, j0, k0), one-cell ghost shell on all
-        six faces filled by the caller (dfg_create_block)."""
+        six faces filled by the caller (dfg_create_block); buffers
+        T[nz+2][ny+2][row_pitch], owned cells from column x_offset
+        (0: x_offset = ghost, row_pitch = x_offset + nx + ghost)."""
         import numpy as np
         from ._dfg import dfg_create_block
         self = cls.__new__(cls)
@@ -56,8 +58,10 @@ class Mesh:
         self.ghost = ghost
         self._coords = (x, y, z)
         self._bound = {}
+        self.x_offset = x_offset or ghost
+        self.row_pitch = row_pitch or self.x_offset + nx + ghost
         self.handle = dfg_create_block(_dtype_code(x.dtype), nx, ny, nz, x, y, z, len(x) - 1, len(y) - 1,
-                                       len(z) - 1, i0, j0, k0, ghost)
+                                       len(z) - 1, i0, j0, k0, ghost, row_pitch, x_offset)
         return self
 
     def bind(self, name, buf, on_device=None):

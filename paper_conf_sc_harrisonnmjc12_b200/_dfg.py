@@ -57,7 +57,7 @@ _SIGS = {
     "dfg_last_error": (C.c_char_p, []),
     "dfg_create_mesh": (C.c_int, [C.c_int, _I64, _I64, _I64, _P, _P, _P, _I64, _I64, C.c_int, C.POINTER(_P)]),
     "dfg_create_block": (C.c_int, [C.c_int, _I64, _I64, _I64, _P, _P, _P, _I64, _I64, _I64, _I64, _I64, _I64,
-                                   C.c_int, C.POINTER(_P)]),
+                                   C.c_int, _I64, _I64, C.POINTER(_P)]),
     "dfg_destroy_mesh": (None, [_P]),
     "dfg_partition": (C.c_int, [_I64, C.c_int, C.c_int, C.POINTER(_I64), C.POINTER(_I64)]),
     "dfg_halo_map": (C.c_int, [_P, C.POINTER(_I64)]),
@@ -142,10 +142,10 @@ def dfg_create_mesh(dtype, nx, ny, nz_local, x, y, z, nz_global=None, z_offset=0
     return h.value
 
 
-def dfg_create_block(dtype, nx, ny, nz, x, y, z, NX, NY, NZ, i0, j0, k0, ghost=1):
+def dfg_create_block(dtype, nx, ny, nz, x, y, z, NX, NY, NZ, i0, j0, k0, ghost=1, row_pitch=0, x_offset=0):
     h = _P()
     _check(_lib.dfg_create_block(dtype, nx, ny, nz, _ptr(x), _ptr(y), _ptr(z), NX, NY, NZ, i0, j0, k0, ghost,
-                                 C.byref(h)))
+                                 row_pitch, x_offset, C.byref(h)))
     return h.value
 
 

@@ -94,11 +94,12 @@ int dfg_create_mesh(dfg_dtype dtype, int64_t nx, int64_t ny, int64_t nz_local, c
 
 int dfg_create_block(dfg_dtype dtype, int64_t nx, int64_t ny, int64_t nz, const void* x, const void* y,
                      const void* z, int64_t NX, int64_t NY, int64_t NZ, int64_t i0, int64_t j0, int64_t k0, int ghost,
-                     dfg_mesh* out) {
+                     int64_t row_pitch, int64_t x_offset, dfg_mesh* out) {
   return guard([&] {
     if (!out) dfg::fail(DFG_E_INVALID, "null output handle");
     *out = nullptr;
-    auto m = dfg::create_block(to_dtype(dtype), nx, ny, nz, x, y, z, NX, NY, NZ, i0, j0, k0, ghost);
+    auto m = dfg::create_block(to_dtype(dtype), nx, ny, nz, x, y, z, NX, NY, NZ, i0, j0, k0, ghost, row_pitch,
+                               x_offset);
     *out = new dfg_mesh_s{std::move(m)};
   });
 }

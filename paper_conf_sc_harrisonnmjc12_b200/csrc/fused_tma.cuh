@@ -228,8 +228,8 @@ extern "C" __global__ void __launch_bounds__((DFG_NCW + 1) * 32, DFG_CTAS)
         const long long ty_ = rest % P.tiles_y;
         const long long zc = rest / P.tiles_y;
         // input coordinates include the block's x/y ghost columns / rows
-        const int x0 = (int)(tx_ * DFG_TX) - DFG_HX + (int)((P.px - P.nx) >> 1);
-        const int y0 = (int)(ty_ * DFG_NCW) - 1 + (int)((P.py - P.ny) >> 1);
+        const int x0 = (int)(tx_ * DFG_TX) - DFG_HX + (int)P.gx;
+        const int y0 = (int)(ty_ * DFG_NCW) - 1 + (int)P.gy;
         const long long kb = P.kbeg + zc * P.kz;
         const long long ke = min(kb + (long long)P.kz, P.kend);
         // pre-plane, kb..ke-1, post-plane; clamped to the global mesh (R1)

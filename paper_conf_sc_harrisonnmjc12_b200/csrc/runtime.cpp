@@ -171,7 +171,7 @@ std::shared_ptr<MeshImpl> create_mesh(DType dt, int64_t nx, int64_t ny, int64_t 
 
 std::shared_ptr<MeshImpl> create_block(DType dt, int64_t nx, int64_t ny, int64_t nz, const void* x, const void* y,
                                        const void* z, int64_t NX, int64_t NY, int64_t NZ, int64_t i0, int64_t j0,
-                                       int64_t k0, int ghost) {
+                                       int64_t k0, int ghost, int64_t pitch, int64_t xoff) {
   if (nx < 1 || ny < 1 || nz < 1 || NX < 1 || NY < 1 || NZ < 1) fail(DFG_E_INVALID, "block sizes must be >= 1");
   if (i0 < 0 || j0 < 0 || k0 < 0 || i0 + nx > NX || j0 + ny > NY || k0 + nz > NZ)
     fail(DFG_E_INVALID, "block outside the global mesh");
@@ -179,8 +179,14 @@ std::shared_ptr<MeshImpl> create_block(DType dt, int64_t nx, int64_t ny, int64_t
   if (ghost == 0 && (nx != NX || ny != NY || nz != NZ))
     fail(DFG_E_INVALID, "a block of a larger mesh needs its one-cell ghost shell");
   if (!x || !y || !z) fail(DFG_E_INVALID, "null coordinate pointer");
+  if (xoff == 0) xoff = ghost;
+  if (pitch == 0) pitch = xoff + nx + ghost;
+  if (xoff < ghost || xoff + nx + ghost > pitch)
+    fail(DFG_E_INVALID, "need ghost <= x_offset and x_offset + nx + ghost <= row_pitch");
   auto m = create_block_impl(dt, nx, ny, nz, x, y, z, NX, NY, NZ, i0, j0, k0, ghost, ghost);
   m->ghosts_supplied = ghost == 1;
+  m->pitch = pitch;
+  m->xoff = xoff;
   return m;
 }
 
@@ -963,7 +969,7 @@ std::vector<uint64_t> pack_params(const std::vector<const void*>& f, void* out, 
   w.push_back(reinterpret_cast<uint64_t>(ty));
   w.push_back(reinterpret_cast<uint64_t>(tz));
   for (int64_t v : {m.nx, m.ny, m.nzl, m.NZ, m.k0, int64_t(m.ghost), kbeg, kend, items, m.NX, m.NY, m.i0, m.j0,
-                    m.px(), m.py()})
+                    m.px(), m.py(), m.gx(), int64_t(m.gxy)})
     w.push_back(uint64_t(v));
   w.push_back(uint64_t(uint32_t(tiles_x)) | (uint64_t(uint32_t(tiles_y)) << 32));
   w.push_back(uint64_t(uint32_t(kz)) | (uint64_t(uint32_t(vec_ok)) << 32));
@@ -1087,7 +1093,7 @@ void PlanImpl::launch_fused(const std::vector<const void*>& fptr, void* dout, co
   const int64_t kbeg = kb < 0 ? m.k0 : kb, kend = ke < 0 ? m.k0 + m.nzl : ke;
   const int64_t N = m.nx * m.ny * (kend - kbeg);
   const int vec = int(16 / ts);
-  bool vec_ok = aligned16(dout) && (N % vec == 0) && m.gxy == 0;
+  bool vec_ok = aligned16(dout) && (N % vec == 0) && m.gxy == 0 && m.px() == m.nx && m.gx() == 0;
   for (auto p : fptr) vec_ok = vec_ok && aligned16(p);
   const char* force = std::getenv("DFG_FUSED_KERNEL");
   bool want_general = force && !std::strcmp(force, "general");
@@ -1103,7 +1109,8 @@ void PlanImpl::launch_fused(const std::vector<const void*>& fptr, void* dout, co
     DFG_CU(drv().LaunchKernel(mod.pointwise, grid, 1, 1, 256, 1, 1, 0, s, args, nullptr));
     DFG_CUDA(cudaEventRecord(ke.second, s));
     last_variant = 3;
-  } else if (mod.tma && !want_general && m.nx % vec == 0 && m.px() % vec == 0 && aligned16(dout) &&
+  } else if (mod.tma && !want_general && m.nx % vec == 0 && m.px() % vec == 0 && m.gx() % vec == 0 &&
+             aligned16(dout) &&
              std::all_of(fptr.begin(), fptr.end(), [](const void* p) { return aligned16(p); })) {
     const int ncw = fsrc.cfg.ncw;
     const int nsf = int(L.stencil_inputs.size() + L.point_inputs.size());  // TMA tiles per stage

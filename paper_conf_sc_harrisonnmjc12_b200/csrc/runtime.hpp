@@ -28,6 +28,8 @@ struct MeshImpl {
   int64_t NX = 0, NY = 0, i0 = 0, j0 = 0;
   int ghost = 0;     // ghost planes in z (slabs, blocks)
   int gxy = 0;       // ghost columns / rows in x and y (VisIt blocks, caller-filled)
+  int64_t pitch = 0; // input row pitch in elements (blocks; 0 = nx + 2*gxy)
+  int64_t xoff = 0;  // column of the first owned cell in an input row (blocks; 0 = gxy)
   bool ghosts_supplied = false;  // blocks: the caller fills every ghost cell (no exchange)
   int device = 0;
   bool markstein_safe = true;        // spacing tables inside the exact-division range
@@ -40,7 +42,8 @@ struct MeshImpl {
   void* nccl = nullptr;              // ncclComm_t
   std::weak_ptr<MeshImpl> link_lo, link_hi;
   ~MeshImpl();
-  int64_t px() const { return nx + 2 * gxy; }        // input row pitch
+  int64_t px() const { return pitch ? pitch : nx + 2 * gxy; }  // input row pitch
+  int64_t gx() const { return xoff ? xoff : gxy; }   // first owned column of an input row
   int64_t py() const { return ny + 2 * gxy; }        // input rows per plane
   int64_t plane() const { return nx * ny; }          // owned cells per plane (output)
   int64_t in_plane() const { return px() * py(); }   // input plane incl. x/y ghosts
@@ -58,10 +61,12 @@ struct SlabView {
   int ghost;
   int64_t NX, NY, i0, j0;
   int gxy;
+  int64_t pitch, xoff;
   static SlabView of(const MeshImpl& m) {
-    return SlabView{m.dt, m.nx, m.ny, m.nzl, m.NZ, m.k0, m.ghost, m.NX, m.NY, m.i0, m.j0, m.gxy};
+    return SlabView{m.dt, m.nx, m.ny, m.nzl, m.NZ, m.k0, m.ghost, m.NX, m.NY, m.i0, m.j0, m.gxy, m.pitch, m.xoff};
   }
-  int64_t px() const { return nx + 2 * gxy; }
+  int64_t px() const { return pitch ? pitch : nx + 2 * gxy; }
+  int64_t gx() const { return xoff ? xoff : gxy; }
   int64_t py() const { return ny + 2 * gxy; }
 };
 
@@ -74,7 +79,7 @@ std::shared_ptr<MeshImpl> create_mesh(DType dt, int64_t nx, int64_t ny, int64_t 
 // on all six faces filled by the caller.
 std::shared_ptr<MeshImpl> create_block(DType dt, int64_t nx, int64_t ny, int64_t nz, const void* x, const void* y,
                                        const void* z, int64_t NX, int64_t NY, int64_t NZ, int64_t i0, int64_t j0,
-                                       int64_t k0, int ghost);
+                                       int64_t k0, int ghost, int64_t pitch, int64_t xoff);
 std::shared_ptr<MeshImpl> create_block_impl(DType dt, int64_t nx, int64_t ny, int64_t nzl, const void* x,
                                             const void* y, const void* z, int64_t NX, int64_t NY, int64_t NZ,
                                             int64_t i0, int64_t j0, int64_t k0, int ghost, int gxy);

@@ -56,7 +56,8 @@ struct DfgParams {
   long long kbeg, kend;     // global planes computed by this launch
   long long items;          // TMA: tiles_x * tiles_y * zchunks
   long long NX, NY, i0, j0; // global x/y cells and this block's offsets (whole mesh: NX = nx, i0 = 0)
-  long long px, py;         // input row pitch and rows per plane (nx / ny + 2 x/y ghosts)
+  long long px, py;         // input row pitch and rows per plane (ny + 2 gy)
+  long long gx, gy;         // column / row of the first owned cell in the input (blocks: x_offset, 1)
   int tiles_x, tiles_y, kz, vec_ok;
   DFG_T nzero;              // -0.0, opaque to the compiler (contraction guard)
 };
@@ -137,8 +138,8 @@ extern "C" __global__ void __launch_bounds__(256) dfg_fused_pointwise(const DfgP
     }
     dfg_store_cells(P.out + (out_off + v * DFG_VEC) * DFG_OUTW, o);
   }
-  const long long gx = (P.px - P.nx) >> 1, gy = (P.py - P.ny) >> 1;
-  const bool pitched = gx != 0 || gy != 0;
+  const long long gx = P.gx, gy = P.gy;
+  const bool pitched = gx != 0 || P.px != P.nx;
   for (long long c = nv * DFG_VEC + tid; c < n; c += stride) {
     // pitched input index (blocks carry x/y ghost columns / rows); 32-bit
     // divisions: nx, ny and the launch's row count stay below 2^32
@@ -166,7 +167,7 @@ extern "C" __global__ void __launch_bounds__(256) dfg_fused_pointwise(const DfgP
 extern "C" __global__ void __launch_bounds__(256) dfg_fused_general(const DfgParams P) {
   const long long plane = P.nx * P.ny;          // output plane (owned cells)
   const long long in_plane = P.px * P.py;       // input plane (with x/y ghosts)
-  const long long gx = (P.px - P.nx) >> 1, gy = (P.py - P.ny) >> 1;
+  const long long gx = P.gx, gy = P.gy;
   const long long total = plane * (P.kend - P.kbeg);
   const long long stride = (long long)gridDim.x * blockDim.x;
   const dfg2 Z = dfg2_splat(P.nzero);

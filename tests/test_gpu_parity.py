@@ -334,14 +334,19 @@ def test_hybrid_edges():
 
 
 @pytest.mark.parametrize("shape,split", [((62, 30, 20), (2, 2, 2)), ((61, 23, 17), (2, 3, 2)),
+                                         ((128, 30, 20), (2, 2, 2)), ((192, 20, 12), (1, 2, 2)),
                                          ((126, 14, 9), (1, 2, 3))])
 @pytest.mark.parametrize("prog", ["qcrit", "intro", "velmag"])
 @pytest.mark.parametrize("strategy", ["fused", "reference"])
-def test_visit_blocks_with_ghost_shells(shape, split, prog, strategy):
+@pytest.mark.parametrize("pitch", ["natural", "padded"])
+def test_visit_blocks_with_ghost_shells(shape, split, prog, strategy, pitch):
     """VisIt-style multi-block (L253-L255, L315; NEXT #4): every block gets a
     one-cell ghost shell on all six faces filled from the global field (what
     VisIt's ghost exchange does); the stitched block interiors equal the
-    whole-mesh result bit for bit (and the oracle)."""
+    whole-mesh result bit for bit (and the oracle).  "padded": owned cells
+    from column 4 (16 bytes), rows padded past a multiple of 16 bytes
+    (padding = NaN, never read), which puts blocks whose width is a multiple
+    of 4 on the TMA kernel."""
     import paper_conf_sc_harrisonnmjc12_b200 as dfg
     if strategy == "reference" and prog == "intro":
         pytest.skip("no reference kernel for the intro expression")
@@ -361,16 +366,23 @@ def test_visit_blocks_with_ghost_shells(shape, split, prog, strategy):
                 i0, i1 = cuts[0][a], cuts[0][a + 1]
                 j0, j1 = cuts[1][b], cuts[1][b + 1]
                 k0, k1 = cuts[2][c], cuts[2][c + 1]
-                m = dfg.Mesh.block(x, y, z, i1 - i0, j1 - j0, k1 - k0, i0, j0, k0, ghost=1)
+                bx = i1 - i0
+                xo = 1 if pitch == "natural" else 4
+                rp = bx + 2 if pitch == "natural" else (xo + bx + 1 + 3) // 4 * 4 + 4
+                m = dfg.Mesh.block(x, y, z, bx, j1 - j0, k1 - k0, i0, j0, k0, ghost=1, row_pitch=rp, x_offset=xo)
                 keep = []
                 for n in names:
-                    t = torch.from_numpy(np.ascontiguousarray(pad[n][k0:k1 + 2, j0:j1 + 2, i0:i1 + 2])).cuda()
+                    buf = np.full((k1 - k0 + 2, j1 - j0 + 2, rp), np.nan, np.float32)
+                    buf[:, :, xo - 1:xo + bx + 1] = pad[n][k0:k1 + 2, j0:j1 + 2, i0:i1 + 2]
+                    t = torch.from_numpy(buf).cuda()
                     keep.append(t)
                     m.bind(n, t)
                 p = dfg.Plan(m, src, strategy)
-                o = torch.empty((k1 - k0, j1 - j0, i1 - i0), device="cuda")
+                o = torch.empty((k1 - k0, j1 - j0, bx), device="cuda")
                 p.execute(o)
                 torch.cuda.synchronize()
+                if pitch == "padded" and bx % 4 == 0 and prog != "velmag":
+                    assert p.info()["variant"] == 1          # TMA kernel on the padded shell
                 got[k0:k1, j0:j1, i0:i1] = o.cpu().numpy()
     assert np.array_equal(got, whole)
 
