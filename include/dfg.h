@@ -231,12 +231,27 @@ void dfg_destroy_plan(dfg_plan plan);
  * the paper's failed GPU cases, L309), DFG_E_CUDA, DFG_E_NCCL. */
 int dfg_execute(dfg_plan plan, void* out, int out_on_device, void* cuda_stream);
 
+/* Several fused plans of ONE network on different meshes of the same device
+ * -- the paper's VisIt sub-grids, 12 per GPU (L253-L255, L315) -- in one
+ * launch: the persistent TMA kernel walks the concatenated tiles of all
+ * meshes, so small blocks do not pay one kernel's fill and drain each.
+ * outs[b]: device output of plans[b].  Used when every plan is DFG_FUSED
+ * with the same generated kernel (same expression, dtype and global mesh),
+ * every input device-resident, no halo exchange needed (whole meshes or
+ * blocks with ghost shells) and every layout TMA-eligible (see
+ * dfg_create_block); otherwise the plans execute one after the other.
+ * Results equal dfg_execute's bit for bit.  Stats: executes +1 on every
+ * plan; the launch and its timing are counted on plans[0].
+ * Errors as dfg_execute; DFG_E_INVALID for n < 1 or null entries. */
+int dfg_execute_blocks(dfg_plan const* plans, int n, void* const* outs, void* cuda_stream);
+
 int dfg_plan_stats(dfg_plan plan, dfg_stats* out);
 int dfg_reset_stats(dfg_plan plan);
 
 /* Plan description: out[0] = strategy, out[1] = result width (1 or 4),
- * out[2] = number of filters, out[3] = fused kernel variant in use
- * (0 none, 1 TMA pipeline, 2 general), out[4] = registers per thread of the
+ * out[2] = number of filters, out[3] = fused kernel variant of the last
+ * execute (0 none, 1 TMA pipeline, 2 general, 3 point-wise, 4 TMA
+ * multi-block via dfg_execute_blocks), out[4] = registers per thread of the
  * fused kernel (0 if none), out[5] = local memory per thread of that kernel
  * (bytes; spills and stack), out[6] = predicted
  * device footprint in bytes for device-resident inputs,

@@ -132,3 +132,12 @@ class Plan:
             self.close()
         except Exception:
             pass
+
+
+def execute_blocks(plans, outs, stream=None):
+    """One launch for fused plans of one network on several meshes (VisIt
+    blocks of a device; dfg_execute_blocks).  outs: device tensors."""
+    from ._dfg import dfg_execute_blocks
+    s = stream if (stream is None or isinstance(stream, int)) else stream.cuda_stream
+    dfg_execute_blocks([p.handle for p in plans], outs, s)
+    return outs

@@ -68,6 +68,7 @@ _SIGS = {
     "dfg_compile": (C.c_int, [_P, C.c_char_p, C.c_int, C.c_size_t, C.POINTER(_P)]),
     "dfg_destroy_plan": (None, [_P]),
     "dfg_execute": (C.c_int, [_P, _P, C.c_int, _P]),
+    "dfg_execute_blocks": (C.c_int, [C.POINTER(_P), C.c_int, C.POINTER(_P), _P]),
     "dfg_plan_stats": (C.c_int, [_P, C.POINTER(dfg_stats)]),
     "dfg_reset_stats": (C.c_int, [_P]),
     "dfg_plan_info": (C.c_int, [_P, C.POINTER(_I64)]),
@@ -244,6 +245,14 @@ def dfg_hybrid_model(expr, inputs, host_mode, cap_units, order=None):
                                  C.byref(n), out))
     events = [(TRANSFER_KINDS[ev[2 * i]], int(ev[2 * i + 1])) for i in range(n.value)]
     return (events,) + tuple(int(v) for v in out)
+
+
+def dfg_execute_blocks(plans, outs, stream=None):
+    """plans: handles; outs: device tensors (or pointers), one per plan."""
+    n = len(plans)
+    ph = (_P * n)(*plans)
+    oh = (_P * n)(*[_ptr(o) for o in outs])
+    _check(_lib.dfg_execute_blocks(ph, n, oh, stream))
 
 
 def dfg_plan_schedule(plan) -> list:

@@ -7,6 +7,7 @@
 #include <cstring>
 #include <memory>
 #include <string>
+#include <vector>
 
 #include "dfg.h"
 #include "runtime.hpp"
@@ -192,6 +193,20 @@ int dfg_execute(dfg_plan plan, void* out, int out_on_device, void* stream) {
   return guard([&] {
     if (!plan) dfg::fail(DFG_E_INVALID, "null plan");
     plan->p->execute(out, out_on_device != 0, static_cast<cudaStream_t>(stream));
+  });
+}
+
+int dfg_execute_blocks(dfg_plan const* plans, int n, void* const* outs, void* stream) {
+  return guard([&] {
+    if (!plans || !outs || n < 1) dfg::fail(DFG_E_INVALID, "need n >= 1 plans and outputs");
+    std::vector<dfg::PlanImpl*> ps;
+    std::vector<void*> os;
+    for (int b = 0; b < n; ++b) {
+      if (!plans[b] || !outs[b]) dfg::fail(DFG_E_INVALID, "null plan or output");
+      ps.push_back(plans[b]->p.get());
+      os.push_back(outs[b]);
+    }
+    dfg::execute_blocks(ps, os, static_cast<cudaStream_t>(stream));
   });
 }
 

@@ -195,17 +195,107 @@ __device__ __forceinline__ void dfg_plane(const DfgCol& C, DfgRing& R, unsigned&
   cur_full = nxt_full;
 }
 
-extern "C" __global__ void __launch_bounds__((DFG_NCW + 1) * 32, DFG_CTAS)
-    dfg_fused_tma(const __grid_constant__ DfgTmaParams TP) {
+// Producer side of one item (x-tile, y-tile, z-chunk) of mesh TP: the
+// pre-plane, planes kb..ke-1 and the post-plane, clamped to the global mesh (R1).
+__device__ __forceinline__ void dfg_produce_item(const DfgTmaParams& TP, long long item, DfgRing& W) {
   const DfgParams& P = TP.p;
+  const long long tx_ = item % P.tiles_x;
+  const long long rest = item / P.tiles_x;
+  const long long ty_ = rest % P.tiles_y;
+  const long long zc = rest / P.tiles_y;
+  // input coordinates include the block's x/y ghost columns / rows
+  const int x0 = (int)(tx_ * DFG_TX) - DFG_HX + (int)P.gx;
+  const int y0 = (int)(ty_ * DFG_NCW) - 1 + (int)P.gy;
+  const long long kb = P.kbeg + zc * P.kz;
+  const long long ke = min(kb + (long long)P.kz, P.kend);
+  for (long long q = kb - 1; q <= ke; ++q) {
+    const long long pg = max(0LL, min(q, P.NZ - 1));
+    // wait until every consumer released this slot (the producer runs
+    // ahead; the suspend hint keeps it off the issue slots)
+    dfg_mbar_wait(DFG_EMPTY(W.full), W.phase ^ 1u, 0x100000u);
+    dfg_mbar_expect_tx(W.full, (unsigned)(DFG_NTF * DFG_TILE_ELEMS * sizeof(DFG_T)));
+    const int zl = (int)(pg - P.k0 + P.ghost);
+#pragma unroll
+    for (int f = 0; f < DFG_NTF; ++f) dfg_tma_load3(W.tile + f * DFG_TILE_BYTES, &TP.map[f], W.full, x0, y0, zl);
+    W.advance();
+  }
+}
+
+// Consumer side of one item: warp w computes tile row w.
+__device__ __forceinline__ void dfg_consume_item(const DfgTmaParams& TP, long long item, DfgRing& R, DfgCol& C,
+                                                 int warp, int lane) {
+  const DfgParams& P = TP.p;
+  const long long plane = P.nx * P.ny;
+  const unsigned c0 = DFG_HX + DFG_VEC * lane;
+  const unsigned r = 1 + warp;
+  const long long tx_ = item % P.tiles_x;
+  const long long rest = item / P.tiles_x;
+  const long long ty_ = rest % P.tiles_y;
+  const long long zc = rest / P.tiles_y;
+  const long long i = tx_ * DFG_TX + DFG_VEC * lane;
+  const long long j = ty_ * DFG_NCW + warp;
+  const long long kb = P.kbeg + zc * P.kz;
+  const long long ke = min(kb + (long long)P.kz, P.kend);
+  C.act = (i < P.nx) && (j < P.ny);
+  const long long ic = min(i, P.nx - DFG_VEC);
+  const long long jc = min(j, P.ny - 1);
+#pragma unroll
+  for (int h = 0; h < DFG_NPAIR; ++h) {
+    // spacing tables are indexed globally (blocks: i0 / j0 offsets)
+    const long long a = P.i0 + ic + h * DFG_LANES, b = P.i0 + ic + h * DFG_LANES + DFG_LANES - 1;
+    C.ndx[h] = dfg2_mk(__ldg(P.tx + DFG_NDSEG_X * P.NX + a), __ldg(P.tx + DFG_NDSEG_X * P.NX + b));
+    C.rx[h] = dfg2_mk(__ldg(P.tx + P.NX + a), __ldg(P.tx + P.NX + b));
+  }
+  C.ndy = dfg2_splat(__ldg(P.ty + DFG_NDSEG_Y * P.NY + P.j0 + jc));
+  C.ry = dfg2_splat(__ldg(P.ty + P.NY + P.j0 + jc));
+  // one-sided differences only at the GLOBAL mesh ends (reading R1)
+  const long long ig = P.i0 + i, jg = P.j0 + j;
+  const unsigned cxm = (ig == 0) ? c0 : c0 - 1;
+  const unsigned cxp = (ig + DFG_VEC >= P.NX) ? c0 + DFG_VEC - 1 : c0 + DFG_VEC;
+  const unsigned rm = (jg == 0) ? r : r - 1;
+  const unsigned rp = (jg >= P.NY - 1) ? r : r + 1;
+  const unsigned TS = (unsigned)sizeof(DFG_T);
+  C.off_c = (r * DFG_ROWW + c0) * TS;
+  C.off_xm = (r * DFG_ROWW + cxm) * TS;
+  C.off_xp = (r * DFG_ROWW + cxp) * TS;
+  C.off_ym = (rm * DFG_ROWW + c0) * TS;
+  C.off_yp = (rp * DFG_ROWW + c0) * TS;
+  const long long cell0 = (kb - P.k0) * plane + jc * P.nx + ic;
+  DFG_T* outp = P.out + cell0 * DFG_OUTW;
+  const DFG_T* tzp = P.tz + kb;
+
+  DFG_T zq[3][DFG_NSF][DFG_VEC];
+  // pre-plane (clamped): its centre becomes z-1 of plane kb
+  dfg_mbar_wait(R.full, R.phase, 0x100000u);
+#pragma unroll
+  for (int f = 0; f < DFG_NSF; ++f) dfg_lds16(zq[0][f], R.tile + f * DFG_TILE_BYTES + C.off_c);
+  dfg_mbar_arrive(DFG_EMPTY(R.full));
+  R.advance();
+  dfg_mbar_wait(R.full, R.phase, 0x100000u);
+  unsigned cur_tile = R.tile, cur_full = R.full;
+#pragma unroll
+  for (int f = 0; f < DFG_NSF; ++f) dfg_lds16(zq[1][f], cur_tile + f * DFG_TILE_BYTES + C.off_c);
+  R.advance();
+  long long k = kb;
+  for (; k + 3 <= ke; k += 3) {
+    dfg_plane<0, 1, 2>(C, R, cur_tile, cur_full, zq, outp, plane, tzp, P.NZ);
+    dfg_plane<1, 2, 0>(C, R, cur_tile, cur_full, zq, outp, plane, tzp, P.NZ);
+    dfg_plane<2, 0, 1>(C, R, cur_tile, cur_full, zq, outp, plane, tzp, P.NZ);
+  }
+  if (k < ke) {
+    dfg_plane<0, 1, 2>(C, R, cur_tile, cur_full, zq, outp, plane, tzp, P.NZ);
+    if (k + 1 < ke) dfg_plane<1, 2, 0>(C, R, cur_tile, cur_full, zq, outp, plane, tzp, P.NZ);
+  }
+  // the post-plane stage was read for its centre only
+  dfg_mbar_arrive(DFG_EMPTY(cur_full));
+}
+
+__device__ __forceinline__ unsigned dfg_ring_init() {
   // dynamic shared memory starts at the (1024-aligned) base of the CTA's
   // window: no static __shared__ in this kernel
   extern __shared__ __align__(1024) unsigned char dfg_smem_raw[];
   const unsigned smem = dfg_smem(dfg_smem_raw);
   const unsigned full0 = smem + DFG_STAGES * DFG_STAGE_BYTES;  // full[s] at full0 + 8s, empty[s] = full[s] + 8*STAGES
-  const int warp = threadIdx.x >> 5;
-  const int lane = threadIdx.x & 31;
-
   if (threadIdx.x == 0) {
     for (int s = 0; s < DFG_STAGES; ++s) {
       dfg_mbar_init(full0 + 8 * s, 1);
@@ -214,7 +304,15 @@ extern "C" __global__ void __launch_bounds__((DFG_NCW + 1) * 32, DFG_CTAS)
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   }
   __syncthreads();
+  return smem;
+}
 
+extern "C" __global__ void __launch_bounds__((DFG_NCW + 1) * 32, DFG_CTAS)
+    dfg_fused_tma(const __grid_constant__ DfgTmaParams TP) {
+  const unsigned smem = dfg_ring_init();
+  const unsigned full0 = smem + DFG_STAGES * DFG_STAGE_BYTES;
+  const int warp = threadIdx.x >> 5;
+  const int lane = threadIdx.x & 31;
   if (warp == DFG_NCW) {
     // ---------------- producer: one lane issues all TMA loads
     if (lane == 0) {
@@ -222,101 +320,52 @@ extern "C" __global__ void __launch_bounds__((DFG_NCW + 1) * 32, DFG_CTAS)
         asm volatile("prefetch.tensormap [%0];" ::"l"(reinterpret_cast<unsigned long long>(&TP.map[f]))
                      : "memory");
       DfgRing W{smem, full0, 0u, 0, smem, full0};
-      for (long long item = blockIdx.x; item < P.items; item += gridDim.x) {
-        const long long tx_ = item % P.tiles_x;
-        const long long rest = item / P.tiles_x;
-        const long long ty_ = rest % P.tiles_y;
-        const long long zc = rest / P.tiles_y;
-        // input coordinates include the block's x/y ghost columns / rows
-        const int x0 = (int)(tx_ * DFG_TX) - DFG_HX + (int)P.gx;
-        const int y0 = (int)(ty_ * DFG_NCW) - 1 + (int)P.gy;
-        const long long kb = P.kbeg + zc * P.kz;
-        const long long ke = min(kb + (long long)P.kz, P.kend);
-        // pre-plane, kb..ke-1, post-plane; clamped to the global mesh (R1)
-        for (long long q = kb - 1; q <= ke; ++q) {
-          const long long pg = max(0LL, min(q, P.NZ - 1));
-          // wait until every consumer released this slot (the producer runs
-          // ahead; the suspend hint keeps it off the issue slots)
-          dfg_mbar_wait(DFG_EMPTY(W.full), W.phase ^ 1u, 0x100000u);
-          dfg_mbar_expect_tx(W.full, (unsigned)(DFG_NTF * DFG_TILE_ELEMS * sizeof(DFG_T)));
-          const int zl = (int)(pg - P.k0 + P.ghost);
-#pragma unroll
-          for (int f = 0; f < DFG_NTF; ++f) dfg_tma_load3(W.tile + f * DFG_TILE_BYTES, &TP.map[f], W.full, x0, y0, zl);
-          W.advance();
-        }
+      for (long long item = blockIdx.x; item < TP.p.items; item += gridDim.x) dfg_produce_item(TP, item, W);
+    }
+    return;
+  }
+  // ------------------- consumers
+  DfgRing R{smem, full0, 0u, 0, smem, full0};
+  DfgCol C;
+  C.Z = dfg2_splat(TP.p.nzero);
+  for (long long item = blockIdx.x; item < TP.p.items; item += gridDim.x) dfg_consume_item(TP, item, R, C, warp, lane);
+}
+
+// Several meshes of one network in one launch (VisIt-style blocks of a
+// device, the paper's 12 sub-grids per GPU, L315): block b's parameters and
+// tensor maps live in global memory; the persistent CTAs walk the
+// concatenated item space, first[b] = first item of block b, first[nb] = total.
+struct DfgMulti {
+  const DfgTmaParams* blocks;
+  const long long* first;
+  int nb;
+};
+
+extern "C" __global__ void __launch_bounds__((DFG_NCW + 1) * 32, DFG_CTAS)
+    dfg_fused_tma_multi(const __grid_constant__ DfgMulti M) {
+  const unsigned smem = dfg_ring_init();
+  const unsigned full0 = smem + DFG_STAGES * DFG_STAGE_BYTES;
+  const int warp = threadIdx.x >> 5;
+  const int lane = threadIdx.x & 31;
+  const long long total = M.first[M.nb];
+  if (warp == DFG_NCW) {
+    if (lane == 0) {
+      DfgRing W{smem, full0, 0u, 0, smem, full0};
+      int b = 0;
+      for (long long item = blockIdx.x; item < total; item += gridDim.x) {
+        while (item >= M.first[b + 1]) ++b;  // items only grow: the block index too
+        dfg_produce_item(M.blocks[b], item - M.first[b], W);
       }
     }
     return;
   }
-
-  // ------------------- consumers: warp w computes tile row w
   DfgRing R{smem, full0, 0u, 0, smem, full0};
   DfgCol C;
-  C.Z = dfg2_splat(P.nzero);
-  const long long plane = P.nx * P.ny;
-  const unsigned c0 = DFG_HX + DFG_VEC * lane;
-  const unsigned r = 1 + warp;
-  for (long long item = blockIdx.x; item < P.items; item += gridDim.x) {
-    const long long tx_ = item % P.tiles_x;
-    const long long rest = item / P.tiles_x;
-    const long long ty_ = rest % P.tiles_y;
-    const long long zc = rest / P.tiles_y;
-    const long long i = tx_ * DFG_TX + DFG_VEC * lane;
-    const long long j = ty_ * DFG_NCW + warp;
-    const long long kb = P.kbeg + zc * P.kz;
-    const long long ke = min(kb + (long long)P.kz, P.kend);
-    C.act = (i < P.nx) && (j < P.ny);
-    const long long ic = min(i, P.nx - DFG_VEC);
-    const long long jc = min(j, P.ny - 1);
-#pragma unroll
-    for (int h = 0; h < DFG_NPAIR; ++h) {
-      // spacing tables are indexed globally (blocks: i0 / j0 offsets)
-      const long long a = P.i0 + ic + h * DFG_LANES, b = P.i0 + ic + h * DFG_LANES + DFG_LANES - 1;
-      C.ndx[h] = dfg2_mk(__ldg(P.tx + DFG_NDSEG_X * P.NX + a), __ldg(P.tx + DFG_NDSEG_X * P.NX + b));
-      C.rx[h] = dfg2_mk(__ldg(P.tx + P.NX + a), __ldg(P.tx + P.NX + b));
-    }
-    C.ndy = dfg2_splat(__ldg(P.ty + DFG_NDSEG_Y * P.NY + P.j0 + jc));
-    C.ry = dfg2_splat(__ldg(P.ty + P.NY + P.j0 + jc));
-    // one-sided differences only at the GLOBAL mesh ends (reading R1)
-    const long long ig = P.i0 + i, jg = P.j0 + j;
-    const unsigned cxm = (ig == 0) ? c0 : c0 - 1;
-    const unsigned cxp = (ig + DFG_VEC >= P.NX) ? c0 + DFG_VEC - 1 : c0 + DFG_VEC;
-    const unsigned rm = (jg == 0) ? r : r - 1;
-    const unsigned rp = (jg >= P.NY - 1) ? r : r + 1;
-    const unsigned TS = (unsigned)sizeof(DFG_T);
-    C.off_c = (r * DFG_ROWW + c0) * TS;
-    C.off_xm = (r * DFG_ROWW + cxm) * TS;
-    C.off_xp = (r * DFG_ROWW + cxp) * TS;
-    C.off_ym = (rm * DFG_ROWW + c0) * TS;
-    C.off_yp = (rp * DFG_ROWW + c0) * TS;
-    const long long cell0 = (kb - P.k0) * plane + jc * P.nx + ic;
-    DFG_T* outp = P.out + cell0 * DFG_OUTW;
-    const DFG_T* tzp = P.tz + kb;
-
-    DFG_T zq[3][DFG_NSF][DFG_VEC];
-    // pre-plane (clamped): its centre becomes z-1 of plane kb
-    dfg_mbar_wait(R.full, R.phase, 0x100000u);
-#pragma unroll
-    for (int f = 0; f < DFG_NSF; ++f) dfg_lds16(zq[0][f], R.tile + f * DFG_TILE_BYTES + C.off_c);
-    dfg_mbar_arrive(DFG_EMPTY(R.full));
-    R.advance();
-    dfg_mbar_wait(R.full, R.phase, 0x100000u);
-    unsigned cur_tile = R.tile, cur_full = R.full;
-#pragma unroll
-    for (int f = 0; f < DFG_NSF; ++f) dfg_lds16(zq[1][f], cur_tile + f * DFG_TILE_BYTES + C.off_c);
-    R.advance();
-    long long k = kb;
-    for (; k + 3 <= ke; k += 3) {
-      dfg_plane<0, 1, 2>(C, R, cur_tile, cur_full, zq, outp, plane, tzp, P.NZ);
-      dfg_plane<1, 2, 0>(C, R, cur_tile, cur_full, zq, outp, plane, tzp, P.NZ);
-      dfg_plane<2, 0, 1>(C, R, cur_tile, cur_full, zq, outp, plane, tzp, P.NZ);
-    }
-    if (k < ke) {
-      dfg_plane<0, 1, 2>(C, R, cur_tile, cur_full, zq, outp, plane, tzp, P.NZ);
-      if (k + 1 < ke) dfg_plane<1, 2, 0>(C, R, cur_tile, cur_full, zq, outp, plane, tzp, P.NZ);
-    }
-    // the post-plane stage was read for its centre only
-    dfg_mbar_arrive(DFG_EMPTY(cur_full));
+  C.Z = dfg2_splat(M.blocks[0].p.nzero);
+  int b = 0;
+  for (long long item = blockIdx.x; item < total; item += gridDim.x) {
+    while (item >= M.first[b + 1]) ++b;
+    dfg_consume_item(M.blocks[b], item - M.first[b], R, C, warp, lane);
   }
 }
 #endif

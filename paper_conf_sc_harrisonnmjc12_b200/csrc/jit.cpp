@@ -144,7 +144,10 @@ LoadedModule load_module(const Cubin& c, bool has_stencil, bool has_tma) {
     DFG_CU(drv().ModuleGetFunction(&m.pointwise, m.mod, "dfg_fused_pointwise"));
   } else {
     DFG_CU(drv().ModuleGetFunction(&m.general, m.mod, "dfg_fused_general"));
-    if (has_tma) DFG_CU(drv().ModuleGetFunction(&m.tma, m.mod, "dfg_fused_tma"));
+    if (has_tma) {
+      DFG_CU(drv().ModuleGetFunction(&m.tma, m.mod, "dfg_fused_tma"));
+      DFG_CU(drv().ModuleGetFunction(&m.tma_multi, m.mod, "dfg_fused_tma_multi"));
+    }
   }
   return m;
 }

@@ -23,6 +23,7 @@ const Cubin& nvrtc_compile(const std::string& source, const std::string& name);
 struct LoadedModule {
   CUmodule mod = nullptr;
   CUfunction pointwise = nullptr, general = nullptr, tma = nullptr;
+  CUfunction tma_multi = nullptr;  // several meshes per launch (dfg_execute_blocks)
 };
 
 // Load into the current context (requires a device).

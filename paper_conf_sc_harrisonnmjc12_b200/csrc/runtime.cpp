@@ -826,6 +826,7 @@ std::unique_ptr<PlanImpl> compile_plan(std::shared_ptr<MeshImpl> mesh, const std
       size_t smem = fused_tma_smem_bytes(mesh->dt, int(plan->fsrc.layout.stencil_inputs.size() + plan->fsrc.layout.point_inputs.size()), plan->fsrc.cfg.ncw,
                                          plan->fsrc.cfg.stages);
       DFG_CU(drv().FuncSetAttribute(plan->mod.tma, CU_FUNC_ATTRIBUTE_MAX_DYNAMIC_SHARED_SIZE_BYTES, int(smem)));
+      DFG_CU(drv().FuncSetAttribute(plan->mod.tma_multi, CU_FUNC_ATTRIBUTE_MAX_DYNAMIC_SHARED_SIZE_BYTES, int(smem)));
     }
   }
   return plan;
@@ -1169,6 +1170,113 @@ void PlanImpl::launch_fused(const std::vector<const void*>& fptr, void* dout, co
     last_variant = 2;
   }
   st.kernel_count += 1;
+}
+
+// Several fused plans of one network (one generated module) in a single
+// launch of dfg_fused_tma_multi: per-block parameter blobs (tensor maps +
+// DfgParams, the layout of DfgTmaParams) go to device memory, the persistent
+// CTAs walk the concatenated item space.  Plans that cannot share the launch
+// run one by one (same results).
+void execute_blocks(const std::vector<PlanImpl*>& plans, const std::vector<void*>& outs, cudaStream_t s) {
+  if (plans.empty()) return;
+  PlanImpl& p0 = *plans[0];
+  const MeshImpl& m0 = *p0.mesh;
+  const size_t ts = dsize(m0.dt);
+  const int vec = int(16 / ts);
+  const FusedLayout& L = p0.fsrc.layout;
+  const char* force = std::getenv("DFG_FUSED_KERNEL");
+  bool batch = plans.size() > 1 && p0.strategy == DFG_FUSED && p0.mod.tma_multi && p0.fsrc.cfg.has_tma &&
+               !(force && !std::strcmp(force, "general"));
+  std::vector<std::vector<const void*>> fptrs(plans.size());
+  for (size_t b = 0; b < plans.size() && batch; ++b) {
+    PlanImpl& p = *plans[b];
+    const MeshImpl& m = *p.mesh;
+    const bool halo = (m.k0 > 0 || m.k0 + m.nzl < m.NZ) && !m.ghosts_supplied;
+    batch = p.strategy == DFG_FUSED && p.fsrc.source == p0.fsrc.source && m.device == m0.device && !halo &&
+            m.nx % vec == 0 && m.px() % vec == 0 && m.gx() % vec == 0 && aligned16(outs[b]);
+    std::vector<int> ins = L.stencil_inputs;
+    ins.insert(ins.end(), L.point_inputs.begin(), L.point_inputs.end());
+    for (int i : ins) {
+      auto it = m.fields.find(p.dag.inputs[size_t(i)]);
+      if (it == m.fields.end() || !it->second.ptr) fail(DFG_E_UNBOUND, "input '" + p.dag.inputs[size_t(i)] + "' is not bound");
+      batch = batch && it->second.on_device && aligned16(it->second.ptr);
+      fptrs[b].push_back(it->second.ptr);
+    }
+  }
+  if (!batch) {
+    for (size_t b = 0; b < plans.size(); ++b) plans[b]->execute(outs[b], true, s);
+    return;
+  }
+  DFG_CUDA(cudaSetDevice(m0.device));
+  const int ncw = p0.fsrc.cfg.ncw;
+  const int nsf = int(L.stencil_inputs.size() + L.point_inputs.size());
+  const size_t smem = fused_tma_smem_bytes(m0.dt, nsf, ncw, p0.fsrc.cfg.stages);
+  int occ = 1;
+  DFG_CU(drv().OccupancyMaxActiveBlocksPerMultiprocessor(&occ, p0.mod.tma_multi, (ncw + 1) * 32, smem));
+  const int64_t slots = int64_t(sm_count(m0.device)) * std::max(occ, 1);
+  // one z-chunk length for the batch: whole rounds of the concatenated items
+  // against the two halo planes per chunk (as launch_fused)
+  int64_t max_range = 1;
+  for (auto* p : plans) max_range = std::max(max_range, p->mesh->nzl);
+  auto items_for = [&](int64_t kz) {
+    int64_t t = 0;
+    for (auto* p : plans) {
+      const MeshImpl& m = *p->mesh;
+      t += int64_t((m.nx + 32 * vec - 1) / (32 * vec)) * ((m.ny + ncw - 1) / ncw) * ((m.nzl + kz - 1) / kz);
+    }
+    return t;
+  };
+  int64_t best_kz = max_range, best_cost = INT64_MAX;
+  for (int64_t kz = 1; kz <= max_range; kz = kz < 8 ? kz + 1 : kz + std::max<int64_t>(1, kz / 8)) {
+    const int64_t cost = (items_for(kz) + slots - 1) / slots * (kz + 2 + 4);
+    if (cost < best_cost) best_cost = cost, best_kz = kz;
+  }
+  // blobs: DfgTmaParams per block, 64-byte aligned stride
+  std::vector<std::vector<uint64_t>> words;
+  std::vector<int64_t> first{0};
+  size_t wmax = 0;
+  for (size_t b = 0; b < plans.size(); ++b) {
+    const MeshImpl& m = *plans[b]->mesh;
+    const SlabView v = SlabView::of(m);
+    const int tx = int((m.nx + 32 * vec - 1) / (32 * vec)), ty = int((m.ny + ncw - 1) / ncw);
+    const int64_t items = int64_t(tx) * ty * ((m.nzl + best_kz - 1) / best_kz);
+    words.push_back(pack_params(fptrs[b], outs[b], m.dev_tab[0], m.dev_tab[1], m.dev_tab[2], v, m.k0, m.k0 + m.nzl,
+                                items, tx, ty, int(best_kz), 0));
+    wmax = std::max(wmax, words.back().size());
+    first.push_back(first.back() + items);
+  }
+  const size_t stride = (size_t(nsf) * 128 + wmax * 8 + 63) / 64 * 64;
+  std::vector<unsigned char> host(stride * plans.size() + sizeof(int64_t) * first.size(), 0);
+  for (size_t b = 0; b < plans.size(); ++b) {
+    unsigned char* blob = host.data() + stride * b;
+    const SlabView v = SlabView::of(*plans[b]->mesh);
+    for (int f = 0; f < nsf; ++f) encode_map(reinterpret_cast<CUtensorMap*>(blob + 128 * f), v, const_cast<void*>(fptrs[b][size_t(f)]), ncw);
+    std::memcpy(blob + 128 * nsf, words[b].data(), words[b].size() * 8);
+  }
+  std::memcpy(host.data() + stride * plans.size(), first.data(), sizeof(int64_t) * first.size());
+  void* dev = dev_alloc(host.size(), m0.device, s);
+  DFG_CUDA(cudaMemcpyAsync(dev, host.data(), host.size(), cudaMemcpyHostToDevice, s));  // pageable: staged now
+  struct {
+    const void* blocks;
+    const void* first;
+    int nb;
+  } arg{dev, static_cast<char*>(dev) + stride * plans.size(), int(plans.size())};
+  void* args[] = {&arg};
+  DFG_CUDA(cudaEventRecord(p0.ev0, s));
+  auto ke = p0.kernel_events();
+  DFG_CUDA(cudaEventRecord(ke.first, s));
+  const unsigned grid = unsigned(std::max<int64_t>(1, std::min(first.back(), slots)));
+  DFG_CU(drv().LaunchKernel(p0.mod.tma_multi, grid, 1, 1, (ncw + 1) * 32, 1, 1, unsigned(smem), s, args, nullptr));
+  DFG_CUDA(cudaEventRecord(ke.second, s));
+  DFG_CUDA(cudaEventRecord(p0.ev1, s));
+  DFG_CUDA(cudaFreeAsync(dev, s));
+  DFG_CUDA(cudaGetLastError());
+  p0.timed = true;
+  p0.st.kernel_count += 1;
+  for (auto* p : plans) {
+    p->st.executes += 1;
+    p->last_variant = 4;
+  }
 }
 
 // ----------------------------------------------------------- streamed

@@ -120,7 +120,7 @@ struct PlanImpl {
   FusedSource fsrc;
   LoadedModule mod;
   int regs = 0, spill = 0;
-  int last_variant = 0;  // 1 TMA, 2 general, 3 pointwise
+  int last_variant = 0;  // 1 TMA, 2 general, 3 pointwise, 4 TMA multi-block (dfg_execute_blocks)
   dfg_stats st{};
   cudaEvent_t ev0 = nullptr, ev1 = nullptr;
   bool timed = false;
@@ -158,6 +158,11 @@ struct PlanImpl {
   void exec_roundtrip(void* out, bool out_dev, cudaStream_t s);
   void halo_exchange(const std::vector<int>& inputs, cudaStream_t s);
 };
+
+// Fused plans of one network on several meshes (VisIt blocks of a device) in
+// one launch when they share the generated module and the TMA layout; else
+// one execute per plan.  Outputs are device pointers.
+void execute_blocks(const std::vector<PlanImpl*>& plans, const std::vector<void*>& outs, cudaStream_t s);
 
 std::unique_ptr<PlanImpl> compile_plan(std::shared_ptr<MeshImpl> mesh, const std::string& expr, dfg_strategy s,
                                        size_t cap);

@@ -359,6 +359,7 @@ def test_visit_blocks_with_ghost_shells(shape, split, prog, strategy, pitch):
     nx, ny, nz = shape
     cuts = [np.linspace(0, n, s + 1).astype(int) for n, s in zip(shape, split)]
     got = np.empty_like(whole)
+    blocks = []
     pad = {n: np.pad(a, 1, mode="edge") for n, a in f.items()}   # ghosts at the global ends are ignored
     for a in range(split[0]):
         for b in range(split[1]):
@@ -384,7 +385,19 @@ def test_visit_blocks_with_ghost_shells(shape, split, prog, strategy, pitch):
                 if pitch == "padded" and bx % 4 == 0 and prog != "velmag":
                     assert p.info()["variant"] == 1          # TMA kernel on the padded shell
                 got[k0:k1, j0:j1, i0:i1] = o.cpu().numpy()
+                blocks.append((p, torch.full_like(o, float("nan")), (k0, k1, j0, j1, i0, i1), m, keep))
     assert np.array_equal(got, whole)
+    # all blocks in one launch (dfg_execute_blocks): the same bits
+    dfg.execute_blocks([b[0] for b in blocks], [b[1] for b in blocks])
+    torch.cuda.synchronize()
+    got2 = np.full_like(whole, np.nan)
+    for p, o, (k0, k1, j0, j1, i0, i1), _, _ in blocks:
+        got2[k0:k1, j0:j1, i0:i1] = o.cpu().numpy()
+    assert np.array_equal(got2, whole)
+    one_launch = (strategy == "fused" and pitch == "padded" and prog != "velmag" and len(blocks) > 1
+                  and all((b[2][5] - b[2][4]) % 4 == 0 for b in blocks))
+    if one_launch:
+        assert blocks[0][0].info()["variant"] == 4
 
 
 def test_memory_cap():

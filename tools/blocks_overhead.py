@@ -76,6 +76,8 @@ def main():
             p.execute(o)
 
     t_blocks = timeit(blocks)
+    t_batched = timeit(lambda: dfg.execute_blocks(plans, outs))
+    batched_variant = plans[0].info()["variant"]
     whole = dfg.Mesh(x, y, z)
     wf = {c: synth.rt_velocity(c, x64, y64, z64, None, torch.float32, "cuda") for c in "uvw"}
     for c, f in wf.items():
@@ -86,6 +88,8 @@ def main():
     same = bool(torch.equal(torch.cat(outs), wo))
     cells = bx * by * NZ
     print(json.dumps({"blocks": B, "block": [bx, by, bz], "row_pitch": rp, "x_offset": xo, "cells": cells, "ms_blocks": t_blocks,
+                      "ms_batched": t_batched, "batched_variant": batched_variant,
+                      "gcells_s_batched": cells / t_batched / 1e6,
                       "ms_one_mesh": t_whole, "overhead": t_blocks / t_whole - 1,
                       "blocks_variant": plans[0].info()["variant"], "bit_identical": same,
                       "gcells_s_blocks": cells / t_blocks / 1e6, "gcells_s_one_mesh": cells / t_whole / 1e6}))
