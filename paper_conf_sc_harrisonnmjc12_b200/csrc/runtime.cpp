@@ -1160,9 +1160,15 @@ void PlanImpl::launch_fused(const std::vector<const void*>& fptr, void* dout, co
     DFG_CUDA(cudaEventRecord(ke.second, s));
     last_variant = 1;
   } else {
-    auto w = pack_params(fptr, dout, tab[0], tab[1], tab[2], m, kbeg, kend, 0, 0, 0, 0, 0);
+    // z-marching columns: enough (column, z-chunk) units to fill the device
+    // (~2048 threads per SM), each chunk as long as that allows
+    const int64_t cols = m.nx * m.ny, range = kend - kbeg;
+    const int64_t chunks = std::max<int64_t>(1, std::min<int64_t>(range, (int64_t(sms) * 2048 + cols - 1) / cols));
+    const int64_t kz = (range + chunks - 1) / chunks;
+    const int64_t units = cols * ((range + kz - 1) / kz);
+    auto w = pack_params(fptr, dout, tab[0], tab[1], tab[2], m, kbeg, kend, 0, 0, 0, int(kz), 0);
     void* args[] = {w.data()};
-    unsigned grid = unsigned(std::max<long long>(1, std::min<long long>((N + 255) / 256, sms * 8LL)));
+    unsigned grid = unsigned(std::max<long long>(1, std::min<long long>((units + 255) / 256, sms * 8LL)));
     auto ke = kernel_events();
     DFG_CUDA(cudaEventRecord(ke.first, s));
     DFG_CU(drv().LaunchKernel(mod.general, grid, 1, 1, 256, 1, 1, 0, s, args, nullptr));

@@ -18,8 +18,8 @@
 //
 // Kernels:
 //   dfg_fused_pointwise -- networks without grad3d: flat, 16-byte I/O.
-//   dfg_fused_general   -- any layout: one cell per thread, clamped direct
-//                          loads (ragged nx, unaligned buffers).
+//   dfg_fused_general   -- any layout (ragged nx, pitched or unaligned
+//                          buffers): z-marching columns, direct loads.
 //   dfg_fused_tma       -- the B200 path: persistent CTAs march z-columns of
 //                          (32*VEC) x DFG_NCW cells; one producer warp streams
 //                          halo'd x-y tiles of every stencil field into a
@@ -164,44 +164,124 @@ extern "C" __global__ void __launch_bounds__(256) dfg_fused_pointwise(const DfgP
 
 #if DFG_NSF > 0
 // ------------------------------------------------------------- general
-extern "C" __global__ void __launch_bounds__(256) dfg_fused_general(const DfgParams P) {
+#ifndef DFG_GEN_MINB
+#if DFG_PAIRS_F32
+#define DFG_GEN_MINB 3   // 24 warps per SM (<= 85 registers): the direct loads need the occupancy
+#else
+#define DFG_GEN_MINB 2   // fp64 would spill at 3
+#endif
+#endif
+// Any layout (ragged nx, pitched or unaligned buffers): a thread owns one
+// (i, j) column of a z-chunk of P.kz planes and marches it, keeping z-1 / z /
+// z+1 of every stencil field in registers; x/y neighbours are direct loads
+// (L1 / L2 hits: the neighbouring threads read the same lines).  fp32: planes
+// k and k+1 are the two lanes of a pair (their x/y spacings are shared).
+extern "C" __global__ void __launch_bounds__(256, DFG_GEN_MINB) dfg_fused_general(const DfgParams P) {
   const long long plane = P.nx * P.ny;          // output plane (owned cells)
   const long long in_plane = P.px * P.py;       // input plane (with x/y ghosts)
-  const long long gx = P.gx, gy = P.gy;
-  const long long total = plane * (P.kend - P.kbeg);
+  const long long range = P.kend - P.kbeg;
+  const long long kz = P.kz > 0 ? (long long)P.kz : range;
+  const long long units = plane * ((range + kz - 1) / kz);
   const long long stride = (long long)gridDim.x * blockDim.x;
   const dfg2 Z = dfg2_splat(P.nzero);
-  for (long long c = (long long)blockIdx.x * blockDim.x + threadIdx.x; c < total; c += stride) {
-    const long long il = c % P.nx;
-    const long long t = c / P.nx;
-    const long long jl = t % P.ny;
-    const long long kg = P.kbeg + t / P.ny;
-    const long long kl = kg - P.k0;
+  for (long long u = (long long)blockIdx.x * blockDim.x + threadIdx.x; u < units; u += stride) {
+    const long long col = u % plane, chunk = u / plane;
+    const long long il = col % P.nx, jl = col / P.nx;
+    const long long kb = P.kbeg + chunk * kz, ke = min(kb + kz, P.kend);
     const long long i = P.i0 + il, j = P.j0 + jl;  // global indices: clamp only at the mesh ends
-    const long long base = ((kl + P.ghost) * P.py + jl + gy) * P.px + il + gx;
     const long long oxm = i > 0 ? 1 : 0, oxp = i < P.NX - 1 ? 1 : 0;
     const long long oym = j > 0 ? P.px : 0, oyp = j < P.NY - 1 ? P.px : 0;
-    const long long ozm = kg > 0 ? in_plane : 0, ozp = kg < P.NZ - 1 ? in_plane : 0;
-    dfg2 s[DFG_NSF_][7], gn[DFG_NSF_][3];
+    const long long cbase = (P.ghost - P.k0) * in_plane + (jl + P.gy) * P.px + il + P.gx;  // + kg * in_plane
+    const dfg2 ndx = dfg2_splat(P.tx[DFG_NDSEG_X * P.NX + i]), rx = dfg2_splat(P.tx[P.NX + i]);
+    const dfg2 ndy = dfg2_splat(P.ty[DFG_NDSEG_Y * P.NY + j]), ry = dfg2_splat(P.ty[P.NY + j]);
+    DFG_T zm[DFG_NSF_], zc[DFG_NSF_];   // planes max(k-1, 0) and k
 #pragma unroll
     for (int f = 0; f < DFG_NSF; ++f) {
-      const DFG_T* F = P.f[f];
-      const DFG_T v[7] = {F[base], F[base - oxm], F[base + oxp], F[base - oym], F[base + oyp], F[base - ozm],
-                          F[base + ozp]};
-#pragma unroll
-      for (int q = 0; q < 7; ++q) s[f][q] = dfg2_splat(v[q]);
-#pragma unroll
-      for (int a = 0; a < 3; ++a) gn[f][a] = dfg2_splat(dfg_sub(v[2 + 2 * a], v[1 + 2 * a]));
+      zm[f] = P.f[f][cbase + max(kb - 1, 0LL) * in_plane];
+      zc[f] = P.f[f][cbase + kb * in_plane];
     }
-    dfg2 p[DFG_NPF_];
+    long long k = kb;
+    for (; k + DFG_LANES <= ke; k += DFG_LANES) {
+      dfg2 s[DFG_NSF_][7], gn[DFG_NSF_][3];
+      DFG_T zn[DFG_NSF_];
 #pragma unroll
-    for (int f = 0; f < DFG_NPF; ++f) p[f] = dfg2_splat(P.f[DFG_NSF + f][base]);
-    dfg2 o[DFG_OUTW];
-    dfg_body(s, gn, p, dfg2_splat(P.tx[DFG_NDSEG_X * P.NX + i]), dfg2_splat(P.tx[P.NX + i]), dfg2_splat(P.ty[DFG_NDSEG_Y * P.NY + j]),
-             dfg2_splat(P.ty[P.NY + j]), dfg2_splat(P.tz[DFG_NDSEG_Z * P.NZ + kg]), dfg2_splat(P.tz[P.NZ + kg]), Z, o);
-    const long long ob = (kl * plane + jl * P.nx + il) * DFG_OUTW;
+      for (int f = 0; f < DFG_NSF; ++f) {
+        const DFG_T* F = P.f[f];
+        const long long b0 = cbase + k * in_plane;
+#if DFG_LANES == 2
+        const long long b1 = b0 + in_plane;
+        const DFG_T c1 = F[b1];                                        // plane k+1 (inside the chunk)
+        const DFG_T c2 = F[cbase + min(k + 2, P.NZ - 1) * in_plane];   // plane min(k+2, NZ-1)
+        s[f][0] = dfg2_mk(zc[f], c1);
+        s[f][1] = dfg2_mk(F[b0 - oxm], F[b1 - oxm]);
+        s[f][2] = dfg2_mk(F[b0 + oxp], F[b1 + oxp]);
+        s[f][3] = dfg2_mk(F[b0 - oym], F[b1 - oym]);
+        s[f][4] = dfg2_mk(F[b0 + oyp], F[b1 + oyp]);
+        s[f][5] = dfg2_mk(zm[f], zc[f]);
+        s[f][6] = dfg2_mk(c1, c2);
+        zm[f] = c1;
+        zn[f] = c2;
+#else
+        const DFG_T c1 = F[cbase + min(k + 1, P.NZ - 1) * in_plane];
+        s[f][0] = zc[f];
+        s[f][1] = F[b0 - oxm];
+        s[f][2] = F[b0 + oxp];
+        s[f][3] = F[b0 - oym];
+        s[f][4] = F[b0 + oyp];
+        s[f][5] = zm[f];
+        s[f][6] = c1;
+        zm[f] = zc[f];
+        zn[f] = c1;
+#endif
 #pragma unroll
-    for (int w = 0; w < DFG_OUTW; ++w) P.out[ob + w] = dfg2_get(o[w], 0);
+        for (int a = 0; a < 3; ++a) gn[f][a] = dfg2_sub(s[f][2 + 2 * a], s[f][1 + 2 * a], Z);
+      }
+#pragma unroll
+      for (int f = 0; f < DFG_NSF; ++f) zc[f] = zn[f];
+      dfg2 p[DFG_NPF_];
+#pragma unroll
+      for (int f = 0; f < DFG_NPF; ++f) {
+        const long long b0 = cbase + k * in_plane;
+        p[f] = dfg2_mk(P.f[DFG_NSF + f][b0], P.f[DFG_NSF + f][b0 + (DFG_LANES == 2 ? in_plane : 0)]);
+      }
+      const dfg2 ndz = dfg2_mk(P.tz[DFG_NDSEG_Z * P.NZ + k], P.tz[DFG_NDSEG_Z * P.NZ + k + DFG_LANES - 1]);
+      const dfg2 rz = dfg2_mk(P.tz[P.NZ + k], P.tz[P.NZ + k + DFG_LANES - 1]);
+      dfg2 o[DFG_OUTW];
+      dfg_body(s, gn, p, ndx, rx, ndy, ry, ndz, rz, Z, o);
+#pragma unroll
+      for (int l = 0; l < DFG_LANES; ++l) {
+        const long long ob = ((k + l - P.k0) * plane + col) * DFG_OUTW;
+#pragma unroll
+        for (int w = 0; w < DFG_OUTW; ++w) P.out[ob + w] = dfg2_get(o[w], l);
+      }
+    }
+#if DFG_LANES == 2
+    if (k < ke) {  // odd tail: plane k on both lanes, stored once
+      dfg2 s[DFG_NSF_][7], gn[DFG_NSF_][3];
+      const long long b0 = cbase + k * in_plane;
+#pragma unroll
+      for (int f = 0; f < DFG_NSF; ++f) {
+        const DFG_T* F = P.f[f];
+        s[f][0] = dfg2_splat(zc[f]);
+        s[f][1] = dfg2_splat(F[b0 - oxm]);
+        s[f][2] = dfg2_splat(F[b0 + oxp]);
+        s[f][3] = dfg2_splat(F[b0 - oym]);
+        s[f][4] = dfg2_splat(F[b0 + oyp]);
+        s[f][5] = dfg2_splat(zm[f]);
+        s[f][6] = dfg2_splat(F[cbase + min(k + 1, P.NZ - 1) * in_plane]);
+#pragma unroll
+        for (int a = 0; a < 3; ++a) gn[f][a] = dfg2_sub(s[f][2 + 2 * a], s[f][1 + 2 * a], Z);
+      }
+      dfg2 p[DFG_NPF_];
+#pragma unroll
+      for (int f = 0; f < DFG_NPF; ++f) p[f] = dfg2_splat(P.f[DFG_NSF + f][b0]);
+      dfg2 o[DFG_OUTW];
+      dfg_body(s, gn, p, ndx, rx, ndy, ry, dfg2_splat(P.tz[DFG_NDSEG_Z * P.NZ + k]), dfg2_splat(P.tz[P.NZ + k]), Z, o);
+      const long long ob = ((k - P.k0) * plane + col) * DFG_OUTW;
+#pragma unroll
+      for (int w = 0; w < DFG_OUTW; ++w) P.out[ob + w] = dfg2_get(o[w], 0);
+    }
+#endif
   }
 }
 #endif
