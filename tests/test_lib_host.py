@@ -278,3 +278,28 @@ def test_hybrid_planner_matches_oracle(dfg, prog, mode):
                                                     want.h2d_units, want.d2h_units)
             compared += 1
     assert compared >= 4
+
+
+def test_new_entry_points_validate_before_device_work(dfg):
+    """Argument errors of the block / batched / hybrid entry points are
+    reported as DFG_E_INVALID without touching a device."""
+    import ctypes
+    import numpy as np
+    x = np.linspace(0, 1, 9).astype(np.float32)
+    # row pitch below x_offset + nx + ghost, x_offset below the ghost width
+    for kw in ({"row_pitch": 9}, {"x_offset": 0, "row_pitch": 5}, {"x_offset": 11, "row_pitch": 12}):
+        with pytest.raises(dfg.DfgError) as e:
+            dfg.dfg_create_block(0, 8, 8, 8, x, x, x, 8, 8, 8, 0, 0, 0, 1, **kw)
+        assert e.value.name == "DFG_E_INVALID", kw
+    # dfg_execute_blocks: no plans / null entries
+    lib = dfg._dfg._lib
+    assert lib.dfg_execute_blocks(None, 0, None, None) == -1
+    plans = (ctypes.c_void_p * 1)(None)
+    outs = (ctypes.c_void_p * 1)(None)
+    assert lib.dfg_execute_blocks(plans, 1, outs, None) == -1
+    # dfg_plan_transfers / dfg_hybrid_model argument checks
+    n = ctypes.c_size_t(0)
+    assert lib.dfg_plan_transfers(None, None, 0, ctypes.byref(n)) == -1
+    with pytest.raises(dfg.DfgError) as e:
+        dfg.dfg_hybrid_model("r = (a + b) * (c + d)\n", ("a", "b", "c", "d"), True, 3, [2, 0, 1])
+    assert e.value.name == "DFG_E_INVALID"   # not a topological order
