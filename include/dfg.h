@@ -259,8 +259,12 @@ int dfg_reset_stats(dfg_plan plan);
  * kernel, bit a set = axis a uses the two-operation exact quotient (fp32,
  * every divisor of the axis verified at mesh creation),
  * clear = the three-operation correction (or IEEE / fast division when
- * DFG_FUSED_VARIANT selects them). */
-int dfg_plan_info(dfg_plan plan, int64_t out[9]);
+ * DFG_FUSED_VARIANT selects them), out[9] = tile rows per consumer warp of
+ * the TMA kernel (1, 2 or 4; 0 without one), out[10] / out[11] = its tile
+ * width (cells along x) / height (rows along y), out[12] = z-chunk length
+ * (planes per work item) of the last TMA launch (0 before one).  `out` must
+ * hold 13 entries. */
+int dfg_plan_info(dfg_plan plan, int64_t out[13]);
 
 /* Execution order of the plan's filters (ids of the canonical text).  Staged
  * plans run the paper's list order unless a dev_mem_cap rejected it and the

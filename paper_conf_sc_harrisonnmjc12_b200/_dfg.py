@@ -212,10 +212,10 @@ def dfg_reset_stats(plan):
 
 
 def dfg_plan_info(plan) -> dict:
-    out = (_I64 * 9)()
+    out = (_I64 * 13)()
     _check(_lib.dfg_plan_info(plan, out))
     keys = ("strategy", "width", "filters", "variant", "regs", "spill", "footprint_device", "footprint_host",
-            "div2_axes")
+            "div2_axes", "rows_per_warp", "tile_w", "tile_h", "kz")
     return dict(zip(keys, list(out)))
 
 

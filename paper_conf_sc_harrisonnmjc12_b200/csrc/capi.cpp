@@ -235,7 +235,7 @@ int dfg_reset_stats(dfg_plan plan) {
   });
 }
 
-int dfg_plan_info(dfg_plan plan, int64_t out[9]) {
+int dfg_plan_info(dfg_plan plan, int64_t out[13]) {
   return guard([&] {
     if (!plan || !out) dfg::fail(DFG_E_INVALID, "null argument");
     auto& p = *plan->p;
@@ -250,6 +250,11 @@ int dfg_plan_info(dfg_plan plan, int64_t out[9]) {
     out[6] = dfg::model(p.dag, p.strategy, false).units * unit;
     out[7] = dfg::model(p.dag, p.strategy, true).units * unit;
     out[8] = p.fsrc.cfg.div2;
+    const bool tma = p.fsrc.cfg.has_tma;
+    out[9] = tma ? p.fsrc.cfg.rpw : 0;
+    out[10] = tma ? dfg::tma_tile_w(m.dt, p.fsrc.cfg.rpw) : 0;
+    out[11] = tma ? dfg::tma_tile_h(p.fsrc.cfg.ncw, p.fsrc.cfg.rpw) : 0;
+    out[12] = p.last_kz;
   });
 }
 

@@ -28,6 +28,7 @@ struct FusedConfig {
   int ncw = 15;        // consumer warps per CTA (tile rows); +1 producer = 512 threads
   int stages = 0;      // smem ring depth (0: choose)
   int ctas = 1;        // resident CTAs per SM the TMA kernel is sized for
+  int rpw = 1;         // tile rows per consumer warp (1, 2, 4): tile = (32*VEC/rpw) x (ncw*rpw)
   bool has_tma = false;
 };
 
@@ -48,6 +49,21 @@ FusedSource generate_fused(const Dag& dag, int64_t nx, int64_t ny, int64_t nz, F
 const char* reference_program(const std::string& which, int* id);
 
 // Dynamic shared memory the TMA kernel needs for a config (bytes).
-size_t fused_tma_smem_bytes(DType dt, int nsf, int ncw, int stages);
+size_t fused_tma_smem_bytes(DType dt, int nsf, int ncw, int stages, int rpw = 1);
+
+// TMA kernel tile: tile_w cells along x, tile_h rows along y (fused_tma.cuh).
+inline int tma_tile_w(DType dt, int rpw) { return 32 * (dt == DType::F32 ? 4 : 2) / rpw; }
+inline int tma_tile_h(int ncw, int rpw) { return ncw * rpw; }
+
+// Rows per consumer warp for a mesh of nx x ny x nz cells on `slots`
+// persistent CTAs: the candidate (1, 2, 4) whose best z-chunking needs the
+// fewest plane-steps, weighted by the halo'd tile it loads per computed cell.
+int choose_rpw(DType dt, int64_t nx, int64_t ny, int64_t nz, int ncw, int64_t slots);
+
+// z-chunk length for `tiles` x-y tiles over `range` planes: whole rounds of
+// items over the persistent CTAs against the two halo planes (and the
+// pipeline fill) each chunk costs.  Returns the chunk length; *cost gets the
+// plane-steps of the slowest CTA.
+int64_t choose_kz(int64_t tiles, int64_t range, int64_t slots, int64_t* cost = nullptr);
 
 }  // namespace dfg

@@ -2,10 +2,12 @@
 // re-designed for sm_100a).  Compiled by NVRTC after skeleton.cuh.
 //
 // Work decomposition: persistent CTAs (grid = #SM x occupancy) walk items
-// (x-tile of 32*VEC cells) x (y-tile of DFG_NCW rows) x (z-chunk of kz
-// planes), item = blockIdx.x + t*gridDim.x.  Warp DFG_NCW is the producer:
+// (x-tile of DFG_TX = 32*VEC/RPW cells) x (y-tile of DFG_TH = NCW*RPW rows)
+// x (z-chunk of kz planes), item = blockIdx.x + t*gridDim.x; RPW (rows per
+// consumer warp: 1, 2 or 4) is chosen on the host so that narrow meshes do
+// not leave lanes idle in a ragged x-tile.  Warp DFG_NCW is the producer:
 // one lane streams, per z-plane, one halo'd x-y tile per stencil field
-// (box (32*VEC + 2*VEC) x (NCW + 2) x 1, cp.async.bulk.tensor.3d) into a
+// (box (TX + 2*VEC) x (TH + 2) x 1, cp.async.bulk.tensor.3d) into a
 // DFG_STAGES-deep ring of shared-memory stages guarded by full/empty
 // mbarriers (complete_tx byte counts; all consumer threads arrive on
 // "empty", so no divergent branch).  For every item the producer loads
@@ -13,7 +15,8 @@
 // min(ke, NZ-1).  At the global ends these duplicate the first / last plane,
 // which is exactly the clamped neighbour of reading R1, so the consumer loop
 // has no boundary branch.
-// Consumers: warp w owns tile row w, lane l owns VEC consecutive x cells;
+// Consumers: warp w owns tile rows w*RPW .. w*RPW+RPW-1 (32/RPW lanes per
+// row), a lane owns VEC consecutive x cells of its row;
 // the z-1 / z / z+1 centres live in a 3-entry register queue whose roles
 // rotate through a 3-way unrolled loop (no register copies); x/y neighbours
 // come from shared memory through per-thread clamped offsets; the network
@@ -27,10 +30,15 @@ struct DfgTmaParams {
   DfgParams p;
 };
 
-#define DFG_TX (32 * DFG_VEC)
+#ifndef DFG_RPW
+#define DFG_RPW 1
+#endif
+#define DFG_LPR (32 / DFG_RPW)          // lanes per tile row
+#define DFG_TX (DFG_LPR * DFG_VEC)      // tile width (cells)
+#define DFG_TH (DFG_NCW * DFG_RPW)      // tile height (rows)
 #define DFG_HX DFG_VEC
 #define DFG_ROWW (DFG_TX + 2 * DFG_HX)
-#define DFG_ROWS (DFG_NCW + 2)
+#define DFG_ROWS (DFG_TH + 2)
 #define DFG_TILE_ELEMS (DFG_ROWW * DFG_ROWS)
 #define DFG_TILE_BYTES ((DFG_TILE_ELEMS * (int)sizeof(DFG_T) + 127) / 128 * 128)
 // every field streams through the ring (point-wise fields: centre only)
@@ -205,7 +213,7 @@ __device__ __forceinline__ void dfg_produce_item(const DfgTmaParams& TP, long lo
   const long long zc = rest / P.tiles_y;
   // input coordinates include the block's x/y ghost columns / rows
   const int x0 = (int)(tx_ * DFG_TX) - DFG_HX + (int)P.gx;
-  const int y0 = (int)(ty_ * DFG_NCW) - 1 + (int)P.gy;
+  const int y0 = (int)(ty_ * DFG_TH) - 1 + (int)P.gy;
   const long long kb = P.kbeg + zc * P.kz;
   const long long ke = min(kb + (long long)P.kz, P.kend);
   for (long long q = kb - 1; q <= ke; ++q) {
@@ -221,19 +229,20 @@ __device__ __forceinline__ void dfg_produce_item(const DfgTmaParams& TP, long lo
   }
 }
 
-// Consumer side of one item: warp w computes tile row w.
+// Consumer side of one item: warp w computes tile rows w*RPW .. w*RPW+RPW-1.
 __device__ __forceinline__ void dfg_consume_item(const DfgTmaParams& TP, long long item, DfgRing& R, DfgCol& C,
                                                  int warp, int lane) {
   const DfgParams& P = TP.p;
   const long long plane = P.nx * P.ny;
-  const unsigned c0 = DFG_HX + DFG_VEC * lane;
-  const unsigned r = 1 + warp;
+  const int col = lane % DFG_LPR, sub = lane / DFG_LPR;
+  const unsigned c0 = DFG_HX + DFG_VEC * col;
+  const unsigned r = 1 + warp * DFG_RPW + sub;
   const long long tx_ = item % P.tiles_x;
   const long long rest = item / P.tiles_x;
   const long long ty_ = rest % P.tiles_y;
   const long long zc = rest / P.tiles_y;
-  const long long i = tx_ * DFG_TX + DFG_VEC * lane;
-  const long long j = ty_ * DFG_NCW + warp;
+  const long long i = tx_ * DFG_TX + DFG_VEC * col;
+  const long long j = ty_ * DFG_TH + warp * DFG_RPW + sub;
   const long long kb = P.kbeg + zc * P.kz;
   const long long ke = min(kb + (long long)P.kz, P.kend);
   C.act = (i < P.nx) && (j < P.ny);

@@ -144,6 +144,14 @@ std::unique_ptr<PlanImpl> compile_plan(std::shared_ptr<MeshImpl> mesh, const std
     if (ctas) cfg.ctas = std::max(1, std::min(4, std::atoi(ctas)));
     const char* st = std::getenv("DFG_STAGES");
     if (st) cfg.stages = std::max(2, std::min(16, std::atoi(st)));
+    // tile shape for this mesh (narrow meshes: several rows per warp)
+    const char* rpw = std::getenv("DFG_RPW");
+    if (rpw) {
+      const int r = std::atoi(rpw);
+      cfg.rpw = (r == 2 || r == 4) ? r : 1;
+    } else {
+      cfg.rpw = choose_rpw(mesh->dt, mesh->nx, mesh->ny, mesh->nzl, cfg.ncw, int64_t(sm_count(mesh->device)) * cfg.ctas);
+    }
     // axis degeneracy (n == 1) is a property of the GLOBAL mesh
     plan->fsrc = generate_fused(dag, mesh->NX, mesh->NY, mesh->NZ, cfg, ref);
     static const std::string kUnit = "dfg_fused.cu";
@@ -163,7 +171,7 @@ std::unique_ptr<PlanImpl> compile_plan(std::shared_ptr<MeshImpl> mesh, const std
     plan->spill = local;
     if (plan->mod.tma) {
       size_t smem = fused_tma_smem_bytes(mesh->dt, int(plan->fsrc.layout.stencil_inputs.size() + plan->fsrc.layout.point_inputs.size()), plan->fsrc.cfg.ncw,
-                                         plan->fsrc.cfg.stages);
+                                         plan->fsrc.cfg.stages, plan->fsrc.cfg.rpw);
       DFG_CU(drv().FuncSetAttribute(plan->mod.tma, CU_FUNC_ATTRIBUTE_MAX_DYNAMIC_SHARED_SIZE_BYTES, int(smem)));
       DFG_CU(drv().FuncSetAttribute(plan->mod.tma_multi, CU_FUNC_ATTRIBUTE_MAX_DYNAMIC_SHARED_SIZE_BYTES, int(smem)));
     }
@@ -284,12 +292,12 @@ void PlanImpl::execute(void* out, bool out_dev, cudaStream_t s) {
 namespace {
 // CUtensorMap for one stencil field: dims {nx, ny, nzl + 2g}, box
 // {32*VEC + 2*VEC, NCW + 2, 1}, OOB fill zero (never read: clamped in smem).
-void encode_map(CUtensorMap* map, const SlabView& m, void* base, int ncw) {
+void encode_map(CUtensorMap* map, const SlabView& m, void* base, int ncw, int rpw) {
   const size_t ts = dsize(m.dt);
   const int vec = int(16 / ts);
   cuuint64_t gdim[3] = {cuuint64_t(m.px()), cuuint64_t(m.py()), cuuint64_t(m.nzl + 2 * m.ghost)};
   cuuint64_t gstride[2] = {cuuint64_t(m.px()) * ts, cuuint64_t(m.px() * m.py()) * ts};
-  cuuint32_t box[3] = {cuuint32_t(32 * vec + 2 * vec), cuuint32_t(ncw + 2), 1};
+  cuuint32_t box[3] = {cuuint32_t(tma_tile_w(m.dt, rpw) + 2 * vec), cuuint32_t(tma_tile_h(ncw, rpw) + 2), 1};
   cuuint32_t estr[3] = {1, 1, 1};
   DFG_CU(drv().TensorMapEncodeTiled(map, m.dt == DType::F32 ? CU_TENSOR_MAP_DATA_TYPE_FLOAT32 : CU_TENSOR_MAP_DATA_TYPE_FLOAT64,
                                 3, base, gdim, gstride, box, estr, CU_TENSOR_MAP_INTERLEAVE_NONE,
@@ -452,32 +460,25 @@ void PlanImpl::launch_fused(const std::vector<const void*>& fptr, void* dout, co
   } else if (mod.tma && !want_general && m.nx % vec == 0 && m.px() % vec == 0 && m.gx() % vec == 0 &&
              aligned16(dout) &&
              std::all_of(fptr.begin(), fptr.end(), [](const void* p) { return aligned16(p); })) {
-    const int ncw = fsrc.cfg.ncw;
+    const int ncw = fsrc.cfg.ncw, rpw = fsrc.cfg.rpw;
     const int nsf = int(L.stencil_inputs.size() + L.point_inputs.size());  // TMA tiles per stage
-    const int tiles_x = int((m.nx + 32 * vec - 1) / (32 * vec));
-    const int tiles_y = int((m.ny + ncw - 1) / ncw);
+    const int tw = tma_tile_w(m.dt, rpw), th = tma_tile_h(ncw, rpw);
+    const int tiles_x = int((m.nx + tw - 1) / tw);
+    const int tiles_y = int((m.ny + th - 1) / th);
     const int64_t range = kend - kbeg;
-    size_t smem = fused_tma_smem_bytes(m.dt, nsf, ncw, fsrc.cfg.stages);
+    size_t smem = fused_tma_smem_bytes(m.dt, nsf, ncw, fsrc.cfg.stages, rpw);
     int occ = 1;
     DFG_CU(drv().OccupancyMaxActiveBlocksPerMultiprocessor(&occ, mod.tma, (ncw + 1) * 32, smem));
     occ = std::max(occ, 1);
     const int64_t slots = int64_t(sms) * occ;
     // z-chunk length: balance whole rounds of items over the persistent CTAs
     // against the two extra (z-halo) planes each chunk loads.
-    int64_t best_kz = range, best_cost = INT64_MAX;
+    int64_t best_kz = range;
     const char* kzenv = std::getenv("DFG_KZ");
     if (kzenv) {
       best_kz = std::max<int64_t>(1, std::min<int64_t>(range, std::atoll(kzenv)));
     } else {
-      for (int64_t kz = 1; kz <= range; kz = kz < 8 ? kz + 1 : kz + std::max<int64_t>(1, kz / 8)) {
-        int64_t items = int64_t(tiles_x) * tiles_y * ((range + kz - 1) / kz);
-        int64_t rounds = (items + slots - 1) / slots;
-        int64_t cost = rounds * (std::min(kz, range) + 2 + 4);  // +4: pipeline fill per item
-        if (cost < best_cost) {
-          best_cost = cost;
-          best_kz = kz;
-        }
-      }
+      best_kz = choose_kz(int64_t(tiles_x) * tiles_y, range, slots);
     }
     const int64_t items = int64_t(tiles_x) * tiles_y * ((range + best_kz - 1) / best_kz);
     const unsigned grid = unsigned(std::min<int64_t>(items, slots));
@@ -490,7 +491,7 @@ void PlanImpl::launch_fused(const std::vector<const void*>& fptr, void* dout, co
     if (pbytes > sizeof(blob)) fail(DFG_E_UNSUPPORTED, "too many stencil fields for the TMA kernel");
     std::memset(blob, 0, sizeof(blob));
     for (int f = 0; f < nsf; ++f)
-      encode_map(reinterpret_cast<CUtensorMap*>(blob + 128 * f), m, const_cast<void*>(fptr[f]), ncw);
+      encode_map(reinterpret_cast<CUtensorMap*>(blob + 128 * f), m, const_cast<void*>(fptr[f]), ncw, rpw);
     std::memcpy(blob + 128 * nsf, w.data(), w.size() * 8);
     void* args[] = {blob};
     auto ke = kernel_events();
@@ -498,6 +499,7 @@ void PlanImpl::launch_fused(const std::vector<const void*>& fptr, void* dout, co
     DFG_CU(drv().LaunchKernel(mod.tma, grid, 1, 1, (ncw + 1) * 32, 1, 1, unsigned(smem), s, args, nullptr));
     DFG_CUDA(cudaEventRecord(ke.second, s));
     last_variant = 1;
+    last_kz = best_kz;
   } else {
     // z-marching columns: enough (column, z-chunk) units to fill the device
     // (~2048 threads per SM), each chunk as long as that allows
@@ -553,9 +555,10 @@ void execute_blocks(const std::vector<PlanImpl*>& plans, const std::vector<void*
     return;
   }
   DFG_CUDA(cudaSetDevice(m0.device));
-  const int ncw = p0.fsrc.cfg.ncw;
+  const int ncw = p0.fsrc.cfg.ncw, rpw = p0.fsrc.cfg.rpw;
+  const int tw = tma_tile_w(m0.dt, rpw), th = tma_tile_h(ncw, rpw);
   const int nsf = int(L.stencil_inputs.size() + L.point_inputs.size());
-  const size_t smem = fused_tma_smem_bytes(m0.dt, nsf, ncw, p0.fsrc.cfg.stages);
+  const size_t smem = fused_tma_smem_bytes(m0.dt, nsf, ncw, p0.fsrc.cfg.stages, rpw);
   int occ = 1;
   DFG_CU(drv().OccupancyMaxActiveBlocksPerMultiprocessor(&occ, p0.mod.tma_multi, (ncw + 1) * 32, smem));
   const int64_t slots = int64_t(sm_count(m0.device)) * std::max(occ, 1);
@@ -567,7 +570,7 @@ void execute_blocks(const std::vector<PlanImpl*>& plans, const std::vector<void*
     int64_t t = 0;
     for (auto* p : plans) {
       const MeshImpl& m = *p->mesh;
-      t += int64_t((m.nx + 32 * vec - 1) / (32 * vec)) * ((m.ny + ncw - 1) / ncw) * ((m.nzl + kz - 1) / kz);
+      t += int64_t((m.nx + tw - 1) / tw) * ((m.ny + th - 1) / th) * ((m.nzl + kz - 1) / kz);
     }
     return t;
   };
@@ -583,7 +586,7 @@ void execute_blocks(const std::vector<PlanImpl*>& plans, const std::vector<void*
   for (size_t b = 0; b < plans.size(); ++b) {
     const MeshImpl& m = *plans[b]->mesh;
     const SlabView v = SlabView::of(m);
-    const int tx = int((m.nx + 32 * vec - 1) / (32 * vec)), ty = int((m.ny + ncw - 1) / ncw);
+    const int tx = int((m.nx + tw - 1) / tw), ty = int((m.ny + th - 1) / th);
     const int64_t items = int64_t(tx) * ty * ((m.nzl + best_kz - 1) / best_kz);
     words.push_back(pack_params(fptrs[b], outs[b], m.dev_tab[0], m.dev_tab[1], m.dev_tab[2], v, m.k0, m.k0 + m.nzl,
                                 items, tx, ty, int(best_kz), 0));
@@ -595,7 +598,7 @@ void execute_blocks(const std::vector<PlanImpl*>& plans, const std::vector<void*
   for (size_t b = 0; b < plans.size(); ++b) {
     unsigned char* blob = host.data() + stride * b;
     const SlabView v = SlabView::of(*plans[b]->mesh);
-    for (int f = 0; f < nsf; ++f) encode_map(reinterpret_cast<CUtensorMap*>(blob + 128 * f), v, const_cast<void*>(fptrs[b][size_t(f)]), ncw);
+    for (int f = 0; f < nsf; ++f) encode_map(reinterpret_cast<CUtensorMap*>(blob + 128 * f), v, const_cast<void*>(fptrs[b][size_t(f)]), ncw, rpw);
     std::memcpy(blob + 128 * nsf, words[b].data(), words[b].size() * 8);
   }
   std::memcpy(host.data() + stride * plans.size(), first.data(), sizeof(int64_t) * first.size());
@@ -621,6 +624,7 @@ void execute_blocks(const std::vector<PlanImpl*>& plans, const std::vector<void*
   for (auto* p : plans) {
     p->st.executes += 1;
     p->last_variant = 4;
+    p->last_kz = best_kz;
   }
 }
 

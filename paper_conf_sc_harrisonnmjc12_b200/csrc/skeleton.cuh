@@ -21,7 +21,7 @@
 //   dfg_fused_general   -- any layout (ragged nx, pitched or unaligned
 //                          buffers): z-marching columns, direct loads.
 //   dfg_fused_tma       -- the B200 path: persistent CTAs march z-columns of
-//                          (32*VEC) x DFG_NCW cells; one producer warp streams
+//                          (32*VEC/RPW) x (DFG_NCW*RPW) cells; one producer warp streams
 //                          halo'd x-y tiles of every stencil field into a
 //                          DFG_STAGES-deep shared-memory ring with TMA
 //                          (cp.async.bulk.tensor.3d + mbarrier complete_tx);

@@ -629,3 +629,52 @@ def test_reference_kernels(prog, T, shape):
     import paper_conf_sc_harrisonnmjc12_b200 as dfg
     with pytest.raises(dfg.DfgError):
         run_lib("intro", f, x, y, z, "reference")
+
+
+@pytest.mark.parametrize("prog", PROGS)
+@pytest.mark.parametrize("T", [np.float32, np.float64])
+@pytest.mark.parametrize("shape", [(132, 40, 33), (67, 45, 37)])
+def test_fast_variant_within_tolerance(prog, T, shape, monkeypatch):
+    """DFG_FUSED_VARIANT=fast (derivative = num * RN(1/d), FMA allowed in the
+    quotient only) is not bit-identical to the literal network, but stays within
+    the R15 bound (1e-5 / 1e-12 normwise) on both kernels (TMA and general)."""
+    x, y, z, f = _inputs(shape, T, NAMES[prog])
+    src = PAPER_PROGRAMS[prog][0]
+    want = run_oracle(src, f, x, y, z)
+    monkeypatch.setenv("DFG_FUSED_VARIANT", "fast")
+    got, plan, *_ = run_lib(src, f, x, y, z, return_plan=True)
+    assert_parity(got, want, exact=False)
+
+
+@pytest.mark.parametrize("rpw", ["1", "2", "4"])
+@pytest.mark.parametrize("T", [np.float32, np.float64])
+@pytest.mark.parametrize("shape", [(200, 37, 21), (132, 40, 33), (8, 70, 9)])
+def test_tma_rows_per_warp(rpw, T, shape, monkeypatch):
+    """Every TMA tile shape (1, 2 or 4 rows per consumer warp: tiles of
+    32*VEC/rpw x 15*rpw cells) gives the oracle's bits, ragged x and y tiles
+    included."""
+    x, y, z, f = _inputs(shape, T)
+    src = PAPER_PROGRAMS["qcrit"][0]
+    want = run_oracle(src, f, x, y, z)
+    monkeypatch.setenv("DFG_RPW", rpw)
+    got, plan, *_ = run_lib(src, f, x, y, z, return_plan=True)
+    info = plan.info()
+    assert info["variant"] == 1 and info["rows_per_warp"] == int(rpw)
+    vec = 4 if T == np.float32 else 2
+    assert info["tile_w"] == 32 * vec // int(rpw) and info["tile_h"] == info["rows_per_warp"] * 15
+    assert_parity(got, want)
+
+
+def test_tile_shape_choice():
+    """Narrow meshes take several rows per warp (no idle lanes in a ragged x
+    tile); the 1024-wide bench mesh keeps one row per warp."""
+    import paper_conf_sc_harrisonnmjc12_b200 as dfg
+    for n, nz, want in ((192, 192, 2), (1024, 64, 1)):
+        x, y, z = synth.rt_coords(n, n, nz, np.float32)
+        mesh = dfg.Mesh(x, y, z)
+        fields = [torch.zeros((nz, n, n), device="cuda") for _ in range(3)]
+        for c, t in zip("uvw", fields):
+            mesh.bind(c, t)
+        plan = dfg.Plan(mesh, PAPER_PROGRAMS["qcrit"][0], "fused")
+        assert plan.info()["rows_per_warp"] == want, (n, plan.info())
+        plan.close()

@@ -1,0 +1,71 @@
+"""Launch overhead of one execute on a tiny mesh (developer tool).
+
+    python tools/launch_overhead.py [--n 32]
+
+For device sleeps of 0, 0.1 and 1 ms before the first event (so the host
+enqueues behind a busy GPU), times a torch zero_() and fused VelMag / Q
+executes between CUDA events, plus the library's own kernel events.
+"""
+import argparse
+import json
+import os
+import sys
+import time
+
+import numpy as np
+import torch
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+sys.path.insert(0, ROOT)
+
+import paper_conf_sc_harrisonnmjc12_b200 as dfg  # noqa: E402
+import synth  # noqa: E402
+from oracle.lang import PAPER_PROGRAMS  # noqa: E402  (program text only)
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--n", type=int, default=32)
+    args = ap.parse_args()
+    n = args.n
+    x, y, z = synth.rt_coords(n, n, n, np.float32)
+    x64, y64, z64 = (a.astype(np.float64) for a in (x, y, z))
+    mesh = dfg.Mesh(x, y, z)
+    bufs = {c: synth.rt_velocity(c, x64, y64, z64, None, torch.float32, "cuda") for c in "uvw"}
+    for c, b in bufs.items():
+        mesh.bind(c, b)
+    out = torch.empty((n, n, n), dtype=torch.float32, device="cuda")
+    plans = {e: dfg.Plan(mesh, PAPER_PROGRAMS[e][0], "fused") for e in ("velmag", "qcrit")}
+    ops = {"torch_zero": lambda: out.zero_()}
+    for e, p in plans.items():
+        ops[e] = p.execute if False else (lambda p=p: p.execute(out))
+    for _ in range(5):
+        for f in ops.values():
+            f()
+    torch.cuda.synchronize()
+    for sleep in (0, 200_000, 2_000_000):
+        for name, f in ops.items():
+            ev, kv, host = [], [], []
+            for _ in range(20):
+                torch.cuda.synchronize()
+                if sleep:
+                    torch.cuda._sleep(sleep)
+                e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+                e0.record()
+                t0 = time.perf_counter()
+                f()
+                host.append((time.perf_counter() - t0) * 1e6)
+                e1.record()
+                e1.synchronize()
+                ev.append(e0.elapsed_time(e1) * 1e3)
+                if name in plans:
+                    kv.append(plans[name].stats()["last_ms"] * 1e3)
+            rec = {"sleep_cycles": sleep, "op": name, "event_us": round(float(np.median(ev)), 2),
+                   "host_call_us": round(float(np.median(host)), 2)}
+            if kv:
+                rec["kernel_event_us"] = round(float(np.median(kv)), 2)
+            print(json.dumps(rec), flush=True)
+
+
+if __name__ == "__main__":
+    main()
