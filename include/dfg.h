@@ -248,6 +248,17 @@ int dfg_execute_blocks(dfg_plan const* plans, int n, void* const* outs, void* cu
 int dfg_plan_stats(dfg_plan plan, dfg_stats* out);
 int dfg_reset_stats(dfg_plan plan);
 
+/* CUDA-event timing of later executes of `plan` (default 1):
+ *   0  no events: last_ms stays at its previous value (-1 after a reset) and
+ *      the kernel timings do not advance -- the cheapest execute;
+ *   1  one event pair around each execute (stats.last_ms);
+ *   2  as 1, plus one event pair around every fused-kernel launch
+ *      (stats.kernel_ms_sum / kernel_launches_timed).
+ * Every timestamped event costs GPU time of its own (measured ~2 us on B200),
+ * which only small meshes notice.  Pending kernel timings are folded into the
+ * stats first.  Errors: DFG_E_INVALID (null plan, level outside 0..2). */
+int dfg_plan_set_timing(dfg_plan plan, int level);
+
 /* Plan description: out[0] = strategy, out[1] = result width (1 or 4),
  * out[2] = number of filters, out[3] = fused kernel variant of the last
  * execute (0 none, 1 TMA pipeline, 2 general, 3 point-wise, 4 TMA

@@ -13,7 +13,7 @@ from ._dfg import *  # noqa: F401,F403
 from ._dfg import (DFG_F32, DFG_F64, DfgError, EXPORTS, LIB_PATH, STRATEGIES,  # noqa: F401
                    dfg_bind_field, dfg_compile, dfg_create_mesh, dfg_destroy_mesh, dfg_destroy_plan,
                    dfg_dump_dag, dfg_dump_kernel, dfg_execute, dfg_halo_map, dfg_plan_info, dfg_plan_stats,
-                   dfg_reset_stats)
+                   dfg_plan_set_timing, dfg_reset_stats)
 
 
 def _dtype_code(dtype) -> int:
@@ -101,6 +101,11 @@ class Plan:
 
     def stats(self):
         return dfg_plan_stats(self.handle)
+
+    def set_timing(self, level: int):
+        """0: no CUDA events, 1: execute interval (default), 2: also per fused launch."""
+        dfg_plan_set_timing(self.handle, level)
+        return self
 
     def reset_stats(self):
         dfg_reset_stats(self.handle)

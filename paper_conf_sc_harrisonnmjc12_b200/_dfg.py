@@ -71,6 +71,7 @@ _SIGS = {
     "dfg_execute_blocks": (C.c_int, [C.POINTER(_P), C.c_int, C.POINTER(_P), _P]),
     "dfg_plan_stats": (C.c_int, [_P, C.POINTER(dfg_stats)]),
     "dfg_reset_stats": (C.c_int, [_P]),
+    "dfg_plan_set_timing": (C.c_int, [_P, C.c_int]),
     "dfg_plan_info": (C.c_int, [_P, C.POINTER(_I64)]),
     "dfg_plan_schedule": (C.c_int, [_P, C.POINTER(C.c_int32), C.c_size_t, C.POINTER(C.c_size_t)]),
     "dfg_plan_transfers": (C.c_int, [_P, C.POINTER(C.c_int32), C.c_size_t, C.POINTER(C.c_size_t)]),
@@ -205,6 +206,10 @@ def dfg_plan_stats(plan) -> dict:
     st = dfg_stats()
     _check(_lib.dfg_plan_stats(plan, C.byref(st)))
     return st.as_dict()
+
+
+def dfg_plan_set_timing(plan, level: int):
+    _check(_lib.dfg_plan_set_timing(plan, int(level)))
 
 
 def dfg_reset_stats(plan):

@@ -225,6 +225,16 @@ int dfg_plan_stats(dfg_plan plan, dfg_stats* out) {
   });
 }
 
+int dfg_plan_set_timing(dfg_plan plan, int level) {
+  return guard([&] {
+    if (!plan) dfg::fail(DFG_E_INVALID, "null plan");
+    if (level < 0 || level > 2) dfg::fail(DFG_E_INVALID, "timing level must be 0, 1 or 2");
+    plan->p->resolve_kernel_times();
+    plan->p->timing = level;
+    if (level == 0) plan->p->timed = false;
+  });
+}
+
 int dfg_reset_stats(dfg_plan plan) {
   return guard([&] {
     if (!plan) dfg::fail(DFG_E_INVALID, "null plan");
@@ -406,6 +416,11 @@ int dfg_fused_source(const char* expr, const char* const* inputs, int n_inputs, 
     dfg::FusedConfig cfg;
     const char* var = std::getenv("DFG_FUSED_VARIANT");
     if (!(var && !std::strcmp(var, "markstein"))) cfg.div2 = 7;
+    // tile rows per warp: DFG_RPW, else the choice for a 148-SM B200
+    const char* rpw = std::getenv("DFG_RPW");
+    cfg.rpw = rpw ? std::atoi(rpw) : dfg::choose_rpw(d.dtype, nx, ny, nz,
+                                                     cfg.ncw, 148);
+    if (cfg.rpw != 2 && cfg.rpw != 4) cfg.rpw = 1;
     dfg::FusedSource fs = dfg::generate_fused(d, nx, ny, nz, cfg);
     if (compile) {
       static const std::string kUnit = "dfg_fused.cu";

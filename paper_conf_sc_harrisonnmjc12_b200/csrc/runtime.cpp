@@ -192,6 +192,17 @@ std::pair<cudaEvent_t, cudaEvent_t> PlanImpl::kernel_events() {
   return e;
 }
 
+std::pair<cudaEvent_t, cudaEvent_t> PlanImpl::kernel_begin(cudaStream_t s) {
+  if (timing < 2) return {nullptr, nullptr};
+  auto e = kernel_events();
+  DFG_CUDA(cudaEventRecord(e.first, s));
+  return e;
+}
+
+void PlanImpl::kernel_end(const std::pair<cudaEvent_t, cudaEvent_t>& e, cudaStream_t s) {
+  if (e.second) DFG_CUDA(cudaEventRecord(e.second, s));
+}
+
 void PlanImpl::resolve_kernel_times() {
   for (auto& e : kev_pending) {
     DFG_CUDA(cudaEventSynchronize(e.second));
@@ -263,7 +274,7 @@ void PlanImpl::execute(void* out, bool out_dev, cudaStream_t s) {
     auto it = m.fields.find(dag.inputs[i]);
     if (it == m.fields.end() || !it->second.ptr) fail(DFG_E_UNBOUND, "input '" + dag.inputs[i] + "' is not bound");
   }
-  DFG_CUDA(cudaEventRecord(ev0, s));
+  if (timing >= 1) DFG_CUDA(cudaEventRecord(ev0, s));
   switch (strategy) {
     case DFG_FUSED: exec_fused(out, out_dev, s); break;
     case DFG_STREAMED: exec_streamed(out, out_dev, s); break;
@@ -272,9 +283,9 @@ void PlanImpl::execute(void* out, bool out_dev, cudaStream_t s) {
     case DFG_HYBRID: exec_hybrid(out, out_dev, s); break;
     case DFG_ROUNDTRIP: exec_roundtrip(out, out_dev, s); break;
   }
-  DFG_CUDA(cudaEventRecord(ev1, s));
+  if (timing >= 1) DFG_CUDA(cudaEventRecord(ev1, s));
   DFG_CUDA(cudaGetLastError());
-  timed = true;
+  timed = timing >= 1;
   st.executes += 1;
   bool any_host = !out_dev;
   for (int i : sources(dag).inputs)
@@ -452,10 +463,9 @@ void PlanImpl::launch_fused(const std::vector<const void*>& fptr, void* dout, co
     void* args[] = {w.data()};
     long long work = vec_ok ? N / vec : N;
     unsigned grid = unsigned(std::max<long long>(1, std::min<long long>((work + 255) / 256, sms * 8LL)));
-    auto ke = kernel_events();
-    DFG_CUDA(cudaEventRecord(ke.first, s));
+    auto ke = kernel_begin(s);
     DFG_CU(drv().LaunchKernel(mod.pointwise, grid, 1, 1, 256, 1, 1, 0, s, args, nullptr));
-    DFG_CUDA(cudaEventRecord(ke.second, s));
+    kernel_end(ke, s);
     last_variant = 3;
   } else if (mod.tma && !want_general && m.nx % vec == 0 && m.px() % vec == 0 && m.gx() % vec == 0 &&
              aligned16(dout) &&
@@ -494,10 +504,9 @@ void PlanImpl::launch_fused(const std::vector<const void*>& fptr, void* dout, co
       encode_map(reinterpret_cast<CUtensorMap*>(blob + 128 * f), m, const_cast<void*>(fptr[f]), ncw, rpw);
     std::memcpy(blob + 128 * nsf, w.data(), w.size() * 8);
     void* args[] = {blob};
-    auto ke = kernel_events();
-    DFG_CUDA(cudaEventRecord(ke.first, s));
+    auto ke = kernel_begin(s);
     DFG_CU(drv().LaunchKernel(mod.tma, grid, 1, 1, (ncw + 1) * 32, 1, 1, unsigned(smem), s, args, nullptr));
-    DFG_CUDA(cudaEventRecord(ke.second, s));
+    kernel_end(ke, s);
     last_variant = 1;
     last_kz = best_kz;
   } else {
@@ -510,10 +519,9 @@ void PlanImpl::launch_fused(const std::vector<const void*>& fptr, void* dout, co
     auto w = pack_params(fptr, dout, tab[0], tab[1], tab[2], m, kbeg, kend, 0, 0, 0, int(kz), 0);
     void* args[] = {w.data()};
     unsigned grid = unsigned(std::max<long long>(1, std::min<long long>((units + 255) / 256, sms * 8LL)));
-    auto ke = kernel_events();
-    DFG_CUDA(cudaEventRecord(ke.first, s));
+    auto ke = kernel_begin(s);
     DFG_CU(drv().LaunchKernel(mod.general, grid, 1, 1, 256, 1, 1, 0, s, args, nullptr));
-    DFG_CUDA(cudaEventRecord(ke.second, s));
+    kernel_end(ke, s);
     last_variant = 2;
   }
   st.kernel_count += 1;
@@ -610,16 +618,15 @@ void execute_blocks(const std::vector<PlanImpl*>& plans, const std::vector<void*
     int nb;
   } arg{dev, static_cast<char*>(dev) + stride * plans.size(), int(plans.size())};
   void* args[] = {&arg};
-  DFG_CUDA(cudaEventRecord(p0.ev0, s));
-  auto ke = p0.kernel_events();
-  DFG_CUDA(cudaEventRecord(ke.first, s));
+  if (p0.timing >= 1) DFG_CUDA(cudaEventRecord(p0.ev0, s));
+  auto ke = p0.kernel_begin(s);
   const unsigned grid = unsigned(std::max<int64_t>(1, std::min(first.back(), slots)));
   DFG_CU(drv().LaunchKernel(p0.mod.tma_multi, grid, 1, 1, (ncw + 1) * 32, 1, 1, unsigned(smem), s, args, nullptr));
-  DFG_CUDA(cudaEventRecord(ke.second, s));
-  DFG_CUDA(cudaEventRecord(p0.ev1, s));
+  p0.kernel_end(ke, s);
+  if (p0.timing >= 1) DFG_CUDA(cudaEventRecord(p0.ev1, s));
   DFG_CUDA(cudaFreeAsync(dev, s));
   DFG_CUDA(cudaGetLastError());
-  p0.timed = true;
+  p0.timed = p0.timing >= 1;
   p0.st.kernel_count += 1;
   for (auto* p : plans) {
     p->st.executes += 1;

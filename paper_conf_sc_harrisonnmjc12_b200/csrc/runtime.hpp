@@ -125,9 +125,16 @@ struct PlanImpl {
   dfg_stats st{};
   cudaEvent_t ev0 = nullptr, ev1 = nullptr;
   bool timed = false;
+  // dfg_plan_set_timing: 0 no events, 1 execute interval (ev0/ev1), 2 also
+  // one event pair per fused-kernel launch.  A timestamped event costs GPU
+  // time of its own (~2 us each, measured), which small meshes notice.
+  int timing = 1;
   // fused-kernel launch timing: event pairs resolved lazily in stats()
   std::vector<std::pair<cudaEvent_t, cudaEvent_t>> kev_free, kev_pending;
   std::pair<cudaEvent_t, cudaEvent_t> kernel_events();
+  // bracket one fused launch with a kernel event pair when timing >= 2
+  std::pair<cudaEvent_t, cudaEvent_t> kernel_begin(cudaStream_t s);
+  void kernel_end(const std::pair<cudaEvent_t, cudaEvent_t>& e, cudaStream_t s);
   void resolve_kernel_times();
   std::map<std::string, std::vector<char>> const_cache;  // roundtrip host constants
   std::vector<int> order;  // staged execution order (list order unless a cap forced a reorder)

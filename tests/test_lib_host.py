@@ -303,3 +303,30 @@ def test_new_entry_points_validate_before_device_work(dfg):
     with pytest.raises(dfg.DfgError) as e:
         dfg.dfg_hybrid_model("r = (a + b) * (c + d)\n", ("a", "b", "c", "d"), True, 3, [2, 0, 1])
     assert e.value.name == "DFG_E_INVALID"   # not a topological order
+
+
+@pytest.mark.parametrize("rpw", ["2", "4"])
+@pytest.mark.parametrize("dtype", [0, 1])
+def test_tile_shapes_compile_without_spills(dfg, rpw, dtype, monkeypatch):
+    """The TMA kernel with 2 or 4 tile rows per consumer warp (narrow meshes)
+    compiles for sm_100a without local memory, like the 1-row tile."""
+    monkeypatch.setenv("DFG_RPW", rpw)
+    src, inputs = PAPER_PROGRAMS["qcrit"]
+    code, regs, spill = dfg.dfg_fused_source(src, inputs, dtype, 192, 192, 192, compile=True)
+    assert f"#define DFG_RPW {rpw}" in code
+    assert regs > 0 and spill == 0, (regs, spill)
+
+
+def test_tile_shape_choice_host(dfg):
+    """Without DFG_RPW the generator takes choose_rpw's tile for a 148-SM part:
+    two rows per warp for the 192-wide meshes of config 2 and the paper's
+    192 x 192 x 256 blocks, one for the 1024^3 bench mesh."""
+    src, inputs = PAPER_PROGRAMS["qcrit"]
+    for dims, want in (((192, 192, 192), 2), ((192, 192, 256), 2), ((1024, 1024, 1024), 1), ((32, 32, 32), 1)):
+        code, _, _ = dfg.dfg_fused_source(src, inputs, 0, *dims)
+        assert f"#define DFG_RPW {want}" in code, dims
+
+
+def test_set_timing_validates(dfg):
+    lib = dfg._dfg._lib
+    assert lib.dfg_plan_set_timing(None, 1) == -1

@@ -35,7 +35,8 @@ def main():
     for c, b in bufs.items():
         mesh.bind(c, b)
     out = torch.empty((n, n, n), dtype=torch.float32, device="cuda")
-    plans = {e: dfg.Plan(mesh, PAPER_PROGRAMS[e][0], "fused") for e in ("velmag", "qcrit")}
+    lvl = int(os.environ.get("DFG_TIMING_LEVEL", "1"))
+    plans = {e: dfg.Plan(mesh, PAPER_PROGRAMS[e][0], "fused").set_timing(lvl) for e in ("velmag", "qcrit")}
     ops = {"torch_zero": lambda: out.zero_()}
     for e, p in plans.items():
         ops[e] = p.execute if False else (lambda p=p: p.execute(out))
@@ -58,13 +59,34 @@ def main():
                 e1.record()
                 e1.synchronize()
                 ev.append(e0.elapsed_time(e1) * 1e3)
-                if name in plans:
+                if name in plans and lvl >= 1:
                     kv.append(plans[name].stats()["last_ms"] * 1e3)
             rec = {"sleep_cycles": sleep, "op": name, "event_us": round(float(np.median(ev)), 2),
                    "host_call_us": round(float(np.median(host)), 2)}
             if kv:
                 rec["kernel_event_us"] = round(float(np.median(kv)), 2)
             print(json.dumps(rec), flush=True)
+    # amortized: 200 back-to-back calls on the default and on a side stream
+    side = torch.cuda.Stream()
+    for sname, st in (("default", None), ("side", side)):
+        for name, f in ops.items():
+            ctx = torch.cuda.stream(st) if st is not None else torch.cuda.stream(torch.cuda.current_stream())
+            with ctx:
+                if name in plans:
+                    g = (lambda p=plans[name]: p.execute(out, stream=torch.cuda.current_stream()))
+                else:
+                    g = f
+                torch.cuda.synchronize()
+                torch.cuda._sleep(20_000_000)
+                e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+                e0.record()
+                for _ in range(200):
+                    g()
+                e1.record()
+                e1.synchronize()
+                rec = {"amortized_stream": sname, "op": name, "us_per_call": round(e0.elapsed_time(e1) * 1e3 / 200, 2)}
+                rec["timing_level"] = lvl
+                print(json.dumps(rec), flush=True)
 
 
 if __name__ == "__main__":
