@@ -383,7 +383,7 @@ def main():
             "config": {"workload": f"fused Q-criterion, {n}^3 fp32 rectilinear mesh per GPU "
                                    f"(mesh {n}x{n}x{NZ}, z-slabs + 1-plane NCCL halo when N>1)",
                        "expression": "qcrit (Fig. 3C completed)", "strategy": "fused",
-                       "cells_per_gpu": cells_rank, "fused_kernel": {1: "tma", 2: "general", 3: "pointwise"}.get(
+                       "cells_per_gpu": cells_rank, "fused_kernel": {1: "tma", 2: "general", 3: "pointwise", 5: "tile"}.get(
                            info["variant"]), "regs": info["regs"],
                        "l2": f"inputs {3 * cells_rank * 4 / 1e9:.1f} GB per GPU >> 126 MB L2; no flush needed",
                        "parallelism": f"zslab{world}",
@@ -485,7 +485,7 @@ def complexity_sweep(dfg, synth, torch):
             res[f"{name}_{dt}"] = {"filters": info["filters"], "kernel_ms": kms, "cells_per_s": n ** 3 / (kms * 1e-3),
                                    "algorithmic_gb_per_s": nbytes * n ** 3 / (kms * 1e-3) / 1e9,
                                    "bytes_per_cell": nbytes, "regs": info["regs"],
-                                   "kernel": {1: "tma", 2: "general", 3: "pointwise"}.get(info["variant"])}
+                                   "kernel": {1: "tma", 2: "general", 3: "pointwise", 5: "tile"}.get(info["variant"])}
             plan.close()
             mesh.close()
         del fields, out

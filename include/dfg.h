@@ -262,7 +262,8 @@ int dfg_plan_set_timing(dfg_plan plan, int level);
 /* Plan description: out[0] = strategy, out[1] = result width (1 or 4),
  * out[2] = number of filters, out[3] = fused kernel variant of the last
  * execute (0 none, 1 TMA pipeline, 2 general, 3 point-wise, 4 TMA
- * multi-block via dfg_execute_blocks), out[4] = registers per thread of the
+ * multi-block via dfg_execute_blocks, 5 tile: the TMA kernel's ring filled
+ * by cp.async, for layouts a tensor map cannot describe), out[4] = registers per thread of the
  * fused kernel (0 if none), out[5] = local memory per thread of that kernel
  * (bytes; spills and stack), out[6] = predicted
  * device footprint in bytes for device-resident inputs,

@@ -129,15 +129,43 @@ struct DfgCol {
   unsigned off_c, off_xm, off_xp, off_ym, off_yp;  // byte offsets in a tile
   dfg2 ndx[DFG_NPAIR], rx[DFG_NPAIR], ndy, ry, Z;  // -d and 1/d spacing entries
   bool act;
+  int nvalid;  // tile kernel: cells of this thread inside the mesh (0..VEC)
+  bool vst;    // tile kernel: 16-byte output stores allowed (aligned rows)
 };
+
+// The TMA kernel's producer warp fills the ring; the tile kernel's consumer
+// threads fill it themselves, one stage per consumed stage (DfgFill below).
+struct DfgNoFill {
+  __device__ __forceinline__ void step() {}
+};
+
+// Masked store of the VEC cells of a thread (tile kernel): 16-byte store
+// when the row is aligned and every cell is inside the mesh, else one scalar
+// store per valid cell.
+__device__ __forceinline__ void dfg_store_masked(DFG_T* dst, const dfg2 (&o)[DFG_NPAIR][DFG_OUTW], const DfgCol& C) {
+  if (C.nvalid == DFG_VEC && C.vst) {
+    dfg_store_cells(dst, o);
+    return;
+  }
+#pragma unroll
+  for (int h = 0; h < DFG_NPAIR; ++h)
+#pragma unroll
+    for (int l = 0; l < DFG_LANES; ++l) {
+      const int c = h * DFG_LANES + l;
+      if (c < C.nvalid) {
+#pragma unroll
+        for (int w = 0; w < DFG_OUTW; ++w) __stcs(dst + c * DFG_OUTW + w, dfg2_get(o[h][w], l));
+      }
+    }
+}
 
 // One z-plane.  `cur` = smem address of the plane's stage (tile, full bar);
 // the next plane's stage is always present (the producer loads a clamped
 // post-plane).  Queue roles are template parameters (no copies).
-template <int ZM, int ZC, int ZN>
+template <int ZM, int ZC, int ZN, bool MASKED = false, class Fill = DfgNoFill>
 __device__ __forceinline__ void dfg_plane(const DfgCol& C, DfgRing& R, unsigned& cur_tile, unsigned& cur_full,
                                           DFG_T (&zq)[3][DFG_NSF][DFG_VEC], DFG_T*& outp,
-                                          long long plane, const DFG_T*& tzp, long long NZ) {
+                                          long long plane, const DFG_T*& tzp, long long NZ, Fill& fill) {
   // x/y neighbours of this plane first (its stage is already resident), then
   // wait for the next plane's stage: the loads overlap the barrier wait
   DFG_T xmv[DFG_NSF], xpv[DFG_NSF], ymv[DFG_NSF][DFG_VEC], ypv[DFG_NSF][DFG_VEC];
@@ -196,9 +224,14 @@ __device__ __forceinline__ void dfg_plane(const DfgCol& C, DfgRing& R, unsigned&
 #pragma unroll
   for (int h = 0; h < DFG_NPAIR; ++h)
     dfg_body(s[h], gn[h], p[h], C.ndx[h], C.rx[h], C.ndy, C.ry, ndz, rz, C.Z, o[h]);
-  if (C.act) dfg_store_cells(outp, o);
+  if (MASKED) {
+    dfg_store_masked(outp, o, C);
+  } else if (C.act) {
+    dfg_store_cells(outp, o);
+  }
   outp += plane * DFG_OUTW;
   dfg_mbar_arrive(DFG_EMPTY(cur_full));  // every consumer thread (count NCW*32)
+  fill.step();
   cur_tile = nxt_tile;
   cur_full = nxt_full;
 }
@@ -285,21 +318,24 @@ __device__ __forceinline__ void dfg_consume_item(const DfgTmaParams& TP, long lo
 #pragma unroll
   for (int f = 0; f < DFG_NSF; ++f) dfg_lds16(zq[1][f], cur_tile + f * DFG_TILE_BYTES + C.off_c);
   R.advance();
+  DfgNoFill nf;
   long long k = kb;
   for (; k + 3 <= ke; k += 3) {
-    dfg_plane<0, 1, 2>(C, R, cur_tile, cur_full, zq, outp, plane, tzp, P.NZ);
-    dfg_plane<1, 2, 0>(C, R, cur_tile, cur_full, zq, outp, plane, tzp, P.NZ);
-    dfg_plane<2, 0, 1>(C, R, cur_tile, cur_full, zq, outp, plane, tzp, P.NZ);
+    dfg_plane<0, 1, 2>(C, R, cur_tile, cur_full, zq, outp, plane, tzp, P.NZ, nf);
+    dfg_plane<1, 2, 0>(C, R, cur_tile, cur_full, zq, outp, plane, tzp, P.NZ, nf);
+    dfg_plane<2, 0, 1>(C, R, cur_tile, cur_full, zq, outp, plane, tzp, P.NZ, nf);
   }
   if (k < ke) {
-    dfg_plane<0, 1, 2>(C, R, cur_tile, cur_full, zq, outp, plane, tzp, P.NZ);
-    if (k + 1 < ke) dfg_plane<1, 2, 0>(C, R, cur_tile, cur_full, zq, outp, plane, tzp, P.NZ);
+    dfg_plane<0, 1, 2>(C, R, cur_tile, cur_full, zq, outp, plane, tzp, P.NZ, nf);
+    if (k + 1 < ke) dfg_plane<1, 2, 0>(C, R, cur_tile, cur_full, zq, outp, plane, tzp, P.NZ, nf);
   }
   // the post-plane stage was read for its centre only
   dfg_mbar_arrive(DFG_EMPTY(cur_full));
 }
 
-__device__ __forceinline__ unsigned dfg_ring_init() {
+// full_count: arrivals that complete a "full" phase (1 for the TMA
+// producer's arrive.expect_tx; every consumer thread for the tile kernel)
+__device__ __forceinline__ unsigned dfg_ring_init(unsigned full_count = 1) {
   // dynamic shared memory starts at the (1024-aligned) base of the CTA's
   // window: no static __shared__ in this kernel
   extern __shared__ __align__(1024) unsigned char dfg_smem_raw[];
@@ -307,7 +343,7 @@ __device__ __forceinline__ unsigned dfg_ring_init() {
   const unsigned full0 = smem + DFG_STAGES * DFG_STAGE_BYTES;  // full[s] at full0 + 8s, empty[s] = full[s] + 8*STAGES
   if (threadIdx.x == 0) {
     for (int s = 0; s < DFG_STAGES; ++s) {
-      dfg_mbar_init(full0 + 8 * s, 1);
+      dfg_mbar_init(full0 + 8 * s, full_count);
       dfg_mbar_init(DFG_EMPTY(full0 + 8 * s), DFG_NCW * 32);
     }
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
@@ -376,5 +412,179 @@ extern "C" __global__ void __launch_bounds__((DFG_NCW + 1) * 32, DFG_CTAS)
     while (item >= M.first[b + 1]) ++b;
     dfg_consume_item(M.blocks[b], item - M.first[b], R, C, warp, lane);
   }
+}
+
+// ---------------------------------------------------------------- tile
+// Layouts the tensor maps cannot describe: rows that are not a multiple of
+// 16 bytes (nx % VEC != 0), packed ghost shells (owned cells from column 1),
+// pitched or unaligned buffers.  TMA needs 16-byte global strides and box
+// starts (an odd start column faults on B200, tools/tma_probe.cu), so the
+// consumer threads fill the same shared-memory ring themselves with 4 / 8-byte
+// cp.async copies, every tile element landing at the position the TMA kernel
+// reads (LDS.128 stays aligned whatever the global alignment).  Elements past
+// the GLOBAL mesh ends are filled with the boundary cell (clamped source
+// index), so a ragged last vector of a row and the one-sided differences of
+// reading R1 need no per-cell selects; inside a block the ghost shell is read
+// as data.  The fill runs STAGES-1 stages ahead of the consumption: every
+// consumed stage releases its slot ("empty") and each thread then issues its
+// share of the next stage (waiting for the slot released one stage earlier)
+// and arrives on that stage's "full" barrier when its copies land
+// (cp.async.mbarrier.arrive.noinc; full count = all consumer threads).
+#define DFG_NT (DFG_NCW * 32)
+#define DFG_FM ((DFG_TILE_ELEMS + DFG_NT - 1) / DFG_NT)  // tile elements per thread
+
+__device__ __forceinline__ void dfg_cp_async(unsigned dst, const DFG_T* src) {
+#if DFG_VEC == 4
+  asm volatile("cp.async.ca.shared.global [%0], [%1], 4;" ::"r"(dst), "l"(src) : "memory");
+#else
+  asm volatile("cp.async.ca.shared.global [%0], [%1], 8;" ::"r"(dst), "l"(src) : "memory");
+#endif
+}
+__device__ __forceinline__ void dfg_cp_async_arrive(unsigned bar) {
+  asm volatile("cp.async.mbarrier.arrive.noinc.shared::cta.b64 [%0];" ::"r"(bar) : "memory");
+}
+
+// Fill cursor of one consumer thread: the stage sequence of the CTA's items
+// (pre-plane, planes kb..ke-1, post-plane of each), its own ring position.
+struct DfgFill {
+  const DfgParams* P;
+  DfgRing W;
+  long long item, q, qe;
+  unsigned off[DFG_FM];  // input element offsets within a plane of this thread's tile elements
+  unsigned tid;
+
+  __device__ __forceinline__ void setup() {
+    const DfgParams& p = *P;
+    const long long tx_ = item % p.tiles_x;
+    const long long rest = item / p.tiles_x;
+    const long long ty_ = rest % p.tiles_y;
+    const long long zc = rest / p.tiles_y;
+    const long long kb = p.kbeg + zc * p.kz;
+    q = kb - 1;
+    qe = min(kb + (long long)p.kz, p.kend);
+    const int x0 = (int)(tx_ * DFG_TX) - DFG_HX + (int)p.gx;  // input column of tile column 0
+    const int y0 = (int)(ty_ * DFG_TH) - 1 + (int)p.gy;      // input row of tile row 0
+    // clamp to the global mesh ends (R1); elsewhere to the input array
+    const int clo = p.i0 == 0 ? (int)p.gx : 0;
+    const int chi = p.i0 + p.nx >= p.NX ? (int)(p.gx + p.nx - 1) : (int)(p.px - 1);
+    const int rlo = p.j0 == 0 ? (int)p.gy : 0;
+    const int rhi = p.j0 + p.ny >= p.NY ? (int)(p.gy + p.ny - 1) : (int)(p.py - 1);
+#pragma unroll
+    for (int m = 0; m < DFG_FM; ++m) {
+      const unsigned e = tid + m * DFG_NT;
+      const int row = (int)(e / DFG_ROWW), col = (int)(e % DFG_ROWW);
+      const int yy = max(rlo, min(y0 + row, rhi)), xx = max(clo, min(x0 + col, chi));
+      off[m] = (unsigned)yy * (unsigned)p.px + (unsigned)xx;
+    }
+  }
+  __device__ __forceinline__ void init(const DfgParams* p, unsigned smem, unsigned full0, unsigned t) {
+    P = p;
+    W = DfgRing{smem, full0, 0u, 0, smem, full0};
+    tid = t;
+    item = blockIdx.x;
+    if (item < p->items) setup();
+  }
+  // issue this thread's share of the next stage of the sequence
+  __device__ __forceinline__ void step() {
+    const DfgParams& p = *P;
+    if (item >= p.items) return;
+    dfg_mbar_wait(DFG_EMPTY(W.full), W.phase ^ 1u, 0x100000u);
+    const long long pg = max(0LL, min(q, p.NZ - 1));
+    const long long pbase = (pg - p.k0 + p.ghost) * p.px * p.py;
+    const unsigned TS = (unsigned)sizeof(DFG_T);
+#pragma unroll
+    for (int f = 0; f < DFG_NTF; ++f) {
+      const DFG_T* src = p.f[f] + pbase;
+      const unsigned dst = W.tile + f * DFG_TILE_BYTES + tid * TS;
+#pragma unroll
+      for (int m = 0; m < DFG_FM; ++m)
+        if (m < DFG_FM - 1 || tid + m * DFG_NT < (unsigned)DFG_TILE_ELEMS) dfg_cp_async(dst + m * DFG_NT * TS, src + off[m]);
+    }
+    dfg_cp_async_arrive(W.full);
+    W.advance();
+    if (++q > qe) {
+      item += gridDim.x;
+      if (item < p.items) setup();
+    }
+  }
+};
+
+__device__ __forceinline__ void dfg_consume_tile(const DfgParams& P, long long item, DfgRing& R, DfgCol& C, int warp,
+                                                 int lane, DfgFill& F) {
+  const long long plane = P.nx * P.ny;
+  const int col = lane % DFG_LPR, sub = lane / DFG_LPR;
+  const unsigned c0 = DFG_HX + DFG_VEC * col;
+  const unsigned r = 1 + warp * DFG_RPW + sub;
+  const long long tx_ = item % P.tiles_x;
+  const long long rest = item / P.tiles_x;
+  const long long ty_ = rest % P.tiles_y;
+  const long long zc = rest / P.tiles_y;
+  const long long i = tx_ * DFG_TX + DFG_VEC * col;
+  const long long j = ty_ * DFG_TH + warp * DFG_RPW + sub;
+  const long long kb = P.kbeg + zc * P.kz;
+  const long long ke = min(kb + (long long)P.kz, P.kend);
+  C.nvalid = j < P.ny ? (int)max(0LL, min((long long)DFG_VEC, P.nx - i)) : 0;
+  C.act = C.nvalid > 0;
+  const long long ic = min(i, P.nx - 1);
+  const long long jc = min(j, P.ny - 1);
+#pragma unroll
+  for (int h = 0; h < DFG_NPAIR; ++h) {
+    // per-cell spacing entries (a ragged vector's outside cells reuse the last)
+    const long long a = min(P.i0 + i + h * DFG_LANES, P.NX - 1);
+    const long long b = min(P.i0 + i + h * DFG_LANES + DFG_LANES - 1, P.NX - 1);
+    C.ndx[h] = dfg2_mk(__ldg(P.tx + DFG_NDSEG_X * P.NX + a), __ldg(P.tx + DFG_NDSEG_X * P.NX + b));
+    C.rx[h] = dfg2_mk(__ldg(P.tx + P.NX + a), __ldg(P.tx + P.NX + b));
+  }
+  C.ndy = dfg2_splat(__ldg(P.ty + DFG_NDSEG_Y * P.NY + P.j0 + jc));
+  C.ry = dfg2_splat(__ldg(P.ty + P.NY + P.j0 + jc));
+  // the fill replicates the boundary cells past the global ends: plain offsets
+  const unsigned TS = (unsigned)sizeof(DFG_T);
+  C.off_c = (r * DFG_ROWW + c0) * TS;
+  C.off_xm = (r * DFG_ROWW + c0 - 1) * TS;
+  C.off_xp = (r * DFG_ROWW + c0 + DFG_VEC) * TS;
+  C.off_ym = ((r - 1) * DFG_ROWW + c0) * TS;
+  C.off_yp = ((r + 1) * DFG_ROWW + c0) * TS;
+  DFG_T* outp = P.out + ((kb - P.k0) * plane + jc * P.nx + ic) * DFG_OUTW;
+  const DFG_T* tzp = P.tz + kb;
+
+  DFG_T zq[3][DFG_NSF][DFG_VEC];
+  dfg_mbar_wait(R.full, R.phase, 0x100000u);
+#pragma unroll
+  for (int f = 0; f < DFG_NSF; ++f) dfg_lds16(zq[0][f], R.tile + f * DFG_TILE_BYTES + C.off_c);
+  dfg_mbar_arrive(DFG_EMPTY(R.full));
+  F.step();
+  R.advance();
+  dfg_mbar_wait(R.full, R.phase, 0x100000u);
+  unsigned cur_tile = R.tile, cur_full = R.full;
+#pragma unroll
+  for (int f = 0; f < DFG_NSF; ++f) dfg_lds16(zq[1][f], cur_tile + f * DFG_TILE_BYTES + C.off_c);
+  R.advance();
+  long long k = kb;
+  for (; k + 3 <= ke; k += 3) {
+    dfg_plane<0, 1, 2, true>(C, R, cur_tile, cur_full, zq, outp, plane, tzp, P.NZ, F);
+    dfg_plane<1, 2, 0, true>(C, R, cur_tile, cur_full, zq, outp, plane, tzp, P.NZ, F);
+    dfg_plane<2, 0, 1, true>(C, R, cur_tile, cur_full, zq, outp, plane, tzp, P.NZ, F);
+  }
+  if (k < ke) {
+    dfg_plane<0, 1, 2, true>(C, R, cur_tile, cur_full, zq, outp, plane, tzp, P.NZ, F);
+    if (k + 1 < ke) dfg_plane<1, 2, 0, true>(C, R, cur_tile, cur_full, zq, outp, plane, tzp, P.NZ, F);
+  }
+  dfg_mbar_arrive(DFG_EMPTY(cur_full));
+  F.step();
+}
+
+extern "C" __global__ void __launch_bounds__(DFG_NCW * 32, DFG_CTAS) dfg_fused_tile(const __grid_constant__ DfgParams P) {
+  const unsigned smem = dfg_ring_init(DFG_NCW * 32);
+  const unsigned full0 = smem + DFG_STAGES * DFG_STAGE_BYTES;
+  const int warp = threadIdx.x >> 5;
+  const int lane = threadIdx.x & 31;
+  DfgFill F;
+  F.init(&P, smem, full0, threadIdx.x);
+  for (int n = 0; n < DFG_STAGES - 1; ++n) F.step();
+  DfgRing R{smem, full0, 0u, 0, smem, full0};
+  DfgCol C;
+  C.Z = dfg2_splat(P.nzero);
+  C.vst = P.vec_ok != 0;
+  for (long long item = blockIdx.x; item < P.items; item += gridDim.x) dfg_consume_tile(P, item, R, C, warp, lane, F);
 }
 #endif

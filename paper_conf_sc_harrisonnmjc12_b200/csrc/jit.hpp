@@ -24,6 +24,7 @@ struct LoadedModule {
   CUmodule mod = nullptr;
   CUfunction pointwise = nullptr, general = nullptr, tma = nullptr;
   CUfunction tma_multi = nullptr;  // several meshes per launch (dfg_execute_blocks)
+  CUfunction tile = nullptr;       // same ring, filled by cp.async (layouts TMA cannot describe)
 };
 
 // Load into the current context (requires a device).

@@ -174,6 +174,7 @@ std::unique_ptr<PlanImpl> compile_plan(std::shared_ptr<MeshImpl> mesh, const std
                                          plan->fsrc.cfg.stages, plan->fsrc.cfg.rpw);
       DFG_CU(drv().FuncSetAttribute(plan->mod.tma, CU_FUNC_ATTRIBUTE_MAX_DYNAMIC_SHARED_SIZE_BYTES, int(smem)));
       DFG_CU(drv().FuncSetAttribute(plan->mod.tma_multi, CU_FUNC_ATTRIBUTE_MAX_DYNAMIC_SHARED_SIZE_BYTES, int(smem)));
+      DFG_CU(drv().FuncSetAttribute(plan->mod.tile, CU_FUNC_ATTRIBUTE_MAX_DYNAMIC_SHARED_SIZE_BYTES, int(smem)));
     }
   }
   return plan;
@@ -455,7 +456,8 @@ void PlanImpl::launch_fused(const std::vector<const void*>& fptr, void* dout, co
   bool vec_ok = aligned16(dout) && (N % vec == 0) && m.gxy == 0 && m.px() == m.nx && m.gx() == 0;
   for (auto p : fptr) vec_ok = vec_ok && aligned16(p);
   const char* force = std::getenv("DFG_FUSED_KERNEL");
-  bool want_general = force && !std::strcmp(force, "general");
+  const bool want_general = force && !std::strcmp(force, "general");
+  const bool want_tile = force && !std::strcmp(force, "tile");
   const int sms = sm_count(mesh->device);
 
   if (L.stencil_inputs.empty()) {
@@ -467,7 +469,7 @@ void PlanImpl::launch_fused(const std::vector<const void*>& fptr, void* dout, co
     DFG_CU(drv().LaunchKernel(mod.pointwise, grid, 1, 1, 256, 1, 1, 0, s, args, nullptr));
     kernel_end(ke, s);
     last_variant = 3;
-  } else if (mod.tma && !want_general && m.nx % vec == 0 && m.px() % vec == 0 && m.gx() % vec == 0 &&
+  } else if (mod.tma && !want_general && !want_tile && m.nx % vec == 0 && m.px() % vec == 0 && m.gx() % vec == 0 &&
              aligned16(dout) &&
              std::all_of(fptr.begin(), fptr.end(), [](const void* p) { return aligned16(p); })) {
     const int ncw = fsrc.cfg.ncw, rpw = fsrc.cfg.rpw;
@@ -509,6 +511,33 @@ void PlanImpl::launch_fused(const std::vector<const void*>& fptr, void* dout, co
     kernel_end(ke, s);
     last_variant = 1;
     last_kz = best_kz;
+  } else if (mod.tile && !want_general && m.px() * m.py() < (int64_t(1) << 32)) {
+    // same ring and consumers, filled by the consumer threads with cp.async
+    const int ncw = fsrc.cfg.ncw, rpw = fsrc.cfg.rpw;
+    const int nsf = int(L.stencil_inputs.size() + L.point_inputs.size());
+    const int tw = tma_tile_w(m.dt, rpw), th = tma_tile_h(ncw, rpw);
+    const int tiles_x = int((m.nx + tw - 1) / tw);
+    const int tiles_y = int((m.ny + th - 1) / th);
+    const int64_t range = kend - kbeg;
+    size_t smem = fused_tma_smem_bytes(m.dt, nsf, ncw, fsrc.cfg.stages, rpw);
+    int occ = 1;
+    DFG_CU(drv().OccupancyMaxActiveBlocksPerMultiprocessor(&occ, mod.tile, ncw * 32, smem));
+    const int64_t slots = int64_t(sms) * std::max(occ, 1);
+    const char* kzenv = std::getenv("DFG_KZ");
+    const int64_t kz = kzenv ? std::max<int64_t>(1, std::min<int64_t>(range, std::atoll(kzenv)))
+                             : choose_kz(int64_t(tiles_x) * tiles_y, range, slots);
+    const int64_t items = int64_t(tiles_x) * tiles_y * ((range + kz - 1) / kz);
+    const unsigned grid = unsigned(std::min<int64_t>(items, slots));
+    // 16-byte output stores need aligned rows (the inputs may be anything)
+    const bool out16 = aligned16(dout) && m.nx % vec == 0;
+    auto w = pack_params(fptr, dout, tab[0], tab[1], tab[2], m, kbeg, kend, items, tiles_x, tiles_y, int(kz),
+                         out16 ? 1 : 0);
+    void* args[] = {w.data()};
+    auto ke = kernel_begin(s);
+    DFG_CU(drv().LaunchKernel(mod.tile, grid, 1, 1, ncw * 32, 1, 1, unsigned(smem), s, args, nullptr));
+    kernel_end(ke, s);
+    last_variant = 5;
+    last_kz = kz;
   } else {
     // z-marching columns: enough (column, z-chunk) units to fill the device
     // (~2048 threads per SM), each chunk as long as that allows

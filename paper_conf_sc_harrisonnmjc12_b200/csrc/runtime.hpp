@@ -120,7 +120,7 @@ struct PlanImpl {
   FusedSource fsrc;
   LoadedModule mod;
   int regs = 0, spill = 0;
-  int last_variant = 0;  // 1 TMA, 2 general, 3 pointwise, 4 TMA multi-block (dfg_execute_blocks)
+  int last_variant = 0;  // 1 TMA, 2 general, 3 pointwise, 4 TMA multi-block (dfg_execute_blocks), 5 tile (cp.async ring)
   int64_t last_kz = 0;   // z-chunk length of the last TMA launch
   dfg_stats st{};
   cudaEvent_t ev0 = nullptr, ev1 = nullptr;

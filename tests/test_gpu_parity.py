@@ -56,6 +56,41 @@ def test_tma_and_general_kernels_identical(T, monkeypatch):
     b, plan2, *_ = run_lib(src, f, x, y, z, return_plan=True)
     assert plan2.info()["variant"] == 2
     assert np.array_equal(a, b)
+    monkeypatch.setenv("DFG_FUSED_KERNEL", "tile")
+    c, plan3, *_ = run_lib(src, f, x, y, z, return_plan=True)
+    assert plan3.info()["variant"] == 5
+    assert np.array_equal(a, c)
+
+
+@pytest.mark.parametrize("prog", PROGS)
+@pytest.mark.parametrize("T", [np.float32, np.float64])
+@pytest.mark.parametrize("shape", [(67, 45, 37), (130, 17, 5), (5, 70, 9), (1, 33, 6), (129, 1, 4), (3, 2, 1)])
+@pytest.mark.parametrize("rpw", ["1", "2", "4"])
+def test_tile_kernel(prog, T, shape, rpw, monkeypatch):
+    """The cp.async-filled ring (layouts a tensor map cannot describe): rows
+    that are not a multiple of 16 bytes, ragged last vectors, degenerate
+    axes, every tile shape -- the oracle's bits."""
+    x, y, z, f = _inputs(shape, T, NAMES[prog])
+    src = PAPER_PROGRAMS[prog][0]
+    want = run_oracle(src, f, x, y, z)
+    monkeypatch.setenv("DFG_RPW", rpw)
+    got, plan, *_ = run_lib(src, f, x, y, z, return_plan=True)
+    if prog != "velmag":
+        vec = 4 if T == np.float32 else 2
+        assert plan.info()["variant"] == (5 if shape[0] % vec else 1)
+    assert_parity(got, want)
+
+
+@pytest.mark.parametrize("kz", ["1", "2", "5", "1000"])
+def test_tile_kernel_z_chunks(kz, monkeypatch):
+    """Every z-chunk length: the fill cursor crosses item boundaries."""
+    x, y, z, f = _inputs((67, 31, 29), np.float32)
+    src = PAPER_PROGRAMS["qcrit"][0]
+    want = run_oracle(src, f, x, y, z)
+    monkeypatch.setenv("DFG_KZ", kz)
+    got, plan, *_ = run_lib(src, f, x, y, z, return_plan=True)
+    assert plan.info()["variant"] == 5 and plan.info()["kz"] == min(int(kz), 29)
+    assert_parity(got, want)
 
 
 @pytest.mark.parametrize("shape", [(132, 40, 33), (67, 45, 37)])
@@ -384,6 +419,8 @@ def test_visit_blocks_with_ghost_shells(shape, split, prog, strategy, pitch):
                 torch.cuda.synchronize()
                 if pitch == "padded" and bx % 4 == 0 and prog != "velmag":
                     assert p.info()["variant"] == 1          # TMA kernel on the padded shell
+                elif prog != "velmag":
+                    assert p.info()["variant"] == 5          # packed shell: the cp.async-filled ring
                 got[k0:k1, j0:j1, i0:i1] = o.cpu().numpy()
                 blocks.append((p, torch.full_like(o, float("nan")), (k0, k1, j0, j1, i0, i1), m, keep))
     assert np.array_equal(got, whole)
