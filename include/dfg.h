@@ -97,7 +97,8 @@ typedef struct {
   int64_t kernel_count;         /* kernel executions ("K-Exe")                */
   int64_t h2d_bytes;
   int64_t d2h_bytes;
-  int64_t halo_bytes;           /* bytes received into ghost planes           */
+  int64_t halo_bytes;           /* bytes received into ghost planes, or read
+                                   from the neighbours' planes (peer halo)    */
   int64_t dev_highwater_bytes;  /* max live problem-sized device arrays, incl.
                                    bound device inputs and the output (Fig. 2) */
   int64_t predicted_highwater_bytes; /* model of the last-executed mode        */
@@ -185,6 +186,36 @@ int dfg_halo_map(dfg_mesh mesh, int64_t out[16]);
  * NCCL is loaded at run time (libnccl.so.2); DFG_E_NCCL if unavailable. */
 int dfg_nccl_unique_id(void* out128);
 int dfg_mesh_init_comm(dfg_mesh mesh, const void* id128, int rank, int nranks);
+
+/* Peer-memory halo, one process per GPU (the B200 path for z-slabs: the
+ * fused kernel reads the neighbours' boundary planes in place over NVLink
+ * instead of receiving copies).
+ *
+ * dfg_mesh_peer_export writes DFG_PEER_BLOB_BYTES bytes describing the slab:
+ * CUDA IPC handles (and offsets) of every field bound with on_device = 1 and
+ * of a small flag block the library allocates, the slab's extent and type.
+ * Bind the fields first; rebinding a field afterwards makes dfg_execute fail
+ * with DFG_E_INVALID until the blob is exported and linked again.  The fields
+ * must be cudaMalloc-backed (IPC), the mesh a z-slab with ghost = 1.
+ *
+ * Every rank exchanges blobs (e.g. torch.distributed all_gather_object) and
+ * calls dfg_mesh_link_peers with the blob of the slab directly below (lo,
+ * NULL on rank 0) and directly above (hi, NULL on the last rank).  Checks:
+ * magic, type, plane size, global depth and adjacency (DFG_E_INVALID);
+ * DFG_E_UNSUPPORTED if CUDA IPC is refused.  The mappings stay open until the
+ * mesh is destroyed (the exporting ranks must keep their fields alive).
+ *
+ * A linked slab's dfg_execute (fused / reference strategies) orders itself
+ * with its neighbours by step flags (stream memory operations: the execute
+ * publishes "ready", waits for the neighbours' "ready" before the boundary
+ * planes, and before returning the stream waits until both neighbours have
+ * read its planes), so every rank must execute the same sequence of plans on
+ * the mesh.  Its ghost planes are not written (TMA reads the neighbours'
+ * buffers), except for layouts the TMA kernel cannot take, which copy the two
+ * planes through the mappings first.  The output must be on the device. */
+#define DFG_PEER_BLOB_BYTES 4096
+int dfg_mesh_peer_export(dfg_mesh mesh, void* blob, size_t cap);
+int dfg_mesh_link_peers(dfg_mesh mesh, const void* lo_blob, const void* hi_blob);
 
 /* Single-process halo transport: slabs that live in one process (one or
  * several devices) exchange ghost planes with device-to-device copies.
@@ -274,9 +305,11 @@ int dfg_plan_set_timing(dfg_plan plan, int level);
  * DFG_FUSED_VARIANT selects them), out[9] = tile rows per consumer warp of
  * the TMA kernel (1, 2 or 4; 0 without one), out[10] / out[11] = its tile
  * width (cells along x) / height (rows along y), out[12] = z-chunk length
- * (planes per work item) of the last TMA launch (0 before one).  `out` must
- * hold 13 entries. */
-int dfg_plan_info(dfg_plan plan, int64_t out[13]);
+ * (planes per work item) of the last TMA launch (0 before one), out[13] =
+ * halo transport of the last execute (0 none, 1 NCCL, 2 local device copies,
+ * 3 peer memory read in place by the kernel, 4 peer memory copied into the
+ * ghost planes).  `out` must hold 14 entries. */
+int dfg_plan_info(dfg_plan plan, int64_t out[14]);
 
 /* Execution order of the plan's filters (ids of the canonical text).  Staged
  * plans run the paper's list order unless a dev_mem_cap rejected it and the

@@ -73,6 +73,16 @@ class Mesh:
     def halo_map(self):
         return dfg_halo_map(self.handle)
 
+    def peer_export(self) -> bytes:
+        """Blob for the z neighbours' link_peers (bind the device fields first)."""
+        from ._dfg import dfg_mesh_peer_export
+        return dfg_mesh_peer_export(self.handle)
+
+    def link_peers(self, lo_blob, hi_blob):
+        """Read the neighbours' boundary planes in place (peer-memory halo)."""
+        from ._dfg import dfg_mesh_link_peers
+        dfg_mesh_link_peers(self.handle, lo_blob, hi_blob)
+
     def close(self):
         if self.handle:
             dfg_destroy_mesh(self.handle)

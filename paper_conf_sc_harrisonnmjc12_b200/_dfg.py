@@ -64,6 +64,8 @@ _SIGS = {
     "dfg_nccl_unique_id": (C.c_int, [_P]),
     "dfg_mesh_init_comm": (C.c_int, [_P, _P, C.c_int, C.c_int]),
     "dfg_mesh_link_local": (C.c_int, [_P, _P]),
+    "dfg_mesh_peer_export": (C.c_int, [_P, _P, C.c_size_t]),
+    "dfg_mesh_link_peers": (C.c_int, [_P, _P, _P]),
     "dfg_bind_field": (C.c_int, [_P, C.c_char_p, _P, C.c_int]),
     "dfg_compile": (C.c_int, [_P, C.c_char_p, C.c_int, C.c_size_t, C.POINTER(_P)]),
     "dfg_destroy_plan": (None, [_P]),
@@ -178,6 +180,22 @@ def dfg_mesh_init_comm(mesh, uid: bytes, rank, nranks):
     _check(_lib.dfg_mesh_init_comm(mesh, buf, rank, nranks))
 
 
+PEER_BLOB_BYTES = 4096
+
+
+def dfg_mesh_peer_export(mesh) -> bytes:
+    buf = C.create_string_buffer(PEER_BLOB_BYTES)
+    _check(_lib.dfg_mesh_peer_export(mesh, buf, PEER_BLOB_BYTES))
+    return buf.raw
+
+
+def dfg_mesh_link_peers(mesh, lo_blob, hi_blob):
+    def arg(b):
+        return None if b is None else C.create_string_buffer(bytes(b), PEER_BLOB_BYTES)
+    lo, hi = arg(lo_blob), arg(hi_blob)
+    _check(_lib.dfg_mesh_link_peers(mesh, lo, hi))
+
+
 def dfg_mesh_link_local(lo, hi):
     _check(_lib.dfg_mesh_link_local(lo, hi))
 
@@ -217,10 +235,10 @@ def dfg_reset_stats(plan):
 
 
 def dfg_plan_info(plan) -> dict:
-    out = (_I64 * 13)()
+    out = (_I64 * 14)()
     _check(_lib.dfg_plan_info(plan, out))
     keys = ("strategy", "width", "filters", "variant", "regs", "spill", "footprint_device", "footprint_host",
-            "div2_axes", "rows_per_warp", "tile_w", "tile_h", "kz")
+            "div2_axes", "rows_per_warp", "tile_w", "tile_h", "kz", "halo")
     return dict(zip(keys, list(out)))
 
 

@@ -145,6 +145,21 @@ int dfg_mesh_init_comm(dfg_mesh mesh, const void* id128, int rank, int nranks) {
   });
 }
 
+int dfg_mesh_peer_export(dfg_mesh mesh, void* blob, size_t cap) {
+  return guard([&] {
+    if (!mesh || !blob) dfg::fail(DFG_E_INVALID, "null argument");
+    if (cap < dfg::kPeerBlobBytes) dfg::fail(DFG_E_RANGE, "peer blob needs DFG_PEER_BLOB_BYTES bytes");
+    dfg::mesh_peer_export(*mesh->m, blob);
+  });
+}
+
+int dfg_mesh_link_peers(dfg_mesh mesh, const void* lo_blob, const void* hi_blob) {
+  return guard([&] {
+    if (!mesh) dfg::fail(DFG_E_INVALID, "null mesh");
+    dfg::mesh_link_peers(*mesh->m, lo_blob, hi_blob);
+  });
+}
+
 int dfg_mesh_link_local(dfg_mesh lo, dfg_mesh hi) {
   return guard([&] {
     if (!lo || !hi) dfg::fail(DFG_E_INVALID, "null mesh");
@@ -245,7 +260,7 @@ int dfg_reset_stats(dfg_plan plan) {
   });
 }
 
-int dfg_plan_info(dfg_plan plan, int64_t out[13]) {
+int dfg_plan_info(dfg_plan plan, int64_t out[14]) {
   return guard([&] {
     if (!plan || !out) dfg::fail(DFG_E_INVALID, "null argument");
     auto& p = *plan->p;
@@ -265,6 +280,7 @@ int dfg_plan_info(dfg_plan plan, int64_t out[13]) {
     out[10] = tma ? dfg::tma_tile_w(m.dt, p.fsrc.cfg.rpw) : 0;
     out[11] = tma ? dfg::tma_tile_h(p.fsrc.cfg.ncw, p.fsrc.cfg.rpw) : 0;
     out[12] = p.last_kz;
+    out[13] = p.last_halo;
   });
 }
 

@@ -27,6 +27,11 @@ struct DriverApi {
                                    const cuuint64_t*, const cuuint32_t*, const cuuint32_t*, CUtensorMapInterleave,
                                    CUtensorMapSwizzle, CUtensorMapL2promotion,
                                    CUtensorMapFloatOOBfill) = nullptr;
+  // peer-memory halo (z-slabs): allocation ranges for IPC export, stream
+  // memory operations for the ready / done flags
+  CUresult (*MemGetAddressRange)(CUdeviceptr*, size_t*, CUdeviceptr) = nullptr;
+  CUresult (*StreamWriteValue32)(CUstream, CUdeviceptr, cuuint32_t, unsigned) = nullptr;
+  CUresult (*StreamWaitValue32)(CUstream, CUdeviceptr, cuuint32_t, unsigned) = nullptr;
 };
 
 inline DriverApi& drv() {
@@ -48,7 +53,10 @@ inline DriverApi& drv() {
          get("cuLaunchKernel", reinterpret_cast<void**>(&api.LaunchKernel)) &&
          get("cuOccupancyMaxActiveBlocksPerMultiprocessor",
              reinterpret_cast<void**>(&api.OccupancyMaxActiveBlocksPerMultiprocessor)) &&
-         get("cuTensorMapEncodeTiled", reinterpret_cast<void**>(&api.TensorMapEncodeTiled));
+         get("cuTensorMapEncodeTiled", reinterpret_cast<void**>(&api.TensorMapEncodeTiled)) &&
+         get("cuMemGetAddressRange", reinterpret_cast<void**>(&api.MemGetAddressRange)) &&
+         get("cuStreamWriteValue32", reinterpret_cast<void**>(&api.StreamWriteValue32)) &&
+         get("cuStreamWaitValue32", reinterpret_cast<void**>(&api.StreamWaitValue32));
     if (!ok) cudaGetLastError();
   });
   if (!ok) fail(DFG_E_CUDA, "CUDA driver API unavailable (no driver / no device); libdfg has no CPU fallback");

@@ -25,8 +25,17 @@
 
 #if DFG_NSF > 0 && DFG_HAS_TMA
 struct __align__(64) DfgTmap { unsigned long long v[16]; };  // CUtensorMap
+// Peer-memory halo of a z-slab: the neighbours' stencil fields, read in place
+// (IPC mappings) for the planes outside [k0, k0 + nzl).
+struct DfgPeerInfo {
+  long long lo_k0, lo_ghost, hi_k0, hi_ghost;
+  int lo_on, hi_on, pad0, pad1;
+};
+// host image: runtime.cpp tma_blob_* (same order, 64-byte aligned maps)
 struct DfgTmaParams {
   DfgTmap map[DFG_NF_];  // stencil fields, then point-wise fields
+  DfgTmap map_lo[DFG_NSF_], map_hi[DFG_NSF_];  // neighbours' stencil fields (peer halo)
+  DfgPeerInfo peer;
   DfgParams p;
 };
 
@@ -256,8 +265,16 @@ __device__ __forceinline__ void dfg_produce_item(const DfgTmaParams& TP, long lo
     dfg_mbar_wait(DFG_EMPTY(W.full), W.phase ^ 1u, 0x100000u);
     dfg_mbar_expect_tx(W.full, (unsigned)(DFG_NTF * DFG_TILE_ELEMS * sizeof(DFG_T)));
     const int zl = (int)(pg - P.k0 + P.ghost);
+    // planes of the z neighbours come from their own buffers when the slab is
+    // linked to peers (stencil fields only; point-wise fields are read at owned planes)
+    const bool lo = TP.peer.lo_on && pg < P.k0, hi = TP.peer.hi_on && pg >= P.k0 + P.nzl;
+    const int zp = lo ? (int)(pg - TP.peer.lo_k0 + TP.peer.lo_ghost) : (int)(pg - TP.peer.hi_k0 + TP.peer.hi_ghost);
 #pragma unroll
-    for (int f = 0; f < DFG_NTF; ++f) dfg_tma_load3(W.tile + f * DFG_TILE_BYTES, &TP.map[f], W.full, x0, y0, zl);
+    for (int f = 0; f < DFG_NTF; ++f) {
+      const bool peer = (lo || hi) && f < DFG_NSF;
+      const DfgTmap* map = !peer ? &TP.map[f] : lo ? &TP.map_lo[f < DFG_NSF ? f : 0] : &TP.map_hi[f < DFG_NSF ? f : 0];
+      dfg_tma_load3(W.tile + f * DFG_TILE_BYTES, map, W.full, x0, y0, peer ? zp : zl);
+    }
     W.advance();
   }
 }

@@ -150,6 +150,8 @@ MeshImpl::~MeshImpl() {
   cudaSetDevice(device);
   for (auto& p : dev_tab)
     if (p) cudaFree(p);
+  for (void* p : ipc_opened) cudaIpcCloseMemHandle(p);
+  if (flags) cudaFree(flags);
   if (nccl) {
     using destroy_fn = ncclResult_t (*)(ncclComm_t);
     void* h = dlopen("libnccl.so.2", RTLD_NOW | RTLD_NOLOAD);
@@ -295,6 +297,115 @@ void mesh_init_comm(MeshImpl& m, const void* id128, int rank, int nranks) {
   m.nccl = comm;
   m.rank = rank;
   m.nranks = nranks;
+}
+
+// ------------------------------------------------------- peer-memory halo
+namespace {
+struct PeerBlobField {
+  char name[48];
+  cudaIpcMemHandle_t h;
+  int64_t off;
+};
+struct PeerBlob {
+  char magic[8];
+  int32_t dtype, nfields;
+  int64_t nx, ny, nzl, NZ, k0, ghost;
+  cudaIpcMemHandle_t flags_h;
+  int64_t flags_off;
+  PeerBlobField f[24];
+};
+static_assert(sizeof(PeerBlob) <= kPeerBlobBytes, "peer blob too large");
+const char kMagic[8] = {'d', 'f', 'g', 'p', 'e', 'e', 'r', '1'};
+
+// IPC handle of the cudaMalloc allocation holding p, and p's offset in it
+void ipc_export(const void* p, cudaIpcMemHandle_t* h, int64_t* off) {
+  CUdeviceptr base = 0;
+  size_t size = 0;
+  DFG_CU(drv().MemGetAddressRange(&base, &size, reinterpret_cast<CUdeviceptr>(p)));
+  cudaError_t e = cudaIpcGetMemHandle(h, reinterpret_cast<void*>(base));
+  if (e != cudaSuccess) {
+    cudaGetLastError();
+    fail(DFG_E_UNSUPPORTED, std::string("cudaIpcGetMemHandle: ") + cudaGetErrorString(e) +
+                                " (peer halo needs cudaMalloc-backed device fields)");
+  }
+  *off = int64_t(reinterpret_cast<CUdeviceptr>(p) - base);
+}
+
+void ensure_flags(MeshImpl& m) {
+  if (m.flags) return;
+  DFG_CUDA(cudaSetDevice(m.device));
+  DFG_CUDA(cudaMalloc(&m.flags, 256));
+  DFG_CUDA(cudaMemset(m.flags, 0, 256));
+  DFG_CUDA(cudaDeviceSynchronize());
+}
+}  // namespace
+
+void mesh_peer_export(MeshImpl& m, void* out) {
+  if (m.ghost != 1 || m.gxy != 0 || m.ghosts_supplied)
+    fail(DFG_E_INVALID, "peer halo: the mesh must be a z-slab with one ghost plane per side (dfg_create_mesh ghost=1)");
+  DFG_CUDA(cudaSetDevice(m.device));
+  ensure_flags(m);
+  PeerBlob b;
+  std::memset(&b, 0, sizeof(b));
+  std::memcpy(b.magic, kMagic, 8);
+  b.dtype = m.dt == DType::F32 ? 0 : 1;
+  b.nx = m.nx, b.ny = m.ny, b.nzl = m.nzl, b.NZ = m.NZ, b.k0 = m.k0, b.ghost = m.ghost;
+  ipc_export(m.flags, &b.flags_h, &b.flags_off);
+  m.exported.clear();
+  for (auto& kv : m.fields) {
+    if (!kv.second.on_device || !kv.second.ptr) continue;
+    if (b.nfields == int32_t(sizeof(b.f) / sizeof(b.f[0]))) fail(DFG_E_UNSUPPORTED, "peer halo: too many bound fields");
+    if (kv.first.size() >= sizeof(b.f[0].name)) fail(DFG_E_UNSUPPORTED, "peer halo: field name too long");
+    PeerBlobField& f = b.f[b.nfields++];
+    std::memcpy(f.name, kv.first.c_str(), kv.first.size());
+    ipc_export(kv.second.ptr, &f.h, &f.off);
+    m.exported[kv.first] = kv.second.ptr;
+  }
+  std::memset(out, 0, kPeerBlobBytes);
+  std::memcpy(out, &b, sizeof(b));
+}
+
+void mesh_link_peers(MeshImpl& m, const void* lo_blob, const void* hi_blob) {
+  const bool has_lo = m.k0 > 0, has_hi = m.k0 + m.nzl < m.NZ;
+  if (has_lo != (lo_blob != nullptr) || has_hi != (hi_blob != nullptr))
+    fail(DFG_E_INVALID, "peer halo: give the blob of every z neighbour and no other");
+  if (m.ghost != 1) fail(DFG_E_INVALID, "peer halo: the mesh needs one ghost plane per side");
+  DFG_CUDA(cudaSetDevice(m.device));
+  ensure_flags(m);
+  std::map<std::string, void*> opened;  // handle bytes -> mapped allocation base
+  auto open = [&](const cudaIpcMemHandle_t& h) -> char* {
+    std::string key(reinterpret_cast<const char*>(&h), sizeof(h));
+    auto it = opened.find(key);
+    if (it != opened.end()) return static_cast<char*>(it->second);
+    void* p = nullptr;
+    cudaError_t e = cudaIpcOpenMemHandle(&p, h, cudaIpcMemLazyEnablePeerAccess);
+    if (e != cudaSuccess) {
+      cudaGetLastError();
+      fail(DFG_E_UNSUPPORTED, std::string("cudaIpcOpenMemHandle: ") + cudaGetErrorString(e));
+    }
+    m.ipc_opened.push_back(p);
+    opened[key] = p;
+    return static_cast<char*>(p);
+  };
+  auto link = [&](const void* blob, MeshImpl::Peer& peer, bool below) {
+    PeerBlob b;
+    std::memcpy(&b, blob, sizeof(b));
+    if (std::memcmp(b.magic, kMagic, 8) != 0) fail(DFG_E_INVALID, "peer halo: not a dfg_mesh_peer_export blob");
+    if (b.dtype != (m.dt == DType::F32 ? 0 : 1) || b.nx != m.nx || b.ny != m.ny || b.NZ != m.NZ || b.ghost != 1)
+      fail(DFG_E_INVALID, "peer halo: neighbour slab has another type, plane size, global depth or ghost width");
+    if (below ? b.k0 + b.nzl != m.k0 : m.k0 + m.nzl != b.k0)
+      fail(DFG_E_INVALID, "peer halo: blob is not the adjacent z slab");
+    peer = MeshImpl::Peer{};
+    peer.k0 = b.k0, peer.nzl = b.nzl, peer.ghost = b.ghost;
+    peer.flags = reinterpret_cast<uint32_t*>(open(b.flags_h) + b.flags_off);
+    for (int i = 0; i < b.nfields && i < int(sizeof(b.f) / sizeof(b.f[0])); ++i) {
+      std::string name(b.f[i].name, strnlen(b.f[i].name, sizeof(b.f[i].name)));
+      peer.fields[name] = open(b.f[i].h) + b.f[i].off;
+    }
+    peer.on = true;
+  };
+  if (lo_blob) link(lo_blob, m.peer_lo, true);
+  if (hi_blob) link(hi_blob, m.peer_hi, false);
 }
 
 }  // namespace dfg

@@ -225,6 +225,7 @@ void PlanImpl::halo_exchange(const std::vector<int>& inputs, cudaStream_t s) {
   const size_t pb = size_t(m.plane()) * ts;
   auto lo = m.link_lo.lock(), hi = m.link_hi.lock();
   if (m.nccl) {
+    last_halo = 1;
     auto& api = nccl();
     ncclComm_t comm = static_cast<ncclComm_t>(m.nccl);
     ncclDataType_t t = m.dt == DType::F32 ? ncclFloat32 : ncclFloat64;
@@ -244,6 +245,7 @@ void PlanImpl::halo_exchange(const std::vector<int>& inputs, cudaStream_t s) {
   } else if (lo || hi || (has_lo && !lo) || (has_hi && !hi)) {
     if ((has_lo && !lo) || (has_hi && !hi))
       fail(DFG_E_INVALID, "slab has neighbours but no halo transport (dfg_mesh_init_comm / dfg_mesh_link_local)");
+    last_halo = 2;
     for (int in : inputs) {
       const std::string& name = dag.inputs[in];
       char* base = static_cast<char*>(m.fields[name].ptr);
@@ -317,6 +319,23 @@ void encode_map(CUtensorMap* map, const SlabView& m, void* base, int ncw, int rp
                                 CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE));
 }
 
+// Host image of DfgTmaParams (fused_tma.cuh): map[NF_] | map_lo[NSF_] |
+// map_hi[NSF_] | DfgPeerInfo (48 B) | DfgParams, each map 128 B (64-aligned),
+// total padded to 64 bytes.
+struct TmaBlobLayout {
+  size_t lo, hi, peer, params, size;
+};
+TmaBlobLayout tma_blob_layout(int nf, int nsf, size_t param_words) {
+  const size_t NF = size_t(std::max(nf, 1)), NSF = size_t(std::max(nsf, 1));
+  TmaBlobLayout b;
+  b.lo = 128 * NF;
+  b.hi = b.lo + 128 * NSF;
+  b.peer = b.hi + 128 * NSF;
+  b.params = b.peer + 48;
+  b.size = (b.params + param_words * 8 + 63) / 64 * 64;
+  return b;
+}
+
 // Host mirror of DfgParams in skeleton.cuh (same field order and widths).
 std::vector<uint64_t> pack_params(const std::vector<const void*>& f, void* out, const void* tx, const void* ty,
                                   const void* tz, const SlabView& m, int64_t kbeg, int64_t kend, int64_t items,
@@ -387,7 +406,16 @@ void PlanImpl::exec_fused(void* out, bool out_dev, cudaStream_t s) {
   const bool need_lo = m.k0 > 0, need_hi = m.k0 + m.nzl < m.NZ;
   const bool halo = !any_host && !L.stencil_inputs.empty() && (need_lo || need_hi) && !m.ghosts_supplied;
   const char* ov = std::getenv("DFG_HALO_OVERLAP");
-  const bool overlap = halo && m.nzl >= 3 && !(ov && !std::strcmp(ov, "0"));
+  // peer-memory halo (dfg_mesh_link_peers): no exchange, the kernel reads the
+  // neighbours' planes in place once their "ready" flag shows this step
+  const bool peer = halo && (need_lo ? m.peer_lo.on : true) && (need_hi ? m.peer_hi.on : true);
+  const bool overlap = halo && !peer && m.nzl >= 3 && !(ov && !std::strcmp(ov, "0"));
+  if (peer) {
+    led.add(size_t(N) * size_t(L.outw) * ts);
+    exec_fused_peer(fptr, out, out_dev, s);
+    st.dev_highwater_bytes = std::max<int64_t>(st.dev_highwater_bytes, int64_t(led.high));
+    return;
+  }
   if (halo && !overlap) halo_exchange(L.stencil_inputs, s);
   if (overlap) {
     if (!sHalo) DFG_CUDA(cudaStreamCreateWithFlags(&sHalo, cudaStreamNonBlocking));
@@ -446,8 +474,87 @@ void PlanImpl::exec_fused(void* out, bool out_dev, cudaStream_t s) {
 
 // One launch of the generated kernel over the owned planes of a slab view
 // (the mesh itself, or one z-chunk of the streamed strategy).
+bool PlanImpl::tma_ok(const std::vector<const void*>& fptr, const void* dout, const SlabView& m) const {
+  const int vec = int(16 / dsize(m.dt));
+  const char* force = std::getenv("DFG_FUSED_KERNEL");
+  if (force && (!std::strcmp(force, "general") || !std::strcmp(force, "tile"))) return false;
+  return mod.tma && !fsrc.layout.stencil_inputs.empty() && m.nx % vec == 0 && m.px() % vec == 0 &&
+         m.gx() % vec == 0 && aligned16(dout) &&
+         std::all_of(fptr.begin(), fptr.end(), [](const void* p) { return aligned16(p); });
+}
+
+// Fused execute of a z-slab linked to its neighbours through peer memory.
+// Per step e (the mesh's execute count, equal on every rank):
+//   write own ready = e           (release: this rank's fields are final)
+//   interior planes               (own planes only)
+//   wait ready(lo), ready(hi) >= e
+//   boundary planes               (TMA reads the neighbours' planes in place)
+//   write lo.hi_done = e, hi.lo_done = e   (done reading their planes)
+//   wait own lo_done, hi_done >= e (the caller may overwrite its fields after)
+// The waits are stream memory operations (no SM spins).  Layouts the TMA
+// kernel cannot take copy the neighbours' planes into the ghost planes
+// (device-to-device through the mappings) and run one launch.
+void PlanImpl::exec_fused_peer(const std::vector<const void*>& fptr, void* out, bool out_dev, cudaStream_t s) {
+  MeshImpl& m = *mesh;
+  if (!out_dev) fail(DFG_E_UNSUPPORTED, "peer halo: the output must be a device buffer");
+  for (auto& kv : m.exported) {
+    auto it = m.fields.find(kv.first);
+    if (it == m.fields.end() || it->second.ptr != kv.second)
+      fail(DFG_E_INVALID, "peer halo: field '" + kv.first + "' was rebound after dfg_mesh_peer_export");
+  }
+  const FusedLayout& L = fsrc.layout;
+  for (int in : L.stencil_inputs)
+    if (!m.exported.count(dag.inputs[size_t(in)]))
+      fail(DFG_E_INVALID, "peer halo: field '" + dag.inputs[size_t(in)] + "' was bound after dfg_mesh_peer_export");
+  const bool lo = m.k0 > 0, hi = m.k0 + m.nzl < m.NZ;
+  const uint32_t e = ++m.epoch;
+  auto dptr = [](const uint32_t* p, int w) { return reinterpret_cast<CUdeviceptr>(p + w); };
+  const CUstream cs = reinterpret_cast<CUstream>(s);
+  DFG_CU(drv().StreamWriteValue32(cs, dptr(m.flags, kFlagReady), e, CU_STREAM_WRITE_VALUE_DEFAULT));
+  const void* tab[3] = {m.dev_tab[0], m.dev_tab[1], m.dev_tab[2]};
+  const SlabView v = SlabView::of(m);
+  auto wait_ready = [&] {
+    if (lo) DFG_CU(drv().StreamWaitValue32(cs, dptr(m.peer_lo.flags, kFlagReady), e, CU_STREAM_WAIT_VALUE_GEQ));
+    if (hi) DFG_CU(drv().StreamWaitValue32(cs, dptr(m.peer_hi.flags, kFlagReady), e, CU_STREAM_WAIT_VALUE_GEQ));
+  };
+  if (tma_ok(fptr, out, v)) {
+    const int64_t a = m.k0 + (lo ? 1 : 0), b = m.k0 + m.nzl - (hi ? 1 : 0);
+    if (a < b) launch_fused(fptr, out, tab, v, s, a, b);
+    wait_ready();
+    if (a >= b) {
+      launch_fused(fptr, out, tab, v, s, m.k0, m.k0 + m.nzl, true);
+    } else {
+      if (lo) launch_fused(fptr, out, tab, v, s, m.k0, m.k0 + 1, true);
+      if (hi) launch_fused(fptr, out, tab, v, s, b, b + 1, true);
+    }
+  } else {
+    wait_ready();
+    const size_t pb = size_t(m.plane()) * dsize(m.dt);
+    for (int in : L.stencil_inputs) {
+      const std::string& name = dag.inputs[size_t(in)];
+      char* base = static_cast<char*>(m.fields[name].ptr);
+      if (lo) {
+        const char* src = static_cast<const char*>(m.peer_lo.fields.at(name)) + size_t(m.peer_lo.nzl) * pb;
+        DFG_CUDA(cudaMemcpyAsync(base, src, pb, cudaMemcpyDeviceToDevice, s));
+      }
+      if (hi) {
+        const char* src = static_cast<const char*>(m.peer_hi.fields.at(name)) + size_t(m.peer_hi.ghost) * pb;
+        DFG_CUDA(cudaMemcpyAsync(base + size_t(m.nzl + 1) * pb, src, pb, cudaMemcpyDeviceToDevice, s));
+      }
+    }
+    launch_fused(fptr, out, tab, v, s);
+  }
+  if (lo) DFG_CU(drv().StreamWriteValue32(cs, dptr(m.peer_lo.flags, kFlagHiDone), e, CU_STREAM_WRITE_VALUE_DEFAULT));
+  if (hi) DFG_CU(drv().StreamWriteValue32(cs, dptr(m.peer_hi.flags, kFlagLoDone), e, CU_STREAM_WRITE_VALUE_DEFAULT));
+  if (lo) DFG_CU(drv().StreamWaitValue32(cs, dptr(m.flags, kFlagLoDone), e, CU_STREAM_WAIT_VALUE_GEQ));
+  if (hi) DFG_CU(drv().StreamWaitValue32(cs, dptr(m.flags, kFlagHiDone), e, CU_STREAM_WAIT_VALUE_GEQ));
+  last_halo = tma_ok(fptr, out, v) ? 3 : 4;
+  st.halo_bytes += int64_t(L.stencil_inputs.size()) * ((lo ? 1 : 0) + (hi ? 1 : 0)) * int64_t(m.plane()) *
+                        int64_t(dsize(m.dt));
+}
+
 void PlanImpl::launch_fused(const std::vector<const void*>& fptr, void* dout, const void* const tab[3],
-                            const SlabView& m, cudaStream_t s, int64_t kb, int64_t ke) {
+                            const SlabView& m, cudaStream_t s, int64_t kb, int64_t ke, bool peer) {
   const size_t ts = dsize(m.dt);
   const FusedLayout& L = fsrc.layout;
   const int64_t kbeg = kb < 0 ? m.k0 : kb, kend = ke < 0 ? m.k0 + m.nzl : ke;
@@ -457,7 +564,6 @@ void PlanImpl::launch_fused(const std::vector<const void*>& fptr, void* dout, co
   for (auto p : fptr) vec_ok = vec_ok && aligned16(p);
   const char* force = std::getenv("DFG_FUSED_KERNEL");
   const bool want_general = force && !std::strcmp(force, "general");
-  const bool want_tile = force && !std::strcmp(force, "tile");
   const int sms = sm_count(mesh->device);
 
   if (L.stencil_inputs.empty()) {
@@ -469,9 +575,7 @@ void PlanImpl::launch_fused(const std::vector<const void*>& fptr, void* dout, co
     DFG_CU(drv().LaunchKernel(mod.pointwise, grid, 1, 1, 256, 1, 1, 0, s, args, nullptr));
     kernel_end(ke, s);
     last_variant = 3;
-  } else if (mod.tma && !want_general && !want_tile && m.nx % vec == 0 && m.px() % vec == 0 && m.gx() % vec == 0 &&
-             aligned16(dout) &&
-             std::all_of(fptr.begin(), fptr.end(), [](const void* p) { return aligned16(p); })) {
+  } else if (tma_ok(fptr, dout, m)) {
     const int ncw = fsrc.cfg.ncw, rpw = fsrc.cfg.rpw;
     const int nsf = int(L.stencil_inputs.size() + L.point_inputs.size());  // TMA tiles per stage
     const int tw = tma_tile_w(m.dt, rpw), th = tma_tile_h(ncw, rpw);
@@ -497,14 +601,40 @@ void PlanImpl::launch_fused(const std::vector<const void*>& fptr, void* dout, co
     // parameter blob: DfgTmap map[NSF_] (128 B each, 64-aligned) then DfgParams
     auto w = pack_params(fptr, dout, tab[0], tab[1], tab[2], m, kbeg, kend, items, tiles_x, tiles_y, int(best_kz),
                          vec_ok ? 1 : 0);
-    size_t pbytes = size_t(nsf) * 128 + w.size() * 8;
-    pbytes = (pbytes + 63) / 64 * 64;
-    alignas(64) unsigned char blob[8 * 128 + 512];
-    if (pbytes > sizeof(blob)) fail(DFG_E_UNSUPPORTED, "too many stencil fields for the TMA kernel");
+    const int nst = int(L.stencil_inputs.size());
+    const TmaBlobLayout bl = tma_blob_layout(nsf, nst, w.size());
+    alignas(64) unsigned char blob[4096];
+    if (bl.size > sizeof(blob)) fail(DFG_E_UNSUPPORTED, "too many fields for the TMA kernel's parameters");
     std::memset(blob, 0, sizeof(blob));
     for (int f = 0; f < nsf; ++f)
       encode_map(reinterpret_cast<CUtensorMap*>(blob + 128 * f), m, const_cast<void*>(fptr[f]), ncw, rpw);
-    std::memcpy(blob + 128 * nsf, w.data(), w.size() * 8);
+    if (peer) {
+      // DfgPeerInfo: lo_k0, lo_ghost, hi_k0, hi_ghost, lo_on, hi_on
+      int64_t info[4] = {0, 0, 0, 0};
+      int32_t on[4] = {0, 0, 0, 0};
+      const MeshImpl::Peer* sides[2] = {&mesh->peer_lo, &mesh->peer_hi};
+      for (int sd = 0; sd < 2; ++sd) {
+        const MeshImpl::Peer& pr = *sides[sd];
+        if (!pr.on) continue;
+        SlabView pv = m;
+        pv.nzl = pr.nzl;
+        pv.k0 = pr.k0;
+        pv.ghost = int(pr.ghost);
+        for (int f = 0; f < nst; ++f) {
+          const std::string& name = dag.inputs[size_t(L.stencil_inputs[size_t(f)])];
+          auto it = pr.fields.find(name);
+          if (it == pr.fields.end()) fail(DFG_E_UNBOUND, "peer slab exported no field '" + name + "'");
+          encode_map(reinterpret_cast<CUtensorMap*>(blob + (sd == 0 ? bl.lo : bl.hi) + 128 * f), pv, it->second, ncw,
+                     rpw);
+        }
+        info[2 * sd] = pr.k0;
+        info[2 * sd + 1] = pr.ghost;
+        on[sd] = 1;
+      }
+      std::memcpy(blob + bl.peer, info, sizeof(info));
+      std::memcpy(blob + bl.peer + sizeof(info), on, sizeof(on));
+    }
+    std::memcpy(blob + bl.params, w.data(), w.size() * 8);
     void* args[] = {blob};
     auto ke = kernel_begin(s);
     DFG_CU(drv().LaunchKernel(mod.tma, grid, 1, 1, (ncw + 1) * 32, 1, 1, unsigned(smem), s, args, nullptr));
@@ -630,13 +760,15 @@ void execute_blocks(const std::vector<PlanImpl*>& plans, const std::vector<void*
     wmax = std::max(wmax, words.back().size());
     first.push_back(first.back() + items);
   }
-  const size_t stride = (size_t(nsf) * 128 + wmax * 8 + 63) / 64 * 64;
+  // DfgTmaParams images (no peer halo: blocks carry their ghost shells)
+  const TmaBlobLayout bl = tma_blob_layout(nsf, int(L.stencil_inputs.size()), wmax);
+  const size_t stride = bl.size;
   std::vector<unsigned char> host(stride * plans.size() + sizeof(int64_t) * first.size(), 0);
   for (size_t b = 0; b < plans.size(); ++b) {
     unsigned char* blob = host.data() + stride * b;
     const SlabView v = SlabView::of(*plans[b]->mesh);
     for (int f = 0; f < nsf; ++f) encode_map(reinterpret_cast<CUtensorMap*>(blob + 128 * f), v, const_cast<void*>(fptrs[b][size_t(f)]), ncw, rpw);
-    std::memcpy(blob + 128 * nsf, words[b].data(), words[b].size() * 8);
+    std::memcpy(blob + bl.params, words[b].data(), words[b].size() * 8);
   }
   std::memcpy(host.data() + stride * plans.size(), first.data(), sizeof(int64_t) * first.size());
   void* dev = dev_alloc(host.size(), m0.device, s);

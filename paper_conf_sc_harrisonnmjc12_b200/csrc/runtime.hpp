@@ -41,6 +41,20 @@ struct MeshImpl {
   int rank = 0, nranks = 1;
   void* nccl = nullptr;              // ncclComm_t
   std::weak_ptr<MeshImpl> link_lo, link_hi;
+  // peer-memory halo (dfg_mesh_peer_export / dfg_mesh_link_peers): the fused
+  // kernel reads the neighbours' boundary planes from their buffers (CUDA IPC
+  // mappings; NVLink between GPUs); step flags order the accesses
+  struct Peer {
+    bool on = false;
+    int64_t k0 = 0, nzl = 0, ghost = 0;
+    std::map<std::string, void*> fields;  // mapped field bases (ghost plane 0 included)
+    uint32_t* flags = nullptr;            // mapped flag words of the peer
+  };
+  Peer peer_lo, peer_hi;
+  uint32_t* flags = nullptr;         // own flags: [0] ready, [16] lo done, [32] hi done (64-byte apart)
+  uint32_t epoch = 0;                // executes of this mesh (every rank runs the same sequence)
+  std::map<std::string, void*> exported;  // bindings at export time (must not change while linked)
+  std::vector<void*> ipc_opened;     // cudaIpcOpenMemHandle bases to close
   ~MeshImpl();
   int64_t px() const { return pitch ? pitch : nx + 2 * gxy; }  // input row pitch
   int64_t gx() const { return xoff ? xoff : gxy; }   // first owned column of an input row
@@ -122,6 +136,7 @@ struct PlanImpl {
   int regs = 0, spill = 0;
   int last_variant = 0;  // 1 TMA, 2 general, 3 pointwise, 4 TMA multi-block (dfg_execute_blocks), 5 tile (cp.async ring)
   int64_t last_kz = 0;   // z-chunk length of the last TMA launch
+  int last_halo = 0;     // halo of the last execute: 0 none, 1 NCCL, 2 local copies, 3 peer (in place), 4 peer copies
   dfg_stats st{};
   cudaEvent_t ev0 = nullptr, ev1 = nullptr;
   bool timed = false;
@@ -156,8 +171,12 @@ struct PlanImpl {
 
  private:
   // kb / ke: global plane range of this launch (default: all owned planes of v)
+  // peer: read the planes outside the slab from the linked neighbours' buffers
+  // (TMA kernel only; the caller checks tma_peer_ok)
   void launch_fused(const std::vector<const void*>& fptr, void* dout, const void* const tab[3], const SlabView& v,
-                    cudaStream_t s, int64_t kb = -1, int64_t ke = -1);
+                    cudaStream_t s, int64_t kb = -1, int64_t ke = -1, bool peer = false);
+  bool tma_ok(const std::vector<const void*>& fptr, const void* dout, const SlabView& v) const;
+  void exec_fused_peer(const std::vector<const void*>& fptr, void* out, bool out_dev, cudaStream_t s);
   void exec_streamed(void* out, bool out_dev, cudaStream_t s);
   void release_stream_buffers();
   void exec_fused(void* out, bool out_dev, cudaStream_t s);
@@ -178,5 +197,13 @@ std::unique_ptr<PlanImpl> compile_plan(std::shared_ptr<MeshImpl> mesh, const std
 // NCCL (loaded with dlopen)
 void nccl_unique_id(void* out128);
 void mesh_init_comm(MeshImpl& m, const void* id128, int rank, int nranks);
+
+// Peer-memory halo: export blob of a z-slab (IPC handles of its bound device
+// fields and of its step flags) and the link to the neighbours' blobs.
+constexpr size_t kPeerBlobBytes = 4096;
+void mesh_peer_export(MeshImpl& m, void* blob);
+void mesh_link_peers(MeshImpl& m, const void* lo_blob, const void* hi_blob);
+// flag word offsets (uint32 units, 64 bytes apart)
+constexpr int kFlagReady = 0, kFlagLoDone = 16, kFlagHiDone = 32;
 
 }  // namespace dfg

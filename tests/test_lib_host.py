@@ -330,3 +330,13 @@ def test_tile_shape_choice_host(dfg):
 def test_set_timing_validates(dfg):
     lib = dfg._dfg._lib
     assert lib.dfg_plan_set_timing(None, 1) == -1
+
+
+def test_peer_entry_points_validate(dfg):
+    import ctypes
+    lib = dfg._dfg._lib
+    buf = ctypes.create_string_buffer(4096)
+    assert lib.dfg_mesh_peer_export(None, buf, 4096) == -1      # DFG_E_INVALID
+    assert lib.dfg_mesh_link_peers(None, None, None) == -1
+    hdr = open(os.path.join(ROOT, "include", "dfg.h")).read()
+    assert "#define DFG_PEER_BLOB_BYTES 4096" in hdr and dfg._dfg.PEER_BLOB_BYTES == 4096
