@@ -196,6 +196,8 @@ def main():
     ap.add_argument("--size", type=int, default=N1, help="cells per axis per GPU (default 1024)")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-strategies", action="store_true")
+    ap.add_argument("--halo", default="peer", choices=["peer", "nccl"],
+                    help="N > 1 z-slab halo: peer memory read in place by the kernel (default) or NCCL send/recv")
     args = ap.parse_args()
     if args.impl == "reference":
         return run_reference(args)
@@ -214,7 +216,7 @@ def main():
     # with its own NCCL_HOSTID (NCCL then uses its socket transport), so the
     # N > 1 path runs end to end on a one-GPU box; its timings mean nothing.
     one_gpu = world > 1 and os.environ.get("DFG_BENCH_ONE_GPU") == "1"
-    if one_gpu:
+    if one_gpu:   # torch's own NCCL process group needs it too
         os.environ.update({"NCCL_HOSTID": f"dfg-bench-{rank}", "NCCL_SOCKET_IFNAME": "lo", "NCCL_IB_DISABLE": "1",
                            "NCCL_P2P_DISABLE": "1", "NCCL_SHM_DISABLE": "1"})
         local = 0
@@ -241,10 +243,35 @@ def main():
     mesh = dfg.Mesh(x, y, z, nz_local=nzl, z_offset=k0, ghost=g)
     for c, b in fields.items():
         mesh.bind(c, b)
+    halo = None
     if world > 1:
-        uid = [dfg.dfg_nccl_unique_id() if rank == 0 else None]
-        dist.broadcast_object_list(uid, src=0)
-        dfg.dfg_mesh_init_comm(mesh.handle, uid[0], rank, world)
+        halo = "nccl"
+        if args.halo == "peer":
+            # the kernel reads the neighbours' boundary planes in place (CUDA IPC
+            # mappings over NVLink); every rank must link or none does
+            blobs, ok = [None] * world, [None] * world
+            try:
+                blob = mesh.peer_export()
+            except dfg.DfgError:
+                blob = None
+            dist.all_gather_object(blobs, blob)
+            linked = False
+            if all(b is not None for b in blobs):
+                try:
+                    mesh.link_peers(blobs[rank - 1] if rank > 0 else None,
+                                    blobs[rank + 1] if rank < world - 1 else None)
+                    linked = True
+                except dfg.DfgError:
+                    pass
+            dist.all_gather_object(ok, linked)
+            if all(ok):
+                halo = "peer"
+            elif linked:
+                mesh.link_peers(None, None)
+        if halo == "nccl":
+            uid = [dfg.dfg_nccl_unique_id() if rank == 0 else None]
+            dist.broadcast_object_list(uid, src=0)
+            dfg.dfg_mesh_init_comm(mesh.handle, uid[0], rank, world)
     plan = dfg.Plan(mesh, QCRIT, "fused").set_timing(2)   # kernel events inside the timed region
     out = torch.empty((nzl, n, n), dtype=torch.float32, device="cuda")
     stream = torch.cuda.Stream()
@@ -362,8 +389,12 @@ def main():
                  "kernel_ms_per_step": [r[1] for r in rows],
                  "step_ms": [r[2] for r in rows],
                  "launches_per_step": [r[3] for r in rows],
-                 "halo": "NCCL send/recv of the first/last owned plane of u, v, w on a side stream, "
-                         "overlapped with the interior planes; boundary planes launched after it"}
+                 "halo_mode": halo,
+                 "halo": ("peer memory: the boundary-plane launches read the neighbours' first/last owned "
+                          "planes of u, v, w in place (CUDA IPC mappings, NVLink), after the interior planes; "
+                          "step flags by stream write/wait-value" if halo == "peer" else
+                          "NCCL send/recv of the first/last owned plane of u, v, w on a side stream, "
+                          "overlapped with the interior planes; boundary planes launched after it")}
 
     strategies = variants = sweep = None
     if rank == 0 and world == 1 and not args.no_strategies:
@@ -381,7 +412,7 @@ def main():
             "ms_per_step": ms_step, "higher_is_better": True, "scaling": "weak", "vs_baseline": None,
             "dtype": "f32", "data": "synthetic",
             "config": {"workload": f"fused Q-criterion, {n}^3 fp32 rectilinear mesh per GPU "
-                                   f"(mesh {n}x{n}x{NZ}, z-slabs + 1-plane NCCL halo when N>1)",
+                                   f"(mesh {n}x{n}x{NZ}, z-slabs + 1-plane halo when N>1: " + (halo or "none") + ")",
                        "expression": "qcrit (Fig. 3C completed)", "strategy": "fused",
                        "cells_per_gpu": cells_rank, "fused_kernel": {1: "tma", 2: "general", 3: "pointwise", 5: "tile"}.get(
                            info["variant"]), "regs": info["regs"],

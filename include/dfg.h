@@ -202,8 +202,10 @@ int dfg_mesh_init_comm(dfg_mesh mesh, const void* id128, int rank, int nranks);
  * calls dfg_mesh_link_peers with the blob of the slab directly below (lo,
  * NULL on rank 0) and directly above (hi, NULL on the last rank).  Checks:
  * magic, type, plane size, global depth and adjacency (DFG_E_INVALID);
- * DFG_E_UNSUPPORTED if CUDA IPC is refused.  The mappings stay open until the
- * mesh is destroyed (the exporting ranks must keep their fields alive).
+ * DFG_E_UNSUPPORTED if CUDA IPC is refused (then neither side is linked).
+ * Both blobs NULL unlinks (the slab falls back to NCCL / local links).  The
+ * mappings stay open until the mesh is destroyed (the exporting ranks must
+ * keep their fields alive).
  *
  * A linked slab's dfg_execute (fused / reference strategies) orders itself
  * with its neighbours by step flags (stream memory operations: the execute

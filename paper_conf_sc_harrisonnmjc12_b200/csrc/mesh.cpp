@@ -367,6 +367,10 @@ void mesh_peer_export(MeshImpl& m, void* out) {
 
 void mesh_link_peers(MeshImpl& m, const void* lo_blob, const void* hi_blob) {
   const bool has_lo = m.k0 > 0, has_hi = m.k0 + m.nzl < m.NZ;
+  if (!lo_blob && !hi_blob) {  // unlink: back to the other halo transports
+    m.peer_lo.on = m.peer_hi.on = false;
+    return;
+  }
   if (has_lo != (lo_blob != nullptr) || has_hi != (hi_blob != nullptr))
     fail(DFG_E_INVALID, "peer halo: give the blob of every z neighbour and no other");
   if (m.ghost != 1) fail(DFG_E_INVALID, "peer halo: the mesh needs one ghost plane per side");
@@ -404,8 +408,12 @@ void mesh_link_peers(MeshImpl& m, const void* lo_blob, const void* hi_blob) {
     }
     peer.on = true;
   };
-  if (lo_blob) link(lo_blob, m.peer_lo, true);
-  if (hi_blob) link(hi_blob, m.peer_hi, false);
+  // both sides or neither: a half-linked slab would wait on flags nobody writes
+  MeshImpl::Peer lo, hi;
+  if (lo_blob) link(lo_blob, lo, true);
+  if (hi_blob) link(hi_blob, hi, false);
+  m.peer_lo = lo;
+  m.peer_hi = hi;
 }
 
 }  // namespace dfg
