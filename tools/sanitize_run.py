@@ -31,6 +31,26 @@ def main():
         dfg.Plan(mesh, "qcrit", "reference").execute(out)
         os.environ["DFG_KZ"] = "2"
         dfg.Plan(mesh, PAPER_PROGRAMS["qcrit"][0], "fused").execute(out)
+        # the cp.async-filled ring (tile kernel), every tile shape, ragged rows
+        for rpw in ("1", "2", "4"):
+            os.environ["DFG_RPW"] = rpw
+            os.environ["DFG_FUSED_KERNEL"] = "tile"
+            dfg.Plan(mesh, PAPER_PROGRAMS["qcrit"][0], "fused").execute(out)
+            os.environ.pop("DFG_FUSED_KERNEL")
+            dfg.Plan(mesh, PAPER_PROGRAMS["qcrit"][0], "fused").execute(out)
+        os.environ.pop("DFG_RPW")
+        rx, ry, rz, rf = synth.rt_inputs(67, 21, 9, dtype=T)
+        rmesh = dfg.Mesh(rx, ry, rz)
+        rdev = {k: v.cuda() for k, v in rf.items()}
+        for k, v in rdev.items():
+            rmesh.bind(k, v)
+        rout = torch.empty((9, 21, 67), dtype=tt, device="cuda")
+        for prog in ("qcrit", "intro"):
+            names = PAPER_PROGRAMS[prog][1]
+            if prog == "intro":
+                for nm, src_name in zip(names, ("u", "v")):
+                    rmesh.bind(nm, rdev[src_name])
+            dfg.Plan(rmesh, PAPER_PROGRAMS[prog][0], "fused").execute(rout)
         os.environ.pop("DFG_KZ")
         # streamed strategy from host fields (3-slot chunk ring, three streams)
         host = dfg.Mesh(x, y, z)
