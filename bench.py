@@ -135,20 +135,29 @@ def _oracle_time(x, y, z, f, win):
     res, valid = oev.evaluate(dag, f, oev.MeshWindow(x, y, z, i0=win[4], j0=win[2], k0=win[0]))
     dt = time.perf_counter() - t0
     cells = int(valid[1:-1, 1:-1, :].sum())
-    return cells, dt
+    return cells, dt, res[1:-1, 1:-1, :]
 
 
-def cpu_baseline_leg(target_s: float = 12.0):
+def cpu_baseline_leg(target_s: float = 12.0, gpu_out=None):
     """The oracle as it stands (numpy, one thread for element-wise ops) on a
-    bounded sample of the bench workload."""
+    bounded sample of the bench workload.  With gpu_out (the fused kernel's
+    1024^3 result of the timed steps), the sample doubles as a full-size parity
+    check: the GPU cells of the same block must equal the oracle's bit for bit."""
     x, y, z, f, win = _oracle_sample(512, 4)
-    cells, dt = _oracle_time(x, y, z, f, win)                 # calibration run
+    cells, dt, _ = _oracle_time(x, y, z, f, win)                 # calibration run
     planes = int(max(1, min(128, round(4 * target_s / max(dt, 1e-3)))))
     x, y, z, f, win = _oracle_sample(512, planes)
-    cells, dt = _oracle_time(x, y, z, f, win)
-    return {"value": cells / dt, "unit": "cells/s", "cores": 1, "kind": "oracle",
+    cells, dt, res = _oracle_time(x, y, z, f, win)
+    line = {"value": cells / dt, "unit": "cells/s", "cores": 1, "kind": "oracle",
             "sample": f"Q-criterion on a 1024 x 512 x {planes} block (+1-cell halo) of the 1024^3 RT-like "
                       f"fp32 workload, numpy oracle, {dt:.1f} s"}
+    if gpu_out is not None:
+        k0, j0 = win[0] + 1, win[2] + 1
+        got = gpu_out[k0:k0 + res.shape[0], j0:j0 + res.shape[1], :].cpu().numpy()
+        line["gpu_parity"] = {"cells_compared": int(res.size),
+                              "mismatches": int(np.count_nonzero(got.view(np.uint32) != res.view(np.uint32))),
+                              "block": f"planes {k0}..{k0 + res.shape[0] - 1}, rows {j0}..{j0 + res.shape[1] - 1}"}
+    return line
 
 
 def run_reference(args):
@@ -159,7 +168,7 @@ def run_reference(args):
     K, W = args.steps, args.warmup
     budget = 150.0
     x, y, z, f, win = _oracle_sample(16, 4)
-    _, dt = _oracle_time(x, y, z, f, win)
+    _, dt, _ = _oracle_time(x, y, z, f, win)
     per_step = budget / (K + W)
     scale = 16 * per_step / max(dt, 1e-3)          # in rows of 1024 x 1 x 4 cells
     rows = int(max(1, min(800, round(scale))))
@@ -169,7 +178,7 @@ def run_reference(args):
         _oracle_time(x, y, z, f, win)
     tot_cells, tot_t = 0, 0.0
     for _ in range(K):
-        c, dt = _oracle_time(x, y, z, f, win)
+        c, dt, _ = _oracle_time(x, y, z, f, win)
         tot_cells += c
         tot_t += dt
     v = tot_cells / tot_t
@@ -404,7 +413,7 @@ def main():
 
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
-        cpu = cpu_baseline_leg()
+        cpu = cpu_baseline_leg(gpu_out=out if n == N1 else None)
 
     if rank == 0:
         line = {
