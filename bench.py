@@ -112,18 +112,24 @@ class ClockSampler:
 
 
 # ------------------------------------------------------------------ oracle
-def _oracle_sample(nx_rows: int, planes: int):
+def _oracle_sample(nx_rows: int, planes: int, k0: int = 100, j0: int = 200, fields=None):
     """Inputs for an oracle sample: a 1024 x nx_rows x planes block of the
-    bench mesh (plus its one-cell halo), generated on the CPU."""
+    bench mesh (plus its one-cell halo): the window of the GPU's own input
+    arrays when given (the same inputs on both sides), else generated on the
+    CPU (the CPU and CUDA generators agree except for rare fp32 rounding
+    flips: their fp64 sin / log differ in the last bit)."""
     import torch
 
     import synth
     x, y, z = synth.rt_coords(N1, N1, N1, np.float32)
     x64, y64, z64 = (a.astype(np.float64) for a in (x, y, z))
-    k0, k1 = 100, 100 + planes
-    j0, j1 = 200, 200 + nx_rows
+    k1 = k0 + planes
+    j1 = j0 + nx_rows
     win = (k0 - 1, k1 + 1, j0 - 1, j1 + 1, 0, N1)
-    f = {c: synth.rt_velocity(c, x64, y64, z64, win, torch.float32).numpy() for c in "uvw"}
+    if fields is not None:
+        f = {c: fields[c][win[0]:win[1], win[2]:win[3], :].cpu().numpy() for c in "uvw"}
+    else:
+        f = {c: synth.rt_velocity(c, x64, y64, z64, win, torch.float32).numpy() for c in "uvw"}
     return x, y, z, f, win
 
 
@@ -138,15 +144,56 @@ def _oracle_time(x, y, z, f, win):
     return cells, dt, res[1:-1, 1:-1, :]
 
 
-def cpu_baseline_leg(target_s: float = 12.0, gpu_out=None):
+def _oracle_mt_worker(i, nworkers, barrier, target_s):
+    """One process of the multi-core oracle timing: its own block of the
+    bench mesh (64 rows x 4 planes, distinct per worker), evaluated by the
+    unchanged oracle repeatedly for about target_s once every worker is ready."""
+    planes, rows = 4, 64
+    k0 = 8 + (i * planes) % (N1 - 16)
+    j0 = 64 + 64 * ((i * planes) // (N1 - 16)) % (N1 - 128)
+    x, y, z, f, win = _oracle_sample(rows, planes, k0, j0)
+    _oracle_time(x, y, z, f, win)                              # warm (page-in, allocator)
+    barrier.wait()
+    t0 = time.time()
+    cells = 0
+    while True:
+        c, _, _ = _oracle_time(x, y, z, f, win)
+        cells += c
+        if time.time() - t0 >= target_s:
+            break
+    return cells, t0, time.time()
+
+
+def cpu_baseline_mt(target_s: float = 8.0):
+    """oracle_mt: the same oracle in one single-threaded process
+    per host core (capped at 64 for memory), each on its own block; throughput =
+    all cells / (last end - first start).  The arithmetic is the oracle's."""
+    import multiprocessing as mp
+    n = max(1, min(64, os.cpu_count() or 1))
+    for k in ("OMP_NUM_THREADS", "OPENBLAS_NUM_THREADS", "MKL_NUM_THREADS"):
+        os.environ[k] = "1"
+    ctx = mp.get_context("spawn")
+    with ctx.Manager() as mgr:
+        barrier = mgr.Barrier(n)
+        with ctx.Pool(n) as pool:
+            res = pool.starmap(_oracle_mt_worker, [(i, n, barrier, target_s) for i in range(n)])
+    cells = sum(r[0] for r in res)
+    wall = max(r[2] for r in res) - min(r[1] for r in res)
+    return {"value": cells / wall, "unit": "cells/s", "cores": n, "kind": "oracle",
+            "sample": f"{n} processes x repeated Q-criterion on 1024 x 64 x 4 blocks of the 1024^3 RT-like fp32 "
+                      f"workload, numpy oracle, {wall:.1f} s wall"}
+
+
+def cpu_baseline_leg(target_s: float = 12.0, gpu_out=None, gpu_fields=None):
     """The oracle as it stands (numpy, one thread for element-wise ops) on a
-    bounded sample of the bench workload.  With gpu_out (the fused kernel's
-    1024^3 result of the timed steps), the sample doubles as a full-size parity
-    check: the GPU cells of the same block must equal the oracle's bit for bit."""
+    bounded sample of the bench workload.  With gpu_out / gpu_fields (the fused
+    kernel's 1024^3 result of the timed steps and its inputs), the sample runs
+    on the GPU's own inputs and doubles as a full-size parity check: the GPU
+    cells of the block must equal the oracle's bit for bit."""
     x, y, z, f, win = _oracle_sample(512, 4)
     cells, dt, _ = _oracle_time(x, y, z, f, win)                 # calibration run
     planes = int(max(1, min(128, round(4 * target_s / max(dt, 1e-3)))))
-    x, y, z, f, win = _oracle_sample(512, planes)
+    x, y, z, f, win = _oracle_sample(512, planes, fields=gpu_fields)
     cells, dt, res = _oracle_time(x, y, z, f, win)
     line = {"value": cells / dt, "unit": "cells/s", "cores": 1, "kind": "oracle",
             "sample": f"Q-criterion on a 1024 x 512 x {planes} block (+1-cell halo) of the 1024^3 RT-like "
@@ -205,6 +252,7 @@ def main():
     ap.add_argument("--size", type=int, default=N1, help="cells per axis per GPU (default 1024)")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-strategies", action="store_true")
+    ap.add_argument("--no-cpu-mt", action="store_true", help="skip the multi-process oracle timing")
     ap.add_argument("--halo", default="peer", choices=["peer", "nccl"],
                     help="N > 1 z-slab halo: peer memory read in place by the kernel (default) or NCCL send/recv")
     args = ap.parse_args()
@@ -413,7 +461,13 @@ def main():
 
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
-        cpu = cpu_baseline_leg(gpu_out=out if n == N1 else None)
+        same = n == N1 and world == 1
+        cpu = cpu_baseline_leg(gpu_out=out if same else None, gpu_fields=fields if same else None)
+        if not args.no_cpu_mt:
+            try:
+                cpu["oracle_mt"] = cpu_baseline_mt()
+            except Exception as e:  # a host without multiprocessing support
+                cpu["oracle_mt"] = {"unavailable": repr(e)[:200]}
 
     if rank == 0:
         line = {

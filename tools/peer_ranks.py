@@ -117,9 +117,16 @@ def main():
     ap.add_argument("--steps", type=int, default=3)
     ap.add_argument("--dtype", default="f32", choices=["f32", "f64"])
     ap.add_argument("--kernel", default="", help="DFG_FUSED_KERNEL for every rank (e.g. tile)")
+    ap.add_argument("--as-rank", type=int, default=-1,
+                    help="run only this rank in this process (start every rank yourself, same --port), "
+                         "e.g. each under compute-sanitizer")
+    ap.add_argument("--port", type=int, default=0)
     args = ap.parse_args()
+    port = args.port or 29500 + (os.getpid() % 2000)
+    if args.as_rank >= 0:
+        worker(args.as_rank, args.ranks, args, port)
+        return
     import torch.multiprocessing as mp
-    port = 29500 + (os.getpid() % 2000)
     mp.spawn(worker, args=(args.ranks, args, port), nprocs=args.ranks, join=True)
 
 
