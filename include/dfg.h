@@ -270,9 +270,11 @@ int dfg_execute(dfg_plan plan, void* out, int out_on_device, void* cuda_stream);
  * meshes, so small blocks do not pay one kernel's fill and drain each.
  * outs[b]: device output of plans[b].  Used when every plan is DFG_FUSED
  * with the same generated kernel (same expression, dtype and global mesh),
- * every input device-resident, no halo exchange needed (whole meshes or
- * blocks with ghost shells) and every layout TMA-eligible (see
- * dfg_create_block); otherwise the plans execute one after the other.
+ * every input device-resident and no halo exchange needed (whole meshes or
+ * blocks with ghost shells): the TMA kernel when every layout is
+ * TMA-eligible (see dfg_create_block), else the same pipeline with the ring
+ * filled by cp.async (packed ghost shells, rows that are not 16-byte
+ * multiples); otherwise the plans execute one after the other.
  * Results equal dfg_execute's bit for bit.  Stats: executes +1 on every
  * plan; the launch and its timing are counted on plans[0].
  * Errors as dfg_execute; DFG_E_INVALID for n < 1 or null entries. */
@@ -296,7 +298,7 @@ int dfg_plan_set_timing(dfg_plan plan, int level);
  * out[2] = number of filters, out[3] = fused kernel variant of the last
  * execute (0 none, 1 TMA pipeline, 2 general, 3 point-wise, 4 TMA
  * multi-block via dfg_execute_blocks, 5 tile: the TMA kernel's ring filled
- * by cp.async, for layouts a tensor map cannot describe), out[4] = registers per thread of the
+ * by cp.async, for layouts a tensor map cannot describe, 6 tile multi-block), out[4] = registers per thread of the
  * fused kernel (0 if none), out[5] = local memory per thread of that kernel
  * (bytes; spills and stack), out[6] = predicted
  * device footprint in bytes for device-resident inputs,

@@ -463,17 +463,28 @@ __device__ __forceinline__ void dfg_cp_async_arrive(unsigned bar) {
 
 // Fill cursor of one consumer thread: the stage sequence of the CTA's items
 // (pre-plane, planes kb..ke-1, post-plane of each), its own ring position.
+// Several meshes (dfg_fused_tile_multi): block b's parameters at blocks[b],
+// its items first[b] .. first[b+1]-1 of the concatenated item space; a
+// single mesh is the case nb = 1 with first = {0, items}.
 struct DfgFill {
-  const DfgParams* P;
+  const DfgParams* P;       // current block
+  const DfgParams* blocks;  // all blocks (single mesh: &P)
+  const long long* first;   // nullptr: single mesh
+  int b;
+  long long item, end;      // global item; end of the item space
+  long long q, qe;
   DfgRing W;
-  long long item, q, qe;
   unsigned off[DFG_FM];  // input element offsets within a plane of this thread's tile elements
   unsigned tid;
 
+  __device__ __forceinline__ long long base() const { return first ? first[b] : 0; }
   __device__ __forceinline__ void setup() {
+    if (first)
+      while (item >= first[b + 1]) P = &blocks[++b];  // items only grow: the block index too
     const DfgParams& p = *P;
-    const long long tx_ = item % p.tiles_x;
-    const long long rest = item / p.tiles_x;
+    const long long li = item - base();
+    const long long tx_ = li % p.tiles_x;
+    const long long rest = li / p.tiles_x;
     const long long ty_ = rest % p.tiles_y;
     const long long zc = rest / p.tiles_y;
     const long long kb = p.kbeg + zc * p.kz;
@@ -494,17 +505,21 @@ struct DfgFill {
       off[m] = (unsigned)yy * (unsigned)p.px + (unsigned)xx;
     }
   }
-  __device__ __forceinline__ void init(const DfgParams* p, unsigned smem, unsigned full0, unsigned t) {
-    P = p;
+  __device__ __forceinline__ void init(const DfgParams* p, const long long* fst, long long total, unsigned smem,
+                                       unsigned full0, unsigned t) {
+    P = blocks = p;
+    first = fst;
+    b = 0;
+    end = total;
     W = DfgRing{smem, full0, 0u, 0, smem, full0};
     tid = t;
     item = blockIdx.x;
-    if (item < p->items) setup();
+    if (item < end) setup();
   }
   // issue this thread's share of the next stage of the sequence
   __device__ __forceinline__ void step() {
+    if (item >= end) return;
     const DfgParams& p = *P;
-    if (item >= p.items) return;
     dfg_mbar_wait(DFG_EMPTY(W.full), W.phase ^ 1u, 0x100000u);
     const long long pg = max(0LL, min(q, p.NZ - 1));
     const long long pbase = (pg - p.k0 + p.ghost) * p.px * p.py;
@@ -521,7 +536,7 @@ struct DfgFill {
     W.advance();
     if (++q > qe) {
       item += gridDim.x;
-      if (item < p.items) setup();
+      if (item < end) setup();
     }
   }
 };
@@ -596,12 +611,42 @@ extern "C" __global__ void __launch_bounds__(DFG_NCW * 32, DFG_CTAS) dfg_fused_t
   const int warp = threadIdx.x >> 5;
   const int lane = threadIdx.x & 31;
   DfgFill F;
-  F.init(&P, smem, full0, threadIdx.x);
+  F.init(&P, nullptr, P.items, smem, full0, threadIdx.x);
   for (int n = 0; n < DFG_STAGES - 1; ++n) F.step();
   DfgRing R{smem, full0, 0u, 0, smem, full0};
   DfgCol C;
   C.Z = dfg2_splat(P.nzero);
   C.vst = P.vec_ok != 0;
   for (long long item = blockIdx.x; item < P.items; item += gridDim.x) dfg_consume_tile(P, item, R, C, warp, lane, F);
+}
+
+// All blocks of a device in one launch on the cp.async ring (packed ghost
+// shells, the paper's VisIt blocks, L315): per-block DfgParams in global
+// memory, first[b] = first item of block b, first[nb] = total.
+struct DfgTileMulti {
+  const DfgParams* blocks;
+  const long long* first;
+  int nb;
+};
+
+extern "C" __global__ void __launch_bounds__(DFG_NCW * 32, DFG_CTAS)
+    dfg_fused_tile_multi(const __grid_constant__ DfgTileMulti M) {
+  const unsigned smem = dfg_ring_init(DFG_NCW * 32);
+  const unsigned full0 = smem + DFG_STAGES * DFG_STAGE_BYTES;
+  const int warp = threadIdx.x >> 5;
+  const int lane = threadIdx.x & 31;
+  const long long total = M.first[M.nb];
+  DfgFill F;
+  F.init(M.blocks, M.first, total, smem, full0, threadIdx.x);
+  for (int n = 0; n < DFG_STAGES - 1; ++n) F.step();
+  DfgRing R{smem, full0, 0u, 0, smem, full0};
+  DfgCol C;
+  C.Z = dfg2_splat(M.blocks[0].nzero);
+  int b = 0;
+  for (long long item = blockIdx.x; item < total; item += gridDim.x) {
+    while (item >= M.first[b + 1]) ++b;
+    C.vst = M.blocks[b].vec_ok != 0;
+    dfg_consume_tile(M.blocks[b], item - M.first[b], R, C, warp, lane, F);
+  }
 }
 #endif

@@ -25,6 +25,7 @@ struct LoadedModule {
   CUfunction pointwise = nullptr, general = nullptr, tma = nullptr;
   CUfunction tma_multi = nullptr;  // several meshes per launch (dfg_execute_blocks)
   CUfunction tile = nullptr;       // same ring, filled by cp.async (layouts TMA cannot describe)
+  CUfunction tile_multi = nullptr; // several meshes per launch on the cp.async ring
 };
 
 // Load into the current context (requires a device).

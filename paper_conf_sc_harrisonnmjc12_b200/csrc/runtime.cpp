@@ -175,6 +175,7 @@ std::unique_ptr<PlanImpl> compile_plan(std::shared_ptr<MeshImpl> mesh, const std
       DFG_CU(drv().FuncSetAttribute(plan->mod.tma, CU_FUNC_ATTRIBUTE_MAX_DYNAMIC_SHARED_SIZE_BYTES, int(smem)));
       DFG_CU(drv().FuncSetAttribute(plan->mod.tma_multi, CU_FUNC_ATTRIBUTE_MAX_DYNAMIC_SHARED_SIZE_BYTES, int(smem)));
       DFG_CU(drv().FuncSetAttribute(plan->mod.tile, CU_FUNC_ATTRIBUTE_MAX_DYNAMIC_SHARED_SIZE_BYTES, int(smem)));
+      DFG_CU(drv().FuncSetAttribute(plan->mod.tile_multi, CU_FUNC_ATTRIBUTE_MAX_DYNAMIC_SHARED_SIZE_BYTES, int(smem)));
     }
   }
   return plan;
@@ -699,21 +700,26 @@ void execute_blocks(const std::vector<PlanImpl*>& plans, const std::vector<void*
   const int vec = int(16 / ts);
   const FusedLayout& L = p0.fsrc.layout;
   const char* force = std::getenv("DFG_FUSED_KERNEL");
-  bool batch = plans.size() > 1 && p0.strategy == DFG_FUSED && p0.mod.tma_multi && p0.fsrc.cfg.has_tma &&
-               !(force && !std::strcmp(force, "general"));
+  // one launch when every block runs the same module on this device: the TMA
+  // kernel if every block's layout suits tensor maps, else the cp.async ring
+  bool batch = plans.size() > 1 && p0.strategy == DFG_FUSED && p0.mod.tma_multi && p0.mod.tile_multi &&
+               p0.fsrc.cfg.has_tma && !(force && !std::strcmp(force, "general"));
+  bool tma = !(force && !std::strcmp(force, "tile"));
   std::vector<std::vector<const void*>> fptrs(plans.size());
   for (size_t b = 0; b < plans.size() && batch; ++b) {
     PlanImpl& p = *plans[b];
     const MeshImpl& m = *p.mesh;
     const bool halo = (m.k0 > 0 || m.k0 + m.nzl < m.NZ) && !m.ghosts_supplied;
     batch = p.strategy == DFG_FUSED && p.fsrc.source == p0.fsrc.source && m.device == m0.device && !halo &&
-            m.nx % vec == 0 && m.px() % vec == 0 && m.gx() % vec == 0 && aligned16(outs[b]);
+            m.px() * m.py() < (int64_t(1) << 32);
+    tma = tma && m.nx % vec == 0 && m.px() % vec == 0 && m.gx() % vec == 0 && aligned16(outs[b]);
     std::vector<int> ins = L.stencil_inputs;
     ins.insert(ins.end(), L.point_inputs.begin(), L.point_inputs.end());
     for (int i : ins) {
       auto it = m.fields.find(p.dag.inputs[size_t(i)]);
       if (it == m.fields.end() || !it->second.ptr) fail(DFG_E_UNBOUND, "input '" + p.dag.inputs[size_t(i)] + "' is not bound");
-      batch = batch && it->second.on_device && aligned16(it->second.ptr);
+      batch = batch && it->second.on_device;
+      tma = tma && aligned16(it->second.ptr);
       fptrs[b].push_back(it->second.ptr);
     }
   }
@@ -726,8 +732,10 @@ void execute_blocks(const std::vector<PlanImpl*>& plans, const std::vector<void*
   const int tw = tma_tile_w(m0.dt, rpw), th = tma_tile_h(ncw, rpw);
   const int nsf = int(L.stencil_inputs.size() + L.point_inputs.size());
   const size_t smem = fused_tma_smem_bytes(m0.dt, nsf, ncw, p0.fsrc.cfg.stages, rpw);
+  CUfunction fn = tma ? p0.mod.tma_multi : p0.mod.tile_multi;
+  const int threads = tma ? (ncw + 1) * 32 : ncw * 32;
   int occ = 1;
-  DFG_CU(drv().OccupancyMaxActiveBlocksPerMultiprocessor(&occ, p0.mod.tma_multi, (ncw + 1) * 32, smem));
+  DFG_CU(drv().OccupancyMaxActiveBlocksPerMultiprocessor(&occ, fn, threads, smem));
   const int64_t slots = int64_t(sm_count(m0.device)) * std::max(occ, 1);
   // one z-chunk length for the batch: whole rounds of the concatenated items
   // against the two halo planes per chunk (as launch_fused)
@@ -755,17 +763,23 @@ void execute_blocks(const std::vector<PlanImpl*>& plans, const std::vector<void*
     const SlabView v = SlabView::of(m);
     const int tx = int((m.nx + tw - 1) / tw), ty = int((m.ny + th - 1) / th);
     const int64_t items = int64_t(tx) * ty * ((m.nzl + best_kz - 1) / best_kz);
+    const bool out16 = aligned16(outs[b]) && m.nx % vec == 0;  // tile kernel: 16-byte output stores
     words.push_back(pack_params(fptrs[b], outs[b], m.dev_tab[0], m.dev_tab[1], m.dev_tab[2], v, m.k0, m.k0 + m.nzl,
-                                items, tx, ty, int(best_kz), 0));
+                                items, tx, ty, int(best_kz), tma ? 0 : (out16 ? 1 : 0)));
     wmax = std::max(wmax, words.back().size());
     first.push_back(first.back() + items);
   }
-  // DfgTmaParams images (no peer halo: blocks carry their ghost shells)
+  // TMA: DfgTmaParams images (no peer halo: blocks carry their ghost
+  // shells); tile: plain DfgParams images
   const TmaBlobLayout bl = tma_blob_layout(nsf, int(L.stencil_inputs.size()), wmax);
-  const size_t stride = bl.size;
+  const size_t stride = tma ? bl.size : wmax * 8;
   std::vector<unsigned char> host(stride * plans.size() + sizeof(int64_t) * first.size(), 0);
   for (size_t b = 0; b < plans.size(); ++b) {
     unsigned char* blob = host.data() + stride * b;
+    if (!tma) {
+      std::memcpy(blob, words[b].data(), words[b].size() * 8);
+      continue;
+    }
     const SlabView v = SlabView::of(*plans[b]->mesh);
     for (int f = 0; f < nsf; ++f) encode_map(reinterpret_cast<CUtensorMap*>(blob + 128 * f), v, const_cast<void*>(fptrs[b][size_t(f)]), ncw, rpw);
     std::memcpy(blob + bl.params, words[b].data(), words[b].size() * 8);
@@ -782,7 +796,7 @@ void execute_blocks(const std::vector<PlanImpl*>& plans, const std::vector<void*
   if (p0.timing >= 1) DFG_CUDA(cudaEventRecord(p0.ev0, s));
   auto ke = p0.kernel_begin(s);
   const unsigned grid = unsigned(std::max<int64_t>(1, std::min(first.back(), slots)));
-  DFG_CU(drv().LaunchKernel(p0.mod.tma_multi, grid, 1, 1, (ncw + 1) * 32, 1, 1, unsigned(smem), s, args, nullptr));
+  DFG_CU(drv().LaunchKernel(fn, grid, 1, 1, threads, 1, 1, unsigned(smem), s, args, nullptr));
   p0.kernel_end(ke, s);
   if (p0.timing >= 1) DFG_CUDA(cudaEventRecord(p0.ev1, s));
   DFG_CUDA(cudaFreeAsync(dev, s));
@@ -791,7 +805,7 @@ void execute_blocks(const std::vector<PlanImpl*>& plans, const std::vector<void*
   p0.st.kernel_count += 1;
   for (auto* p : plans) {
     p->st.executes += 1;
-    p->last_variant = 4;
+    p->last_variant = tma ? 4 : 6;
     p->last_kz = best_kz;
   }
 }

@@ -134,7 +134,7 @@ struct PlanImpl {
   FusedSource fsrc;
   LoadedModule mod;
   int regs = 0, spill = 0;
-  int last_variant = 0;  // 1 TMA, 2 general, 3 pointwise, 4 TMA multi-block (dfg_execute_blocks), 5 tile (cp.async ring)
+  int last_variant = 0;  // 1 TMA, 2 general, 3 pointwise, 4 TMA multi-block (dfg_execute_blocks), 5 tile (cp.async ring), 6 tile multi-block
   int64_t last_kz = 0;   // z-chunk length of the last TMA launch
   int last_halo = 0;     // halo of the last execute: 0 none, 1 NCCL, 2 local copies, 3 peer (in place), 4 peer copies
   dfg_stats st{};
