@@ -467,10 +467,9 @@ __device__ __forceinline__ void dfg_cp_async_arrive(unsigned bar) {
 // its items first[b] .. first[b+1]-1 of the concatenated item space; a
 // single mesh is the case nb = 1 with first = {0, items}.
 struct DfgFill {
-  const DfgParams* P;       // current block
-  const DfgParams* blocks;  // all blocks (single mesh: &P)
+  const DfgParams* blocks;  // all blocks (single mesh: the kernel parameter)
   const long long* first;   // nullptr: single mesh
-  int b;
+  int b;                    // current block
   long long item, end;      // global item; end of the item space
   long long q, qe;
   DfgRing W;
@@ -480,8 +479,8 @@ struct DfgFill {
   __device__ __forceinline__ long long base() const { return first ? first[b] : 0; }
   __device__ __forceinline__ void setup() {
     if (first)
-      while (item >= first[b + 1]) P = &blocks[++b];  // items only grow: the block index too
-    const DfgParams& p = *P;
+      while (item >= first[b + 1]) ++b;  // items only grow: the block index too
+    const DfgParams& p = blocks[b];
     const long long li = item - base();
     const long long tx_ = li % p.tiles_x;
     const long long rest = li / p.tiles_x;
@@ -507,7 +506,7 @@ struct DfgFill {
   }
   __device__ __forceinline__ void init(const DfgParams* p, const long long* fst, long long total, unsigned smem,
                                        unsigned full0, unsigned t) {
-    P = blocks = p;
+    blocks = p;
     first = fst;
     b = 0;
     end = total;
@@ -519,7 +518,7 @@ struct DfgFill {
   // issue this thread's share of the next stage of the sequence
   __device__ __forceinline__ void step() {
     if (item >= end) return;
-    const DfgParams& p = *P;
+    const DfgParams& p = blocks[b];
     dfg_mbar_wait(DFG_EMPTY(W.full), W.phase ^ 1u, 0x100000u);
     const long long pg = max(0LL, min(q, p.NZ - 1));
     const long long pbase = (pg - p.k0 + p.ghost) * p.px * p.py;
