@@ -107,7 +107,9 @@ class ClockSampler:
         mx = [float(r[1]) for r in self.rows if r[1].replace(".", "").isdigit()]
         names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
         reasons = sorted({names[i] for r in self.rows for i in range(4) if len(r) > 3 + i and r[3 + i] == "Active"})
+        pw = [float(r[2]) for r in self.rows if len(r) > 2 and r[2].replace(".", "").isdigit()]
         return {"sm_mhz": float(np.median(sm)) if sm else None, "sm_max_mhz": max(mx) if mx else None,
+                "power_w": float(np.median(pw)) if pw else None,
                 "reasons": reasons, "samples": len(self.rows), "source": getattr(self, "source", None)}
 
 
@@ -368,6 +370,29 @@ def main():
     value = cells_rank * world / (ms_step * 1e-3)
     info = plan.info()
 
+    # context for the roofline: a plain device copy (torch copy_, 4 GiB read +
+    # 4 GiB written) back to back for ~1 s, i.e. HBM bandwidth under the same
+    # board power cap a long step runs in (MEASURED_PEAKS is a burst figure)
+    sustained = None
+    if world == 1 and not args.no_strategies:
+        a = torch.empty(1 << 30, dtype=torch.float32, device="cuda")
+        b = torch.empty_like(a)
+        b.copy_(a)
+        torch.cuda.synchronize()
+        reps = max(10, int(1.0 / (kern_ms * 1e-3 * 2.6)))
+        with ClockSampler(local) as cclk:
+            c0, c1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            c0.record()
+            for _ in range(reps):
+                b.copy_(a)
+            c1.record()
+            c1.synchronize()
+        sustained = {"gb_per_s": 2 * a.numel() * 4 * reps / (c0.elapsed_time(c1) * 1e-3) / 1e9,
+                     "reps": reps, "clocks": cclk.summary(),
+                     "how": "torch copy_ of 4 GiB fp32, back to back, CUDA events (read + write bytes)"}
+        del a, b
+        torch.cuda.empty_cache()
+
     # roofline of the dominant kernel (the only kernel of the step)
     peak, peak_src = _peak()
     achieved = ALGO_BYTES_PER_CELL * cells_rank / (kern_ms * 1e-3) / 1e9
@@ -406,6 +431,26 @@ def main():
                "d2h_bytes_per_step": hs["d2h_bytes"] // hs["executes"],
                "ms_per_step": te * 1e3, "matches_device_result": ok, "strategy": "streamed",
                "pcie_gb_per_s": (hs["h2d_bytes"] + hs["d2h_bytes"]) / hs["executes"] / te / 1e9}
+        # the PCIe bound of this leg: pinned copies alone (CUDA events), inputs
+        # up and the result down overlapping (full duplex)
+        scratch = torch.empty_like(fields["u"])
+        bw = {}
+        for name, dst, src in (("h2d", scratch, hostf["u"]), ("d2h", hout, out)):
+            dst.copy_(src, non_blocking=True)
+            torch.cuda.synchronize()
+            c0, c1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            c0.record()
+            for _ in range(3):
+                dst.copy_(src, non_blocking=True)
+            c1.record()
+            c1.synchronize()
+            bw[name] = 3 * src.numel() * src.element_size() / (c0.elapsed_time(c1) * 1e-3) / 1e9
+        del scratch
+        bound_s = max(e2e["h2d_bytes_per_step"] / (bw["h2d"] * 1e9), e2e["d2h_bytes_per_step"] / (bw["d2h"] * 1e9))
+        e2e["pcie_bound"] = {"h2d_gb_per_s": bw["h2d"], "d2h_gb_per_s": bw["d2h"], "bound_ms": bound_s * 1e3,
+                             "frac": bound_s / te,
+                             "how": "pinned torch copies of 4 GiB alone; bound = max(h2d bytes / h2d rate, "
+                                    "d2h bytes / d2h rate), i.e. full-duplex overlap"}
         hplan.close()
         hmesh.close()
         del hostf, hout
@@ -486,7 +531,9 @@ def main():
             "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
                          "frac": achieved / peak, "traffic": traffic, "peak_source": peak_src,
                          "kernel": "dfg_fused_tma", "kernel_ms": kern_ms,
-                         "algorithmic_bytes_per_launch": ALGO_BYTES_PER_CELL * cells_rank},
+                         "algorithmic_bytes_per_launch": ALGO_BYTES_PER_CELL * cells_rank,
+                         **({"sustained_copy": sustained, "frac_of_sustained_copy": achieved / sustained["gb_per_s"]}
+                            if sustained else {})},
             "e2e": e2e,
             "multi_gpu": multi,
             "gpu_launches": st["kernel_count"],
