@@ -382,6 +382,18 @@ def test_visit_blocks_with_ghost_shells(shape, split, prog, strategy, pitch):
     from column 4 (16 bytes), rows padded past a multiple of 16 bytes
     (padding = NaN, never read), which puts blocks whose width is a multiple
     of 4 on the TMA kernel."""
+    _visit_blocks(shape, split, prog, strategy, pitch)
+
+
+@pytest.mark.parametrize("pitch", ["natural", "padded"])
+def test_visit_blocks_several_items_per_cta(pitch):
+    """27 blocks of 128 x 128 x 16 (243 tile columns for 148 persistent CTAs):
+    in the one-launch multi-block kernels a CTA's items, and the ring fill
+    running ahead of its consumers, cross from one block into the next."""
+    _visit_blocks((384, 384, 48), (3, 3, 3), "qcrit", "fused", pitch)
+
+
+def _visit_blocks(shape, split, prog, strategy, pitch):
     import paper_conf_sc_harrisonnmjc12_b200 as dfg
     if strategy == "reference" and prog == "intro":
         pytest.skip("no reference kernel for the intro expression")

@@ -78,7 +78,38 @@ def main():
             o = torch.empty((m.nz, shape[1], shape[0]), dtype=tt, device="cuda")
             dfg.Plan(m, PAPER_PROGRAMS["qcrit"][0], "fused").execute(o)
         torch.cuda.synchronize()
+    blocks_one_launch()
     print("sanitize run done")
+
+
+def blocks_one_launch():
+    """VisIt blocks of one device in one launch: packed ghost shells (the
+    cp.async-filled ring, dfg_fused_tile_multi) and 16-byte padded shells
+    (dfg_fused_tma_multi); 8 blocks of 32 x 10 x 7."""
+    shape, split = (64, 20, 14), (2, 2, 2)
+    x, y, z, f = synth.rt_inputs(*shape, dtype=np.float32)
+    f = {k: v.numpy() for k, v in f.items()}
+    pad = {n: np.pad(a, 1, mode="edge") for n, a in f.items()}
+    for xo in (1, 4):
+        plans, outs, keep = [], [], []
+        for a in range(2):
+            for b in range(2):
+                for c in range(2):
+                    i0, j0, k0 = 32 * a, 10 * b, 7 * c
+                    rp = 34 if xo == 1 else 40
+                    m = dfg.Mesh.block(x, y, z, 32, 10, 7, i0, j0, k0, ghost=1, row_pitch=rp, x_offset=xo)
+                    for n in "uvw":
+                        buf = np.zeros((9, 12, rp), np.float32)
+                        buf[:, :, xo - 1:xo + 33] = pad[n][k0:k0 + 9, j0:j0 + 12, i0:i0 + 34]
+                        t = torch.from_numpy(buf).cuda()
+                        keep.append(t)
+                        m.bind(n, t)
+                    keep.append(m)
+                    plans.append(dfg.Plan(m, PAPER_PROGRAMS["qcrit"][0], "fused"))
+                    outs.append(torch.empty((7, 10, 32), device="cuda"))
+        dfg.execute_blocks(plans, outs)
+        torch.cuda.synchronize()
+        print("blocks one launch, variant", plans[0].info()["variant"])
 
 
 if __name__ == "__main__":
