@@ -382,7 +382,7 @@ int dfg_hybrid_model(const char* expr, const char* const* inputs, int n_inputs,
 /* Generate the fused kernel source for `expr` on an nx x ny x nz mesh and,
  * if compile != 0, NVRTC-compile it for sm_100a (no device needed); on
  * success *regs / *spill (may be NULL) get the ptxas figures of the TMA
- * kernel.  fp32 sources use the two-operation quotient on every axis (the
+ * kernel.  Sources use the two-operation quotient on every axis (the
  * kernel of a mesh whose divisors all verified) unless the environment sets
  * DFG_FUSED_VARIANT=markstein.  Writes the source with the buffer protocol
  * above. */
@@ -390,6 +390,24 @@ int dfg_fused_source(const char* expr, const char* const* inputs, int n_inputs,
                      dfg_dtype dtype, int64_t nx, int64_t ny, int64_t nz,
                      int compile, char* buf, size_t cap, size_t* needed,
                      int* regs, int* spill);
+
+/* Two-operation quotient check, exposed for tests (DESIGN.md section 5,
+ * csrc/div2.hpp).  A fused kernel forms a grad3d derivative num / d (L99,
+ * reading R1) as RN(num*r + RN(num*yl)) with r = RN(1/d), yl = RN(1/d - r)
+ * on every axis whose divisors all pass this check, else with Markstein's
+ * three-operation correction.  For each of the n divisors d[i] (host array
+ * of T = dtype; positive normal numbers, else DFG_E_INVALID) the library
+ * forms r and yl as the spacing tables do and sets ok[i] = 1 if the scheme
+ * equals RN(num / d) for every numerator in the normal range:
+ *   method 0: certification by candidate numerators (fp32 and fp64; the
+ *             handful of numerators whose quotient lies within the scheme's
+ *             error bound of a rounding boundary; what fp64 meshes use);
+ *   method 1: exhaustive, all 2^23 fp32 significands on the host (fp32
+ *             only, else DFG_E_UNSUPPORTED; ~10 ms per divisor; fp32 meshes
+ *             run the same enumeration on the device).
+ * tested (may be NULL): candidate numerators evaluated per divisor (method 0;
+ * 0 for method 1).  Host only, no device needed; caller owns all arrays. */
+int dfg_div2_check(dfg_dtype dtype, const void* d, int64_t n, int method, uint8_t* ok, int64_t* tested);
 
 #ifdef __cplusplus
 }

@@ -86,6 +86,7 @@ _SIGS = {
                                C.POINTER(C.c_size_t)]),
     "dfg_model": (C.c_int, [C.c_char_p, C.POINTER(C.c_char_p), C.c_int, C.c_int, C.c_int, C.POINTER(_I64)]),
     "dfg_points3d_to_axes": (C.c_int, [C.c_int, _I64, _I64, _I64, _P, _P, _P, _P, _P, _P]),
+    "dfg_div2_check": (C.c_int, [C.c_int, _P, _I64, C.c_int, _P, _P]),
     "dfg_fused_source": (C.c_int, [C.c_char_p, C.POINTER(C.c_char_p), C.c_int, C.c_int, _I64, _I64, _I64, C.c_int,
                                    C.c_char_p, C.c_size_t, C.POINTER(C.c_size_t), C.POINTER(C.c_int),
                                    C.POINTER(C.c_int)]),
@@ -319,6 +320,17 @@ def dfg_points3d_to_axes(x3, y3, z3):
     _check(_lib.dfg_points3d_to_axes(dt, px - 1, py - 1, pz - 1, _ptr(x3), _ptr(y3), _ptr(z3),
                                      _ptr(x), _ptr(y), _ptr(z)))
     return x, y, z
+
+
+def dfg_div2_check(d, method=0):
+    """numpy divisors (float32 / float64) -> (ok uint8[n], candidates tested int64[n])."""
+    import numpy as np
+    d = np.ascontiguousarray(d)
+    ok = np.zeros(d.shape[0], np.uint8)
+    tested = np.zeros(d.shape[0], np.int64)
+    dt = DFG_F32 if d.dtype == np.float32 else DFG_F64
+    _check(_lib.dfg_div2_check(dt, _ptr(d), d.shape[0], method, _ptr(ok), _ptr(tested)))
+    return ok, tested
 
 
 def dfg_fused_source(expr, inputs, dtype, nx, ny, nz, compile=False):

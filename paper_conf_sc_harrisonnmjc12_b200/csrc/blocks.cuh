@@ -186,5 +186,7 @@ DFG_DEVICE dfg2 dfg2_eq(dfg2 a, dfg2 b, dfg2) { return dfg_eq(a, b); }
 DFG_DEVICE dfg2 dfg2_ne(dfg2 a, dfg2 b, dfg2) { return dfg_ne(a, b); }
 DFG_DEVICE dfg2 dfg2_select(dfg2 c, dfg2 a, dfg2 b, dfg2) { return dfg_select(c, a, b); }
 DFG_DEVICE dfg2 dfg2_gradq(dfg2 num, dfg2 nd, dfg2 r, dfg2) { return dfg_grad1q(num, -nd, r); }
+// two-operation quotient (fp64 axes certified by candidates, div2.hpp)
+DFG_DEVICE dfg2 dfg2_gradq2(dfg2 num, dfg2 yl, dfg2 yh, dfg2) { return __fma_rn(num, yh, __dmul_rn(num, yl)); }
 #endif
 #endif  // DFG_PAIRS

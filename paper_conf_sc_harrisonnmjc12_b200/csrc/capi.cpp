@@ -3,6 +3,7 @@
 // returns the status; nothing throws across the ABI.
 #include <cuda_runtime.h>
 
+#include <cmath>
 #include <cstdlib>
 #include <cstring>
 #include <memory>
@@ -10,6 +11,7 @@
 #include <vector>
 
 #include "dfg.h"
+#include "div2.hpp"
 #include "runtime.hpp"
 
 struct dfg_mesh_s {
@@ -359,6 +361,31 @@ int dfg_points3d_to_axes(dfg_dtype dtype, int64_t nx, int64_t ny, int64_t nz, co
   });
 }
 
+int dfg_div2_check(dfg_dtype dtype, const void* d, int64_t n, int method, uint8_t* ok, int64_t* tested) {
+  return guard([&] {
+    if (!d || !ok || n < 0) dfg::fail(DFG_E_INVALID, "null pointer or negative count");
+    if (method != 0 && method != 1) dfg::fail(DFG_E_INVALID, "method must be 0 (candidates) or 1 (exhaustive)");
+    if (method == 1 && to_dtype(dtype) != dfg::DType::F32) dfg::fail(DFG_E_UNSUPPORTED, "exhaustive check is fp32 only");
+    for (int64_t i = 0; i < n; ++i) {
+      long c = 0;
+      bool v;
+      if (to_dtype(dtype) == dfg::DType::F32) {
+        const float di = static_cast<const float*>(d)[i];
+        if (!(di > 0.0f) || !std::isnormal(di)) dfg::fail(DFG_E_INVALID, "divisors must be positive normal numbers");
+        const float r = 1.0f / di, yl = dfg::div2_low_part(di, r);
+        v = method == 0 ? dfg::certify_div2<float>(di, r, yl, 16, &c) : dfg::exhaustive_div2_f32(di, r, yl);
+      } else {
+        const double di = static_cast<const double*>(d)[i];
+        if (!(di > 0.0) || !std::isnormal(di)) dfg::fail(DFG_E_INVALID, "divisors must be positive normal numbers");
+        const double r = 1.0 / di, yl = dfg::div2_low_part(di, r);
+        v = dfg::certify_div2<double>(di, r, yl, 16, &c);
+      }
+      ok[i] = v ? 1 : 0;
+      if (tested) tested[i] = c;
+    }
+  });
+}
+
 int dfg_dag_dump(const char* expr, const char* const* inputs, int n_inputs, dfg_dtype dtype, char* buf, size_t cap,
                  size_t* needed) {
   return guard([&] {
@@ -428,7 +455,7 @@ int dfg_fused_source(const char* expr, const char* const* inputs, int n_inputs, 
     if (nx < 1 || ny < 1 || nz < 1) dfg::fail(DFG_E_INVALID, "mesh sizes must be >= 1");
     dfg::Dag d = dfg::build_dag(expr, names_of(inputs, n_inputs), to_dtype(dtype));
     // no mesh here: describe the kernel of a mesh whose divisors all verified
-    // (fp32 two-operation quotient), unless DFG_FUSED_VARIANT=markstein
+    // (two-operation quotient on every axis), unless DFG_FUSED_VARIANT=markstein
     dfg::FusedConfig cfg;
     const char* var = std::getenv("DFG_FUSED_VARIANT");
     if (!(var && !std::strcmp(var, "markstein"))) cfg.div2 = 7;

@@ -11,6 +11,7 @@
 #include <mutex>
 #include <set>
 
+#include "div2.hpp"
 #include "driver.hpp"
 #include "kernels.hpp"
 #include "runtime_detail.hpp"
@@ -35,7 +36,7 @@ void build_axis(const T* p, int64_t n, std::vector<char>& tab, bool& safe) {
   T* d = reinterpret_cast<T*>(tab.data());
   T* r = d + n;
   T* nd = r + n;  // exact negation: the fused kernels form num - q0*d with one FFMA2
-  T* yl = nd + n; // low part of 1/d for the two-operation quotient (fp32 only)
+  T* yl = nd + n; // low part of 1/d for the two-operation quotient
   for (int64_t i = 0; i < n; ++i) {
     if (n == 1) {  // derivative is 0 by definition; the kernels never read these
       d[i] = T(1);
@@ -48,11 +49,9 @@ void build_axis(const T* p, int64_t n, std::vector<char>& tab, bool& safe) {
     if (!(d[i] > T(0))) fail(DFG_E_INVALID, "cell centres coincide (coordinates too close for T)");
     r[i] = T(1) / d[i];
     nd[i] = -d[i];
-    // yl = RN(1/d - r): 1/d in double is within 2^-53 of the real quotient and
-    // the subtraction is exact (Sterbenz); the kernels only use yl on axes whose
-    // every divisor passed the exhaustive check (verify_div2 below), so its last
-    // bit needs no argument.
-    if (sizeof(T) == 4) yl[i] = T(1.0 / double(d[i]) - double(r[i]));
+    // yl = RN(1/d - r) = RN(e / d) with the exact remainder e = 1 - r d (div2.hpp);
+    // the kernels use it only on axes whose every divisor is certified below
+    yl[i] = div2_low_part(d[i], r[i]);
     // Markstein's exact-quotient argument needs d and r well inside the normal range.
     double ad = double(d[i]);
     if (!(ad > 0x1p-60 && ad < 0x1p60) || !std::isfinite(double(r[i]))) safe = false;
@@ -109,6 +108,33 @@ bool axis_div2(const std::vector<char>& tab, int64_t n) {
   for (int64_t i = 0; i < n; ++i)
     if (!g_div2_ok[div2_key(d[i], yl[i])]) return false;
   return true;
+}
+
+// fp64 axes: certification by candidates on the host (div2.hpp); 2^52
+// significands cannot be enumerated.  Cached per divisor like the fp32 check.
+std::map<uint64_t, bool> g_div2_ok64;  // key: d bits (r and yl are functions of d)
+
+bool axis_div2_f64(const std::vector<char>& tab, int64_t n) {
+  const double* d = reinterpret_cast<const double*>(tab.data());
+  const double* r = d + n;
+  const double* yl = d + 3 * n;
+  if (n == 1) return true;
+  std::lock_guard<std::mutex> lk(g_div2_mu);
+  bool all = true;
+  for (int64_t i = 0; i < n; ++i) {
+    uint64_t b;
+    std::memcpy(&b, &d[i], 8);
+    auto it = g_div2_ok64.find(b);
+    bool ok;
+    if (it != g_div2_ok64.end() && yl[i] == div2_low_part(d[i], r[i])) {
+      ok = it->second;
+    } else {
+      ok = certify_div2<double>(d[i], r[i], yl[i]);
+      if (yl[i] == div2_low_part(d[i], r[i])) g_div2_ok64[b] = ok;
+    }
+    all = all && ok;
+  }
+  return all;
 }
 
 std::mutex g_pool_mu;
@@ -227,16 +253,19 @@ std::shared_ptr<MeshImpl> create_block_impl(DType dt, int64_t nx, int64_t ny, in
   // unless every divisor is a power of two
   const char* d2 = std::getenv("DFG_DIV2");
   const bool div2_off = d2 && !std::strcmp(d2, "0");
-  if (dt == DType::F32 && d2 && !std::strcmp(d2, "test-1op"))
-    for (int a = 0; a < 3; ++a)
-      std::fill_n(reinterpret_cast<float*>(m->host_tab[a].data()) + 3 * N[a], N[a], 0.0f);
+  if (d2 && !std::strcmp(d2, "test-1op"))
+    for (int a = 0; a < 3; ++a) {
+      if (dt == DType::F32) std::fill_n(reinterpret_cast<float*>(m->host_tab[a].data()) + 3 * N[a], N[a], 0.0f);
+      else std::fill_n(reinterpret_cast<double*>(m->host_tab[a].data()) + 3 * N[a], N[a], 0.0);
+    }
   for (int a = 0; a < 3; ++a) {
     DFG_CUDA(cudaMalloc(&m->dev_tab[a], m->host_tab[a].size()));
     DFG_CUDA(cudaMemcpy(m->dev_tab[a], m->host_tab[a].data(), m->host_tab[a].size(), cudaMemcpyHostToDevice));
   }
-  if (dt == DType::F32 && m->markstein_safe && !div2_off)
+  if (m->markstein_safe && !div2_off)
     for (int a = 0; a < 3; ++a)
-      if (axis_div2(m->host_tab[a], N[a])) m->div2_mask |= 1 << a;
+      if (dt == DType::F32 ? axis_div2(m->host_tab[a], N[a]) : axis_div2_f64(m->host_tab[a], N[a]))
+        m->div2_mask |= 1 << a;
   return m;
 }
 

@@ -134,7 +134,7 @@ std::unique_ptr<PlanImpl> compile_plan(std::shared_ptr<MeshImpl> mesh, const std
     // exact quotient with two operations on the axes whose divisors all verified;
     // DFG_FUSED_VARIANT=markstein keeps the three-operation correction everywhere
     const bool markstein_only = var && !std::strcmp(var, "markstein");
-    if (cfg.div_mode == 1 && mesh->dt == DType::F32 && !markstein_only) cfg.div2 = mesh->div2_mask;
+    if (cfg.div_mode == 1 && !markstein_only) cfg.div2 = mesh->div2_mask;
     // scale folding is exact in the normal range only; "ieee" keeps every op
     const char* fold = std::getenv("DFG_SCALE_FOLD");
     cfg.fold = cfg.div_mode != 0 && !(fold && !std::strcmp(fold, "0"));

@@ -33,7 +33,7 @@ struct MeshImpl {
   bool ghosts_supplied = false;  // blocks: the caller fills every ghost cell (no exchange)
   int device = 0;
   bool markstein_safe = true;        // spacing tables inside the exact-division range
-  int div2_mask = 0;                 // bit a: every divisor of axis a passed verify_div2 (fp32)
+  int div2_mask = 0;                 // bit a: every divisor of axis a passed verify_div2 (fp32) / certify_div2 (fp64)
   std::vector<char> host_tab[3];     // per axis over the GLOBAL mesh: d | r | -d | yl (T), reading R1
   void* dev_tab[3] = {nullptr, nullptr, nullptr};
   std::map<std::string, Binding> fields;

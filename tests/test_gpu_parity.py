@@ -93,50 +93,71 @@ def test_tile_kernel_z_chunks(kz, monkeypatch):
     assert_parity(got, want)
 
 
+@pytest.mark.parametrize("T", [np.float32, np.float64])
 @pytest.mark.parametrize("shape", [(132, 40, 33), (67, 45, 37)])
-def test_two_operation_quotient(shape, monkeypatch):
-    """on fp32 axes whose every divisor passed the
-    exhaustive check the fused kernels form d f/d axis as
+def test_two_operation_quotient(shape, T, monkeypatch):
+    """on axes whose every divisor passed the check
+    (fp32: exhaustive enumeration on the device; fp64: certification by
+    candidate numerators) the fused kernels form d f/d axis as
     RN(num*r + RN(num*yl)); the bits equal the oracle's IEEE division and the
     three-operation correction's (TMA and general kernels)."""
-    x, y, z, f = _inputs(shape, np.float32)
+    x, y, z, f = _inputs(shape, T)
     src = PAPER_PROGRAMS["qcrit"][0]
     want = run_oracle(src, f, x, y, z)
     a, plan, *_ = run_lib(src, f, x, y, z, return_plan=True)
     assert plan.info()["div2_axes"] == 7
     assert_parity(a, want)
+    u = np.uint32 if T == np.float32 else np.uint64
     monkeypatch.setenv("DFG_FUSED_VARIANT", "markstein")
     b, plan2, *_ = run_lib(src, f, x, y, z, return_plan=True)
     assert plan2.info()["div2_axes"] == 0
-    assert np.array_equal(a.view(np.uint32), b.view(np.uint32))
+    assert np.array_equal(a.view(u), b.view(u))
     monkeypatch.delenv("DFG_FUSED_VARIANT")
     monkeypatch.setenv("DFG_DIV2", "0")
     c, plan3, *_ = run_lib(src, f, x, y, z, return_plan=True)
     assert plan3.info()["div2_axes"] == 0
-    assert np.array_equal(a.view(np.uint32), c.view(np.uint32))
+    assert np.array_equal(a.view(u), c.view(u))
 
 
-def test_two_operation_check_rejects_one_operation(monkeypatch):
-    """The device check is not vacuous: with yl = 0 (the one-operation
-    RN(num*r), not correctly rounded for most divisors) it rejects every axis
-    of the RT mesh, while on a uniform mesh with power-of-two spacing, where
-    r = 1/d exactly and RN(num*r) = RN(num/d), it accepts all three."""
+@pytest.mark.parametrize("T", [np.float32, np.float64])
+def test_two_operation_check_rejects_one_operation(T, monkeypatch):
+    """The checks are not vacuous: with yl = 0 (the one-operation RN(num*r),
+    not correctly rounded for most divisors) every axis of the RT mesh is
+    rejected, while on a uniform mesh with power-of-two spacing, where
+    r = 1/d exactly and RN(num*r) = RN(num/d), all three are accepted."""
     monkeypatch.setenv("DFG_DIV2", "test-1op")
     src = PAPER_PROGRAMS["vortmag"][0]
-    x, y, z, f = _inputs((64, 24, 20), np.float32)
+    x, y, z, f = _inputs((64, 24, 20), T)
     got, plan, *_ = run_lib(src, f, x, y, z, return_plan=True)
     assert plan.info()["div2_axes"] == 0
     assert_parity(got, run_oracle(src, f, x, y, z))
-    x, y, z = (synth.uniform_coords(n, dtype=np.float32) for n in (64, 24, 20))
+    x, y, z = (synth.uniform_coords(n, dtype=T) for n in (64, 24, 20))
     got, plan, *_ = run_lib(src, f, x, y, z, return_plan=True)
     assert plan.info()["div2_axes"] == 7
     assert_parity(got, run_oracle(src, f, x, y, z))
 
 
-def test_two_operation_quotient_fp32_only():
-    x, y, z, f = _inputs((40, 24, 20), np.float64)
-    _, plan, *_ = run_lib(PAPER_PROGRAMS["qcrit"][0], f, x, y, z, return_plan=True)
-    assert plan.info()["div2_axes"] == 0
+def test_two_operation_quotient_fp64_mixed_axes():
+    """fp64 x axis with jittered geometric spacing (ratio ~1.35: divisors with
+    full-precision significands; with seed 1 the certificate rejects one of
+    them): that axis keeps the three-operation correction, the others use two
+    operations, and the mesh's choice equals the host checker's verdict on
+    the same spacing table; bit-exact parity."""
+    from paper_conf_sc_harrisonnmjc12_b200._dfg import dfg_div2_check
+    nx, ny, nz = 120, 24, 20
+    _, y, z, f = _inputs((nx, ny, nz), np.float64)
+    x = np.exp(0.3 * np.arange(nx + 1) + 0.1 * np.random.default_rng(1).uniform(size=nx + 1))
+    want_mask = 0
+    for a, p in enumerate((x, y, z)):
+        c = (p[:-1] + p[1:]) * 0.5
+        i = np.arange(c.size)
+        d = c[np.minimum(i + 1, c.size - 1)] - c[np.maximum(i - 1, 0)]
+        want_mask |= int(dfg_div2_check(d, 0)[0].all()) << a
+    assert want_mask == 6, "the geometric x axis should contain a rejected divisor"
+    src = PAPER_PROGRAMS["qcrit"][0]
+    got, plan, *_ = run_lib(src, f, x, y, z, return_plan=True)
+    assert plan.info()["div2_axes"] == want_mask
+    assert_parity(got, run_oracle(src, f, x, y, z))
 
 
 @pytest.mark.parametrize("kz", ["1", "3", "7", "1000"])

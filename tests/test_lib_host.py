@@ -209,7 +209,7 @@ def test_fused_kernel_compiles_without_spills(dfg, name, dtype, variant, monkeyp
     src, inputs = PAPER_PROGRAMS[name]
     code, regs, spill = dfg.dfg_fused_source(src, inputs, dtype, 64, 48, 40, compile=True)
     assert "dfg_body" in code and "extern \"C\" __global__" in code
-    two_op = dtype == 0 and not variant and name != "velmag"
+    two_op = not variant and name != "velmag"
     assert ("dfg2_gradq2(gn" in code) == two_op
     assert regs > 0
     assert spill == 0, (regs, spill)
@@ -340,3 +340,50 @@ def test_peer_entry_points_validate(dfg):
     assert lib.dfg_mesh_link_peers(None, None, None) == -1
     hdr = open(os.path.join(ROOT, "include", "dfg.h")).read()
     assert "#define DFG_PEER_BLOB_BYTES 4096" in hdr and dfg._dfg.PEER_BLOB_BYTES == 4096
+
+
+def test_div2_certificate_matches_exhaustive(dfg):
+    """The two-operation quotient RN(x*r + RN(x*yl)) (Brisebarre-Muller-Raina)
+    is not RN(x/d) for every divisor.  fp64 axes are certified by testing
+    the few numerators whose quotient can lie within the scheme's error of a
+    rounding boundary (csrc/div2.hpp); the same method at fp32 precision must
+    reach the verdict of exhaustive enumeration of all 2^23 significands for
+    every divisor -- including the ones that fail, found here among seeded
+    random divisors, so a wrong candidate set cannot pass unnoticed."""
+    import numpy as np
+    from paper_conf_sc_harrisonnmjc12_b200._dfg import dfg_div2_check
+    rng = np.random.default_rng(2012)
+    d = rng.uniform(1.0, 2.0, 320) * np.exp2(rng.integers(-12, 4, 320))
+    d = d.astype(np.float32)
+    cand, tested = dfg_div2_check(d, 0)
+    exh, _ = dfg_div2_check(d, 1)
+    assert (exh == 0).sum() >= 2, "the sample should contain failing divisors"
+    assert np.array_equal(cand, exh)
+    assert tested.max() > 0
+    # power-of-two divisors: r is exact, no candidate, always certified
+    ok, tested = dfg_div2_check(np.exp2(np.arange(-20, 20)).astype(np.float64), 0)
+    assert ok.all() and tested.max() == 0
+
+
+def test_div2_certificate_fp64_axes(dfg):
+    """fp64: the RT-like mesh spacings (differences of nearby coordinates,
+    many trailing zero bits) all certify; a rejection is always a genuine
+    counterexample, and random full-precision divisors fail at about the fp32
+    rate (~1 %)."""
+    import numpy as np
+    import synth
+    from paper_conf_sc_harrisonnmjc12_b200._dfg import dfg_div2_check
+    for a in synth.rt_coords(1024, 1024, 1024, np.float64):
+        c = (a[:-1] + a[1:]) * 0.5
+        i = np.arange(c.size)
+        dd = c[np.minimum(i + 1, c.size - 1)] - c[np.maximum(i - 1, 0)]
+        ok, _ = dfg_div2_check(dd, 0)
+        assert ok.all()
+    rng = np.random.default_rng(7)
+    d = rng.uniform(1.0, 2.0, 4000)
+    ok, _ = dfg_div2_check(d, 0)
+    assert 0.002 < (ok == 0).mean() < 0.03
+    with pytest.raises(Exception):
+        dfg_div2_check(d[:3], 1)          # exhaustive is fp32 only
+    with pytest.raises(Exception):
+        dfg_div2_check(np.array([0.0, 1.0]), 0)
