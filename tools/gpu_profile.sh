@@ -2,7 +2,7 @@
 # capture of the top kernel (dfg_fused_tma, fused Q 1024^3 fp32)
 python -c "import __graft_entry__ as g; g.build()" > /dev/null 2>&1
 TAG=${TAG:-r01h}
-timeout 900 ncu --metrics gpu__time_duration.sum --clock-control none -c 4000 --csv \
+timeout 900 ncu --metrics gpu__time_duration.sum --clock-control none -k regex:dfg -c 400 --csv \
   --log-file gpurun_out/${TAG}_launches.csv python bench.py --steps 20 --warmup 3 --no-cpu-baseline --no-strategies \
   > gpurun_out/${TAG}_launches_bench.log 2>&1; echo launches=$?
 timeout 900 ncu --set full --clock-control none --import-source on -k regex:dfg_fused_tma -s 3 -c 1 \
