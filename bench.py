@@ -257,6 +257,9 @@ def main():
     ap.add_argument("--no-cpu-mt", action="store_true", help="skip the multi-process oracle timing")
     ap.add_argument("--halo", default="peer", choices=["peer", "nccl"],
                     help="N > 1 z-slab halo: peer memory read in place by the kernel (default) or NCCL send/recv")
+    ap.add_argument("--scaling", default="weak", choices=["weak", "strong"],
+                    help="weak: size^3 cells per GPU (mesh size x size x size*N); strong: one size^3 mesh "
+                         "split into N z-slabs (config 4 of BASELINE.json runs both)")
     args = ap.parse_args()
     if args.impl == "reference":
         return run_reference(args)
@@ -284,7 +287,7 @@ def main():
         dist.init_process_group("nccl", device_id=torch.device("cuda", local))
     assert world == args.gpus or world == 1, "launch with torchrun --nproc-per-node N for --gpus N"
     n = args.size
-    NZ = n * world
+    NZ = n * world if args.scaling == "weak" else n
     K, W = args.steps, args.warmup
     assert W >= 3, "at least 3 warm-up steps"
 
@@ -367,7 +370,7 @@ def main():
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
     ms, kern_ms = float(t[0]), float(t[1])
     ms_step = ms / K
-    value = cells_rank * world / (ms_step * 1e-3)
+    value = n * n * NZ / (ms_step * 1e-3)          # every cell of the job once per step
     info = plan.info()
 
     # context for the roofline: a plain device copy (torch copy_, 4 GiB read +
@@ -517,10 +520,11 @@ def main():
     if rank == 0:
         line = {
             "metric": METRIC, "value": value, "unit": "cells/s", "n_gpus": world, "steps": K, "warmup": W,
-            "ms_per_step": ms_step, "higher_is_better": True, "scaling": "weak", "vs_baseline": None,
+            "ms_per_step": ms_step, "higher_is_better": True, "scaling": args.scaling, "vs_baseline": None,
             "dtype": "f32", "data": "synthetic",
-            "config": {"workload": f"fused Q-criterion, {n}^3 fp32 rectilinear mesh per GPU "
-                                   f"(mesh {n}x{n}x{NZ}, z-slabs + 1-plane halo when N>1: " + (halo or "none") + ")",
+            "config": {"workload": (f"fused Q-criterion, {n}^3 fp32 rectilinear mesh per GPU " if args.scaling == "weak"
+                                    else f"fused Q-criterion, one {n}^3 fp32 rectilinear mesh over {world} GPU(s) ")
+                                   + f"(mesh {n}x{n}x{NZ}, z-slabs + 1-plane halo when N>1: " + (halo or "none") + ")",
                        "expression": "qcrit (Fig. 3C completed)", "strategy": "fused",
                        "cells_per_gpu": cells_rank, "fused_kernel": {1: "tma", 2: "general", 3: "pointwise", 5: "tile"}.get(
                            info["variant"]), "regs": info["regs"],
