@@ -501,11 +501,12 @@ def main():
                           "NCCL send/recv of the first/last owned plane of u, v, w on a side stream, "
                           "overlapped with the interior planes; boundary planes launched after it")}
 
-    strategies = variants = sweep = None
+    strategies = variants = sweep = blocks = None
     if rank == 0 and world == 1 and not args.no_strategies:
         variants = variant_leg(dfg, mesh, out, QCRIT, torch, n)
         strategies = strategy_sweep(dfg, synth, torch)
         sweep = complexity_sweep(dfg, synth, torch)
+        blocks = blocks_leg(torch)
 
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
@@ -546,6 +547,7 @@ def main():
             "variants": variants,
             "strategies": strategies,
             "complexity_sweep_768": sweep,
+            "visit_blocks": blocks,
             "cpu_baseline": cpu,
         }
         print(json.dumps(line), flush=True)
@@ -604,6 +606,23 @@ def variant_leg(dfg, mesh, out_exact, src, torch, n):
                                "normwise_diff_vs_exact": diff}
     plan.close()
     del out
+    return res
+
+
+def blocks_leg(torch):
+    """the paper's VisIt decomposition (Fig. 7,
+    L315: blocks of 192 x 192 x 256 with ghost shells, 12 sub-grids per GPU)
+    -- one plan per block back to back vs all blocks of the device in one
+    persistent launch (TMA kernel on 16-byte padded shells, cp.async ring on
+    packed shells) vs one mesh of the same cells; 16 algorithmic B / cell."""
+    sys.path.insert(0, os.path.join(ROOT, "tools"))
+    import blocks_overhead
+    res = {}
+    for pad, name in ((1, "padded_shells"), (0, "packed_shells")):
+        r = blocks_overhead.measure(12, 192, 192, 256, pad)
+        r["algorithmic_gb_per_s_one_launch"] = ALGO_BYTES_PER_CELL * r["cells"] / (r["ms_batched"] * 1e-3) / 1e9
+        res[name] = r
+        torch.cuda.empty_cache()
     return res
 
 

@@ -43,7 +43,16 @@ def main():
     ap.add_argument("--bz", type=int, default=256)
     ap.add_argument("--pad", type=int, default=1, help="pad shell rows to a multiple of 16 bytes (TMA path)")
     a = ap.parse_args()
-    B, bx, by, bz = a.blocks, a.bx, a.by, a.bz
+    print(json.dumps(measure(a.blocks, a.bx, a.by, a.bz, a.pad)))
+
+
+def measure(B=12, bx=192, by=192, bz=256, pad=1):
+    """B blocks of bx x by x bz stacked in z, one-cell ghost shells: one plan
+    per block back to back, all blocks in one launch (dfg_execute_blocks) and
+    one mesh of the same cells; returns a dict (times in ms)."""
+    class a:  # noqa: N801
+        pass
+    a.pad = pad
     NZ = bz * B                       # blocks stacked in z: global mesh bx x by x (bz*B)
     x, y, z = synth.rt_coords(bx, by, NZ, np.float32)
     x64, y64, z64 = (v.astype(np.float64) for v in (x, y, z))
@@ -76,6 +85,7 @@ def main():
             p.execute(o)
 
     t_blocks = timeit(blocks)
+    blocks_variant = plans[0].info()["variant"]
     t_batched = timeit(lambda: dfg.execute_blocks(plans, outs))
     batched_variant = plans[0].info()["variant"]
     whole = dfg.Mesh(x, y, z)
@@ -87,12 +97,15 @@ def main():
     t_whole = timeit(lambda: wp.execute(wo))
     same = bool(torch.equal(torch.cat(outs), wo))
     cells = bx * by * NZ
-    print(json.dumps({"blocks": B, "block": [bx, by, bz], "row_pitch": rp, "x_offset": xo, "cells": cells, "ms_blocks": t_blocks,
-                      "ms_batched": t_batched, "batched_variant": batched_variant,
-                      "gcells_s_batched": cells / t_batched / 1e6,
-                      "ms_one_mesh": t_whole, "overhead": t_blocks / t_whole - 1,
-                      "blocks_variant": plans[0].info()["variant"], "bit_identical": same,
-                      "gcells_s_blocks": cells / t_blocks / 1e6, "gcells_s_one_mesh": cells / t_whole / 1e6}))
+    res = {"blocks": B, "block": [bx, by, bz], "row_pitch": rp, "x_offset": xo, "cells": cells, "ms_blocks": t_blocks,
+           "ms_batched": t_batched, "batched_variant": batched_variant,
+           "gcells_s_batched": cells / t_batched / 1e6,
+           "ms_one_mesh": t_whole, "overhead": t_blocks / t_whole - 1,
+           "blocks_variant": blocks_variant, "bit_identical": same,
+           "gcells_s_blocks": cells / t_blocks / 1e6, "gcells_s_one_mesh": cells / t_whole / 1e6}
+    for p in plans + [wp]:
+        p.close()
+    return res
 
 
 if __name__ == "__main__":
