@@ -91,6 +91,15 @@ bool axis_div2(const std::vector<char>& tab, int64_t n) {
     const int m = int(qd.size());
     float* buf = nullptr;
     unsigned* bad = nullptr;
+    struct Free {
+      float*& b;
+      unsigned*& u;
+      bool armed = true;
+      ~Free() {
+        if (armed && b) cudaFree(b);
+        if (armed && u) cudaFree(u);
+      }
+    } guard{buf, bad};  // frees both if a CUDA call below throws
     DFG_CUDA(cudaMalloc(&buf, 3 * size_t(m) * sizeof(float)));
     DFG_CUDA(cudaMalloc(&bad, size_t(m) * sizeof(unsigned)));
     DFG_CUDA(cudaMemcpy(buf, qd.data(), m * sizeof(float), cudaMemcpyHostToDevice));
@@ -100,6 +109,7 @@ bool axis_div2(const std::vector<char>& tab, int64_t n) {
     kern::verify_div2(buf, buf + m, buf + 2 * m, m, bad, nullptr);
     std::vector<unsigned> hb(m);
     cudaError_t e = cudaMemcpy(hb.data(), bad, m * sizeof(unsigned), cudaMemcpyDeviceToHost);
+    guard.armed = false;
     cudaFree(buf);
     cudaFree(bad);
     DFG_CUDA(e);
