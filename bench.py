@@ -529,6 +529,9 @@ def main():
                        "expression": "qcrit (Fig. 3C completed)", "strategy": "fused",
                        "cells_per_gpu": cells_rank, "fused_kernel": {1: "tma", 2: "general", 3: "pointwise", 5: "tile"}.get(
                            info["variant"]), "regs": info["regs"],
+                       "arithmetic": "exact: every cell bit-identical to the fp32 oracle (two-operation grad3d quotient "
+                                     f"on verified axes, mask {info.get('div2_axes')}); the within-tolerance 'fast' "
+                                     "quotient and the hand-written reference kernel are under 'variants'",
                        "l2": f"inputs {3 * cells_rank * 4 / 1e9:.1f} GB per GPU >> 126 MB L2; no flush needed",
                        "parallelism": f"zslab{world}",
                        **({"one_gpu_functional_test": True} if one_gpu else {})},
