@@ -629,6 +629,27 @@ def blocks_leg(torch):
     return res
 
 
+def _window_parity(src, names, dt, fields, out, x, y, z, n):
+    """Sampled full-size parity of a sweep case: the oracle on three windows
+    of the GPU's own inputs (the low corner with the global one-sided
+    boundaries, an interior block, the high corner), full rows in x, compared
+    bit for bit with the fused kernel's output over the window cells whose
+    stencil lies inside the window (oracle.evaluate's valid mask)."""
+    from oracle import evaluate as oev
+    from oracle.lang import build_dag
+    dag = build_dag(src, tuple(names), dt)
+    u = np.uint32 if dt == "f32" else np.uint64
+    cells = bad = 0
+    for k0, j0 in ((0, 0), (n // 2 - 3, n // 2 - 4), (n - 6, n - 8)):
+        win = {nm: fields[c][k0:k0 + 6, j0:j0 + 8, :].cpu().numpy() for nm, c in zip(names, "uvw")}
+        ref, valid = oev.evaluate(dag, win, oev.MeshWindow(x, y, z, i0=0, j0=j0, k0=k0))
+        got = out[k0:k0 + 6, j0:j0 + 8, :].cpu().numpy()
+        cells += int(valid.sum())
+        bad += int(np.count_nonzero(got[valid].view(u) != ref[valid].view(u)))
+    return {"cells_compared": cells, "mismatches": bad, "windows": "6 planes x 8 rows x all columns at the low "
+            "corner, the centre and the high corner"}
+
+
 def complexity_sweep(dfg, synth, torch):
     """Config 5: the expression-complexity sweep (intro -> VelMag -> VortMag
     -> Q) at 768^3, fp32 and fp64, fused strategy, device-resident inputs."""
@@ -652,7 +673,8 @@ def complexity_sweep(dfg, synth, torch):
             res[f"{name}_{dt}"] = {"filters": info["filters"], "kernel_ms": kms, "cells_per_s": n ** 3 / (kms * 1e-3),
                                    "algorithmic_gb_per_s": nbytes * n ** 3 / (kms * 1e-3) / 1e9,
                                    "bytes_per_cell": nbytes, "regs": info["regs"],
-                                   "kernel": {1: "tma", 2: "general", 3: "pointwise", 5: "tile"}.get(info["variant"])}
+                                   "kernel": {1: "tma", 2: "general", 3: "pointwise", 5: "tile"}.get(info["variant"]),
+                                   "oracle_parity": _window_parity(src, names, dt, fields, out, x, y, z, n)}
             plan.close()
             mesh.close()
         del fields, out
@@ -762,6 +784,7 @@ def _strategies_at(dfg, synth, torch, n, src, strategies, runs):
                   "highwater_bytes": st["dev_highwater_bytes"]}
         if ref is None:
             ref = out.clone()
+            res[s]["oracle_parity"] = _window_parity(src, ("u", "v", "w"), "f32", bufs, out, x, y, z, n)
         else:
             res[s]["bit_identical_to_fused"] = bool(torch.equal(ref, out))
         plan.close()
