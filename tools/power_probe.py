@@ -55,7 +55,7 @@ for c in cases:
         prog, strat = c[:-4], "reference"
     for k, v in env.items():
         os.environ[k] = v
-    for k, v in [kv.split("=") for kv in os.environ.get("EXTRA", "").split(",") if kv]:
+    for k, v in [kv.split("=") for kv in os.environ.get("EXTRA", "").split(",") if "=" in kv]:
         os.environ[k] = v
     try:
         plan = dfg.Plan(mesh, PAPER_PROGRAMS[prog][0] if strat == "fused" else prog, strat)
