@@ -459,10 +459,10 @@ int dfg_fused_source(const char* expr, const char* const* inputs, int n_inputs, 
     dfg::FusedConfig cfg;
     const char* var = std::getenv("DFG_FUSED_VARIANT");
     if (!(var && !std::strcmp(var, "markstein"))) cfg.div2 = 7;
-    // tile rows per warp: DFG_RPW, else the choice for a 148-SM B200
+    // tile shape: DFG_RPW (15 warps), else the planner's choice for a 148-SM B200
     const char* rpw = std::getenv("DFG_RPW");
-    cfg.rpw = rpw ? std::atoi(rpw) : dfg::choose_rpw(d.dtype, nx, ny, nz,
-                                                     cfg.ncw, 148);
+    if (rpw) cfg.rpw = std::atoi(rpw);
+    else dfg::choose_tile(d.dtype, nx, ny, nz, 148, &cfg.ncw, &cfg.rpw);
     if (cfg.rpw != 2 && cfg.rpw != 4) cfg.rpw = 1;
     dfg::FusedSource fs = dfg::generate_fused(d, nx, ny, nz, cfg);
     if (compile) {

@@ -58,7 +58,11 @@ inline int tma_tile_h(int ncw, int rpw) { return ncw * rpw; }
 // Rows per consumer warp for a mesh of nx x ny x nz cells on `slots`
 // persistent CTAs: the candidate (1, 2, 4) whose best z-chunking needs the
 // fewest plane-steps, weighted by the halo'd tile it loads per computed cell.
-int choose_rpw(DType dt, int64_t nx, int64_t ny, int64_t nz, int ncw, int64_t slots);
+int choose_rpw(DType dt, int64_t nx, int64_t ny, int64_t nz, int ncw, int64_t slots, double* cost = nullptr);
+// Tile shape of the fused kernel for a mesh: consumer warps (15, or 12 when the
+// plane-step model -- steps per CTA x halo'd tile area -- is >= 5 % cheaper,
+// e.g. 192 rows = 8 tiles of 24) and rows per warp.
+void choose_tile(DType dt, int64_t nx, int64_t ny, int64_t nz, int64_t slots, int* ncw, int* rpw);
 
 // z-chunk length for `tiles` x-y tiles over `range` planes: whole rounds of
 // items over the persistent CTAs against the two halo planes (and the

@@ -146,11 +146,14 @@ std::unique_ptr<PlanImpl> compile_plan(std::shared_ptr<MeshImpl> mesh, const std
     if (st) cfg.stages = std::max(2, std::min(16, std::atoi(st)));
     // tile shape for this mesh (narrow meshes: several rows per warp)
     const char* rpw = std::getenv("DFG_RPW");
+    const int64_t slots = int64_t(sm_count(mesh->device)) * cfg.ctas;
     if (rpw) {
       const int r = std::atoi(rpw);
       cfg.rpw = (r == 2 || r == 4) ? r : 1;
+    } else if (ncw) {
+      cfg.rpw = choose_rpw(mesh->dt, mesh->nx, mesh->ny, mesh->nzl, cfg.ncw, slots);
     } else {
-      cfg.rpw = choose_rpw(mesh->dt, mesh->nx, mesh->ny, mesh->nzl, cfg.ncw, int64_t(sm_count(mesh->device)) * cfg.ctas);
+      choose_tile(mesh->dt, mesh->nx, mesh->ny, mesh->nzl, slots, &cfg.ncw, &cfg.rpw);
     }
     // axis degeneracy (n == 1) is a property of the GLOBAL mesh
     plan->fsrc = generate_fused(dag, mesh->NX, mesh->NY, mesh->NZ, cfg, ref);

@@ -736,7 +736,8 @@ def test_tma_rows_per_warp(rpw, T, shape, monkeypatch):
 
 def test_tile_shape_choice():
     """Narrow meshes take several rows per warp (no idle lanes in a ragged x
-    tile); the 1024-wide bench mesh keeps one row per warp."""
+    tile); the 1024-wide bench mesh keeps one row per warp; 192^3 (config 2)
+    takes 12 warps x 2 rows (8 whole tiles of 24 rows), bit-exact."""
     import paper_conf_sc_harrisonnmjc12_b200 as dfg
     for n, nz, want in ((192, 192, 2), (1024, 64, 1)):
         x, y, z = synth.rt_coords(n, n, nz, np.float32)
@@ -746,4 +747,6 @@ def test_tile_shape_choice():
             mesh.bind(c, t)
         plan = dfg.Plan(mesh, PAPER_PROGRAMS["qcrit"][0], "fused")
         assert plan.info()["rows_per_warp"] == want, (n, plan.info())
+        if n == 192:
+            assert plan.info()["tile_h"] == 24, plan.info()
         plan.close()

@@ -318,13 +318,15 @@ def test_tile_shapes_compile_without_spills(dfg, rpw, dtype, monkeypatch):
 
 
 def test_tile_shape_choice_host(dfg):
-    """Without DFG_RPW the generator takes choose_rpw's tile for a 148-SM part:
-    two rows per warp for the 192-wide meshes of config 2 and the paper's
-    192 x 192 x 256 blocks, one for the 1024^3 bench mesh."""
+    """Without DFG_RPW the generator takes choose_tile's shape for a 148-SM
+    part: 12 warps x 2 rows for config 2's 192^3 (8 tiles of 24 rows, no
+    ragged tile; measured -12 %), 15 x 2 for the paper's 192 x 192 x 256
+    blocks, 15 x 1 for the 1024^3 bench mesh."""
     src, inputs = PAPER_PROGRAMS["qcrit"]
-    for dims, want in (((192, 192, 192), 2), ((192, 192, 256), 2), ((1024, 1024, 1024), 1), ((32, 32, 32), 1)):
+    for dims, ncw, rpw in (((192, 192, 192), 12, 2), ((192, 192, 256), 15, 2), ((1024, 1024, 1024), 15, 1),
+                           ((768, 768, 768), 15, 1), ((32, 32, 32), 12, 1)):
         code, _, _ = dfg.dfg_fused_source(src, inputs, 0, *dims)
-        assert f"#define DFG_RPW {want}" in code, dims
+        assert f"#define DFG_RPW {rpw}" in code and f"#define DFG_NCW {ncw}" in code, dims
 
 
 def test_set_timing_validates(dfg):
