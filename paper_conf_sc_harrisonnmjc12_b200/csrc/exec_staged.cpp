@@ -413,8 +413,10 @@ void PlanImpl::exec_roundtrip(void* out, bool out_dev, cudaStream_t s) {
 
   auto host_const = [&](const Filter& f) -> void* {
     void* h = hp.get(sb);
-    if (m.dt == DType::F32) std::fill_n(static_cast<float*>(h), N, float(f.cval));
-    else std::fill_n(static_cast<double*>(h), N, f.cval);
+    parallel_for(N, [&](int64_t a, int64_t b) {
+      if (m.dt == DType::F32) std::fill(static_cast<float*>(h) + a, static_cast<float*>(h) + b, float(f.cval));
+      else std::fill(static_cast<double*>(h) + a, static_cast<double*>(h) + b, f.cval);
+    });
     return h;
   };
   auto release = [&](const Ref& r) {
@@ -433,15 +435,18 @@ void PlanImpl::exec_roundtrip(void* out, bool out_dev, cudaStream_t s) {
     if (f.op == Op::Decompose) {  // on the host, no transfer (L289)
       const Ref& a = f.in[0];
       void* h = hp.get(sb);
-      if (m.dt == DType::F32) {
-        const float* v = static_cast<const float*>(hval[a.id]);
-        float* o = static_cast<float*>(h);
-        for (int64_t e = 0; e < N; ++e) o[e] = v[4 * e + f.k];
-      } else {
-        const double* v = static_cast<const double*>(hval[a.id]);
-        double* o = static_cast<double*>(h);
-        for (int64_t e = 0; e < N; ++e) o[e] = v[4 * e + f.k];
-      }
+      const int lane = f.k;
+      parallel_for(N, [&](int64_t lo, int64_t hi) {
+        if (m.dt == DType::F32) {
+          const float* v = static_cast<const float*>(hval[a.id]);
+          float* o = static_cast<float*>(h);
+          for (int64_t e = lo; e < hi; ++e) o[e] = v[4 * e + lane];
+        } else {
+          const double* v = static_cast<const double*>(hval[a.id]);
+          double* o = static_cast<double*>(h);
+          for (int64_t e = lo; e < hi; ++e) o[e] = v[4 * e + lane];
+        }
+      });
       hval[k] = h;
       release(a);
       continue;
@@ -549,7 +554,10 @@ void PlanImpl::exec_roundtrip(void* out, bool out_dev, cudaStream_t s) {
     st.h2d_count += 1;
     st.h2d_bytes += int64_t(rb);
   } else {
-    std::memcpy(out, hval[res.id], rb);
+    const char* hsrc = static_cast<const char*>(hval[res.id]);
+    parallel_for(int64_t(rb), [&](int64_t lo, int64_t hi) {
+      std::memcpy(static_cast<char*>(out) + lo, hsrc + lo, size_t(hi - lo));
+    });
   }
   DFG_CUDA(cudaStreamSynchronize(s));
   release(res);

@@ -9,6 +9,7 @@
 #include <map>
 #include <mutex>
 #include <string>
+#include <thread>
 #include <vector>
 
 #include "common.hpp"
@@ -84,6 +85,23 @@ struct HostPool {
   }
 };
 HostPool& host_pool();
+
+// Host loops of the roundtrip strategy (constant fills, decompose on the host,
+// L289) over problem-sized arrays: split [0, n) over the host cores.  Element
+// order does not matter (each index is written once from its own inputs).
+template <class F>
+void parallel_for(int64_t n, F f) {
+  const int64_t hw = int64_t(std::max(1u, std::thread::hardware_concurrency()));
+  const int64_t T = std::max<int64_t>(1, std::min<int64_t>({hw, 32, n / (1 << 16)}));
+  if (T == 1) {
+    f(int64_t(0), n);
+    return;
+  }
+  std::vector<std::thread> th;
+  for (int64_t t = 1; t < T; ++t) th.emplace_back(f, n * t / T, n * (t + 1) / T);
+  f(int64_t(0), n / T);
+  for (auto& x : th) x.join();
+}
 extern std::mutex g_host_mu;
 
 }  // namespace detail
