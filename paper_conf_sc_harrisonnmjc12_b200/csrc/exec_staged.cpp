@@ -384,6 +384,55 @@ void PlanImpl::exec_staged(void* out, bool out_dev, cudaStream_t s) {
   st.dev_highwater_bytes = std::max<int64_t>(st.dev_highwater_bytes, int64_t(led.high));
 }
 
+// Device-resident staged execute as a CUDA graph: the first execute for an
+// (output, inputs) binding captures exec_staged on a private stream (the
+// kernels, the stream-ordered allocations and frees of the intermediates)
+// and every execute launches the instantiated graph on the caller's stream:
+// one host call instead of one launch + allocation + free per filter.
+void PlanImpl::exec_staged_graph(void* out, cudaStream_t s) {
+  MeshImpl& m = *mesh;
+  std::vector<const void*> key{out};
+  for (int i : sources(dag).inputs) key.push_back(m.fields[dag.inputs[i]].ptr);
+  if (!gexec || key != gkey) {
+    if (gexec) {
+      DFG_CUDA(cudaGraphExecDestroy(gexec));
+      gexec = nullptr;
+    }
+    if (!sCap) DFG_CUDA(cudaStreamCreateWithFlags(&sCap, cudaStreamNonBlocking));
+    pool_for(m.device);  // created outside the capture (pool creation is not capturable)
+    const dfg_stats before = st;
+    DFG_CUDA(cudaStreamBeginCapture(sCap, cudaStreamCaptureModeThreadLocal));
+    cudaGraph_t g = nullptr;
+    try {
+      exec_staged(out, true, sCap);
+    } catch (...) {
+      cudaStreamEndCapture(sCap, &g);  // leave the stream usable
+      if (g) cudaGraphDestroy(g);
+      cudaGetLastError();
+      throw;
+    }
+    DFG_CUDA(cudaStreamEndCapture(sCap, &g));
+    cudaError_t e = cudaGraphInstantiate(&gexec, g, 0);
+    cudaGraphDestroy(g);
+    DFG_CUDA(e);
+    gdelta = dfg_stats{};
+    gdelta.kernel_count = st.kernel_count - before.kernel_count;
+    gdelta.h2d_count = st.h2d_count - before.h2d_count;
+    gdelta.d2h_count = st.d2h_count - before.d2h_count;
+    gdelta.h2d_bytes = st.h2d_bytes - before.h2d_bytes;
+    gdelta.d2h_bytes = st.d2h_bytes - before.d2h_bytes;
+    gkey = key;
+  } else {
+    st.kernel_count += gdelta.kernel_count;
+    st.h2d_count += gdelta.h2d_count;
+    st.d2h_count += gdelta.d2h_count;
+    st.h2d_bytes += gdelta.h2d_bytes;
+    st.d2h_bytes += gdelta.d2h_bytes;
+    graph_launches += 1;
+  }
+  DFG_CUDA(cudaGraphLaunch(gexec, s));
+}
+
 // ---------------------------------------------------------- roundtrip
 void PlanImpl::exec_roundtrip(void* out, bool out_dev, cudaStream_t s) {
   MeshImpl& m = *mesh;

@@ -63,6 +63,8 @@ PlanImpl::~PlanImpl() {
   if (sHalo) cudaStreamDestroy(sHalo);
   if (evHaloIn) cudaEventDestroy(evHaloIn);
   if (evHaloOut) cudaEventDestroy(evHaloOut);
+  if (gexec) cudaGraphExecDestroy(gexec);
+  if (sCap) cudaStreamDestroy(sCap);
   if (cur >= 0) cudaSetDevice(cur);
 }
 
@@ -286,7 +288,14 @@ void PlanImpl::execute(void* out, bool out_dev, cudaStream_t s) {
     case DFG_FUSED: exec_fused(out, out_dev, s); break;
     case DFG_STREAMED: exec_streamed(out, out_dev, s); break;
     case DFG_REFERENCE: exec_fused(out, out_dev, s); break;
-    case DFG_STAGED: exec_staged(out, out_dev, s); break;
+    case DFG_STAGED: {
+      const char* g = std::getenv("DFG_GRAPH");
+      bool device = out_dev;
+      for (int i : sources(dag).inputs) device = device && m.fields[dag.inputs[i]].on_device;
+      if (device && !(g && !std::strcmp(g, "0"))) exec_staged_graph(out, s);
+      else exec_staged(out, out_dev, s);
+      break;
+    }
     case DFG_HYBRID: exec_hybrid(out, out_dev, s); break;
     case DFG_ROUNDTRIP: exec_roundtrip(out, out_dev, s); break;
   }

@@ -166,6 +166,15 @@ struct PlanImpl {
   // with the interior planes
   cudaStream_t sHalo = nullptr;
   cudaEvent_t evHaloIn = nullptr, evHaloOut = nullptr;
+  // staged strategy, everything device-resident: the execute's launches,
+  // stream-ordered allocations and frees captured once into a CUDA graph and
+  // replayed while the output and input pointers stay the same (DFG_GRAPH=0:
+  // off).  gdelta = the counters one execute adds.
+  cudaGraphExec_t gexec = nullptr;
+  std::vector<const void*> gkey;
+  cudaStream_t sCap = nullptr;
+  dfg_stats gdelta{};
+  int64_t graph_launches = 0;   // executes served by a replay
   ~PlanImpl();
   void execute(void* out, bool out_dev, cudaStream_t s);
 
@@ -181,6 +190,7 @@ struct PlanImpl {
   void release_stream_buffers();
   void exec_fused(void* out, bool out_dev, cudaStream_t s);
   void exec_staged(void* out, bool out_dev, cudaStream_t s);
+  void exec_staged_graph(void* out, cudaStream_t s);
   void exec_hybrid(void* out, bool out_dev, cudaStream_t s);
   void exec_roundtrip(void* out, bool out_dev, cudaStream_t s);
   void halo_exchange(const std::vector<int>& inputs, cudaStream_t s);
