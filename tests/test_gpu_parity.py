@@ -798,3 +798,42 @@ def test_staged_graph_replay(T, monkeypatch):
     plan.execute(out3)
     torch.cuda.synchronize()
     assert torch.equal(out2, out3)
+
+
+@pytest.mark.parametrize("seed", range(4))
+def test_differential_fuzz_fused(seed, monkeypatch):
+    """Random well-formed programs (the parser fuzz generator of
+    test_lib_host: arithmetic, sqrt, unary minus, grad3d / decompose, norm,
+    compose, if / comparisons, constants incl. 1e39 and 0) through the
+    generated fused kernel -- value numbering, scale folding and the
+    verified two-operation quotient included -- on TMA-aligned and ragged
+    (cp.async ring) meshes in fp32 and fp64: the oracle's bits wherever no
+    intermediate leaves the normal range, and always with
+    DFG_FUSED_VARIANT=ieee."""
+    import random
+    from test_lib_host import _rand_program
+    from oracle.lang import DfgError as OracleError
+    rng = random.Random(1000 + seed)
+    n_run = 0
+    for it in range(24):
+        src = _rand_program(rng)
+        T = np.float32 if it % 2 == 0 else np.float64
+        shape = (24, 13, 9) if it % 4 < 2 else (23, 13, 9)
+        x, y, z, f = _inputs(shape, T)
+        try:
+            want = run_oracle(src, f, x, y, z)
+        except OracleError:
+            continue
+        with np.errstate(all="ignore"):
+            tiny = np.finfo(T).tiny
+            fin = want[np.isfinite(want)]
+            normal = bool(np.all(np.isfinite(want)) and np.all((fin == 0) | (np.abs(fin) >= tiny)))
+        monkeypatch.setenv("DFG_FUSED_VARIANT", "ieee")
+        got = run_lib(src, f, x, y, z, "fused")
+        assert_parity(got, want), ("ieee", src)
+        monkeypatch.delenv("DFG_FUSED_VARIANT")
+        if normal:
+            got = run_lib(src, f, x, y, z, "fused")
+            assert_parity(got, want), ("exact", src)
+        n_run += 1
+    assert n_run >= 12
