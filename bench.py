@@ -683,10 +683,13 @@ def complexity_sweep(dfg, synth, torch):
 
 
 def strategy_sweep(dfg, synth, torch):
-    """Config 2 (192^3: fused vs staged vs roundtrip, VelMag / VortMag / Q) and
-    config 3 (512^3 Q: staged under device-memory caps vs fused)."""
+    """Config 1 (32^3 VortMag, the three strategies: launch-bound), config 2
+    (192^3: fused vs staged vs roundtrip, VelMag / VortMag / Q) and config 3
+    (512^3 Q: staged under device-memory caps vs fused)."""
     from oracle.lang import PAPER_PROGRAMS
-    out = {"config2_192": {}}
+    out = {"config1_32_vortmag": _strategies_at(dfg, synth, torch, 32, PAPER_PROGRAMS["vortmag"][0],
+                                                ("fused", "staged", "roundtrip"), 7),
+           "config2_192": {}}
     for name in ("velmag", "vortmag", "qcrit"):
         out["config2_192"][name] = _strategies_at(dfg, synth, torch, 192, PAPER_PROGRAMS[name][0],
                                                   ("fused", "staged", "roundtrip"), 7)
