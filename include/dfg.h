@@ -39,7 +39,11 @@ typedef struct dfg_plan_s* dfg_plan;
 /* Execution strategies, L88-L105. */
 typedef enum {
   DFG_ROUNDTRIP = 0, /* one kernel per primitive, every result to the host (L92) */
-  DFG_STAGED = 1,    /* one kernel per primitive, intermediates on the device (L96) */
+  DFG_STAGED = 1,    /* one kernel per primitive, intermediates on the device (L96); with the
+                        inputs and the output on the device the first execute for a binding
+                        is captured into a CUDA graph (kernels + stream-ordered allocations
+                        and frees) that later executes replay while the output and input
+                        pointers stay the same (environment DFG_GRAPH=0: plain launches) */
   DFG_FUSED = 2,     /* one generated kernel, intermediates in registers (L97) */
   DFG_STREAMED = 3,  /* fusion over z-chunks streamed through a 3-slot device ring with
                         overlapped upload / kernel / download (the paper's future-work
