@@ -504,7 +504,7 @@ def main():
     strategies = variants = sweep = blocks = None
     if rank == 0 and world == 1 and not args.no_strategies:
         variants = variant_leg(dfg, mesh, out, QCRIT, torch, n)
-        strategies = strategy_sweep(dfg, synth, torch)
+        strategies = strategy_sweep(dfg, synth, torch, (e2e or {}).get("pcie_bound"))
         sweep = complexity_sweep(dfg, synth, torch)
         blocks = blocks_leg(torch)
 
@@ -682,17 +682,17 @@ def complexity_sweep(dfg, synth, torch):
     return res
 
 
-def strategy_sweep(dfg, synth, torch):
+def strategy_sweep(dfg, synth, torch, pcie=None):
     """Config 1 (32^3 VortMag, the three strategies: launch-bound), config 2
     (192^3: fused vs staged vs roundtrip, VelMag / VortMag / Q) and config 3
     (512^3 Q: staged under device-memory caps vs fused)."""
     from oracle.lang import PAPER_PROGRAMS
     out = {"config1_32_vortmag": _strategies_at(dfg, synth, torch, 32, PAPER_PROGRAMS["vortmag"][0],
-                                                ("fused", "staged", "roundtrip"), 7),
+                                                ("fused", "staged", "roundtrip"), 7, pcie),
            "config2_192": {}}
     for name in ("velmag", "vortmag", "qcrit"):
         out["config2_192"][name] = _strategies_at(dfg, synth, torch, 192, PAPER_PROGRAMS[name][0],
-                                                  ("fused", "staged", "roundtrip"), 7)
+                                                  ("fused", "staged", "roundtrip"), 7, pcie)
     GiB = 1 << 30
     c3 = _strategies_at(dfg, synth, torch, 512, PAPER_PROGRAMS["qcrit"][0], ("fused", "staged"), 3)
     # staged under device-memory caps: the paper's list order fails below its
@@ -745,7 +745,7 @@ def strategy_sweep(dfg, synth, torch):
     return out
 
 
-def _strategies_at(dfg, synth, torch, n, src, strategies, runs):
+def _strategies_at(dfg, synth, torch, n, src, strategies, runs, pcie=None):
     x, y, z = synth.rt_coords(n, n, n, np.float32)
     x64, y64, z64 = (a.astype(np.float64) for a in (x, y, z))
     mesh = dfg.Mesh(x, y, z)
@@ -783,6 +783,11 @@ def _strategies_at(dfg, synth, torch, n, src, strategies, runs):
                   "device_gb_per_s": st["predicted_hbm_bytes"] / (ms * 1e-3) / 1e9,
                   "predicted_device_bytes": st["predicted_hbm_bytes"],
                   "pcie_bytes": (st["h2d_bytes"] + st["d2h_bytes"]) // ex,
+                  **({"pcie_bound_ms": 1e3 * (st["h2d_bytes"] / ex / (pcie["h2d_gb_per_s"] * 1e9)
+                                              + st["d2h_bytes"] / ex / (pcie["d2h_gb_per_s"] * 1e9)),
+                      "pcie_bound_how": "h2d bytes / pinned h2d rate + d2h bytes / pinned d2h rate (the "
+                                        "roundtrip's transfers are serial: every filter waits for its result)"}
+                     if pcie and st["h2d_bytes"] + st["d2h_bytes"] > 0 else {}),
                   "kernels_per_execute": st["kernel_count"] // ex,
                   "highwater_bytes": st["dev_highwater_bytes"]}
         if ref is None:
