@@ -6,6 +6,7 @@
 #include <nccl.h>
 
 #include <algorithm>
+#include <cstdlib>
 #include <map>
 #include <mutex>
 #include <string>
@@ -91,8 +92,12 @@ HostPool& host_pool();
 // order does not matter (each index is written once from its own inputs).
 template <class F>
 void parallel_for(int64_t n, F f) {
+  static const int64_t cap = [] {
+    const char* e = std::getenv("DFG_HOST_THREADS");
+    return e ? std::max<int64_t>(1, std::atoll(e)) : int64_t(32);
+  }();
   const int64_t hw = int64_t(std::max(1u, std::thread::hardware_concurrency()));
-  const int64_t T = std::max<int64_t>(1, std::min<int64_t>({hw, 32, n / (1 << 16)}));
+  const int64_t T = std::max<int64_t>(1, std::min<int64_t>({hw, cap, n / (1 << 16)}));
   if (T == 1) {
     f(int64_t(0), n);
     return;
