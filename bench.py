@@ -263,13 +263,15 @@ def main():
     args = ap.parse_args()
     if args.impl == "reference":
         return run_reference(args)
+    global ORACLE_CHECKS
+    ORACLE_CHECKS = not args.no_cpu_baseline
 
     import torch
     import torch.distributed as dist
 
     import paper_conf_sc_harrisonnmjc12_b200 as dfg
     import synth
-    from oracle.lang import QCRIT  # the program text only (a string constant)
+    QCRIT = dfg.paper_program("qcrit")  # the paper's program text, from the library
 
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
@@ -629,12 +631,17 @@ def blocks_leg(torch):
     return res
 
 
+ORACLE_CHECKS = True   # bench.py --no-cpu-baseline: no oracle use at all
+
+
 def _window_parity(src, names, dt, fields, out, x, y, z, n):
     """Sampled full-size parity of a sweep case: the oracle on three windows
     of the GPU's own inputs (the low corner with the global one-sided
     boundaries, an interior block, the high corner), full rows in x, compared
     bit for bit with the fused kernel's output over the window cells whose
     stencil lies inside the window (oracle.evaluate's valid mask)."""
+    if not ORACLE_CHECKS:
+        return None
     from oracle import evaluate as oev
     from oracle.lang import build_dag
     dag = build_dag(src, tuple(names), dt)
@@ -653,7 +660,7 @@ def _window_parity(src, names, dt, fields, out, x, y, z, n):
 def complexity_sweep(dfg, synth, torch):
     """Config 5: the expression-complexity sweep (intro -> VelMag -> VortMag
     -> Q) at 768^3, fp32 and fp64, fused strategy, device-resident inputs."""
-    from oracle.lang import PAPER_PROGRAMS
+    PAPER_PROGRAMS = {k: (dfg.paper_program(k), dfg.PAPER_INPUTS[k]) for k in dfg.PAPER_INPUTS}
     n = 768
     res = {}
     for dt, tt, npt in (("f32", torch.float32, np.float32), ("f64", torch.float64, np.float64)):
@@ -686,7 +693,7 @@ def strategy_sweep(dfg, synth, torch, pcie=None):
     """Config 1 (32^3 VortMag, the three strategies: launch-bound), config 2
     (192^3: fused vs staged vs roundtrip, VelMag / VortMag / Q) and config 3
     (512^3 Q: staged under device-memory caps vs fused)."""
-    from oracle.lang import PAPER_PROGRAMS
+    PAPER_PROGRAMS = {k: (dfg.paper_program(k), dfg.PAPER_INPUTS[k]) for k in dfg.PAPER_INPUTS}
     out = {"config1_32_vortmag": _strategies_at(dfg, synth, torch, 32, PAPER_PROGRAMS["vortmag"][0],
                                                 ("fused", "staged", "roundtrip"), 7, pcie),
            "config2_192": {}}

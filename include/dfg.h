@@ -395,6 +395,13 @@ int dfg_fused_source(const char* expr, const char* const* inputs, int n_inputs,
                      int compile, char* buf, size_t cap, size_t* needed,
                      int* regs, int* spill);
 
+/* The paper's programs as text, for callers: "velmag", "vortmag", "qcrit"
+ * (Fig. 3; Q completed per DESIGN.md readings G1-G3; inputs u,
+ * v, w) and "intro" (L19; inputs b, c).  Buffer protocol as dfg_dump_dag:
+ * *needed = bytes incl. the terminating NUL; DFG_E_RANGE if cap is too
+ * small; DFG_E_INVALID for an unknown name.  Host only. */
+int dfg_paper_program(const char* which, char* buf, size_t cap, size_t* needed);
+
 /* Two-operation quotient check, exposed for tests (DESIGN.md section 5,
  * csrc/div2.hpp).  A fused kernel forms a grad3d derivative num / d (L99,
  * reading R1) as RN(num*r + RN(num*yl)) with r = RN(1/d), yl = RN(1/d - r)

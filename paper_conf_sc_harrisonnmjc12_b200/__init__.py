@@ -156,3 +156,13 @@ def execute_blocks(plans, outs, stream=None):
     s = stream if (stream is None or isinstance(stream, int)) else stream.cuda_stream
     dfg_execute_blocks([p.handle for p in plans], outs, s)
     return outs
+
+
+PAPER_INPUTS = {"velmag": ("u", "v", "w"), "vortmag": ("u", "v", "w"), "qcrit": ("u", "v", "w"), "intro": ("b", "c")}
+
+
+def paper_program(which: str) -> str:
+    """The paper's program text (dfg_paper_program): velmag, vortmag, qcrit
+    (Fig. 3, inputs u, v, w) or intro (L19, inputs b, c)."""
+    from ._dfg import dfg_paper_program
+    return dfg_paper_program(which)

@@ -87,6 +87,7 @@ _SIGS = {
     "dfg_model": (C.c_int, [C.c_char_p, C.POINTER(C.c_char_p), C.c_int, C.c_int, C.c_int, C.POINTER(_I64)]),
     "dfg_points3d_to_axes": (C.c_int, [C.c_int, _I64, _I64, _I64, _P, _P, _P, _P, _P, _P]),
     "dfg_div2_check": (C.c_int, [C.c_int, _P, _I64, C.c_int, _P, _P]),
+    "dfg_paper_program": (C.c_int, [C.c_char_p, C.c_char_p, C.c_size_t, C.POINTER(C.c_size_t)]),
     "dfg_fused_source": (C.c_int, [C.c_char_p, C.POINTER(C.c_char_p), C.c_int, C.c_int, _I64, _I64, _I64, C.c_int,
                                    C.c_char_p, C.c_size_t, C.POINTER(C.c_size_t), C.POINTER(C.c_int),
                                    C.POINTER(C.c_int)]),
@@ -320,6 +321,17 @@ def dfg_points3d_to_axes(x3, y3, z3):
     _check(_lib.dfg_points3d_to_axes(dt, px - 1, py - 1, pz - 1, _ptr(x3), _ptr(y3), _ptr(z3),
                                      _ptr(x), _ptr(y), _ptr(z)))
     return x, y, z
+
+
+def dfg_paper_program(which):
+    """The paper's program text: "velmag", "vortmag", "qcrit" (inputs u, v, w), "intro" (b, c)."""
+    need = C.c_size_t(0)
+    st = _lib.dfg_paper_program(which.encode(), None, 0, C.byref(need))
+    if st not in (0, -11):
+        _check(st)
+    buf = C.create_string_buffer(need.value)
+    _check(_lib.dfg_paper_program(which.encode(), buf, need.value, C.byref(need)))
+    return buf.value.decode()
 
 
 def dfg_div2_check(d, method=0):

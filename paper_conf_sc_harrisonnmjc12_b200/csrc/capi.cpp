@@ -361,6 +361,16 @@ int dfg_points3d_to_axes(dfg_dtype dtype, int64_t nx, int64_t ny, int64_t nz, co
   });
 }
 
+int dfg_paper_program(const char* which, char* buf, size_t cap, size_t* needed) {
+  return guard([&] {
+    if (!which) dfg::fail(DFG_E_INVALID, "null name");
+    int id = 0;
+    const char* prog = dfg::reference_program(which, &id);
+    if (!prog) dfg::fail(DFG_E_INVALID, "paper programs: \"velmag\", \"vortmag\", \"qcrit\", \"intro\"");
+    copy_out(prog, buf, cap, needed);
+  });
+}
+
 int dfg_div2_check(dfg_dtype dtype, const void* d, int64_t n, int method, uint8_t* ok, int64_t* tested) {
   return guard([&] {
     if (!d || !ok || n < 0) dfg::fail(DFG_E_INVALID, "null pointer or negative count");
@@ -402,7 +412,7 @@ int dfg_model(const char* expr, const char* const* inputs, int n_inputs, dfg_str
     if (strategy < DFG_ROUNDTRIP || strategy > DFG_HYBRID) dfg::fail(DFG_E_INVALID, "bad strategy");
     int ref = 0;
     const char* prog = strategy == DFG_REFERENCE ? dfg::reference_program(expr, &ref) : expr;
-    if (!prog) dfg::fail(DFG_E_INVALID, "reference kernels exist for velmag, vortmag and qcrit");
+    if (strategy == DFG_REFERENCE && ref == 0) dfg::fail(DFG_E_INVALID, "reference kernels exist for velmag, vortmag and qcrit");
     dfg::Dag d = dfg::build_dag(prog, names_of(inputs, n_inputs), dfg::DType::F32);
     dfg::Model m = dfg::model(d, strategy, host_mode != 0);
     out[0] = m.h2d;

@@ -82,7 +82,7 @@ std::unique_ptr<PlanImpl> compile_plan(std::shared_ptr<MeshImpl> mesh, const std
   int ref = 0;
   if (s == DFG_REFERENCE) {
     const char* prog = reference_program(expr, &ref);
-    if (!prog) fail(DFG_E_INVALID, "reference kernels exist for \"velmag\", \"vortmag\" and \"qcrit\"");
+    if (!prog || ref == 0) fail(DFG_E_INVALID, "reference kernels exist for \"velmag\", \"vortmag\" and \"qcrit\"");
     plan->dag = build_dag(prog, names, mesh->dt);
   } else {
     plan->dag = build_dag(expr, names, mesh->dt);

@@ -389,3 +389,15 @@ def test_div2_certificate_fp64_axes(dfg):
         dfg_div2_check(d[:3], 1)          # exhaustive is fp32 only
     with pytest.raises(Exception):
         dfg_div2_check(np.array([0.0, 1.0]), 0)
+
+
+def test_paper_program_texts(dfg):
+    """dfg_paper_program: the library's copies of the paper's programs build the
+    same networks as the oracle's (Fig. 3 and L19); unknown names are errors."""
+    for name, (src, inputs) in PAPER_PROGRAMS.items():
+        text = dfg.paper_program(name)
+        assert tuple(dfg.PAPER_INPUTS[name]) == tuple(inputs)
+        for dt in ("f32", "f64"):
+            assert _lib_dump(dfg, text, inputs, dt) == _oracle_dump(src, inputs, dt)
+    with pytest.raises(Exception):
+        dfg.paper_program("lambda2")

@@ -19,7 +19,7 @@ sys.path.insert(0, ROOT)
 
 import paper_conf_sc_harrisonnmjc12_b200 as dfg  # noqa: E402
 import synth  # noqa: E402
-from oracle.lang import QCRIT  # noqa: E402
+QCRIT = dfg.paper_program("qcrit")
 
 
 def timeit(fn, iters=20):
