@@ -5,7 +5,7 @@ sys.path.insert(0, os.path.join(os.path.dirname(__file__), "..", "tests"))
 import numpy as np, torch
 import paper_conf_sc_harrisonnmjc12_b200 as dfg
 import synth
-from oracle.lang import PAPER_PROGRAMS
+PAPER_PROGRAMS = {k: (dfg.paper_program(k), dfg.PAPER_INPUTS[k]) for k in dfg.PAPER_INPUTS}
 from dfg_testutil import run_lib
 
 shape = (62, 30, 20); split = tuple(int(c) for c in os.environ.get("SPLIT", "222"))

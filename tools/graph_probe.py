@@ -6,7 +6,7 @@ sys.path.insert(0, os.path.join(os.path.dirname(__file__), ".."))
 import numpy as np, torch
 import paper_conf_sc_harrisonnmjc12_b200 as dfg
 import synth
-from oracle.lang import PAPER_PROGRAMS
+PAPER_PROGRAMS = {k: (dfg.paper_program(k), dfg.PAPER_INPUTS[k]) for k in dfg.PAPER_INPUTS}
 
 for n in (32, 192):
     x, y, z = synth.rt_coords(n, n, n, np.float32)

@@ -35,7 +35,7 @@ def worker(rank, world, args, port):
 
     import paper_conf_sc_harrisonnmjc12_b200 as dfg
     import synth
-    from oracle.lang import PAPER_PROGRAMS
+    PAPER_PROGRAMS = {k: (dfg.paper_program(k), dfg.PAPER_INPUTS[k]) for k in dfg.PAPER_INPUTS}
 
     torch.cuda.set_device(0)
     dist.init_process_group("gloo", rank=rank, world_size=world)

@@ -7,7 +7,7 @@ import numpy as np, torch
 import paper_conf_sc_harrisonnmjc12_b200 as dfg
 import synth
 from bench import ClockSampler
-from oracle.lang import PAPER_PROGRAMS
+PAPER_PROGRAMS = {k: (dfg.paper_program(k), dfg.PAPER_INPUTS[k]) for k in dfg.PAPER_INPUTS}
 
 n = int(os.environ.get("N", "1024"))
 x, y, z = synth.rt_coords(n, n, n, np.float32)

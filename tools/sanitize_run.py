@@ -13,7 +13,7 @@ sys.path.insert(0, ROOT)
 
 import paper_conf_sc_harrisonnmjc12_b200 as dfg  # noqa: E402
 import synth  # noqa: E402
-from oracle.lang import PAPER_PROGRAMS  # noqa: E402
+PAPER_PROGRAMS = {k: (dfg.paper_program(k), dfg.PAPER_INPUTS[k]) for k in dfg.PAPER_INPUTS}
 
 
 def main():

@@ -22,7 +22,7 @@ sys.path.insert(0, ROOT)
 
 import paper_conf_sc_harrisonnmjc12_b200 as dfg  # noqa: E402
 import synth  # noqa: E402
-from oracle.lang import PAPER_PROGRAMS  # noqa: E402  (program text only)
+PAPER_PROGRAMS = {k: (dfg.paper_program(k), dfg.PAPER_INPUTS[k]) for k in dfg.PAPER_INPUTS}
 
 KNOBS = ("DFG_FUSED_VARIANT", "DFG_NCW", "DFG_STAGES", "DFG_KZ", "DFG_FUSED_KERNEL", "DFG_CTAS", "DFG_ROWS_PER_WARP")
 

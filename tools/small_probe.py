@@ -7,7 +7,7 @@ import torch
 import paper_conf_sc_harrisonnmjc12_b200 as dfg
 import synth
 from bench import _strategies_at
-from oracle.lang import PAPER_PROGRAMS
+PAPER_PROGRAMS = {k: (dfg.paper_program(k), dfg.PAPER_INPUTS[k]) for k in dfg.PAPER_INPUTS}
 
 for n in [int(a) for a in (sys.argv[1:] or ["192", "256"])]:
     for prog in ("vortmag", "qcrit"):

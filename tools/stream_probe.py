@@ -5,7 +5,7 @@ sys.path.insert(0, os.path.join(os.path.dirname(__file__), ".."))
 import numpy as np, torch
 import paper_conf_sc_harrisonnmjc12_b200 as dfg
 import synth
-from oracle.lang import QCRIT
+QCRIT = dfg.paper_program("qcrit")
 
 n = 1024
 x, y, z = synth.rt_coords(n, n, n, np.float32)
