@@ -401,3 +401,27 @@ def test_paper_program_texts(dfg):
             assert _lib_dump(dfg, text, inputs, dt) == _oracle_dump(src, inputs, dt)
     with pytest.raises(Exception):
         dfg.paper_program("lambda2")
+
+
+def test_oracle_only_in_checks():
+    """The oracle is test infrastructure: the package never imports it, and
+    bench.py imports it only inside its CPU-baseline / reference-arm and
+    parity-check functions (the product legs take program texts from the
+    library, dfg_paper_program)."""
+    import ast
+    pkg = os.path.join(ROOT, "paper_conf_sc_harrisonnmjc12_b200")
+    for name in os.listdir(pkg):
+        if name.endswith(".py"):
+            assert "oracle" not in open(os.path.join(pkg, name)).read().replace("no CPU", ""), name
+    tree = ast.parse(open(os.path.join(ROOT, "bench.py")).read())
+    allowed = {"_oracle_time", "_window_parity"}
+    for fn in ast.walk(tree):
+        if isinstance(fn, ast.FunctionDef):
+            for node in ast.walk(fn):
+                if isinstance(node, (ast.Import, ast.ImportFrom)):
+                    mods = [a.name for a in node.names] if isinstance(node, ast.Import) else [node.module or ""]
+                    if any(m.split(".")[0] == "oracle" for m in mods):
+                        assert fn.name in allowed, fn.name
+    top = [n for n in tree.body if isinstance(n, (ast.Import, ast.ImportFrom))]
+    assert not any((getattr(n, "module", None) or "").startswith("oracle") or
+                   any(a.name.startswith("oracle") for a in n.names) for n in top)
