@@ -244,6 +244,74 @@ def run_reference(args):
     return 0
 
 
+def slab_boundary_parity(dist, torch, rank, world, fields, out, x, y, z, n, nzl, g, target_s=10.0):
+    """N > 1: the oracle against the GPU on rank 0's slab where the halo
+    matters -- a block of full rows ending at the slab's LAST owned plane,
+    whose z+1 neighbours live on rank 1 (ghost data lets the
+    gradient compute the proper values on the boundaries).  Rank 1 sends its
+    first owned plane of u, v, w (the window's rows) to rank 0; rank 0 runs
+    the unchanged oracle on its own planes + that plane and compares the
+    last planes of its output bit for bit.  Every other rank only joins the
+    exchange.  Returns the rank-0 cpu_baseline line (or None elsewhere)."""
+    j0 = min(200, n // 4)
+    rows = min(512, n - j0 - 1)
+    win_rows = slice(j0 - 1, j0 + rows + 1)
+    if rank == 1:
+        t = torch.stack([fields[c][g, win_rows, :] for c in "uvw"]).contiguous()
+        dist.send(t, dst=0)
+        return None
+    if rank != 0:
+        return None
+    recv = torch.empty((3, rows + 2, n), dtype=torch.float32, device="cuda")
+    dist.recv(recv, src=1)
+    from oracle import evaluate as oev
+    from oracle.lang import QCRIT, build_dag
+    dag = build_dag(QCRIT, ("u", "v", "w"), "f32")
+
+    def sample(planes):
+        k0 = nzl - planes                            # global = local on rank 0 (z_offset 0)
+        f = {}
+        for i, c in enumerate("uvw"):
+            own = fields[c][g + k0 - 1:g + nzl, win_rows, :].cpu().numpy()
+            f[c] = np.concatenate([own, recv[i:i + 1].cpu().numpy()], axis=0)
+        t0 = time.perf_counter()
+        res, valid = oev.evaluate(dag, f, oev.MeshWindow(x, y, z, i0=0, j0=j0 - 1, k0=k0 - 1))
+        return k0, res[1:-1, 1:-1, :], int(valid[1:-1, 1:-1, :].sum()), time.perf_counter() - t0
+
+    _, _, _, dt = sample(2)                          # calibration
+    planes = int(max(2, min(64, nzl - 1, round(2 * target_s / max(dt, 1e-3)))))
+    k0, res, cells, dt = sample(planes)
+    got = out[k0:nzl, j0:j0 + rows, :].cpu().numpy()
+    bad = int(np.count_nonzero(got.view(np.uint32) != res.view(np.uint32)))
+    return {"value": cells / dt, "unit": "cells/s", "cores": 1, "kind": "oracle",
+            "sample": f"Q-criterion on a {n} x {rows} x {planes} block of rank 0's slab ending at its last owned "
+                      f"plane (z+1 neighbours from rank 1), numpy oracle, {dt:.1f} s",
+            "slab_boundary_parity": {"cells_compared": int(res.size), "mismatches": bad,
+                                     "block": f"planes {k0}..{nzl - 1} (slab boundary at {nzl - 1}|{nzl}), "
+                                              f"rows {j0}..{j0 + rows - 1}"}}
+
+
+def _self_launch(args):
+    """--gpus N > 1 outside torchrun: run this script under
+    torch.distributed.run with N ranks (one per GPU, rendezvous on
+    127.0.0.1), the launch the driver uses; fail loudly when the node has
+    fewer GPUs (DFG_BENCH_ONE_GPU=1: every rank on cuda:0, functional test)."""
+    import socket
+
+    import torch
+    have = torch.cuda.device_count()
+    if os.environ.get("DFG_BENCH_ONE_GPU") != "1" and have < args.gpus:
+        sys.stderr.write(f"bench.py: --gpus {args.gpus} needs {args.gpus} CUDA devices, this node has {have} "
+                         "(DFG_BENCH_ONE_GPU=1 runs every rank on cuda:0 as a functional test)\n")
+        return 2
+    with socket.socket() as sk:
+        sk.bind(("127.0.0.1", 0))
+        port = sk.getsockname()[1]
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", f"--nproc-per-node={args.gpus}",
+           "--master-addr", "127.0.0.1", "--master-port", str(port), os.path.abspath(__file__)] + sys.argv[1:]
+    return subprocess.call(cmd)
+
+
 # ---------------------------------------------------------------- our arm
 def main():
     ap = argparse.ArgumentParser()
@@ -255,14 +323,20 @@ def main():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-strategies", action="store_true")
     ap.add_argument("--no-cpu-mt", action="store_true", help="skip the multi-process oracle timing")
-    ap.add_argument("--halo", default="peer", choices=["peer", "nccl"],
-                    help="N > 1 z-slab halo: peer memory read in place by the kernel (default) or NCCL send/recv")
+    ap.add_argument("--halo", default="auto", choices=["auto", "peer", "nccl"],
+                    help="N > 1 z-slab halo: peer memory read in place by the kernel, NCCL send/recv, or auto "
+                         "(default): peer when every rank's isolated probe of the in-place TMA read passes, else NCCL")
     ap.add_argument("--scaling", default="weak", choices=["weak", "strong"],
                     help="weak: size^3 cells per GPU (mesh size x size x size*N); strong: one size^3 mesh "
                          "split into N z-slabs (config 4 of BASELINE.json runs both)")
     args = ap.parse_args()
     if args.impl == "reference":
         return run_reference(args)
+    if "WORLD_SIZE" not in os.environ and args.gpus > 1:
+        return _self_launch(args)
+    if int(os.environ.get("WORLD_SIZE", "1")) != args.gpus:
+        sys.stderr.write(f"bench.py: WORLD_SIZE={os.environ.get('WORLD_SIZE')} but --gpus {args.gpus}\n")
+        return 2
     global ORACLE_CHECKS
     ORACLE_CHECKS = not args.no_cpu_baseline
 
@@ -287,7 +361,6 @@ def main():
     torch.cuda.set_device(local)
     if world > 1:
         dist.init_process_group("nccl", device_id=torch.device("cuda", local))
-    assert world == args.gpus or world == 1, "launch with torchrun --nproc-per-node N for --gpus N"
     n = args.size
     NZ = n * world if args.scaling == "weak" else n
     K, W = args.steps, args.warmup
@@ -308,27 +381,38 @@ def main():
     for c, b in fields.items():
         mesh.bind(c, b)
     halo = None
+    probe = None
     if world > 1:
         halo = "nccl"
-        if args.halo == "peer":
+        if args.halo in ("peer", "auto"):
             # the kernel reads the neighbours' boundary planes in place (CUDA IPC
-            # mappings over NVLink); every rank must link or none does
+            # mappings over NVLink); every rank must link or none does.  auto:
+            # first an isolated probe (a child process per rank TMA-reads the
+            # neighbours' probe blocks through the mappings), so a transport
+            # that faults or misreads costs a fallback to NCCL, not the run
             blobs, ok = [None] * world, [None] * world
             try:
                 blob = mesh.peer_export()
             except dfg.DfgError:
                 blob = None
             dist.all_gather_object(blobs, blob)
+            lo_b = blobs[rank - 1] if rank > 0 else None
+            hi_b = blobs[rank + 1] if rank < world - 1 else None
             linked = False
             if all(b is not None for b in blobs):
-                try:
-                    mesh.link_peers(blobs[rank - 1] if rank > 0 else None,
-                                    blobs[rank + 1] if rank < world - 1 else None)
-                    linked = True
-                except dfg.DfgError:
-                    pass
-            dist.all_gather_object(ok, linked)
-            if all(ok):
+                good, detail = True, "forced (--halo peer)"
+                if args.halo == "auto":
+                    good, detail = dfg.probe_peer_transport([lo_b, hi_b], local)
+                probe = {"rank": rank, "ok": good, "detail": detail}
+                if good:
+                    try:
+                        mesh.link_peers(lo_b, hi_b)
+                        linked = True
+                    except dfg.DfgError as e:
+                        probe["detail"] = f"link refused: {e}"
+            dist.all_gather_object(ok, (linked, probe))
+            probe = [p for _, p in ok]
+            if all(lk for lk, _ in ok):
                 halo = "peer"
             elif linked:
                 mesh.link_peers(None, None)
@@ -367,6 +451,7 @@ def main():
     # plus the one or two boundary-plane launches that follow the halo exchange
     launches_per_step = st["kernel_count"] / max(1, K)
     kern_ms = st["kernel_ms_sum"] / max(1, st["kernel_launches_timed"]) * launches_per_step
+    kern_ms_rank, ms_rank = kern_ms, ms
     t = torch.tensor([ms, kern_ms], device="cuda", dtype=torch.float64)
     if world > 1:
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
@@ -487,7 +572,9 @@ def main():
     multi = None
     if world > 1:
         # per-rank halo bytes, kernel time and step time; max over ranks
-        per = torch.tensor([st["halo_bytes"] / max(1, K), kern_ms, ms_step, launches_per_step],
+        hm = mesh.halo_map()
+        per = torch.tensor([st["halo_bytes"] / max(1, K), kern_ms_rank, ms_rank / K, launches_per_step, dist.get_world_size(), dist.get_rank(),
+                            (ALGO_BYTES_PER_CELL * cells_rank / (kern_ms_rank * 1e-3) / 1e9), hm[1]],
                            dtype=torch.float64, device="cuda")
         allr = [torch.zeros_like(per) for _ in range(world)]
         dist.all_gather(allr, per)
@@ -496,7 +583,16 @@ def main():
                  "kernel_ms_per_step": [r[1] for r in rows],
                  "step_ms": [r[2] for r in rows],
                  "launches_per_step": [r[3] for r in rows],
+                 "comm_rank_of_rank": [int(r[5]) for r in rows],
+                 "comm_ranks": [int(r[4]) for r in rows],
+                 "nccl_comm_ranks": [int(r[7]) for r in rows],
+                 "comm": "comm_ranks: torch process group size seen by each rank; nccl_comm_ranks: libdfg's own "
+                         "NCCL communicator (1 = none: the peer halo needs no communicator)",
+                 "world_size": world,
+                 "achieved_gb_per_s_per_rank": [r[6] for r in rows],
+                 "roofline_frac_per_rank": [r[6] / _peak()[0] for r in rows],
                  "halo_mode": halo,
+                 "halo_probe": probe,
                  "halo": ("peer memory: the boundary-plane launches read the neighbours' first/last owned "
                           "planes of u, v, w in place (CUDA IPC mappings, NVLink), after the interior planes; "
                           "step flags by stream write/wait-value" if halo == "peer" else
@@ -511,6 +607,9 @@ def main():
         blocks = blocks_leg(torch)
 
     cpu = None
+    if world > 1 and not args.no_cpu_baseline:
+        cpu = slab_boundary_parity(dist, torch, rank, world, fields, out, x, y, z, n, nzl, g)
+        barrier()
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
         same = n == N1 and world == 1
         cpu = cpu_baseline_leg(gpu_out=out if same else None, gpu_fields=fields if same else None)

@@ -223,6 +223,19 @@ int dfg_mesh_init_comm(dfg_mesh mesh, const void* id128, int rank, int nranks);
 int dfg_mesh_peer_export(dfg_mesh mesh, void* blob, size_t cap);
 int dfg_mesh_link_peers(dfg_mesh mesh, const void* lo_blob, const void* hi_blob);
 
+/* Probe of the in-place transport before a link:
+ * opens the flag allocation of the slab that exported `blob` (host pointer,
+ * DFG_PEER_BLOB_BYTES) through CUDA IPC on the CURRENT device, reads its
+ * 8 KiB probe block (a pattern the exporter wrote) with one TMA load through
+ * a tensor map over the mapping -- the access the boundary-plane launches
+ * make -- and sets *ok = 1 if every word matches, 0 otherwise; the mapping
+ * is closed again.  Run it in a separate short-lived process (bench.py does):
+ * the caller of dfg_mesh_link_peers must not be the process a faulting
+ * transport takes down.  The exporter must keep its mesh alive meanwhile.
+ * Errors: DFG_E_INVALID (null argument, not an export blob),
+ * DFG_E_UNSUPPORTED (IPC refused), DFG_E_CUDA. */
+int dfg_peer_probe(const void* blob, int* ok);
+
 /* Single-process halo transport: slabs that live in one process (one or
  * several devices) exchange ghost planes with device-to-device copies.
  * `lo` must hold the slab directly below `hi` (lo.k1 == hi.k0). */

@@ -9,6 +9,8 @@ memory and streams.
 
 from __future__ import annotations
 
+import sys
+
 from ._dfg import *  # noqa: F401,F403
 from ._dfg import (DFG_F32, DFG_F64, DfgError, EXPORTS, LIB_PATH, STRATEGIES,  # noqa: F401
                    dfg_bind_field, dfg_compile, dfg_create_mesh, dfg_destroy_mesh, dfg_destroy_plan,
@@ -25,6 +27,43 @@ def _dtype_code(dtype) -> int:
     raise ValueError(f"unsupported dtype {dtype}")
 
 
+def _current_device():
+    """The CUDA device current now (the one dfg_create_mesh takes), or None
+    when torch or CUDA is absent."""
+    torch = sys.modules.get("torch")
+    if torch is None or not torch.cuda.is_available():
+        return None
+    return torch.cuda.current_device()
+
+
+def _check_buffer(buf, dtype, numel, device, what):
+    """Validate a torch tensor / numpy array before its raw pointer crosses
+    the C ABI (which cannot see dtype, size, strides or device): contiguous,
+    the mesh's element type, exactly the layout's element count (dfg.h) and,
+    for a CUDA tensor, the mesh's device.  Plain integer pointers pass
+    unchecked.  Raises ValueError."""
+    import numpy as np
+    if isinstance(buf, int) or buf is None:
+        return
+    if hasattr(buf, "is_contiguous"):                       # torch.Tensor
+        if not buf.is_contiguous():
+            raise ValueError(f"{what}: tensor is not contiguous")
+        got = np.dtype(str(buf.dtype).replace("torch.", ""))
+        n = buf.numel()
+        if buf.is_cuda and device is not None and buf.device.index != device:
+            raise ValueError(f"{what}: tensor on cuda:{buf.device.index}, mesh on cuda:{device}")
+    elif isinstance(buf, np.ndarray):
+        if not buf.flags["C_CONTIGUOUS"]:
+            raise ValueError(f"{what}: array is not C-contiguous")
+        got, n = buf.dtype, buf.size
+    else:
+        return
+    if got != np.dtype(dtype):
+        raise ValueError(f"{what}: dtype {got}, mesh type {np.dtype(dtype)}")
+    if n != numel:
+        raise ValueError(f"{what}: {n} elements, the layout needs {numel}")
+
+
 class Mesh:
     """Owns a dfg_mesh.  x, y, z: point coordinates (numpy, T); for a z slab
     pass the GLOBAL z and (nz_global, z_offset, ghost)."""
@@ -38,6 +77,9 @@ class Mesh:
         self.nz = self.nz_global if nz_local is None else nz_local
         self.ghost = ghost
         self._coords = (x, y, z)
+        self.device = _current_device()
+        # bound field layout T[nz_local + 2 ghost][ny][nx] (dfg.h)
+        self.field_numel = (self.nz + 2 * ghost) * self.ny * self.nx
         self.handle = dfg_create_mesh(_dtype_code(x.dtype), self.nx, self.ny, self.nz, x, y, z,
                                       self.nz_global, z_offset, ghost)
         self._bound = {}
@@ -60,6 +102,9 @@ class Mesh:
         self._bound = {}
         self.x_offset = x_offset or ghost
         self.row_pitch = row_pitch or self.x_offset + nx + ghost
+        self.device = _current_device()
+        # T[nz + 2 ghost][ny + 2 ghost][row_pitch] (dfg_create_block)
+        self.field_numel = (nz + 2 * ghost) * (ny + 2 * ghost) * self.row_pitch
         self.handle = dfg_create_block(_dtype_code(x.dtype), nx, ny, nz, x, y, z, len(x) - 1, len(y) - 1,
                                        len(z) - 1, i0, j0, k0, ghost, row_pitch, x_offset)
         return self
@@ -67,6 +112,8 @@ class Mesh:
     def bind(self, name, buf, on_device=None):
         if on_device is None:
             on_device = bool(getattr(buf, "is_cuda", False))
+        if buf is not None:
+            _check_buffer(buf, self.dtype, self.field_numel, self.device, f"field '{name}'")
         self._bound[name] = buf          # keep the borrowed buffer alive
         dfg_bind_field(self.handle, name, buf, on_device)
 
@@ -105,6 +152,8 @@ class Plan:
     def execute(self, out, out_on_device=None, stream=None):
         if out_on_device is None:
             out_on_device = bool(getattr(out, "is_cuda", False))
+        m = self.mesh
+        _check_buffer(out, m.dtype, m.nz * m.ny * m.nx * self.info()["width"], m.device, "output")
         s = stream if (stream is None or isinstance(stream, int)) else stream.cuda_stream
         dfg_execute(self.handle, out, out_on_device, s)
         return out
@@ -156,6 +205,34 @@ def execute_blocks(plans, outs, stream=None):
     s = stream if (stream is None or isinstance(stream, int)) else stream.cuda_stream
     dfg_execute_blocks([p.handle for p in plans], outs, s)
     return outs
+
+
+def probe_peer_transport(blobs, device: int, timeout: float = 120.0):
+    """dfg_peer_probe on every neighbour blob, in a child process on CUDA
+    device ``device`` (dfg.h: a transport that faults must not take the
+    caller down).  Returns (ok, detail)."""
+    import os
+    import subprocess
+    blobs = [b for b in blobs if b is not None]
+    if not blobs:
+        return True, "no neighbours"
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    code = ("import sys; sys.path.insert(0, sys.argv[1]); import torch; torch.cuda.set_device(int(sys.argv[2]))\n"
+            "from paper_conf_sc_harrisonnmjc12_b200._dfg import dfg_peer_probe\n"
+            "oks = [dfg_peer_probe(bytes.fromhex(h)) for h in sys.stdin.read().split()]\n"
+            "print('probe', ' '.join(str(int(o)) for o in oks))\n")
+    try:
+        r = subprocess.run([sys.executable, "-c", code, root, str(device)], input=" ".join(b.hex() for b in blobs),
+                           capture_output=True, text=True, timeout=timeout)
+    except subprocess.TimeoutExpired:
+        return False, "probe process timed out"
+    lines = [ln for ln in r.stdout.splitlines() if ln.startswith("probe ")]
+    if r.returncode != 0 or not lines:
+        return False, f"probe process exit {r.returncode}: {(r.stderr or r.stdout).strip()[-300:]}"
+    oks = lines[-1].split()[1:]
+    if len(oks) != len(blobs) or any(o != "1" for o in oks):
+        return False, f"probe read a wrong pattern ({' '.join(oks)})"
+    return True, f"{len(blobs)} neighbour(s): TMA read through the IPC mapping returned the pattern"
 
 
 PAPER_INPUTS = {"velmag": ("u", "v", "w"), "vortmag": ("u", "v", "w"), "qcrit": ("u", "v", "w"), "intro": ("b", "c")}

@@ -66,6 +66,7 @@ _SIGS = {
     "dfg_mesh_link_local": (C.c_int, [_P, _P]),
     "dfg_mesh_peer_export": (C.c_int, [_P, _P, C.c_size_t]),
     "dfg_mesh_link_peers": (C.c_int, [_P, _P, _P]),
+    "dfg_peer_probe": (C.c_int, [_P, C.POINTER(C.c_int)]),
     "dfg_bind_field": (C.c_int, [_P, C.c_char_p, _P, C.c_int]),
     "dfg_compile": (C.c_int, [_P, C.c_char_p, C.c_int, C.c_size_t, C.POINTER(_P)]),
     "dfg_destroy_plan": (None, [_P]),
@@ -196,6 +197,12 @@ def dfg_mesh_link_peers(mesh, lo_blob, hi_blob):
         return None if b is None else C.create_string_buffer(bytes(b), PEER_BLOB_BYTES)
     lo, hi = arg(lo_blob), arg(hi_blob)
     _check(_lib.dfg_mesh_link_peers(mesh, lo, hi))
+
+
+def dfg_peer_probe(blob) -> bool:
+    ok = C.c_int(0)
+    _check(_lib.dfg_peer_probe(C.create_string_buffer(bytes(blob), PEER_BLOB_BYTES), C.byref(ok)))
+    return bool(ok.value)
 
 
 def dfg_mesh_link_local(lo, hi):

@@ -162,6 +162,14 @@ int dfg_mesh_link_peers(dfg_mesh mesh, const void* lo_blob, const void* hi_blob)
   });
 }
 
+int dfg_peer_probe(const void* blob, int* ok) {
+  return guard([&] {
+    if (!blob || !ok) dfg::fail(DFG_E_INVALID, "null argument");
+    *ok = 0;
+    *ok = dfg::peer_probe(blob) ? 1 : 0;
+  });
+}
+
 int dfg_mesh_link_local(dfg_mesh lo, dfg_mesh hi) {
   return guard([&] {
     if (!lo || !hi) dfg::fail(DFG_E_INVALID, "null mesh");

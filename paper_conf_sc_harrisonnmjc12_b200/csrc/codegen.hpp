@@ -50,6 +50,9 @@ const char* reference_program(const std::string& which, int* id);
 
 // Dynamic shared memory the TMA kernel needs for a config (bytes).
 size_t fused_tma_smem_bytes(DType dt, int nsf, int ncw, int stages, int rpw = 1);
+// the row-copy kernel's ring (fused_tma.cuh DFG_R*): rows per warp 1, smem
+// row pitch = halo'd tile row + 3 chunks
+size_t fused_rows_smem_bytes(DType dt, int nsf, int ncw, int stages);
 
 // TMA kernel tile: tile_w cells along x, tile_h rows along y (fused_tma.cuh).
 inline int tma_tile_w(DType dt, int rpw) { return 32 * (dt == DType::F32 ? 4 : 2) / rpw; }

@@ -401,6 +401,8 @@ void PlanImpl::exec_staged_graph(void* out, cudaStream_t s) {
     if (!sCap) DFG_CUDA(cudaStreamCreateWithFlags(&sCap, cudaStreamNonBlocking));
     pool_for(m.device);  // created outside the capture (pool creation is not capturable)
     const dfg_stats before = st;
+    // the captured execute's own ledger high-water (replays repeat it)
+    st.dev_highwater_bytes = 0;
     DFG_CUDA(cudaStreamBeginCapture(sCap, cudaStreamCaptureModeThreadLocal));
     cudaGraph_t g = nullptr;
     try {
@@ -409,8 +411,11 @@ void PlanImpl::exec_staged_graph(void* out, cudaStream_t s) {
       cudaStreamEndCapture(sCap, &g);  // leave the stream usable
       if (g) cudaGraphDestroy(g);
       cudaGetLastError();
+      st.dev_highwater_bytes = std::max(st.dev_highwater_bytes, before.dev_highwater_bytes);
       throw;
     }
+    const int64_t captured_high = st.dev_highwater_bytes;
+    st.dev_highwater_bytes = std::max(captured_high, before.dev_highwater_bytes);
     DFG_CUDA(cudaStreamEndCapture(sCap, &g));
     cudaError_t e = cudaGraphInstantiate(&gexec, g, 0);
     cudaGraphDestroy(g);
@@ -421,6 +426,7 @@ void PlanImpl::exec_staged_graph(void* out, cudaStream_t s) {
     gdelta.d2h_count = st.d2h_count - before.d2h_count;
     gdelta.h2d_bytes = st.h2d_bytes - before.h2d_bytes;
     gdelta.d2h_bytes = st.d2h_bytes - before.d2h_bytes;
+    gdelta.dev_highwater_bytes = captured_high;
     gkey = key;
   } else {
     st.kernel_count += gdelta.kernel_count;
@@ -428,6 +434,7 @@ void PlanImpl::exec_staged_graph(void* out, cudaStream_t s) {
     st.d2h_count += gdelta.d2h_count;
     st.h2d_bytes += gdelta.h2d_bytes;
     st.d2h_bytes += gdelta.d2h_bytes;
+    st.dev_highwater_bytes = std::max(st.dev_highwater_bytes, gdelta.dev_highwater_bytes);
     graph_launches += 1;
   }
   DFG_CUDA(cudaGraphLaunch(gexec, s));

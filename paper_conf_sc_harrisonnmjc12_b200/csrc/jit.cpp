@@ -149,6 +149,8 @@ LoadedModule load_module(const Cubin& c, bool has_stencil, bool has_tma) {
       DFG_CU(drv().ModuleGetFunction(&m.tma_multi, m.mod, "dfg_fused_tma_multi"));
       DFG_CU(drv().ModuleGetFunction(&m.tile, m.mod, "dfg_fused_tile"));
       DFG_CU(drv().ModuleGetFunction(&m.tile_multi, m.mod, "dfg_fused_tile_multi"));
+      DFG_CU(drv().ModuleGetFunction(&m.rows, m.mod, "dfg_fused_rows"));
+      DFG_CU(drv().ModuleGetFunction(&m.rows_multi, m.mod, "dfg_fused_rows_multi"));
     }
   }
   return m;

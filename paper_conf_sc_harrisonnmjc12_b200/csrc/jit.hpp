@@ -26,6 +26,8 @@ struct LoadedModule {
   CUfunction tma_multi = nullptr;  // several meshes per launch (dfg_execute_blocks)
   CUfunction tile = nullptr;       // same ring, filled by cp.async (layouts TMA cannot describe)
   CUfunction tile_multi = nullptr; // several meshes per launch on the cp.async ring
+  CUfunction rows = nullptr;       // same ring, one bulk copy per tile row (packed / unaligned rows)
+  CUfunction rows_multi = nullptr; // several meshes per launch on the row-copy ring
 };
 
 // Load into the current context (requires a device).

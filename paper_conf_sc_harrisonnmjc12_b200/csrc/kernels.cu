@@ -6,6 +6,7 @@
 // All element kernels are HBM-bound streams: grid-stride loops over 16-byte
 // vectors (float4 / double2), grids sized to a multiple of the SM count,
 // 64-bit indices (a 1024^3 vector array has 2^32 elements).
+#include <cuda.h>
 #include <cuda_runtime.h>
 
 #include <cstdint>
@@ -252,6 +253,43 @@ void verify_div2(const float* d, const float* yh, const float* yl, int n, unsign
   dim3 grid(64, unsigned(n < 32768 ? n : 32768));
   k_verify_div2<<<grid, 256, 0, s>>>(d, yh, yl, n, bad);
 }
+
+namespace {
+// Peer-halo probe: one TMA box of kProbeCols x
+// kProbeRows 32-bit words through `map` (a tensor map over a neighbour's
+// IPC-mapped probe block) into shared memory, then out to `out` -- the
+// in-place read of the peer halo path, on a known pattern.
+__global__ void __launch_bounds__(256) k_tma_probe(const __grid_constant__ CUtensorMap map, uint32_t* out) {
+  __shared__ alignas(128) uint32_t buf[kProbeRows * kProbeCols];
+  __shared__ alignas(8) unsigned long long bar;
+  const unsigned b = unsigned(__cvta_generic_to_shared(&bar));
+  const unsigned d = unsigned(__cvta_generic_to_shared(buf));
+  if (threadIdx.x == 0) {
+    asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(b) : "memory");
+    asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+  }
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(b), "r"(unsigned(sizeof(buf)))
+                 : "memory");
+    asm volatile(
+        "cp.async.bulk.tensor.2d.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1, {%3, %4}], [%2];" ::"r"(d),
+        "l"(reinterpret_cast<unsigned long long>(&map)), "r"(b), "r"(0), "r"(0)
+        : "memory");
+  }
+  unsigned done = 0;
+  while (!done)
+    asm volatile(
+        "{\n\t.reg .pred p;\n\tmbarrier.try_wait.parity.shared::cta.b64 p, [%1], 0, 1000000;\n\t"
+        "selp.u32 %0, 1, 0, p;\n\t}"
+        : "=r"(done)
+        : "r"(b)
+        : "memory");
+  for (int i = threadIdx.x; i < kProbeRows * kProbeCols; i += blockDim.x) out[i] = buf[i];
+}
+}  // namespace
+
+void tma_probe(const CUtensorMap* map, uint32_t* out, cudaStream_t s) { k_tma_probe<<<1, 256, 0, s>>>(*map, out); }
 
 }  // namespace kern
 }  // namespace dfg

@@ -2,7 +2,10 @@
 // counts; vector arrays are AoS 4-wide.  All launches are asynchronous on `s`.
 #pragma once
 
+#include <cuda.h>
 #include <cuda_runtime.h>
+
+#include <cstdint>
 
 #include "lang.hpp"
 
@@ -24,6 +27,14 @@ void grad3d(DType dt, const void* f, void* o4, const void* tx, const void* ty, c
 // a in [1, 2), RN(a*yh[k] + RN(a*yl[k])) == RN(a / d[k]).  Device pointers;
 // bad must be zeroed by the caller.
 void verify_div2(const float* d, const float* yh, const float* yl, int n, unsigned* bad, cudaStream_t s);
+
+// Peer-halo probe block: kProbeRows rows of kProbeCols 32-bit words, word i =
+// probe_word(i), placed kProbeOffset bytes into a mesh's flag allocation.
+constexpr int kProbeRows = 32, kProbeCols = 64, kProbeOffset = 256;
+inline uint32_t probe_word(uint32_t i) { return (i + 1u) * 2654435761u ^ 0x5bd1e995u; }
+// One TMA load of the whole probe box through `map` (host copy of a
+// CUtensorMap) into out[kProbeRows * kProbeCols] (device).
+void tma_probe(const CUtensorMap* map, uint32_t* out, cudaStream_t s);
 
 }  // namespace kern
 }  // namespace dfg

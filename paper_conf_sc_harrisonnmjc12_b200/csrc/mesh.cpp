@@ -370,11 +370,17 @@ void ipc_export(const void* p, cudaIpcMemHandle_t* h, int64_t* off) {
   *off = int64_t(reinterpret_cast<CUdeviceptr>(p) - base);
 }
 
+// flag words (256 bytes) followed by the probe block dfg_peer_probe reads
 void ensure_flags(MeshImpl& m) {
   if (m.flags) return;
   DFG_CUDA(cudaSetDevice(m.device));
-  DFG_CUDA(cudaMalloc(&m.flags, 256));
-  DFG_CUDA(cudaMemset(m.flags, 0, 256));
+  const size_t words = size_t(kern::kProbeRows) * kern::kProbeCols;
+  DFG_CUDA(cudaMalloc(&m.flags, kern::kProbeOffset + words * 4));
+  DFG_CUDA(cudaMemset(m.flags, 0, kern::kProbeOffset));
+  std::vector<uint32_t> pat(words);
+  for (size_t i = 0; i < words; ++i) pat[i] = kern::probe_word(uint32_t(i));
+  DFG_CUDA(cudaMemcpy(reinterpret_cast<char*>(m.flags) + kern::kProbeOffset, pat.data(), words * 4,
+                      cudaMemcpyHostToDevice));
   DFG_CUDA(cudaDeviceSynchronize());
 }
 }  // namespace
@@ -453,6 +459,52 @@ void mesh_link_peers(MeshImpl& m, const void* lo_blob, const void* hi_blob) {
   if (hi_blob) link(hi_blob, hi, false);
   m.peer_lo = lo;
   m.peer_hi = hi;
+}
+
+// Open the flag allocation of an exported slab on the current device, read
+// its probe block with one TMA load (the access the in-place halo makes) and
+// compare it with the pattern.  Meant to run in a short-lived process: a
+// transport that faults takes down that process, not the caller's.
+bool peer_probe(const void* blob) {
+  PeerBlob b;
+  std::memcpy(&b, blob, sizeof(b));
+  if (std::memcmp(b.magic, kMagic, 8) != 0) fail(DFG_E_INVALID, "peer probe: not a dfg_mesh_peer_export blob");
+  DFG_CUDA(cudaFree(0));
+  void* base = nullptr;
+  cudaError_t e = cudaIpcOpenMemHandle(&base, b.flags_h, cudaIpcMemLazyEnablePeerAccess);
+  if (e != cudaSuccess) {
+    cudaGetLastError();
+    fail(DFG_E_UNSUPPORTED, std::string("cudaIpcOpenMemHandle: ") + cudaGetErrorString(e));
+  }
+  struct Close {
+    void* p;
+    ~Close() { cudaIpcCloseMemHandle(p); }
+  } close{base};
+  char* probe = static_cast<char*>(base) + b.flags_off + kern::kProbeOffset;
+  CUtensorMap map;
+  cuuint64_t gdim[2] = {cuuint64_t(kern::kProbeCols), cuuint64_t(kern::kProbeRows)};
+  cuuint64_t gstride[1] = {cuuint64_t(kern::kProbeCols) * 4};
+  cuuint32_t box[2] = {cuuint32_t(kern::kProbeCols), cuuint32_t(kern::kProbeRows)};
+  cuuint32_t estr[2] = {1, 1};
+  DFG_CU(drv().TensorMapEncodeTiled(&map, CU_TENSOR_MAP_DATA_TYPE_UINT32, 2, probe, gdim, gstride, box, estr,
+                                    CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE,
+                                    CU_TENSOR_MAP_L2_PROMOTION_NONE, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE));
+  const size_t words = size_t(kern::kProbeRows) * kern::kProbeCols;
+  uint32_t* out = nullptr;
+  DFG_CUDA(cudaMalloc(&out, words * 4));
+  struct Free {
+    void* p;
+    ~Free() { cudaFree(p); }
+  } fr{out};
+  DFG_CUDA(cudaMemset(out, 0, words * 4));
+  kern::tma_probe(&map, out, nullptr);
+  DFG_CUDA(cudaGetLastError());
+  DFG_CUDA(cudaDeviceSynchronize());
+  std::vector<uint32_t> got(words);
+  DFG_CUDA(cudaMemcpy(got.data(), out, words * 4, cudaMemcpyDeviceToHost));
+  for (size_t i = 0; i < words; ++i)
+    if (got[i] != kern::probe_word(uint32_t(i))) return false;
+  return true;
 }
 
 }  // namespace dfg

@@ -145,7 +145,8 @@ std::unique_ptr<PlanImpl> compile_plan(std::shared_ptr<MeshImpl> mesh, const std
     const char* ctas = std::getenv("DFG_CTAS");
     if (ctas) cfg.ctas = std::max(1, std::min(4, std::atoi(ctas)));
     const char* st = std::getenv("DFG_STAGES");
-    if (st) cfg.stages = std::max(2, std::min(16, std::atoi(st)));
+    // >= 3: the cp.async tile ring waits on stage n+1 before it fills stage n+2
+    if (st) cfg.stages = std::max(3, std::min(16, std::atoi(st)));
     // tile shape for this mesh (narrow meshes: several rows per warp)
     const char* rpw = std::getenv("DFG_RPW");
     const int64_t slots = int64_t(sm_count(mesh->device)) * cfg.ctas;
@@ -181,6 +182,14 @@ std::unique_ptr<PlanImpl> compile_plan(std::shared_ptr<MeshImpl> mesh, const std
       DFG_CU(drv().FuncSetAttribute(plan->mod.tma_multi, CU_FUNC_ATTRIBUTE_MAX_DYNAMIC_SHARED_SIZE_BYTES, int(smem)));
       DFG_CU(drv().FuncSetAttribute(plan->mod.tile, CU_FUNC_ATTRIBUTE_MAX_DYNAMIC_SHARED_SIZE_BYTES, int(smem)));
       DFG_CU(drv().FuncSetAttribute(plan->mod.tile_multi, CU_FUNC_ATTRIBUTE_MAX_DYNAMIC_SHARED_SIZE_BYTES, int(smem)));
+      const size_t rsmem = fused_rows_smem_bytes(mesh->dt, int(plan->fsrc.layout.stencil_inputs.size() +
+                                                               plan->fsrc.layout.point_inputs.size()),
+                                                 plan->fsrc.cfg.ncw, plan->fsrc.cfg.stages);
+      if (rsmem <= 227 * 1024) {
+        plan->rows_smem = rsmem;
+        DFG_CU(drv().FuncSetAttribute(plan->mod.rows, CU_FUNC_ATTRIBUTE_MAX_DYNAMIC_SHARED_SIZE_BYTES, int(rsmem)));
+        DFG_CU(drv().FuncSetAttribute(plan->mod.rows_multi, CU_FUNC_ATTRIBUTE_MAX_DYNAMIC_SHARED_SIZE_BYTES, int(rsmem)));
+      }
     }
   }
   return plan;
@@ -306,6 +315,9 @@ void PlanImpl::execute(void* out, bool out_dev, cudaStream_t s) {
   bool any_host = !out_dev;
   for (int i : sources(dag).inputs)
     if (!m.fields[dag.inputs[i]].on_device) any_host = true;
+  // any host buffer makes the call synchronous (dfg.h): the uploads have read
+  // the caller's inputs and the result is in place when dfg_execute returns
+  if (any_host) DFG_CUDA(cudaStreamSynchronize(s));
   const int64_t unit_b = m.cells() * int64_t(dsize(m.dt));
   const int64_t units = strategy == DFG_HYBRID   ? hyb.high
                         : strategy == DFG_STAGED ? staged_units(dag, order, any_host)
@@ -490,9 +502,19 @@ void PlanImpl::exec_fused(void* out, bool out_dev, cudaStream_t s) {
 bool PlanImpl::tma_ok(const std::vector<const void*>& fptr, const void* dout, const SlabView& m) const {
   const int vec = int(16 / dsize(m.dt));
   const char* force = std::getenv("DFG_FUSED_KERNEL");
-  if (force && (!std::strcmp(force, "general") || !std::strcmp(force, "tile"))) return false;
+  if (force && (!std::strcmp(force, "general") || !std::strcmp(force, "tile") || !std::strcmp(force, "rows")))
+    return false;
   return mod.tma && !fsrc.layout.stencil_inputs.empty() && m.nx % vec == 0 && m.px() % vec == 0 &&
          m.gx() % vec == 0 && aligned16(dout) &&
+         std::all_of(fptr.begin(), fptr.end(), [](const void* p) { return aligned16(p); });
+}
+
+bool PlanImpl::rows_ok(const std::vector<const void*>& fptr, const SlabView& m) const {
+  const char* force = std::getenv("DFG_FUSED_KERNEL");
+  if (force && (!std::strcmp(force, "general") || !std::strcmp(force, "tile"))) return false;
+  return mod.rows && rows_smem && !fsrc.layout.stencil_inputs.empty() &&
+         (m.px() * m.py() * int64_t(dsize(m.dt))) % 16 == 0 && m.px() * m.py() < (int64_t(1) << 32) &&
+         m.px() < (int64_t(1) << 30) &&
          std::all_of(fptr.begin(), fptr.end(), [](const void* p) { return aligned16(p); });
 }
 
@@ -520,17 +542,31 @@ void PlanImpl::exec_fused_peer(const std::vector<const void*>& fptr, void* out, 
     if (!m.exported.count(dag.inputs[size_t(in)]))
       fail(DFG_E_INVALID, "peer halo: field '" + dag.inputs[size_t(in)] + "' was bound after dfg_mesh_peer_export");
   const bool lo = m.k0 > 0, hi = m.k0 + m.nzl < m.NZ;
+  const SlabView v = SlabView::of(m);
+  // every check that can fail runs before this rank publishes "ready": a
+  // throw after it would leave the neighbours waiting for the done flags.
+  // In-place TMA reads need the neighbours' mapped fields 16-byte aligned too
+  // (their tensor maps), else the planes are copied into the ghost planes.
+  bool use_tma = tma_ok(fptr, out, v);
+  for (const MeshImpl::Peer* pr : {lo ? &m.peer_lo : nullptr, hi ? &m.peer_hi : nullptr}) {
+    if (!pr) continue;
+    for (int in : L.stencil_inputs) {
+      auto it = pr->fields.find(dag.inputs[size_t(in)]);
+      if (it == pr->fields.end() || !it->second)
+        fail(DFG_E_UNBOUND, "peer slab exported no field '" + dag.inputs[size_t(in)] + "'");
+      use_tma = use_tma && aligned16(it->second);
+    }
+  }
   const uint32_t e = ++m.epoch;
   auto dptr = [](const uint32_t* p, int w) { return reinterpret_cast<CUdeviceptr>(p + w); };
   const CUstream cs = reinterpret_cast<CUstream>(s);
   DFG_CU(drv().StreamWriteValue32(cs, dptr(m.flags, kFlagReady), e, CU_STREAM_WRITE_VALUE_DEFAULT));
   const void* tab[3] = {m.dev_tab[0], m.dev_tab[1], m.dev_tab[2]};
-  const SlabView v = SlabView::of(m);
   auto wait_ready = [&] {
     if (lo) DFG_CU(drv().StreamWaitValue32(cs, dptr(m.peer_lo.flags, kFlagReady), e, CU_STREAM_WAIT_VALUE_GEQ));
     if (hi) DFG_CU(drv().StreamWaitValue32(cs, dptr(m.peer_hi.flags, kFlagReady), e, CU_STREAM_WAIT_VALUE_GEQ));
   };
-  if (tma_ok(fptr, out, v)) {
+  if (use_tma) {
     const int64_t a = m.k0 + (lo ? 1 : 0), b = m.k0 + m.nzl - (hi ? 1 : 0);
     if (a < b) launch_fused(fptr, out, tab, v, s, a, b);
     wait_ready();
@@ -561,7 +597,7 @@ void PlanImpl::exec_fused_peer(const std::vector<const void*>& fptr, void* out, 
   if (hi) DFG_CU(drv().StreamWriteValue32(cs, dptr(m.peer_hi.flags, kFlagLoDone), e, CU_STREAM_WRITE_VALUE_DEFAULT));
   if (lo) DFG_CU(drv().StreamWaitValue32(cs, dptr(m.flags, kFlagLoDone), e, CU_STREAM_WAIT_VALUE_GEQ));
   if (hi) DFG_CU(drv().StreamWaitValue32(cs, dptr(m.flags, kFlagHiDone), e, CU_STREAM_WAIT_VALUE_GEQ));
-  last_halo = tma_ok(fptr, out, v) ? 3 : 4;
+  last_halo = use_tma ? 3 : 4;
   st.halo_bytes += int64_t(L.stencil_inputs.size()) * ((lo ? 1 : 0) + (hi ? 1 : 0)) * int64_t(m.plane()) *
                         int64_t(dsize(m.dt));
 }
@@ -573,7 +609,12 @@ void PlanImpl::launch_fused(const std::vector<const void*>& fptr, void* dout, co
   const int64_t kbeg = kb < 0 ? m.k0 : kb, kend = ke < 0 ? m.k0 + m.nzl : ke;
   const int64_t N = m.nx * m.ny * (kend - kbeg);
   const int vec = int(16 / ts);
-  bool vec_ok = aligned16(dout) && (N % vec == 0) && m.gxy == 0 && m.px() == m.nx && m.gx() == 0;
+  // 16-byte point-wise loads / stores: aligned bases, whole vectors, and the
+  // input / output offsets of plane kbeg (ghost planes shift the input) on
+  // vector boundaries
+  const int64_t in_off = (kbeg - m.k0 + m.ghost) * m.nx * m.ny, out_off = (kbeg - m.k0) * m.nx * m.ny;
+  bool vec_ok = aligned16(dout) && (N % vec == 0) && m.gxy == 0 && m.px() == m.nx && m.gx() == 0 &&
+                in_off % vec == 0 && out_off % vec == 0;
   for (auto p : fptr) vec_ok = vec_ok && aligned16(p);
   const char* force = std::getenv("DFG_FUSED_KERNEL");
   const bool want_general = force && !std::strcmp(force, "general");
@@ -654,6 +695,30 @@ void PlanImpl::launch_fused(const std::vector<const void*>& fptr, void* dout, co
     kernel_end(ke, s);
     last_variant = 1;
     last_kz = best_kz;
+  } else if (rows_ok(fptr, m)) {
+    // the same ring filled by one bulk copy per tile row (rows per warp 1)
+    const int ncw = fsrc.cfg.ncw;
+    const int tw = tma_tile_w(m.dt, 1), th = tma_tile_h(ncw, 1);
+    const int tiles_x = int((m.nx + tw - 1) / tw);
+    const int tiles_y = int((m.ny + th - 1) / th);
+    const int64_t range = kend - kbeg;
+    int occ = 1;
+    DFG_CU(drv().OccupancyMaxActiveBlocksPerMultiprocessor(&occ, mod.rows, (ncw + 1) * 32, rows_smem));
+    const int64_t slots = int64_t(sms) * std::max(occ, 1);
+    const char* kzenv = std::getenv("DFG_KZ");
+    const int64_t kz = kzenv ? std::max<int64_t>(1, std::min<int64_t>(range, std::atoll(kzenv)))
+                             : choose_kz(int64_t(tiles_x) * tiles_y, range, slots);
+    const int64_t items = int64_t(tiles_x) * tiles_y * ((range + kz - 1) / kz);
+    const unsigned grid = unsigned(std::min<int64_t>(items, slots));
+    const bool out16 = aligned16(dout) && m.nx % vec == 0;
+    auto w = pack_params(fptr, dout, tab[0], tab[1], tab[2], m, kbeg, kend, items, tiles_x, tiles_y, int(kz),
+                         out16 ? 1 : 0);
+    void* args[] = {w.data()};
+    auto ke = kernel_begin(s);
+    DFG_CU(drv().LaunchKernel(mod.rows, grid, 1, 1, (ncw + 1) * 32, 1, 1, unsigned(rows_smem), s, args, nullptr));
+    kernel_end(ke, s);
+    last_variant = 7;
+    last_kz = kz;
   } else if (mod.tile && !want_general && m.px() * m.py() < (int64_t(1) << 32)) {
     // same ring and consumers, filled by the consumer threads with cp.async
     const int ncw = fsrc.cfg.ncw, rpw = fsrc.cfg.rpw;
@@ -716,7 +781,7 @@ void execute_blocks(const std::vector<PlanImpl*>& plans, const std::vector<void*
   // kernel if every block's layout suits tensor maps, else the cp.async ring
   bool batch = plans.size() > 1 && p0.strategy == DFG_FUSED && p0.mod.tma_multi && p0.mod.tile_multi &&
                p0.fsrc.cfg.has_tma && !(force && !std::strcmp(force, "general"));
-  bool tma = !(force && !std::strcmp(force, "tile"));
+  bool tma = !(force && (!std::strcmp(force, "tile") || !std::strcmp(force, "rows")));
   std::vector<std::vector<const void*>> fptrs(plans.size());
   for (size_t b = 0; b < plans.size() && batch; ++b) {
     PlanImpl& p = *plans[b];
@@ -739,13 +804,17 @@ void execute_blocks(const std::vector<PlanImpl*>& plans, const std::vector<void*
     for (size_t b = 0; b < plans.size(); ++b) plans[b]->execute(outs[b], true, s);
     return;
   }
+  // layouts a tensor map cannot describe: the row-copy ring when every block
+  // meets its alignment preconditions, else the cp.async ring
+  bool rows = !tma && p0.mod.rows_multi && p0.rows_smem;
+  for (size_t b = 0; b < plans.size() && rows; ++b) rows = plans[b]->rows_ok(fptrs[b], SlabView::of(*plans[b]->mesh));
   DFG_CUDA(cudaSetDevice(m0.device));
-  const int ncw = p0.fsrc.cfg.ncw, rpw = p0.fsrc.cfg.rpw;
+  const int ncw = p0.fsrc.cfg.ncw, rpw = rows ? 1 : p0.fsrc.cfg.rpw;
   const int tw = tma_tile_w(m0.dt, rpw), th = tma_tile_h(ncw, rpw);
   const int nsf = int(L.stencil_inputs.size() + L.point_inputs.size());
-  const size_t smem = fused_tma_smem_bytes(m0.dt, nsf, ncw, p0.fsrc.cfg.stages, rpw);
-  CUfunction fn = tma ? p0.mod.tma_multi : p0.mod.tile_multi;
-  const int threads = tma ? (ncw + 1) * 32 : ncw * 32;
+  const size_t smem = rows ? p0.rows_smem : fused_tma_smem_bytes(m0.dt, nsf, ncw, p0.fsrc.cfg.stages, rpw);
+  CUfunction fn = tma ? p0.mod.tma_multi : rows ? p0.mod.rows_multi : p0.mod.tile_multi;
+  const int threads = tma || rows ? (ncw + 1) * 32 : ncw * 32;
   int occ = 1;
   DFG_CU(drv().OccupancyMaxActiveBlocksPerMultiprocessor(&occ, fn, threads, smem));
   const int64_t slots = int64_t(sm_count(m0.device)) * std::max(occ, 1);
@@ -817,7 +886,7 @@ void execute_blocks(const std::vector<PlanImpl*>& plans, const std::vector<void*
   p0.st.kernel_count += 1;
   for (auto* p : plans) {
     p->st.executes += 1;
-    p->last_variant = tma ? 4 : 6;
+    p->last_variant = tma ? 4 : rows ? 8 : 6;
     p->last_kz = best_kz;
   }
 }

@@ -134,7 +134,9 @@ struct PlanImpl {
   FusedSource fsrc;
   LoadedModule mod;
   int regs = 0, spill = 0;
-  int last_variant = 0;  // 1 TMA, 2 general, 3 pointwise, 4 TMA multi-block (dfg_execute_blocks), 5 tile (cp.async ring), 6 tile multi-block
+  int last_variant = 0;  // 1 TMA, 2 general, 3 pointwise, 4 TMA multi-block (dfg_execute_blocks), 5 tile (cp.async ring), 6 tile multi-block,
+                         // 7 rows (bulk row copies), 8 rows multi-block
+  size_t rows_smem = 0;  // dynamic smem of the rows kernel (0: unavailable)
   int64_t last_kz = 0;   // z-chunk length of the last TMA launch
   int last_halo = 0;     // halo of the last execute: 0 none, 1 NCCL, 2 local copies, 3 peer (in place), 4 peer copies
   dfg_stats st{};
@@ -185,6 +187,11 @@ struct PlanImpl {
   void launch_fused(const std::vector<const void*>& fptr, void* dout, const void* const tab[3], const SlabView& v,
                     cudaStream_t s, int64_t kb = -1, int64_t ke = -1, bool peer = false);
   bool tma_ok(const std::vector<const void*>& fptr, const void* dout, const SlabView& v) const;
+ public:
+  // the row-copy kernel's preconditions: 16-byte aligned field bases and
+  // plane strides (DFG_FUSED_KERNEL=tile / general turn it off)
+  bool rows_ok(const std::vector<const void*>& fptr, const SlabView& v) const;
+ private:
   void exec_fused_peer(const std::vector<const void*>& fptr, void* out, bool out_dev, cudaStream_t s);
   void exec_streamed(void* out, bool out_dev, cudaStream_t s);
   void release_stream_buffers();
@@ -213,6 +220,9 @@ void mesh_init_comm(MeshImpl& m, const void* id128, int rank, int nranks);
 constexpr size_t kPeerBlobBytes = 4096;
 void mesh_peer_export(MeshImpl& m, void* blob);
 void mesh_link_peers(MeshImpl& m, const void* lo_blob, const void* hi_blob);
+// One TMA read of an exported slab's probe block on the current device;
+// true when it returns the pattern (dfg_peer_probe).
+bool peer_probe(const void* blob);
 // flag word offsets (uint32 units, 64 bytes apart)
 constexpr int kFlagReady = 0, kFlagLoDone = 16, kFlagHiDone = 32;
 

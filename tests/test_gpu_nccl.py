@@ -30,7 +30,7 @@ def test_nccl_slabs_match_single_slab(ranks, overlap, prog, dtype):
     r = subprocess.run(cmd, capture_output=True, text=True, timeout=600, cwd=ROOT)
     assert r.returncode == 0, r.stdout[-3000:] + r.stderr[-3000:]
     line = json.loads([ln for ln in r.stdout.splitlines() if ln.startswith("{")][-1])
-    assert line["bit_identical_to_single_slab"] and line["halo_bytes_ok"]
+    assert line["bit_identical_to_single_slab"] and line["bit_identical_to_oracle"] and line["halo_bytes_ok"]
     # interior launch + one boundary launch per halo side when overlapped
     want = [1 + (r_ > 0) + (r_ < ranks - 1) if overlap else 1 for r_ in range(ranks)]
     assert line["kernels_per_execute"] == want

@@ -530,6 +530,7 @@ def test_zslab_emulation_matches_single_gpu(G, T, overlap, monkeypatch):
     torch.cuda.synchronize()
     got = torch.cat(outs).cpu().numpy()
     assert np.array_equal(got, whole)
+    assert_parity(got, run_oracle(src, f, x, y, z))       # the stitched slabs against the oracle itself
     for r, p in enumerate(plans):
         sides = (r > 0) + (r < G - 1)
         st = p.stats()
@@ -652,6 +653,21 @@ def test_streamed_strategy(planes, prog, shape, monkeypatch):
     assert st["d2h_count"] == nch
     # device-resident everything: identical to fusion
     assert_parity(run_lib(src, f, x, y, z, "streamed", host=False), want)
+
+
+@pytest.mark.parametrize("planes", ["4", "12"])
+@pytest.mark.parametrize("prog", ["velmag", "qcrit"])
+def test_streamed_odd_plane_vector_offsets(planes, prog, monkeypatch):
+    """a chunk of 4 or 12 planes of a 67 x 9 plane holds a whole
+    number of 16-byte vectors, but its first owned plane sits one odd plane
+    (the ghost) into the slot: the point-wise kernel must not take its
+    16-byte path there (it would load misaligned)."""
+    monkeypatch.setenv("DFG_STREAM_PLANES", planes)
+    shape = (67, 9, 12)
+    x, y, z, f = _inputs(shape, np.float32, NAMES[prog])
+    src = PAPER_PROGRAMS[prog][0]
+    got = run_lib(src, f, x, y, z, "streamed", host=True)
+    assert_parity(got, run_oracle(src, f, x, y, z))
 
 
 def test_streamed_pinned_large(monkeypatch):
@@ -777,6 +793,17 @@ def test_staged_graph_replay(T, monkeypatch):
         assert_parity(out.cpu().numpy(), want)
     st = plan.stats()
     assert st["executes"] == 3 and st["kernel_count"] == 3 * 67
+    # the ledger high-water survives a stats reset on the replay path (row a10)
+    units = omodel.footprint(build_dag(src, ("u", "v", "w")), "staged", "device")
+    elem = int(np.prod(shape)) * np.dtype(T).itemsize
+    assert st["dev_highwater_bytes"] == units * elem
+    plan.reset_stats()
+    assert plan.stats()["dev_highwater_bytes"] == 0
+    plan.execute(out)
+    torch.cuda.synchronize()
+    st = plan.stats()
+    assert st["executes"] == 1 and st["kernel_count"] == 67
+    assert st["dev_highwater_bytes"] == units * elem
     # new data under the same pointer: the replay reads it
     f2 = {k: (v * 2).astype(T) for k, v in f.items()}
     for k in dev:

@@ -414,7 +414,7 @@ def test_oracle_only_in_checks():
         if name.endswith(".py"):
             assert "oracle" not in open(os.path.join(pkg, name)).read().replace("no CPU", ""), name
     tree = ast.parse(open(os.path.join(ROOT, "bench.py")).read())
-    allowed = {"_oracle_time", "_window_parity"}
+    allowed = {"_oracle_time", "_window_parity", "slab_boundary_parity"}
     for fn in ast.walk(tree):
         if isinstance(fn, ast.FunctionDef):
             for node in ast.walk(fn):
@@ -425,3 +425,23 @@ def test_oracle_only_in_checks():
     top = [n for n in tree.body if isinstance(n, (ast.Import, ast.ImportFrom))]
     assert not any((getattr(n, "module", None) or "").startswith("oracle") or
                    any(a.name.startswith("oracle") for a in n.names) for n in top)
+
+
+def test_python_binding_validates_buffers(dfg):
+    """the C ABI sees raw pointers only, so Mesh.bind /
+    Plan.execute check contiguity, dtype, element count and device before
+    passing one (ValueError, nothing reaches the library)."""
+    import numpy as np
+    import torch
+    from paper_conf_sc_harrisonnmjc12_b200 import _check_buffer
+    n = 2 * 3 * 5
+    _check_buffer(np.zeros((2, 3, 5), np.float32), np.float32, n, None, "f")
+    _check_buffer(torch.zeros(2, 3, 5, dtype=torch.float64), np.float64, n, None, "f")
+    _check_buffer(12345, np.float32, n, None, "f")             # raw pointers pass
+    bad = [(np.zeros((2, 3, 5), np.float64), "dtype"), (np.zeros((2, 3, 4), np.float32), "elements"),
+           (np.zeros((2, 3, 10), np.float32)[:, :, ::2], "contiguous"),
+           (torch.zeros(2, 5, 3).transpose(1, 2), "contiguous"), (torch.zeros(31), "elements"),
+           (torch.zeros(30, dtype=torch.float64), "dtype")]
+    for buf, why in bad:
+        with pytest.raises(ValueError, match=why):
+            _check_buffer(buf, np.float32, n, None, "f")

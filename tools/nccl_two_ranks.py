@@ -75,14 +75,19 @@ def worker(rank, world, args, port):
         torch.cuda.synchronize()
         whole = wout.cpu().numpy()
         stitched = np.concatenate([p[3] for p in sorted(parts, key=lambda p: p[1])])
-        ok = bool(np.array_equal(stitched, whole))
+        from oracle import evaluate as oev
+        from oracle.lang import build_dag
+        want = oev.evaluate_full(build_dag(src, tuple(recipe), args.dtype),
+                                 {k: v.cpu().numpy() for k, v in wf.items()}, x, y, z)
+        oracle_ok = bool(np.array_equal(stitched, want))      # the oracle itself
+        ok = bool(np.array_equal(stitched, whole)) and oracle_ok
         pb = n * n * np.dtype(T).itemsize
         # halo fields = the stencil inputs: the same whole number on every rank
         per = [p[4] / (args.reps * pb * ((p[0] > 0) + (p[0] < world - 1))) for p in parts]
         halo_ok = all(v == per[0] and v == int(v) and v >= 1 for v in per)
         print(json.dumps({"ranks": world, "n": n, "nz": NZ, "prog": args.prog, "dtype": args.dtype,
                           "overlap": args.overlap,
-                          "bit_identical_to_single_slab": ok, "halo_bytes_ok": halo_ok, "halo_fields": per[0],
+                          "bit_identical_to_single_slab": ok, "bit_identical_to_oracle": oracle_ok, "halo_bytes_ok": halo_ok, "halo_fields": per[0],
                           "kernels_per_execute": [p[5] / args.reps for p in parts],
                           "transport": "NCCL socket (loopback), one GPU, per-rank NCCL_HOSTID"}), flush=True)
     plan.close()

@@ -80,7 +80,10 @@ def worker(rank, world, args, port):
         for c, b in wf.items():
             whole_mesh.bind(c, b)
         wplan = dfg.Plan(whole_mesh, src, "fused")
-        ok = True
+        from oracle import evaluate as oev
+        from oracle.lang import build_dag
+        dag = build_dag(src, tuple(recipe), args.dtype)
+        ok = oracle_ok = True
         for t in range(args.steps):
             for name in recipe:
                 wf[name].copy_(wbase[name] * (1 + t))
@@ -89,10 +92,15 @@ def worker(rank, world, args, port):
             torch.cuda.synchronize()
             stitched = np.concatenate([p[3][t] for p in sorted(parts, key=lambda p: p[1])])
             ok = ok and bool(np.array_equal(stitched, wout.cpu().numpy()))
+            # and against the oracle on the same step's arrays
+            want = oev.evaluate_full(dag, {k: v.cpu().numpy() for k, v in wf.items()}, x, y, z)
+            oracle_ok = oracle_ok and bool(np.array_equal(stitched, want))
+        ok = ok and oracle_ok
         pb = n * nx * np.dtype(T).itemsize
         per = [p[4] / (args.steps * pb * ((p[0] > 0) + (p[0] < world - 1))) for p in parts]
         print(json.dumps({"ranks": world, "nx": nx, "n": n, "nz": NZ, "prog": args.prog, "dtype": args.dtype,
                           "steps": args.steps, "bit_identical_to_single_slab": ok,
+                          "bit_identical_to_oracle": oracle_ok,
                           "halo_fields": per[0], "halo_modes": [p[6] for p in parts],
                           "ghost_planes_untouched": [p[7] for p in parts],
                           "kernels_per_execute": [p[5] / args.steps for p in parts],
