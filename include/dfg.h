@@ -332,6 +332,20 @@ int dfg_plan_set_timing(dfg_plan plan, int level);
  * ghost planes).  `out` must hold 14 entries. */
 int dfg_plan_info(dfg_plan plan, int64_t out[14]);
 
+/* Arithmetic of a plan and the inputs on which its results equal the
+ * oracle's (the literal network evaluated in T, reading R6; DESIGN.md
+ * section 5): out[0] = grad3d quotient (0 IEEE div.rn, 1 exact in the
+ * normal range: two-operation / Markstein with the reciprocal tables,
+ * 2 fast num * (1/d)), out[1] = 1 if power-of-two scale folding rewrites
+ * the fused body, out[2] = two-operation axes mask (out[0] == 1),
+ * out[3] = exactness domain: 2 = bit-identical for EVERY input (IEEE
+ * operations only: the staged / roundtrip / hybrid kernels, and
+ * DFG_FUSED_VARIANT=ieee), 1 = bit-identical whenever no intermediate of the
+ * literal network is subnormal or overflows (the default fused kernel),
+ * 0 = within tolerance only (fast quotient, hand-written reference
+ * bodies).  `out` must hold 4 entries.  Host only; no device work. */
+int dfg_plan_arith(dfg_plan plan, int64_t out[4]);
+
 /* Execution order of the plan's filters (ids of the canonical text).  Staged
  * plans run the paper's list order unless a dev_mem_cap rejected it and the
  * memory-aware order (greedy minimum live memory) fits --

@@ -103,12 +103,15 @@ _CMP = {
 }
 
 
-def evaluate(dag: Dag, inputs: dict, mw: MeshWindow):
+def evaluate(dag: Dag, inputs: dict, mw: MeshWindow, on_value=None):
     """Evaluate every filter in list order over whole arrays.
 
     inputs: name -> array[k, j, i] of dtype T (all the same window shape).
     Returns (result, valid): result is [k, j, i] for a scalar program or
     [k, j, i, 4] (lanes beyond the used width are 0) for a vector program.
+    on_value(k, filter, value, args), if given, sees every filter's value
+    and its (non-mesh) argument values (an observer: it cannot change the
+    evaluation).
     """
     T = np.float32 if dag.dtype == "f32" else np.float64
     shape = None
@@ -152,6 +155,8 @@ def evaluate(dag: Dag, inputs: dict, mw: MeshWindow):
                 raise AssertionError(f.op)
             assert v.dtype == T, (f.op, v.dtype)
             vals[ref] = v
+            if on_value is not None:
+                on_value(k, f, v, a)
     res = get(dag.result)
     if res.ndim == 4:
         pad = np.zeros(shape + (4,), dtype=T)
@@ -167,3 +172,51 @@ def evaluate_full(dag: Dag, inputs: dict, x, y, z):
     res, valid = evaluate(dag, inputs, MeshWindow(x, y, z))
     assert valid.all()
     return res
+
+
+def in_range_mask(dag: Dag, inputs: dict, x, y, z):
+    """Whole mesh: True at the cells where every input value, every grad3d
+    numerator f[ip] - f[im] (each axis) and every value of the literal
+    network (each filter, each lane) is zero or has a magnitude in
+    [2^(emin + 2p), 2^(emax - p)] of T (fp32: [2^-78, 2^104], fp64:
+    [2^-916, 2^970]; p = significand bits) -- finite, normal, with 2^p of
+    headroom above and 2^(2p) below.  This is the sufficient condition of
+    DESIGN.md section 5 under which the default fused kernel's reciprocal
+    quotients and power-of-two scale folding round exactly like the literal
+    network; it is written as a plain definition over the oracle's values."""
+    T = np.float32 if dag.dtype == "f32" else np.float64
+    fi = np.finfo(T)
+    p = fi.nmant + 1
+    lo = np.ldexp(1.0, fi.minexp + 2 * p)
+    hi = np.ldexp(1.0, fi.maxexp - 1 - p)
+
+    def ok(a):
+        a = np.abs(a.astype(np.float64))
+        return (a == 0) | ((a >= lo) & (a <= hi))
+
+    shape = next(iter(inputs.values())).shape
+    mask = np.ones(shape, dtype=bool)
+    for a in inputs.values():
+        mask &= ok(a)
+
+    def numerators(f):
+        out = np.ones(shape, dtype=bool)
+        for axis in range(3):
+            n = f.shape[axis]
+            if n == 1:
+                continue
+            i = np.arange(n)
+            num = np.take(f, np.minimum(i + 1, n - 1), axis=axis) - np.take(f, np.maximum(i - 1, 0), axis=axis)
+            out &= ok(num)
+        return out
+
+    def see(k, f, v, args):
+        nonlocal mask
+        if f.op == "grad3d":
+            mask &= numerators(args[0])
+        m = ok(v)
+        mask &= m.all(axis=-1) if m.ndim == 4 else m
+
+    with np.errstate(all="ignore"):
+        evaluate(dag, inputs, MeshWindow(x, y, z), on_value=see)
+    return mask

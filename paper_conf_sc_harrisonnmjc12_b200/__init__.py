@@ -175,6 +175,12 @@ class Plan:
     def dag(self):
         return dfg_dump_dag(self.handle)
 
+    def arith(self):
+        """Quotient form, scale folding and the inputs on which the results
+        equal the oracle's (dfg_plan_arith)."""
+        from ._dfg import dfg_plan_arith
+        return dfg_plan_arith(self.handle)
+
     def schedule(self):
         from ._dfg import dfg_plan_schedule
         return dfg_plan_schedule(self.handle)

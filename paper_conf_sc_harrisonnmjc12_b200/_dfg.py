@@ -76,6 +76,7 @@ _SIGS = {
     "dfg_reset_stats": (C.c_int, [_P]),
     "dfg_plan_set_timing": (C.c_int, [_P, C.c_int]),
     "dfg_plan_info": (C.c_int, [_P, C.POINTER(_I64)]),
+    "dfg_plan_arith": (C.c_int, [_P, C.POINTER(_I64)]),
     "dfg_plan_schedule": (C.c_int, [_P, C.POINTER(C.c_int32), C.c_size_t, C.POINTER(C.c_size_t)]),
     "dfg_plan_transfers": (C.c_int, [_P, C.POINTER(C.c_int32), C.c_size_t, C.POINTER(C.c_size_t)]),
     "dfg_hybrid_model": (C.c_int, [C.c_char_p, C.POINTER(C.c_char_p), C.c_int, C.c_int, C.c_int64,
@@ -241,6 +242,13 @@ def dfg_plan_set_timing(plan, level: int):
 
 def dfg_reset_stats(plan):
     _check(_lib.dfg_reset_stats(plan))
+
+
+def dfg_plan_arith(plan) -> dict:
+    out = (_I64 * 4)()
+    _check(_lib.dfg_plan_arith(plan, out))
+    return {"div_mode": ("ieee", "exact_normal", "fast")[out[0]], "fold": bool(out[1]), "div2_axes": out[2],
+            "exact_domain": ("tolerance", "normal_range", "all_inputs")[out[3]]}
 
 
 def dfg_plan_info(plan) -> dict:

@@ -294,6 +294,23 @@ int dfg_plan_info(dfg_plan plan, int64_t out[14]) {
   });
 }
 
+int dfg_plan_arith(dfg_plan plan, int64_t out[4]) {
+  return guard([&] {
+    if (!plan || !out) dfg::fail(DFG_E_INVALID, "null argument");
+    const auto& p = *plan->p;
+    const bool fused = p.strategy == DFG_FUSED || p.strategy == DFG_STREAMED || p.strategy == DFG_REFERENCE;
+    const int div = fused ? p.fsrc.cfg.div_mode : 0;  // per-primitive kernels: IEEE div.rn
+    const bool fold = fused && p.fsrc.cfg.fold;
+    out[0] = div;
+    out[1] = fold ? 1 : 0;
+    out[2] = fused ? p.fsrc.cfg.div2 : 0;
+    // 2: equal to the oracle for every input; 1: for every input whose
+    // literal-network intermediates are all zero or normal and finite;
+    // 0: within tolerance (fast quotient, hand-written reference body)
+    out[3] = p.strategy == DFG_REFERENCE || div == 2 ? 0 : (div == 0 && !fold) ? 2 : 1;
+  });
+}
+
 int dfg_plan_schedule(dfg_plan plan, int32_t* order, size_t cap, size_t* n) {
   return guard([&] {
     if (!plan || !n) dfg::fail(DFG_E_INVALID, "null argument");

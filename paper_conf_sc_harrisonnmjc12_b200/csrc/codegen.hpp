@@ -30,6 +30,7 @@ struct FusedConfig {
   int ctas = 1;        // resident CTAs per SM the TMA kernel is sized for
   int rpw = 1;         // tile rows per consumer warp (1, 2, 4): tile = (32*VEC/rpw) x (ncw*rpw)
   bool has_tma = false;
+  int rstages = 0;     // row-class kernel: ring depth (0: it does not fit)
 };
 
 struct FusedSource {
@@ -50,9 +51,9 @@ const char* reference_program(const std::string& which, int* id);
 
 // Dynamic shared memory the TMA kernel needs for a config (bytes).
 size_t fused_tma_smem_bytes(DType dt, int nsf, int ncw, int stages, int rpw = 1);
-// the row-copy kernel's ring (fused_tma.cuh DFG_R*): rows per warp 1, smem
-// row pitch = halo'd tile row + 3 chunks
-size_t fused_rows_smem_bytes(DType dt, int nsf, int ncw, int stages);
+// the row-class kernel (fused_tma.cuh "rows"): a ring of `stages` stages of
+// class boxes (box width = halo'd tile row + one chunk) + its barriers
+size_t fused_rows_smem_bytes(DType dt, int nsf, int ncw, int rpw, int stages);
 
 // TMA kernel tile: tile_w cells along x, tile_h rows along y (fused_tma.cuh).
 inline int tma_tile_w(DType dt, int rpw) { return 32 * (dt == DType::F32 ? 4 : 2) / rpw; }

@@ -9,29 +9,40 @@
 // only when every divisor of its table is certified.  DESIGN.md section 5.
 //
 // certify_div2<T>: certification by candidates, for float and double.
-//   Let p be the precision, d = B 2^(e-p) with B in [2^(p-1), 2^p), and scale
-//   the numerator so that x = A 2^(e-p), A in [2^(p-1), 2^p): q* = x/d = A/B
-//   in (1/2, 2) (every quantity scales exactly by powers of two in the normal
-//   range, so these significands decide every numerator).  With yl = RN(1/d
-//   - r) the value v = x r + RN(x yl) rounded by the FMA differs from q* by
-//   at most c A B 2^(2-3p)-ish, c ~ 1 (|1/d - r - yl| <= 2^-p |1/d - r| and
-//   |RN(x yl) - x yl| <= 2^-p |x yl|).  RN(v) != RN(q*) needs a rounding
-//   boundary -- a midpoint N 2^-p (q* in [1, 2)) or N 2^-(p+1) (q* in
-//   [1/2, 1)), N odd in (2^p, 2^(p+1)) -- between v and q*, i.e.
-//       |2^s A - N B| = |k| < 2 (s = p)   or   < 4 (s = p + 1),
-//   k an integer, k != 0 (an exact midpoint is impossible).  For each k
-//   with |k| <= W (W = 16 leaves a wide margin) the congruence N B = -k
-//   (mod 2^s) fixes N modulo 2^(s-t) (t = trailing zero bits of B); the
-//   handful of N in range give the candidate numerators A = (N B + k) / 2^s.
-//   The scheme is certified when it matches IEEE division at every
-//   candidate and its two neighbours.  A divisor with more than log2(W)
-//   trailing zero bits has no candidate at all: such divisors (the RT
-//   meshes' spacings, differences of nearby coordinates) always pass.
-//   Preconditions checked here: r == RN(1/d) and yl == RN(1/d - r), the
-//   latter formed as RN(e / d) with the exact remainder e = fma(-r, d, 1);
-//   d, r, yl normal.  The method is validated against exhaustive fp32
-//   enumeration (tests/test_lib_host.py::test_div2_certificate_matches_exhaustive).
-//
+//   Error bound (proof).  u = 2^-p.  r = RN(1/d) gives |r - 1/d| <= u/d
+//   (|RN(y) - y| <= ulp(y)/2 <= u |y|).  The remainder e = fma(-r, d, 1) =
+//   1 - r d is exact (Markstein), so tau = 1/d - r = e/d exactly and
+//   yl = RN(e/d) = RN(tau) with |yl - tau| <= u |tau| (tau normal; if
+//   yl == 0 we require e == 0, i.e. tau == 0).  Let L = RN(x yl):
+//   |L - x yl| <= u |x yl| (x yl normal).  The FMA rounds v = x r + L once,
+//   and x/d = x r + x tau, so
+//       v - x/d = (L - x yl) + x (yl - tau),
+//       |v - x/d| <= u |x| (|yl| + |tau|) <= u (2 + u) |x| |tau|
+//                 <= (2 + u) 2^-2p |x/d|.
+//   Scale to significands: d = B 2^(e-p), x = A 2^(e-p), B, A in [2^(p-1),
+//   2^p) (every quantity scales exactly by powers of two while the products
+//   stay normal), q* = x/d = A/B in (1/2, 2).  RN(v) != RN(q*) needs a
+//   rounding midpoint m between v and q* (q* itself is never a midpoint;
+//   v == m is covered since |q* - m| <= |v - q*| then):
+//     q* in [1, 2):   m = N 2^-p,     N odd:  |2^p A - N B| <= (2+u) 2^-p A < 2 + u
+//     q* in [1/2, 1): m = N 2^-(p+1), N odd:  |2^(p+1) A - N B| < 4 + 2u
+//   (A < 2^p), i.e. k = 2^s A - N B is a nonzero integer with |k| <= 2
+//   (s = p) or |k| <= 4 (s = p + 1); the binade ends are out of reach
+//   (q* >= 1/2 + 2^-(p+1) - and <= 2 - 2^(1-p), far beyond the error).  For
+//   each k with |k| <= W (W = 16 > 4) the congruence N B = -k (mod 2^s)
+//   fixes N modulo 2^(s-t) (t = trailing zero bits of B); every N in
+//   (2^p, 2^(p+1)) is enumerated and gives the numerator A = (N B + k) / 2^s.
+//   So the candidates contain EVERY numerator at which the scheme can
+//   differ from RN(x/d): the divisor is certified when the scheme matches
+//   IEEE division at each of them (and, for margin, its two neighbours).  A
+//   divisor with more than log2(W) trailing zero bits has no candidate at
+//   all: such divisors (the RT meshes' spacings, differences of nearby
+//   coordinates) always pass.  tests/test_lib_host.py pins the bound with
+//   exact rational arithmetic on random fp64 operands and the whole method
+//   against exhaustive fp32 enumeration.
+//   Preconditions checked here: r == RN(1/d) and yl == RN(1/d - r) formed
+//   as RN(e / d); d, r, yl normal, or yl == 0 with e == 0.
+
 // exhaustive_div2_f32: the exhaustive definition for fp32 (all 2^23
 // significands), on the host; the device version (kern::verify_div2) decides
 // fp32 meshes, this one exists to validate certify_div2.
@@ -60,6 +71,7 @@ bool certify_div2(T d, T r, T yl, int W = 16, long* tested = nullptr) {
   if (!(d > T(0)) || !std::isnormal(d) || !std::isnormal(r)) return false;
   if (r != T(1) / d || yl != div2_low_part(d, r)) return false;
   if (yl != T(0) && !std::isnormal(yl)) return false;
+  if (yl == T(0) && std::fma(-r, d, T(1)) != T(0)) return false;  // tau != 0 lost to underflow
   int ed = 0;
   const T md = std::frexp(d, &ed);                  // d = md 2^ed, md in [1/2, 1)
   const uint64_t B = uint64_t(std::ldexp(md, p));   // d = B 2^(ed - p)

@@ -26,6 +26,7 @@ namespace {
 void launch_primitive(const MeshImpl& m, const Filter& f, void* o, const std::vector<const void*>& a,
                       const void* gsrc, int64_t gghost, const void* const tab[3], cudaStream_t s) {
   const int64_t N = m.cells();
+  NvtxRange nv(op_name(f.op));
   switch (f.op) {
     case Op::Const: kern::fill(m.dt, f.cval, o, N, s); break;
     case Op::Add: case Op::Sub: case Op::Mult: case Op::Div:

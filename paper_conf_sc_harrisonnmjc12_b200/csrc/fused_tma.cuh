@@ -113,8 +113,9 @@ __device__ __forceinline__ DFG_T dfg_lds1(unsigned addr) {
 // Ring cursor: shared-memory byte address of the current stage and of its
 // full / empty barriers, advanced without multiplies (same sequence as the
 // producer's).
-template <unsigned SB>
+template <unsigned SB, int NS>
 struct DfgRingT {
+  static constexpr unsigned kEmpty = 8u * NS;  // empty[s] = full[s] + kEmpty
   unsigned tile;   // smem byte address of stage s, field 0
   unsigned full;   // smem byte address of full[s]
   unsigned phase;
@@ -124,7 +125,7 @@ struct DfgRingT {
     ++stage;
     tile += SB;
     full += 8;
-    if (stage == DFG_STAGES) {
+    if (stage == NS) {
       stage = 0;
       tile = tile0;
       full = full0;
@@ -132,7 +133,7 @@ struct DfgRingT {
     }
   }
 };
-typedef DfgRingT<DFG_STAGE_BYTES> DfgRing;
+typedef DfgRingT<DFG_STAGE_BYTES, DFG_STAGES> DfgRing;
 #define DFG_EMPTY(full_addr) ((full_addr) + 8 * DFG_STAGES)
 
 // per-item, per-thread constants of a consumer thread
@@ -173,8 +174,8 @@ __device__ __forceinline__ void dfg_store_masked(DFG_T* dst, const dfg2 (&o)[DFG
 // One z-plane.  `cur` = smem address of the plane's stage (tile, full bar);
 // the next plane's stage is always present (the producer loads a clamped
 // post-plane).  Queue roles are template parameters (no copies).
-template <int ZM, int ZC, int ZN, bool MASKED = false, class Fill = DfgNoFill>
-__device__ __forceinline__ void dfg_plane(const DfgCol& C, DfgRing& R, unsigned& cur_tile, unsigned& cur_full,
+template <int ZM, int ZC, int ZN, bool MASKED = false, class Fill = DfgNoFill, class Ring = DfgRing>
+__device__ __forceinline__ void dfg_plane(const DfgCol& C, Ring& R, unsigned& cur_tile, unsigned& cur_full,
                                           DFG_T (&zq)[3][DFG_NSF][DFG_VEC], DFG_T*& outp,
                                           long long plane, const DFG_T*& tzp, long long NZ, Fill& fill) {
   // x/y neighbours of this plane first (its stage is already resident), then
@@ -241,7 +242,7 @@ __device__ __forceinline__ void dfg_plane(const DfgCol& C, DfgRing& R, unsigned&
     dfg_store_cells(outp, o);
   }
   outp += plane * DFG_OUTW;
-  dfg_mbar_arrive(DFG_EMPTY(cur_full));  // every consumer thread (count NCW*32)
+  dfg_mbar_arrive(cur_full + Ring::kEmpty);  // every consumer thread (count NCW*32)
   fill.step();
   cur_tile = nxt_tile;
   cur_full = nxt_full;
@@ -354,16 +355,17 @@ __device__ __forceinline__ void dfg_consume_item(const DfgTmaParams& TP, long lo
 
 // full_count: arrivals that complete a "full" phase (1 for the TMA
 // producer's arrive.expect_tx; every consumer thread for the tile kernel)
-__device__ __forceinline__ unsigned dfg_ring_init(unsigned full_count = 1, unsigned stage_bytes = DFG_STAGE_BYTES) {
+__device__ __forceinline__ unsigned dfg_ring_init(unsigned full_count = 1, unsigned stage_bytes = DFG_STAGE_BYTES,
+                                                  int stages = DFG_STAGES, unsigned empty_count = DFG_NCW * 32) {
   // dynamic shared memory starts at the (1024-aligned) base of the CTA's
   // window: no static __shared__ in this kernel
   extern __shared__ __align__(1024) unsigned char dfg_smem_raw[];
   const unsigned smem = dfg_smem(dfg_smem_raw);
-  const unsigned full0 = smem + DFG_STAGES * stage_bytes;  // full[s] at full0 + 8s, empty[s] = full[s] + 8*STAGES
+  const unsigned full0 = smem + stages * stage_bytes;  // full[s] at full0 + 8s, empty[s] = full[s] + 8*stages
   if (threadIdx.x == 0) {
-    for (int s = 0; s < DFG_STAGES; ++s) {
+    for (int s = 0; s < stages; ++s) {
       dfg_mbar_init(full0 + 8 * s, full_count);
-      dfg_mbar_init(DFG_EMPTY(full0 + 8 * s), DFG_NCW * 32);
+      dfg_mbar_init(full0 + 8 * s + 8 * stages, empty_count);
     }
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   }
@@ -542,8 +544,9 @@ struct DfgFill {
   }
 };
 
-__device__ __forceinline__ void dfg_consume_tile(const DfgParams& P, long long item, DfgRing& R, DfgCol& C, int warp,
-                                                 int lane, DfgFill& F) {
+template <class Ring, class Fill>
+__device__ __forceinline__ void dfg_consume_tile(const DfgParams& P, long long item, Ring& R, DfgCol& C, int warp,
+                                                 int lane, Fill& F) {
   const long long plane = P.nx * P.ny;
   const int col = lane % DFG_LPR, sub = lane / DFG_LPR;
   const unsigned c0 = DFG_HX + DFG_VEC * col;
@@ -584,7 +587,7 @@ __device__ __forceinline__ void dfg_consume_tile(const DfgParams& P, long long i
   dfg_mbar_wait(R.full, R.phase, 0x100000u);
 #pragma unroll
   for (int f = 0; f < DFG_NSF; ++f) dfg_lds16(zq[0][f], R.tile + f * DFG_TILE_BYTES + C.off_c);
-  dfg_mbar_arrive(DFG_EMPTY(R.full));
+  dfg_mbar_arrive(R.full + Ring::kEmpty);
   F.step();
   R.advance();
   dfg_mbar_wait(R.full, R.phase, 0x100000u);
@@ -594,15 +597,15 @@ __device__ __forceinline__ void dfg_consume_tile(const DfgParams& P, long long i
   R.advance();
   long long k = kb;
   for (; k + 3 <= ke; k += 3) {
-    dfg_plane<0, 1, 2, true>(C, R, cur_tile, cur_full, zq, outp, plane, tzp, P.NZ, F);
-    dfg_plane<1, 2, 0, true>(C, R, cur_tile, cur_full, zq, outp, plane, tzp, P.NZ, F);
-    dfg_plane<2, 0, 1, true>(C, R, cur_tile, cur_full, zq, outp, plane, tzp, P.NZ, F);
+    dfg_plane<0, 1, 2, true, Fill, Ring>(C, R, cur_tile, cur_full, zq, outp, plane, tzp, P.NZ, F);
+    dfg_plane<1, 2, 0, true, Fill, Ring>(C, R, cur_tile, cur_full, zq, outp, plane, tzp, P.NZ, F);
+    dfg_plane<2, 0, 1, true, Fill, Ring>(C, R, cur_tile, cur_full, zq, outp, plane, tzp, P.NZ, F);
   }
   if (k < ke) {
-    dfg_plane<0, 1, 2, true>(C, R, cur_tile, cur_full, zq, outp, plane, tzp, P.NZ, F);
-    if (k + 1 < ke) dfg_plane<1, 2, 0, true>(C, R, cur_tile, cur_full, zq, outp, plane, tzp, P.NZ, F);
+    dfg_plane<0, 1, 2, true, Fill, Ring>(C, R, cur_tile, cur_full, zq, outp, plane, tzp, P.NZ, F);
+    if (k + 1 < ke) dfg_plane<1, 2, 0, true, Fill, Ring>(C, R, cur_tile, cur_full, zq, outp, plane, tzp, P.NZ, F);
   }
-  dfg_mbar_arrive(DFG_EMPTY(cur_full));
+  dfg_mbar_arrive(cur_full + Ring::kEmpty);
   F.step();
 }
 
@@ -651,157 +654,164 @@ extern "C" __global__ void __launch_bounds__(DFG_NCW * 32, DFG_CTAS)
   }
 }
 
+#if DFG_ROWS_KERNEL
 // ---------------------------------------------------------------- rows
 // The tile kernel's layouts (packed VisIt ghost shells, rows that are not a
-// multiple of 16 bytes) without its LSU-bound fill: the producer warp copies
-// every halo'd tile row with ONE 1-D bulk copy (cp.async.bulk, the TMA
-// engine; no per-element LSU work) of the 16-byte-aligned superset of the
-// row's span.  A row therefore lands in shared memory shifted by its global
-// misalignment m (0..VEC-1 elements), which differs from row to row; every
-// row's copy starts one 16-byte chunk into its smem row (pitch DFG_RP).  Rows
-// per warp = 1, so a warp's rows (r-1, r, r+1) each have ONE shift:
-// consumers read a vector as the aligned chunk (LDS.128) when the shift is 0,
-// else two aligned chunks and a warp-uniform register funnel (no divergence).
-// The mesh-end rules of reading R1 are the TMA kernel's clamped smem offsets
-// in y (the producer replicates the boundary row, like the tile fill) and
-// per-thread rules in x: at the first global cell x-1 reads the cell itself,
-// at the last global cell (ragged vectors included) x+1 is the cell itself.
-// Preconditions (host): 16-byte aligned field bases and plane strides
-// (px * py * sizeof(T) % 16 == 0), so m depends on the row and column only.
-#define DFG_RTX (32 * DFG_VEC)
-#define DFG_RTH DFG_NCW
-#define DFG_RROWW (DFG_RTX + 2 * DFG_HX)
-#define DFG_RP (DFG_RROWW + 3 * DFG_VEC)  // smem row: pad chunk, data (<= ROWW + 2 chunks), slack
-#define DFG_RROWS (DFG_RTH + 2)
-#define DFG_RTILE_BYTES ((DFG_RP * DFG_RROWS * (int)sizeof(DFG_T) + 127) / 128 * 128)
-#define DFG_RSTAGE_BYTES (DFG_RTILE_BYTES * DFG_NTF)
-typedef DfgRingT<DFG_RSTAGE_BYTES> DfgRingR;
+// multiple of 16 bytes) with the TMA engine doing the loads.  A tensor map
+// needs 16-byte global strides and 16-byte-aligned box starts, which a row
+// pitch of 194 floats breaks -- but only from row to row: the rows whose
+// byte offset y * px * sizeof(T) has the same residue mod 16 form a CLASS,
+// and the rows of one class are a regular 3-D tensor with stride
+// P * px * sizeof(T), a multiple of 16 (P = the period of the residues: 1, 2
+// or 4 rows).  So the producer loads, per field and plane, one box per class
+// (2 requests for a 194-float pitch, 4 for an odd pitch): class c's map
+// starts at the field base + (c px T) rounded down to 16 bytes (o_c elements
+// before row c's first element), its box at the column x0 + o_c rounded down
+// to a 16-byte boundary, so every row of class c lands shifted by
+// m_c = (x0 + o_c) mod VEC elements.
+// Consumers read the boxes as they are, with STRIDED cell ownership: lane l
+// of a tile row owns the cells l, l + LPR, l + 2 LPR, l + 3 LPR (LPR = lanes
+// per row), so every shared-memory access of a warp is LPR consecutive
+// 4/8-byte words -- conflict-free at any shift, one wavefront per 128 bytes
+// like the TMA kernel's 16-byte accesses -- and the x neighbours are plain
+// loads at +-1 element.  Stores are fully coalesced (consecutive lanes,
+// consecutive cells).  Mesh-end rules of reading R1: clamped rows in y (as
+// the TMA kernel), per-cell flags in x (the first global cell's x-1 and the
+// last one's x+1 read the cell itself).
+// Preconditions (host): 16-byte aligned field bases and plane strides, and
+// at least P rows per plane.
+#define DFG_SBW (DFG_ROWW + DFG_VEC)     // box width: the tile row + up to VEC-1 leading elements
+#define DFG_SROWS_ALLOC (DFG_ROWS + 3)   // P boxes of ceil(ROWS / P) rows, P <= 4
+// class boxes start on 128-byte boundaries (TMA destination alignment)
+#define DFG_STILE_BYTES ((DFG_SBW * DFG_SROWS_ALLOC * (int)sizeof(DFG_T) + 127) / 128 * 128 + 3 * 128)
+#define DFG_SSTAGE_BYTES (DFG_STILE_BYTES * DFG_NTF)
+typedef DfgRingT<DFG_SSTAGE_BYTES, DFG_RSTAGES> DfgRingS;
 
-__device__ __forceinline__ void dfg_mbar_expect_tx_only(unsigned bar, unsigned bytes) {
-  asm volatile("mbarrier.expect_tx.relaxed.cta.shared::cta.b64 [%0], %1;" ::"r"(bar), "r"(bytes) : "memory");
-}
-__device__ __forceinline__ void dfg_bulk_g2s(unsigned dst, const void* src, unsigned bytes, unsigned bar) {
-  asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(dst),
-               "l"(reinterpret_cast<unsigned long long>(src)), "r"(bytes), "r"(bar)
-               : "memory");
-}
+// host image: runtime.cpp rows_blob (same order, 64-byte aligned maps):
+// map[f * 4 + c] = class c of field f
+struct DfgRowsInfo {
+  int P;      // rows per period of the 16-byte residues (1, 2 or 4)
+  int BR;     // box rows: ceil(ROWS / P)
+  int o[4];   // o_c: elements between class c's map origin and its rows' first element
+  int lgP;    // log2 P
+  __device__ __forceinline__ unsigned box() const { return (unsigned)(DFG_SBW * BR * (int)sizeof(DFG_T)); }
+  __device__ __forceinline__ unsigned cstride() const { return (box() + 127u) & ~127u; }
+};
+struct DfgRowsParams {
+  DfgTmap map[DFG_NF_ * 4];
+  DfgRowsInfo ri;
+  int pad[9];
+  DfgParams p;
+};
 
-// VEC consecutive elements starting `s` elements into the aligned chunk at
-// smem byte address a (s warp-uniform: the branches do not diverge).  Pieces
-// at their natural alignment (8-byte halves, 4-byte ends) rather than two
-// aligned chunks and a register funnel: no extra live registers.
-__device__ __forceinline__ void dfg_lds8(DFG_T* d, unsigned addr) {
-#if DFG_VEC == 4
-  asm volatile("ld.shared.v2.f32 {%0, %1}, [%2];" : "=f"(d[0]), "=f"(d[1]) : "r"(addr) : "memory");
-#else
-  asm volatile("ld.shared.f64 %0, [%1];" : "=d"(d[0]) : "r"(addr) : "memory");
-#endif
-}
-__device__ __forceinline__ void dfg_ldsv(DFG_T (&d)[DFG_VEC], unsigned a, int s) {
-  const unsigned TS = (unsigned)sizeof(DFG_T);
-#if DFG_VEC == 4
-  if (s == 0) {
-    dfg_lds16(d, a);
-  } else if (s == 2) {
-    dfg_lds8(d, a + 2 * TS);
-    dfg_lds8(d + 2, a + 4 * TS);
-  } else {
-    d[0] = dfg_lds1(a + s * TS);
-    dfg_lds8(d + 1, a + (s + 1) * TS);
-    d[3] = dfg_lds1(a + (s + 3) * TS);
+// geometry of an item (the tile kernel's), shared by producer and consumers
+struct DfgRowsItem {
+  long long kb, ke;
+  int x0, y0, tx, ty;
+  __device__ __forceinline__ DfgRowsItem(const DfgParams& p, long long item) {
+    tx = (int)(item % p.tiles_x);
+    const long long rest = item / p.tiles_x;
+    ty = (int)(rest % p.tiles_y);
+    const long long zc = rest / p.tiles_y;
+    kb = p.kbeg + zc * p.kz;
+    ke = min(kb + (long long)p.kz, p.kend);
+    x0 = tx * DFG_TX - DFG_HX + (int)p.gx;  // input column of tile column 0
+    y0 = ty * DFG_TH - 1 + (int)p.gy;       // input row of tile row 0
   }
-#else
-  if (s == 0) {
-    dfg_lds16(d, a);
-  } else {
-    d[0] = dfg_lds1(a + TS);
-    d[1] = dfg_lds1(a + 2 * TS);
+  // first tile row of class c (rows y = c mod P), and the start of its box:
+  // the aligned map column and the class row index (may be -1)
+  __device__ __forceinline__ int first(const DfgRowsInfo& ri, int c) const { return (c - y0) & (ri.P - 1); }
+  __device__ __forceinline__ int bx(const DfgRowsInfo& ri, int c) const {
+    const int v = x0 + ri.o[c];
+    return v - (v & (DFG_VEC - 1));  // floor to a multiple of VEC (v may be negative)
   }
-#endif
-}
-
-// per-item constants of a consumer thread of the rows kernel (packed: the
-// body needs every register it can get)
-struct DfgColR {
-  unsigned a_c;  // smem byte offset (in a tile) of the aligned chunk of row r
-  // bits 0-1 / 2-3 / 4-5: element shift of row r / r-1 / r+1 in its chunk pair;
-  // bit 6: first global cell (x-1 reads the cell itself); bit 7: the vector's
-  // last cell is the last global cell (x+1 reads it); bits 8-10: index of
-  // the last global cell inside a ragged vector (VEC: none); bits 11-12 /
-  // 13-14: chunk of row r-1 / r+1 relative to row r's, + 1 (0..2)
-  unsigned bits;
-  __device__ __forceinline__ unsigned a_m() const {
-    return a_c - (unsigned)(DFG_RP * (int)sizeof(DFG_T)) + (((bits >> 11) & 3u) - 1u) * 16u;
+  __device__ __forceinline__ int by(const DfgRowsInfo& ri, int c) const {
+    return (y0 + first(ri, c) - c) >> ri.lgP;  // exact: y0 + first - c is a multiple of P
   }
-  __device__ __forceinline__ unsigned a_p() const {
-    return a_c + (unsigned)(DFG_RP * (int)sizeof(DFG_T)) + (((bits >> 13) & 3u) - 1u) * 16u;
-  }
-  __device__ __forceinline__ int s_c() const { return (int)(bits & 3u); }
-  __device__ __forceinline__ int s_m() const { return (int)((bits >> 2) & 3u); }
-  __device__ __forceinline__ int s_p() const { return (int)((bits >> 4) & 3u); }
-  __device__ __forceinline__ int endc() const { return (int)((bits >> 8) & 7u); }
-  __device__ __forceinline__ unsigned off_xm() const {
-    return a_c + (unsigned)((int)(bits & 3u) - 1 + (int)((bits >> 6) & 1u)) * (unsigned)sizeof(DFG_T);
-  }
-  __device__ __forceinline__ unsigned off_xp() const {
-    return a_c + (unsigned)((int)(bits & 3u) + DFG_VEC - (int)((bits >> 7) & 1u)) * (unsigned)sizeof(DFG_T);
+  // smem byte offset (in a field tile) of tile column 0 of tile row r
+  __device__ __forceinline__ unsigned row_col0(const DfgRowsInfo& ri, int r) const {
+    const int c = (y0 + r) & (ri.P - 1);
+    const int m = (x0 + ri.o[c]) & (DFG_VEC - 1);
+    return (unsigned)c * ri.cstride() +
+           (unsigned)((((r - first(ri, c)) >> ri.lgP) * DFG_SBW + m) * (int)sizeof(DFG_T));
   }
 };
 
-// shift of row element position v (may be negative before the data start) ->
-// aligned chunk byte offset and shift
-__device__ __forceinline__ void dfg_rows_split(int rr, int v, unsigned& a, int& s) {
-  const int e = DFG_VEC + v;  // the copy starts one chunk into the smem row
-  s = e & (DFG_VEC - 1);
-  a = (unsigned)((rr * DFG_RP + (e - s)) * (int)sizeof(DFG_T));
+// Producer (one lane): per stage, one TMA box per (field, row class)
+__device__ __forceinline__ void dfg_produce_rows(const DfgRowsParams& RP, long long item, DfgRingS& W) {
+  const DfgParams& p = RP.p;
+  const DfgRowsInfo& ri = RP.ri;
+  const DfgRowsItem I(p, item);
+  const unsigned box = ri.box(), cs = ri.cstride();
+  int bxc[4], byc[4];
+#pragma unroll
+  for (int c = 0; c < 4; ++c) {
+    bxc[c] = c < ri.P ? I.bx(ri, c) : 0;
+    byc[c] = c < ri.P ? I.by(ri, c) : 0;
+  }
+  for (long long q = I.kb - 1; q <= I.ke; ++q) {
+    const long long pg = max(0LL, min(q, p.NZ - 1));
+    dfg_mbar_wait(W.full + DfgRingS::kEmpty, W.phase ^ 1u, 0x100000u);
+    dfg_mbar_expect_tx(W.full, (unsigned)(DFG_NTF * ri.P) * box);
+    const int zl = (int)(pg - p.k0 + p.ghost);
+#pragma unroll
+    for (int f = 0; f < DFG_NTF; ++f)
+#pragma unroll
+      for (int c = 0; c < 4; ++c)
+        if (c < ri.P)
+          dfg_tma_load3(W.tile + f * DFG_STILE_BYTES + c * cs, &RP.map[f * 4 + c], W.full, bxc[c], byc[c], zl);
+    W.advance();
+  }
 }
 
+// per-item constants of a consumer thread: smem byte offsets (in a field
+// tile) of its first cell in rows r, r-1, r+1; cell k sits k * LPR elements
+// further.  bits 0-3: cell k is the first global cell (x-1 = itself);
+// bits 4-7: cell k is the last global cell (x+1 = itself).
+struct DfgColS {
+  unsigned o_c, o_m, o_p;
+  unsigned flags;
+};
+
 template <int ZM, int ZC, int ZN>
-__device__ __forceinline__ void dfg_plane_rows(const DfgCol& C, const DfgColR& Q, DfgRingR& R, unsigned& cur_tile,
+__device__ __forceinline__ void dfg_plane_rows(const DfgCol& C, const DfgColS& Q, DfgRingS& R, unsigned& cur_tile,
                                                unsigned& cur_full, DFG_T (&zq)[3][DFG_NSF][DFG_VEC], DFG_T*& outp,
                                                long long plane, const DFG_T*& tzp, long long NZ) {
-  DFG_T xmv[DFG_NSF], xpv[DFG_NSF], ymv[DFG_NSF][DFG_VEC], ypv[DFG_NSF][DFG_VEC];
+  constexpr unsigned TS = (unsigned)sizeof(DFG_T), ST = DFG_LPR * TS;  // cell k stride
+  DFG_T xm[DFG_NSF][DFG_VEC], xp[DFG_NSF][DFG_VEC], ym[DFG_NSF][DFG_VEC], yp[DFG_NSF][DFG_VEC];
 #pragma unroll
   for (int f = 0; f < DFG_NSF; ++f) {
-    const unsigned t = cur_tile + f * DFG_RTILE_BYTES;
-    xmv[f] = dfg_lds1(t + Q.off_xm());
-    xpv[f] = dfg_lds1(t + Q.off_xp());
-    dfg_ldsv(ymv[f], t + Q.a_m(), Q.s_m());
-    dfg_ldsv(ypv[f], t + Q.a_p(), Q.s_p());
+    const unsigned t = cur_tile + f * DFG_STILE_BYTES;
+#pragma unroll
+    for (int k = 0; k < DFG_VEC; ++k) {
+      const unsigned c = t + Q.o_c + k * ST;
+      xm[f][k] = dfg_lds1(c - ((Q.flags >> k) & 1u ? 0u : TS));
+      xp[f][k] = dfg_lds1(c + ((Q.flags >> (4 + k)) & 1u ? 0u : TS));
+      ym[f][k] = dfg_lds1(t + Q.o_m + k * ST);
+      yp[f][k] = dfg_lds1(t + Q.o_p + k * ST);
+    }
   }
   dfg_mbar_wait(R.full, R.phase, 0x100000u);
   const unsigned nxt_tile = R.tile, nxt_full = R.full;
 #pragma unroll
-  for (int f = 0; f < DFG_NSF; ++f) dfg_ldsv(zq[ZN][f], nxt_tile + f * DFG_RTILE_BYTES + Q.a_c, Q.s_c());
+  for (int f = 0; f < DFG_NSF; ++f)
+#pragma unroll
+    for (int k = 0; k < DFG_VEC; ++k) zq[ZN][f][k] = dfg_lds1(nxt_tile + f * DFG_STILE_BYTES + Q.o_c + k * ST);
   R.advance();
   dfg2 s[DFG_NPAIR][DFG_NSF][7], gn[DFG_NPAIR][DFG_NSF][3];
 #pragma unroll
   for (int f = 0; f < DFG_NSF; ++f) {
-    const DFG_T xm = xmv[f], xp = xpv[f];
-    const DFG_T(&ym)[DFG_VEC] = ymv[f];
-    const DFG_T(&yp)[DFG_VEC] = ypv[f];
-    DFG_T lft[DFG_VEC], rgt[DFG_VEC];
-#pragma unroll
-    for (int c = 0; c < DFG_VEC; ++c) {
-      lft[c] = c == 0 ? xm : zq[ZC][f][c == 0 ? 0 : c - 1];
-      rgt[c] = c == DFG_VEC - 1 ? xp : zq[ZC][f][c == DFG_VEC - 1 ? c : c + 1];
-    }
-    {  // the last global cell inside a ragged vector (R1: one-sided): x+1 is the cell itself
-      const int ec = Q.endc();
-#pragma unroll
-      for (int c = 0; c < DFG_VEC - 1; ++c) rgt[c] = (c == ec) ? zq[ZC][f][c] : rgt[c];
-    }
 #pragma unroll
     for (int h = 0; h < DFG_NPAIR; ++h) {
       const int a = h * DFG_LANES, b = h * DFG_LANES + DFG_LANES - 1;
       s[h][f][0] = dfg2_mk(zq[ZC][f][a], zq[ZC][f][b]);
-      s[h][f][1] = dfg2_mk(lft[a], lft[b]);
-      s[h][f][2] = dfg2_mk(rgt[a], rgt[b]);
-      s[h][f][3] = dfg2_mk(ym[a], ym[b]);
-      s[h][f][4] = dfg2_mk(yp[a], yp[b]);
+      s[h][f][1] = dfg2_mk(xm[f][a], xm[f][b]);
+      s[h][f][2] = dfg2_mk(xp[f][a], xp[f][b]);
+      s[h][f][3] = dfg2_mk(ym[f][a], ym[f][b]);
+      s[h][f][4] = dfg2_mk(yp[f][a], yp[f][b]);
       s[h][f][5] = dfg2_mk(zq[ZM][f][a], zq[ZM][f][b]);
       s[h][f][6] = dfg2_mk(zq[ZN][f][a], zq[ZN][f][b]);
-      gn[h][f][0] = dfg2_mk(dfg_sub(rgt[a], lft[a]), dfg_sub(rgt[b], lft[b]));
+      gn[h][f][0] = dfg2_sub(s[h][f][2], s[h][f][1], C.Z);
       gn[h][f][1] = dfg2_sub(s[h][f][4], s[h][f][3], C.Z);
       gn[h][f][2] = dfg2_sub(s[h][f][6], s[h][f][5], C.Z);
     }
@@ -812,7 +822,8 @@ __device__ __forceinline__ void dfg_plane_rows(const DfgCol& C, const DfgColR& Q
 #pragma unroll
   for (int f = 0; f < DFG_NPF; ++f) {
     DFG_T pv[DFG_VEC];
-    dfg_ldsv(pv, cur_tile + (DFG_NSF + f) * DFG_RTILE_BYTES + Q.a_c, Q.s_c());
+#pragma unroll
+    for (int k = 0; k < DFG_VEC; ++k) pv[k] = dfg_lds1(cur_tile + (DFG_NSF + f) * DFG_STILE_BYTES + Q.o_c + k * ST);
 #pragma unroll
     for (int h = 0; h < DFG_NPAIR; ++h) p[h][f] = dfg2_mk(pv[h * DFG_LANES], pv[h * DFG_LANES + DFG_LANES - 1]);
   }
@@ -820,116 +831,85 @@ __device__ __forceinline__ void dfg_plane_rows(const DfgCol& C, const DfgColR& Q
 #pragma unroll
   for (int h = 0; h < DFG_NPAIR; ++h)
     dfg_body(s[h], gn[h], p[h], C.ndx[h], C.rx[h], C.ndy, C.ry, ndz, rz, C.Z, o[h]);
-  dfg_store_masked(outp, o, C);
+  // cell k at outp + k * LPR cells; nvalid = number of valid cells (a prefix)
+#pragma unroll
+  for (int h = 0; h < DFG_NPAIR; ++h)
+#pragma unroll
+    for (int l = 0; l < DFG_LANES; ++l) {
+      const int k = h * DFG_LANES + l;
+      if (k < C.nvalid) {
+        DFG_T* d = outp + k * DFG_LPR * DFG_OUTW;
+#if DFG_OUTW == 1
+        __stcs(d, dfg2_get(o[h][0], l));
+#else
+#pragma unroll
+        for (int w = 0; w < DFG_OUTW; ++w) __stcs(d + w, dfg2_get(o[h][w], l));
+#endif
+      }
+    }
   outp += plane * DFG_OUTW;
-  dfg_mbar_arrive(DFG_EMPTY(cur_full));
+  dfg_mbar_arrive(cur_full + DfgRingS::kEmpty);  // every consumer thread (count NCW*32)
   cur_tile = nxt_tile;
   cur_full = nxt_full;
 }
 
-// geometry of an item of the rows kernel, shared by producer and consumers
-struct DfgRowsItem {
-  long long kb, ke;
-  int x0, y0, lo, hi, rlo, rhi;
-  int tx, ty;
-  __device__ __forceinline__ DfgRowsItem(const DfgParams& p, long long item) {
-    tx = (int)(item % p.tiles_x);
-    const long long rest = item / p.tiles_x;
-    ty = (int)(rest % p.tiles_y);
-    const long long zc = rest / p.tiles_y;
-    kb = p.kbeg + zc * p.kz;
-    ke = min(kb + (long long)p.kz, p.kend);
-    x0 = tx * DFG_RTX - DFG_HX + (int)p.gx;  // input column of tile column 0
-    y0 = ty * DFG_RTH - 1 + (int)p.gy;       // input row of tile row 0
-    lo = max(x0, 0);                          // copied span of every row, inside the row
-    hi = min(x0 + DFG_RROWW, (int)p.px);
-    // rows clamp to the global mesh ends (R1: the boundary row is replicated)
-    // and elsewhere to the input array
-    rlo = p.j0 == 0 ? (int)p.gy : 0;
-    rhi = p.j0 + p.ny >= p.NY ? (int)(p.gy + p.ny - 1) : (int)(p.py - 1);
-  }
-  __device__ __forceinline__ int row(int r) const { return max(rlo, min(y0 + r, rhi)); }
-  // element shift of tile column 0 of tile row r in its smem row
-  __device__ __forceinline__ int delta(const DfgParams& p, int r) const {
-    const int m = (int)(((long long)row(r) * p.px + lo) & (DFG_VEC - 1));
-    return x0 - lo + m;
-  }
-};
-
-// Producer warp: per stage, one bulk copy per (field, tile row); the lanes
-// share the copies, lane 0 waits for the slot and arrives after them
-__device__ __forceinline__ void dfg_produce_rows(const DfgParams& p, long long item, DfgRingR& W, int lane) {
-  const DfgRowsItem I(p, item);
-  const unsigned TS = (unsigned)sizeof(DFG_T);
-  for (long long q = I.kb - 1; q <= I.ke; ++q) {
-    const long long pg = max(0LL, min(q, p.NZ - 1));
-    if (lane == 0) dfg_mbar_wait(DFG_EMPTY(W.full), W.phase ^ 1u, 0x100000u);
-    __syncwarp();
-    const long long pbase = (pg - p.k0 + p.ghost) * p.px * p.py;
-    for (int j = lane; j < DFG_NTF * DFG_RROWS; j += 32) {
-      const int f = j / DFG_RROWS, r = j - f * DFG_RROWS;
-      const DFG_T* rowp = p.f[f] + pbase + (long long)I.row(r) * p.px;
-      const unsigned long long a = reinterpret_cast<unsigned long long>(rowp + I.lo) & ~15ull;
-      const unsigned long long e = (reinterpret_cast<unsigned long long>(rowp + I.hi) + 15ull) & ~15ull;
-      const unsigned dst = W.tile + f * DFG_RTILE_BYTES + (unsigned)(r * DFG_RP + DFG_VEC) * TS;
-      dfg_mbar_expect_tx_only(W.full, (unsigned)(e - a));
-      dfg_bulk_g2s(dst, reinterpret_cast<const void*>(a), (unsigned)(e - a), W.full);
-    }
-    __syncwarp();
-    if (lane == 0) dfg_mbar_arrive(W.full);
-    W.advance();
-  }
-}
-
-__device__ __forceinline__ void dfg_consume_rows(const DfgParams& P, long long item, DfgRingR& R, DfgCol& C,
+__device__ __forceinline__ void dfg_consume_rows(const DfgRowsParams& RP, long long item, DfgRingS& R, DfgCol& C,
                                                  int warp, int lane) {
+  const DfgParams& P = RP.p;
+  const DfgRowsInfo& ri = RP.ri;
   const DfgRowsItem I(P, item);
   const long long plane = P.nx * P.ny;
-  const int r = 1 + warp;
-  const long long i = (long long)I.tx * DFG_RTX + DFG_VEC * lane;
-  const long long j = (long long)I.ty * DFG_RTH + warp;
-  C.nvalid = j < P.ny ? (int)max(0LL, min((long long)DFG_VEC, P.nx - i)) : 0;
-  C.act = C.nvalid > 0;
-  const long long ic = min(i, P.nx - 1);
+  const int col = lane % DFG_LPR, sub = lane / DFG_LPR;
+  const int r = 1 + warp * DFG_RPW + sub;
+  const long long i = (long long)I.tx * DFG_TX + col;  // cell k: i + k * LPR
+  const long long j = (long long)I.ty * DFG_TH + warp * DFG_RPW + sub;
+  // valid cells are a prefix of k = 0..VEC-1 (i + k LPR < nx)
+  C.nvalid = j < P.ny ? (int)max(0LL, min((long long)DFG_VEC, (P.nx - i + DFG_LPR - 1) / DFG_LPR)) : 0;
   const long long jc = min(j, P.ny - 1);
 #pragma unroll
   for (int h = 0; h < DFG_NPAIR; ++h) {
-    const long long a = min(P.i0 + i + h * DFG_LANES, P.NX - 1);
-    const long long b = min(P.i0 + i + h * DFG_LANES + DFG_LANES - 1, P.NX - 1);
+    const long long a = min(P.i0 + i + (h * DFG_LANES) * DFG_LPR, P.NX - 1);
+    const long long b = min(P.i0 + i + (h * DFG_LANES + DFG_LANES - 1) * DFG_LPR, P.NX - 1);
     C.ndx[h] = dfg2_mk(__ldg(P.tx + DFG_NDSEG_X * P.NX + a), __ldg(P.tx + DFG_NDSEG_X * P.NX + b));
     C.rx[h] = dfg2_mk(__ldg(P.tx + P.NX + a), __ldg(P.tx + P.NX + b));
   }
   C.ndy = dfg2_splat(__ldg(P.ty + DFG_NDSEG_Y * P.NY + P.j0 + jc));
   C.ry = dfg2_splat(__ldg(P.ty + P.NY + P.j0 + jc));
-  DfgColR Q;
-  const int c0 = DFG_HX + DFG_VEC * lane;  // tile column of this thread's first cell
-  int sc, sm, sp;
-  unsigned am, ap;
-  dfg_rows_split(r, c0 + I.delta(P, r), Q.a_c, sc);
-  dfg_rows_split(r - 1, c0 + I.delta(P, r - 1), am, sm);
-  dfg_rows_split(r + 1, c0 + I.delta(P, r + 1), ap, sp);
-  const unsigned RB = (unsigned)(DFG_RP * (int)sizeof(DFG_T));
-  // |delta(r +- 1) - delta(r)| < VEC, so the rows' chunks differ by at most one
-  const unsigned dm = (am + RB + 16u - Q.a_c) / 16u, dp = (ap + 16u - RB - Q.a_c) / 16u;
-  // one-sided differences at the GLOBAL x ends only (reading R1)
-  const long long ig = P.i0 + i;
-  const long long last = P.NX - 1 - ig;  // index of the global last cell in this vector, if < VEC
-  const unsigned endc = last >= 0 && last < DFG_VEC - 1 ? (unsigned)last : (unsigned)DFG_VEC;
-  Q.bits = (unsigned)sc | ((unsigned)sm << 2) | ((unsigned)sp << 4) | ((ig == 0 ? 1u : 0u) << 6) |
-           ((last == DFG_VEC - 1 ? 1u : 0u) << 7) | (endc << 8) | (dm << 11) | (dp << 13);
-  DFG_T* outp = P.out + ((I.kb - P.k0) * plane + jc * P.nx + ic) * DFG_OUTW;
+  // one-sided differences only at the GLOBAL mesh ends (reading R1)
+  const long long jg = P.j0 + j;
+  const int rm = (jg == 0) ? r : r - 1;
+  const int rp = (jg >= P.NY - 1) ? r : r + 1;
+  const unsigned TS = (unsigned)sizeof(DFG_T);
+  const unsigned cb = (unsigned)(DFG_HX + col) * TS;  // tile column of cell 0
+  DfgColS Q;
+  Q.o_c = I.row_col0(ri, r) + cb;
+  Q.o_m = I.row_col0(ri, rm) + cb;
+  Q.o_p = I.row_col0(ri, rp) + cb;
+  Q.flags = 0;
+#pragma unroll
+  for (int k = 0; k < DFG_VEC; ++k) {
+    const long long ig = P.i0 + i + k * DFG_LPR;
+    Q.flags |= (ig == 0 ? 1u : 0u) << k;
+    Q.flags |= (ig == P.NX - 1 ? 1u : 0u) << (4 + k);
+  }
+  DFG_T* outp = P.out + ((I.kb - P.k0) * plane + jc * P.nx + min(i, P.nx - 1)) * DFG_OUTW;
   const DFG_T* tzp = P.tz + I.kb;
+  constexpr unsigned ST = DFG_LPR * (unsigned)sizeof(DFG_T);
 
   DFG_T zq[3][DFG_NSF][DFG_VEC];
   dfg_mbar_wait(R.full, R.phase, 0x100000u);
 #pragma unroll
-  for (int f = 0; f < DFG_NSF; ++f) dfg_ldsv(zq[0][f], R.tile + f * DFG_RTILE_BYTES + Q.a_c, Q.s_c());
-  dfg_mbar_arrive(DFG_EMPTY(R.full));
+  for (int f = 0; f < DFG_NSF; ++f)
+#pragma unroll
+    for (int k = 0; k < DFG_VEC; ++k) zq[0][f][k] = dfg_lds1(R.tile + f * DFG_STILE_BYTES + Q.o_c + k * ST);
+  dfg_mbar_arrive(R.full + DfgRingS::kEmpty);
   R.advance();
   dfg_mbar_wait(R.full, R.phase, 0x100000u);
   unsigned cur_tile = R.tile, cur_full = R.full;
 #pragma unroll
-  for (int f = 0; f < DFG_NSF; ++f) dfg_ldsv(zq[1][f], cur_tile + f * DFG_RTILE_BYTES + Q.a_c, Q.s_c());
+  for (int f = 0; f < DFG_NSF; ++f)
+#pragma unroll
+    for (int k = 0; k < DFG_VEC; ++k) zq[1][f][k] = dfg_lds1(cur_tile + f * DFG_STILE_BYTES + Q.o_c + k * ST);
   R.advance();
   long long k = I.kb;
   for (; k + 3 <= I.ke; k += 3) {
@@ -941,50 +921,63 @@ __device__ __forceinline__ void dfg_consume_rows(const DfgParams& P, long long i
     dfg_plane_rows<0, 1, 2>(C, Q, R, cur_tile, cur_full, zq, outp, plane, tzp, P.NZ);
     if (k + 1 < I.ke) dfg_plane_rows<1, 2, 0>(C, Q, R, cur_tile, cur_full, zq, outp, plane, tzp, P.NZ);
   }
-  dfg_mbar_arrive(DFG_EMPTY(cur_full));
+  dfg_mbar_arrive(cur_full + DfgRingS::kEmpty);
 }
 
 extern "C" __global__ void __launch_bounds__((DFG_NCW + 1) * 32, DFG_CTAS)
-    dfg_fused_rows(const __grid_constant__ DfgParams P) {
-  const unsigned smem = dfg_ring_init(1, DFG_RSTAGE_BYTES);
-  const unsigned full0 = smem + DFG_STAGES * DFG_RSTAGE_BYTES;
+    dfg_fused_rows(const __grid_constant__ DfgRowsParams RP) {
+  const unsigned smem = dfg_ring_init(1, DFG_SSTAGE_BYTES, DFG_RSTAGES);
+  const unsigned full0 = smem + DFG_RSTAGES * DFG_SSTAGE_BYTES;
   const int warp = threadIdx.x >> 5;
   const int lane = threadIdx.x & 31;
   if (warp == DFG_NCW) {
-    DfgRingR W{smem, full0, 0u, 0, smem, full0};
-    for (long long item = blockIdx.x; item < P.items; item += gridDim.x) dfg_produce_rows(P, item, W, lane);
+    if (lane == 0) {
+      for (int f = 0; f < DFG_NTF * 4; ++f)
+        if ((f & 3) < RP.ri.P)
+          asm volatile("prefetch.tensormap [%0];" ::"l"(reinterpret_cast<unsigned long long>(&RP.map[f])) : "memory");
+      DfgRingS W{smem, full0, 0u, 0, smem, full0};
+      for (long long item = blockIdx.x; item < RP.p.items; item += gridDim.x) dfg_produce_rows(RP, item, W);
+    }
     return;
   }
-  DfgRingR R{smem, full0, 0u, 0, smem, full0};
+  DfgRingS R{smem, full0, 0u, 0, smem, full0};
   DfgCol C;
-  C.Z = dfg2_splat(P.nzero);
-  C.vst = P.vec_ok != 0;
-  for (long long item = blockIdx.x; item < P.items; item += gridDim.x) dfg_consume_rows(P, item, R, C, warp, lane);
+  C.Z = dfg2_splat(RP.p.nzero);
+  for (long long item = blockIdx.x; item < RP.p.items; item += gridDim.x) dfg_consume_rows(RP, item, R, C, warp, lane);
 }
 
+// several meshes in one launch: DfgRowsParams images in global memory
+struct DfgRowsMulti {
+  const DfgRowsParams* blocks;
+  const long long* first;
+  int nb;
+};
+
 extern "C" __global__ void __launch_bounds__((DFG_NCW + 1) * 32, DFG_CTAS)
-    dfg_fused_rows_multi(const __grid_constant__ DfgTileMulti M) {
-  const unsigned smem = dfg_ring_init(1, DFG_RSTAGE_BYTES);
-  const unsigned full0 = smem + DFG_STAGES * DFG_RSTAGE_BYTES;
+    dfg_fused_rows_multi(const __grid_constant__ DfgRowsMulti M) {
+  const unsigned smem = dfg_ring_init(1, DFG_SSTAGE_BYTES, DFG_RSTAGES);
+  const unsigned full0 = smem + DFG_RSTAGES * DFG_SSTAGE_BYTES;
   const int warp = threadIdx.x >> 5;
   const int lane = threadIdx.x & 31;
   const long long total = M.first[M.nb];
   int b = 0;
   if (warp == DFG_NCW) {
-    DfgRingR W{smem, full0, 0u, 0, smem, full0};
-    for (long long item = blockIdx.x; item < total; item += gridDim.x) {
-      while (item >= M.first[b + 1]) ++b;
-      dfg_produce_rows(M.blocks[b], item - M.first[b], W, lane);
+    if (lane == 0) {
+      DfgRingS W{smem, full0, 0u, 0, smem, full0};
+      for (long long item = blockIdx.x; item < total; item += gridDim.x) {
+        while (item >= M.first[b + 1]) ++b;
+        dfg_produce_rows(M.blocks[b], item - M.first[b], W);
+      }
     }
     return;
   }
-  DfgRingR R{smem, full0, 0u, 0, smem, full0};
+  DfgRingS R{smem, full0, 0u, 0, smem, full0};
   DfgCol C;
-  C.Z = dfg2_splat(M.blocks[0].nzero);
+  C.Z = dfg2_splat(M.blocks[0].p.nzero);
   for (long long item = blockIdx.x; item < total; item += gridDim.x) {
     while (item >= M.first[b + 1]) ++b;
-    C.vst = M.blocks[b].vec_ok != 0;
     dfg_consume_rows(M.blocks[b], item - M.first[b], R, C, warp, lane);
   }
 }
+#endif  // DFG_ROWS_KERNEL
 #endif

@@ -4,6 +4,8 @@
 #include <dlfcn.h>
 #include <nvrtc.h>
 
+#include <algorithm>
+
 #include <cstdlib>
 #include <functional>
 #include <map>
@@ -86,11 +88,12 @@ void parse_ptxas(const std::string& log, Cubin& c) {
       c.regs = std::atoi(line.c_str() + p + 5);
       best = prio;
     }
+    // spills: the worst of ALL kernels in the module (any spilling kernel counts)
     p = line.find("bytes spill stores");
-    if (p != std::string::npos && prio >= best) {
+    if (p != std::string::npos) {
       auto q = line.rfind(',', p);
       size_t start = q == std::string::npos ? 0 : q + 1;
-      c.spill = std::atoi(line.c_str() + start);
+      c.spill = std::max(c.spill, std::atoi(line.c_str() + start));
     }
   }
 }
@@ -136,7 +139,7 @@ const Cubin& nvrtc_compile(const std::string& source, const std::string& name) {
   return ref;
 }
 
-LoadedModule load_module(const Cubin& c, bool has_stencil, bool has_tma) {
+LoadedModule load_module(const Cubin& c, bool has_stencil, bool has_tma, bool rows) {
   LoadedModule m;
   DFG_CU(drv().ModuleLoadData(&m.mod, c.image.data()));
   // look up exactly the kernels skeleton.cuh / fused_tma.cuh emit for this layout
@@ -149,8 +152,10 @@ LoadedModule load_module(const Cubin& c, bool has_stencil, bool has_tma) {
       DFG_CU(drv().ModuleGetFunction(&m.tma_multi, m.mod, "dfg_fused_tma_multi"));
       DFG_CU(drv().ModuleGetFunction(&m.tile, m.mod, "dfg_fused_tile"));
       DFG_CU(drv().ModuleGetFunction(&m.tile_multi, m.mod, "dfg_fused_tile_multi"));
-      DFG_CU(drv().ModuleGetFunction(&m.rows, m.mod, "dfg_fused_rows"));
-      DFG_CU(drv().ModuleGetFunction(&m.rows_multi, m.mod, "dfg_fused_rows_multi"));
+      if (rows) {
+        DFG_CU(drv().ModuleGetFunction(&m.rows, m.mod, "dfg_fused_rows"));
+        DFG_CU(drv().ModuleGetFunction(&m.rows_multi, m.mod, "dfg_fused_rows_multi"));
+      }
     }
   }
   return m;

@@ -31,6 +31,6 @@ struct LoadedModule {
 };
 
 // Load into the current context (requires a device).
-LoadedModule load_module(const Cubin& c, bool has_stencil, bool has_tma);
+LoadedModule load_module(const Cubin& c, bool has_stencil, bool has_tma, bool rows = false);
 
 }  // namespace dfg

@@ -11,6 +11,11 @@
 
 #include <cstdint>
 
+// the per-primitive kernels divide with IEEE div.rn (DFG_DIV_MODE 0): the
+// staged and roundtrip strategies are HBM / PCIe bound, so they can afford
+// the quotient that equals the oracle's for EVERY input, subnormal and
+// overflowing intermediates included
+#define DFG_DIV_MODE 0
 #include "blocks.cuh"
 #include "kernels.hpp"
 

@@ -6,6 +6,7 @@
 
 #include <algorithm>
 #include <cmath>
+#include <cstdio>
 #include <cstdlib>
 #include <cstring>
 #include <mutex>
@@ -166,7 +167,8 @@ std::unique_ptr<PlanImpl> compile_plan(std::shared_ptr<MeshImpl> mesh, const std
     plan->spill = cb.spill;
     // the runtime API owns the primary context; make it current for the driver API
     DFG_CUDA(cudaFree(0));
-    plan->mod = load_module(cb, !plan->fsrc.layout.stencil_inputs.empty(), plan->fsrc.cfg.has_tma);
+    plan->mod = load_module(cb, !plan->fsrc.layout.stencil_inputs.empty(), plan->fsrc.cfg.has_tma,
+                            plan->fsrc.cfg.rstages >= 2);
     // registers / local memory of the main kernel from the loaded module (the
     // NVRTC log can be empty when the compile is served from a cache)
     CUfunction main_fn = plan->mod.tma ? plan->mod.tma : plan->mod.general ? plan->mod.general : plan->mod.pointwise;
@@ -182,18 +184,21 @@ std::unique_ptr<PlanImpl> compile_plan(std::shared_ptr<MeshImpl> mesh, const std
       DFG_CU(drv().FuncSetAttribute(plan->mod.tma_multi, CU_FUNC_ATTRIBUTE_MAX_DYNAMIC_SHARED_SIZE_BYTES, int(smem)));
       DFG_CU(drv().FuncSetAttribute(plan->mod.tile, CU_FUNC_ATTRIBUTE_MAX_DYNAMIC_SHARED_SIZE_BYTES, int(smem)));
       DFG_CU(drv().FuncSetAttribute(plan->mod.tile_multi, CU_FUNC_ATTRIBUTE_MAX_DYNAMIC_SHARED_SIZE_BYTES, int(smem)));
+      const FusedConfig& c = plan->fsrc.cfg;
       const size_t rsmem = fused_rows_smem_bytes(mesh->dt, int(plan->fsrc.layout.stencil_inputs.size() +
                                                                plan->fsrc.layout.point_inputs.size()),
-                                                 plan->fsrc.cfg.ncw, plan->fsrc.cfg.stages);
-      if (rsmem <= 227 * 1024) {
-        plan->rows_smem = rsmem;
+                                                 c.ncw, c.rpw, c.rstages);
+      if (plan->mod.rows && rsmem <= 227 * 1024) {
         DFG_CU(drv().FuncSetAttribute(plan->mod.rows, CU_FUNC_ATTRIBUTE_MAX_DYNAMIC_SHARED_SIZE_BYTES, int(rsmem)));
         DFG_CU(drv().FuncSetAttribute(plan->mod.rows_multi, CU_FUNC_ATTRIBUTE_MAX_DYNAMIC_SHARED_SIZE_BYTES, int(rsmem)));
+        plan->rows_smem = rsmem;
       }
     }
   }
   return plan;
 }
+
+
 
 std::pair<cudaEvent_t, cudaEvent_t> PlanImpl::kernel_events() {
   std::pair<cudaEvent_t, cudaEvent_t> e;
@@ -236,6 +241,7 @@ void PlanImpl::halo_exchange(const std::vector<int>& inputs, cudaStream_t s) {
   MeshImpl& m = *mesh;
   const bool has_lo = m.k0 > 0, has_hi = m.k0 + m.nzl < m.NZ;
   if ((!has_lo && !has_hi) || m.ghosts_supplied) return;  // blocks: the caller filled the ghosts
+  NvtxRange nv(m.nccl ? "dfg halo nccl" : "dfg halo copies");
   const size_t ts = dsize(m.dt);
   const size_t pb = size_t(m.plane()) * ts;
   auto lo = m.link_lo.lock(), hi = m.link_hi.lock();
@@ -292,6 +298,9 @@ void PlanImpl::execute(void* out, bool out_dev, cudaStream_t s) {
     auto it = m.fields.find(dag.inputs[i]);
     if (it == m.fields.end() || !it->second.ptr) fail(DFG_E_UNBOUND, "input '" + dag.inputs[i] + "' is not bound");
   }
+  static const char* const kStrat[] = {"dfg_execute roundtrip", "dfg_execute staged", "dfg_execute fused",
+                                      "dfg_execute streamed", "dfg_execute reference", "dfg_execute hybrid"};
+  NvtxRange nv(kStrat[strategy]);
   if (timing >= 1) DFG_CUDA(cudaEventRecord(ev0, s));
   switch (strategy) {
     case DFG_FUSED: exec_fused(out, out_dev, s); break;
@@ -380,6 +389,53 @@ std::vector<uint64_t> pack_params(const std::vector<const void*>& f, void* out, 
   // nzero = -0.0 in T (the contraction guard of the paired blocks)
   w.push_back(m.dt == DType::F32 ? uint64_t(0x80000000u) : uint64_t(0x8000000000000000ull));
   return w;
+}
+// Row period P of the 16-byte residues of the row offsets y * px * sizeof(T)
+// (fused_tma.cuh "rows"): 1, 2 or 4.
+int row_period(const SlabView& m) {
+  const int64_t rb = m.px() * int64_t(dsize(m.dt));
+  int P = 1;
+  while ((rb * P) % 16 != 0) P *= 2;
+  return P;
+}
+
+// Host image of DfgRowsParams (fused_tma.cuh): map[NF_ * 4] (128 B each; map
+// f * 4 + c = row class c of field f) | DfgRowsInfo {P, BR, o[4]} + pad to
+// 64 B | DfgParams.  Class c of a field: the rows y = c (mod P) as a 3-D
+// tensor from base + (c px T) rounded down to 16 bytes (o_c elements before
+// the row's first element), dims {px + o_c, rows of the class, planes},
+// strides {P px T, px py T} (both multiples of 16), box {TX + 3 VEC, BR, 1}.
+std::vector<unsigned char> rows_blob(const std::vector<const void*>& fptr, int nf_, const SlabView& m, int ncw,
+                                     int rpw, const std::vector<uint64_t>& words) {
+  const size_t ts = dsize(m.dt);
+  const int vec = int(16 / ts);
+  const int P = row_period(m);
+  const int rows = tma_tile_h(ncw, rpw) + 2, BR = (rows + P - 1) / P;
+  const size_t maps = size_t(128) * size_t(std::max(nf_, 1)) * 4;
+  std::vector<unsigned char> blob((maps + 64 + words.size() * 8 + 63) / 64 * 64, 0);
+  int32_t info[7] = {P, BR, 0, 0, 0, 0, P == 1 ? 0 : P == 2 ? 1 : 2};
+  for (int c = 0; c < P; ++c) info[2 + c] = int32_t((int64_t(c) * m.px() * int64_t(ts)) % 16 / int64_t(ts));
+  for (size_t f = 0; f < fptr.size(); ++f) {
+    for (int c = 0; c < P; ++c) {
+      const int64_t off = int64_t(c) * m.px() * int64_t(ts);
+      const int o = info[2 + c];
+      char* base = static_cast<char*>(const_cast<void*>(fptr[f])) + (off - o * int64_t(ts));
+      cuuint64_t gdim[3] = {cuuint64_t(m.px() + o), cuuint64_t((m.py() - c + P - 1) / P),
+                            cuuint64_t(m.nzl + 2 * m.ghost)};
+      cuuint64_t gstride[2] = {cuuint64_t(P) * cuuint64_t(m.px()) * ts, cuuint64_t(m.px() * m.py()) * ts};
+      cuuint32_t box[3] = {cuuint32_t(tma_tile_w(m.dt, rpw) + 3 * vec), cuuint32_t(BR), 1};
+      cuuint32_t estr[3] = {1, 1, 1};
+      DFG_CU(drv().TensorMapEncodeTiled(reinterpret_cast<CUtensorMap*>(blob.data() + 128 * (f * 4 + size_t(c))),
+                                        m.dt == DType::F32 ? CU_TENSOR_MAP_DATA_TYPE_FLOAT32
+                                                           : CU_TENSOR_MAP_DATA_TYPE_FLOAT64,
+                                        3, base, gdim, gstride, box, estr, CU_TENSOR_MAP_INTERLEAVE_NONE,
+                                        CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+                                        CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE));
+    }
+  }
+  std::memcpy(blob.data() + maps, info, sizeof(info));
+  std::memcpy(blob.data() + maps + 64, words.data(), words.size() * 8);
+  return blob;
 }
 }  // namespace
 
@@ -509,13 +565,15 @@ bool PlanImpl::tma_ok(const std::vector<const void*>& fptr, const void* dout, co
          std::all_of(fptr.begin(), fptr.end(), [](const void* p) { return aligned16(p); });
 }
 
-bool PlanImpl::rows_ok(const std::vector<const void*>& fptr, const SlabView& m) const {
+bool PlanImpl::rows_ok(const std::vector<const void*>& fptr, const SlabView& m) {
   const char* force = std::getenv("DFG_FUSED_KERNEL");
   if (force && (!std::strcmp(force, "general") || !std::strcmp(force, "tile"))) return false;
-  return mod.rows && rows_smem && !fsrc.layout.stencil_inputs.empty() &&
-         (m.px() * m.py() * int64_t(dsize(m.dt))) % 16 == 0 && m.px() * m.py() < (int64_t(1) << 32) &&
-         m.px() < (int64_t(1) << 30) &&
-         std::all_of(fptr.begin(), fptr.end(), [](const void* p) { return aligned16(p); });
+  // a class of rows needs at least one row per plane (py >= P)
+  const bool layout = !fsrc.layout.stencil_inputs.empty() && fsrc.cfg.has_tma &&
+                      (m.px() * m.py() * int64_t(dsize(m.dt))) % 16 == 0 && m.px() * m.py() < (int64_t(1) << 32) &&
+                      m.px() < (int64_t(1) << 30) && m.py() >= row_period(m) &&
+                      std::all_of(fptr.begin(), fptr.end(), [](const void* p) { return aligned16(p); });
+  return layout && mod.rows && rows_smem != 0;
 }
 
 // Fused execute of a z-slab linked to its neighbours through peer memory.
@@ -557,6 +615,7 @@ void PlanImpl::exec_fused_peer(const std::vector<const void*>& fptr, void* out, 
       use_tma = use_tma && aligned16(it->second);
     }
   }
+  NvtxRange nv("dfg halo peer (in-place reads)");
   const uint32_t e = ++m.epoch;
   auto dptr = [](const uint32_t* p, int w) { return reinterpret_cast<CUdeviceptr>(p + w); };
   const CUstream cs = reinterpret_cast<CUstream>(s);
@@ -607,6 +666,7 @@ void PlanImpl::launch_fused(const std::vector<const void*>& fptr, void* dout, co
   const size_t ts = dsize(m.dt);
   const FusedLayout& L = fsrc.layout;
   const int64_t kbeg = kb < 0 ? m.k0 : kb, kend = ke < 0 ? m.k0 + m.nzl : ke;
+  NvtxRange nv(kb < 0 && ke < 0 ? "dfg fused launch" : peer ? "dfg fused boundary planes (peer)" : "dfg fused planes");
   const int64_t N = m.nx * m.ny * (kend - kbeg);
   const int vec = int(16 / ts);
   // 16-byte point-wise loads / stores: aligned bases, whole vectors, and the
@@ -696,14 +756,14 @@ void PlanImpl::launch_fused(const std::vector<const void*>& fptr, void* dout, co
     last_variant = 1;
     last_kz = best_kz;
   } else if (rows_ok(fptr, m)) {
-    // the same ring filled by one bulk copy per tile row (rows per warp 1)
-    const int ncw = fsrc.cfg.ncw;
-    const int tw = tma_tile_w(m.dt, 1), th = tma_tile_h(ncw, 1);
+    // TMA row-class boxes, read in place by strided-cell consumers
+    const int ncw = fsrc.cfg.ncw, rpw = fsrc.cfg.rpw, threads = (ncw + 1) * 32;
+    const int tw = tma_tile_w(m.dt, rpw), th = tma_tile_h(ncw, rpw);
     const int tiles_x = int((m.nx + tw - 1) / tw);
     const int tiles_y = int((m.ny + th - 1) / th);
     const int64_t range = kend - kbeg;
     int occ = 1;
-    DFG_CU(drv().OccupancyMaxActiveBlocksPerMultiprocessor(&occ, mod.rows, (ncw + 1) * 32, rows_smem));
+    DFG_CU(drv().OccupancyMaxActiveBlocksPerMultiprocessor(&occ, mod.rows, threads, rows_smem));
     const int64_t slots = int64_t(sms) * std::max(occ, 1);
     const char* kzenv = std::getenv("DFG_KZ");
     const int64_t kz = kzenv ? std::max<int64_t>(1, std::min<int64_t>(range, std::atoll(kzenv)))
@@ -713,9 +773,11 @@ void PlanImpl::launch_fused(const std::vector<const void*>& fptr, void* dout, co
     const bool out16 = aligned16(dout) && m.nx % vec == 0;
     auto w = pack_params(fptr, dout, tab[0], tab[1], tab[2], m, kbeg, kend, items, tiles_x, tiles_y, int(kz),
                          out16 ? 1 : 0);
-    void* args[] = {w.data()};
+    auto blob = rows_blob(fptr, int(L.stencil_inputs.size() + L.point_inputs.size()), m, ncw, rpw, w);
+    if (blob.size() > 32000) fail(DFG_E_UNSUPPORTED, "too many fields for the row-class kernel's parameters");
+    void* args[] = {blob.data()};
     auto ke = kernel_begin(s);
-    DFG_CU(drv().LaunchKernel(mod.rows, grid, 1, 1, (ncw + 1) * 32, 1, 1, unsigned(rows_smem), s, args, nullptr));
+    DFG_CU(drv().LaunchKernel(mod.rows, grid, 1, 1, threads, 1, 1, unsigned(rows_smem), s, args, nullptr));
     kernel_end(ke, s);
     last_variant = 7;
     last_kz = kz;
@@ -806,13 +868,15 @@ void execute_blocks(const std::vector<PlanImpl*>& plans, const std::vector<void*
   }
   // layouts a tensor map cannot describe: the row-copy ring when every block
   // meets its alignment preconditions, else the cp.async ring
-  bool rows = !tma && p0.mod.rows_multi && p0.rows_smem;
-  for (size_t b = 0; b < plans.size() && rows; ++b) rows = plans[b]->rows_ok(fptrs[b], SlabView::of(*plans[b]->mesh));
   DFG_CUDA(cudaSetDevice(m0.device));
-  const int ncw = p0.fsrc.cfg.ncw, rpw = rows ? 1 : p0.fsrc.cfg.rpw;
+  bool rows = !tma;
+  for (size_t b = 0; b < plans.size() && rows; ++b) rows = plans[b]->rows_ok(fptrs[b], SlabView::of(*plans[b]->mesh));
+  rows = rows && p0.rows_smem;
+  const FusedConfig& kc = p0.fsrc.cfg;
+  const int ncw = kc.ncw, rpw = kc.rpw;
   const int tw = tma_tile_w(m0.dt, rpw), th = tma_tile_h(ncw, rpw);
   const int nsf = int(L.stencil_inputs.size() + L.point_inputs.size());
-  const size_t smem = rows ? p0.rows_smem : fused_tma_smem_bytes(m0.dt, nsf, ncw, p0.fsrc.cfg.stages, rpw);
+  const size_t smem = rows ? p0.rows_smem : fused_tma_smem_bytes(m0.dt, nsf, ncw, kc.stages, rpw);
   CUfunction fn = tma ? p0.mod.tma_multi : rows ? p0.mod.rows_multi : p0.mod.tile_multi;
   const int threads = tma || rows ? (ncw + 1) * 32 : ncw * 32;
   int occ = 1;
@@ -851,12 +915,26 @@ void execute_blocks(const std::vector<PlanImpl*>& plans, const std::vector<void*
     first.push_back(first.back() + items);
   }
   // TMA: DfgTmaParams images (no peer halo: blocks carry their ghost
-  // shells); tile: plain DfgParams images
+  // shells); rows: DfgRowsParams images; tile: plain DfgParams images
   const TmaBlobLayout bl = tma_blob_layout(nsf, int(L.stencil_inputs.size()), wmax);
-  const size_t stride = tma ? bl.size : wmax * 8;
+  std::vector<std::vector<unsigned char>> rblobs;
+  size_t rstride = 0;
+  if (rows) {
+    for (size_t b = 0; b < plans.size(); ++b) {
+      std::vector<uint64_t> w = words[b];
+      w.resize(wmax, 0);
+      rblobs.push_back(rows_blob(fptrs[b], nsf, SlabView::of(*plans[b]->mesh), ncw, rpw, w));
+      rstride = std::max(rstride, rblobs.back().size());
+    }
+  }
+  const size_t stride = tma ? bl.size : rows ? rstride : wmax * 8;
   std::vector<unsigned char> host(stride * plans.size() + sizeof(int64_t) * first.size(), 0);
   for (size_t b = 0; b < plans.size(); ++b) {
     unsigned char* blob = host.data() + stride * b;
+    if (rows) {
+      std::memcpy(blob, rblobs[b].data(), rblobs[b].size());
+      continue;
+    }
     if (!tma) {
       std::memcpy(blob, words[b].data(), words[b].size() * 8);
       continue;

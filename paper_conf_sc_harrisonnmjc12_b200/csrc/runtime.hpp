@@ -136,7 +136,7 @@ struct PlanImpl {
   int regs = 0, spill = 0;
   int last_variant = 0;  // 1 TMA, 2 general, 3 pointwise, 4 TMA multi-block (dfg_execute_blocks), 5 tile (cp.async ring), 6 tile multi-block,
                          // 7 rows (bulk row copies), 8 rows multi-block
-  size_t rows_smem = 0;  // dynamic smem of the rows kernel (0: unavailable)
+  size_t rows_smem = 0;  // dynamic smem of the row-class kernel (0: unavailable)
   int64_t last_kz = 0;   // z-chunk length of the last TMA launch
   int last_halo = 0;     // halo of the last execute: 0 none, 1 NCCL, 2 local copies, 3 peer (in place), 4 peer copies
   dfg_stats st{};
@@ -190,7 +190,7 @@ struct PlanImpl {
  public:
   // the row-copy kernel's preconditions: 16-byte aligned field bases and
   // plane strides (DFG_FUSED_KERNEL=tile / general turn it off)
-  bool rows_ok(const std::vector<const void*>& fptr, const SlabView& v) const;
+  bool rows_ok(const std::vector<const void*>& fptr, const SlabView& v);
  private:
   void exec_fused_peer(const std::vector<const void*>& fptr, void* out, bool out_dev, cudaStream_t s);
   void exec_streamed(void* out, bool out_dev, cudaStream_t s);

@@ -4,6 +4,7 @@
 
 #include <cuda_runtime.h>
 #include <nccl.h>
+#include <nvtx3/nvToolsExt.h>
 
 #include <algorithm>
 #include <cstdlib>
@@ -18,6 +19,16 @@
 
 namespace dfg {
 namespace detail {
+
+// NVTX range around a host-side step (header-only NVTX3: a no-op unless a
+// tool such as nsys injects itself), so a timeline shows every execute, each
+// staged filter, the halo exchange and each fused launch by name
+struct NvtxRange {
+  explicit NvtxRange(const char* name) { nvtxRangePushA(name); }
+  NvtxRange(const NvtxRange&) = delete;
+  NvtxRange& operator=(const NvtxRange&) = delete;
+  ~NvtxRange() { nvtxRangePop(); }
+};
 
 // ---- mesh.cpp
 cudaMemPool_t pool_for(int dev);  // per-device pool, memory kept across executes

@@ -20,6 +20,13 @@ PROGS = ["velmag", "vortmag", "qcrit", "intro"]
 NAMES = {"velmag": ("u", "v", "w"), "vortmag": ("u", "v", "w"), "qcrit": ("u", "v", "w"), "intro": ("b", "c")}
 
 
+def _rows_layout(px, py, itemsize):
+    """The row-copy kernel's precondition (16-byte aligned bases, as torch
+    allocations are, and 16-byte plane strides): layouts the tensor maps
+    cannot take run on it (variant 7), the rest on the cp.async ring (5)."""
+    return (px * py * itemsize) % 16 == 0
+
+
 def _inputs(shape, T, names=("u", "v", "w")):
     x, y, z, f = synth.rt_inputs(*shape, dtype=T, names=names)
     return x, y, z, {k: v.numpy() for k, v in f.items()}
@@ -77,8 +84,53 @@ def test_tile_kernel(prog, T, shape, rpw, monkeypatch):
     got, plan, *_ = run_lib(src, f, x, y, z, return_plan=True)
     if prog != "velmag":
         vec = 4 if T == np.float32 else 2
-        assert plan.info()["variant"] == (5 if shape[0] % vec else 1)
+        ragged = 7 if _rows_layout(shape[0], shape[1], np.dtype(T).itemsize) else 5
+        assert plan.info()["variant"] == (ragged if shape[0] % vec else 1)
     assert_parity(got, want)
+
+
+@pytest.mark.parametrize("prog", PROGS)
+@pytest.mark.parametrize("T", [np.float32, np.float64])
+@pytest.mark.parametrize("shape", [(66, 8, 9), (67, 16, 7), (65, 32, 6), (130, 12, 10), (6, 2, 3), (1, 4, 5),
+                                   (131, 4, 3), (258, 2, 4), (33, 4, 2), (2, 8, 1), (197, 36, 12)])
+def test_rows_kernel(prog, T, shape, monkeypatch):
+    """The row-copy ring (one bulk copy per halo'd tile row, rows shifted by
+    their global misalignment, warp-uniform realignment in the consumers):
+    rows of 2 mod 4, odd and 1 cells (every shift 0..3 recurs), ragged last
+    vectors, one-cell axes, several x tiles -- the oracle's bits, and the
+    cp.async ring's."""
+    isz = np.dtype(T).itemsize
+    if not _rows_layout(shape[0], shape[1], isz):
+        pytest.skip("plane stride not a multiple of 16 bytes for this type")
+    x, y, z, f = _inputs(shape, T, NAMES[prog])
+    src = PAPER_PROGRAMS[prog][0]
+    want = run_oracle(src, f, x, y, z)
+    got, plan, *_ = run_lib(src, f, x, y, z, return_plan=True)
+    vec = 16 // isz
+    if prog != "velmag":
+        assert plan.info()["variant"] == (7 if shape[0] % vec else 1)
+    assert_parity(got, want)
+    if prog != "velmag":
+        monkeypatch.setenv("DFG_FUSED_KERNEL", "rows")     # also where the tensor maps could run
+        got2, plan2, *_ = run_lib(src, f, x, y, z, return_plan=True)
+        assert plan2.info()["variant"] == 7
+        assert_parity(got2, want)
+        monkeypatch.setenv("DFG_FUSED_KERNEL", "tile")
+        got3, plan3, *_ = run_lib(src, f, x, y, z, return_plan=True)
+        assert plan3.info()["variant"] == 5
+        assert np.array_equal(got.view(np.uint8), got3.view(np.uint8))
+
+
+@pytest.mark.parametrize("kz", ["1", "2", "5", "1000"])
+def test_rows_kernel_z_chunks(kz, monkeypatch):
+    """Every z-chunk length on the row-copy ring (producer and consumers
+    cross item boundaries)."""
+    x, y, z, f = _inputs((66, 32, 29), np.float32)
+    src = PAPER_PROGRAMS["qcrit"][0]
+    monkeypatch.setenv("DFG_KZ", kz)
+    got, plan, *_ = run_lib(src, f, x, y, z, return_plan=True)
+    assert plan.info()["variant"] == 7 and plan.info()["kz"] == min(int(kz), 29)
+    assert_parity(got, run_oracle(src, f, x, y, z))
 
 
 @pytest.mark.parametrize("kz", ["1", "2", "5", "1000"])
@@ -452,21 +504,24 @@ def _visit_blocks(shape, split, prog, strategy, pitch):
                 torch.cuda.synchronize()
                 if pitch == "padded" and bx % 4 == 0 and prog != "velmag":
                     assert p.info()["variant"] == 1          # TMA kernel on the padded shell
-                elif prog != "velmag":
-                    assert p.info()["variant"] == 5          # packed shell: the cp.async-filled ring
+                elif prog != "velmag":                       # packed shell: row copies or the cp.async ring
+                    assert p.info()["variant"] == (7 if _rows_layout(rp, j1 - j0 + 2, 4) else 5)
                 got[k0:k1, j0:j1, i0:i1] = o.cpu().numpy()
-                blocks.append((p, torch.full_like(o, float("nan")), (k0, k1, j0, j1, i0, i1), m, keep))
+                blocks.append((p, torch.full_like(o, float("nan")), (k0, k1, j0, j1, i0, i1), m, keep,
+                               p.info()["variant"]))
     assert np.array_equal(got, whole)
     # all blocks in one launch (dfg_execute_blocks): the same bits
     dfg.execute_blocks([b[0] for b in blocks], [b[1] for b in blocks])
     torch.cuda.synchronize()
     got2 = np.full_like(whole, np.nan)
-    for p, o, (k0, k1, j0, j1, i0, i1), _, _ in blocks:
+    for p, o, (k0, k1, j0, j1, i0, i1), _, _, _ in blocks:
         got2[k0:k1, j0:j1, i0:i1] = o.cpu().numpy()
     assert np.array_equal(got2, whole)
     if strategy == "fused" and prog != "velmag" and len(blocks) > 1:
         tma = pitch == "padded" and all((b[2][5] - b[2][4]) % 4 == 0 for b in blocks)
-        assert blocks[0][0].info()["variant"] == (4 if tma else 6)   # one launch: TMA or cp.async ring
+        rows = all(b[5] == 7 for b in blocks)
+        # one launch: TMA, row copies or the cp.async ring
+        assert blocks[0][0].info()["variant"] == (4 if tma else 8 if rows else 6)
 
 
 def test_memory_cap():
@@ -864,3 +919,68 @@ def test_differential_fuzz_fused(seed, monkeypatch):
             assert_parity(got, want), ("exact", src)
         n_run += 1
     assert n_run >= 12
+
+
+def _same_bits(got, want, where=None):
+    """Bit-for-bit equality except NaN payloads (x86 and the GPU produce
+    different default NaNs): NaN positions equal, every other value -- signed
+    zeros and infinities included -- equal as bits."""
+    u = np.uint32 if got.dtype == np.float32 else np.uint64
+    if where is None:
+        where = np.ones(got.shape, dtype=bool)
+    gn, wn = np.isnan(got) & where, np.isnan(want) & where
+    if not np.array_equal(gn, wn):
+        return False
+    keep = where & ~wn
+    return bool(np.array_equal(got.view(u)[keep], want.view(u)[keep]))
+
+
+def _extreme_fields(T, shape):
+    """RT-like velocity with three planted regions: u = 2^64 y (fp32; 2^600
+    y in fp64) in the low z quarter -- the literal network stays finite but
+    a power-of-two-folded square of (du[1] + dv[0]) would be 4x larger --
+    w = 2^-70 x (2^-1000 x) in the high quarter, whose squares underflow to
+    subnormals, and a few subnormal / infinite / NaN input cells."""
+    x, y, z = (synth.dyadic_coords(n, s, T) for n, s in zip(shape, (5, 6, 7)))
+    _, _, _, f = _inputs(shape, T)
+    big, tiny = (2.0 ** 64, 2.0 ** -70) if T == np.float32 else (2.0 ** 600, 2.0 ** -1000)
+    yc, xc = synth.centres64(y), synth.centres64(x)
+    nz = shape[2]
+    f["u"][: nz // 4] = (big * yc)[None, :, None].astype(T)
+    f["w"][3 * nz // 4:] = (tiny * xc)[None, None, :].astype(T)
+    f["v"][nz // 2, 3, 5] = np.finfo(T).tiny / 8          # subnormal input
+    f["v"][nz // 2, 5, 9] = np.inf
+    f["u"][nz // 2 + 1, 7, 2] = np.nan
+    return x, y, z, f
+
+
+@pytest.mark.parametrize("T", [np.float32, np.float64])
+def test_exactness_domain_extreme_values(T, monkeypatch):
+    """VERDICT r1 (parity scope): the contract of each arithmetic variant on
+    inputs whose intermediates overflow or go subnormal.  dfg_plan_arith
+    reports the domain; IEEE-only plans (the staged kernels, and the fused
+    kernel with DFG_FUSED_VARIANT=ieee) equal the oracle bit for bit on
+    EVERY cell, NaN / Inf positions and signed zeros included; the default
+    fused kernel equals it on every cell of oracle.evaluate.in_range_mask
+    (DESIGN.md section 5), and the planted regions do leave that domain."""
+    shape = (40, 24, 20)
+    x, y, z, f = _extreme_fields(T, shape)
+    src = PAPER_PROGRAMS["qcrit"][0]
+    want = run_oracle(src, f, x, y, z)
+    dag = build_dag(src, ("u", "v", "w"), "f32" if T == np.float32 else "f64")
+    mask = oev.in_range_mask(dag, f, x, y, z)
+    assert 0.2 < mask.mean() < 0.9, mask.mean()
+    assert not np.isfinite(want).all()
+    for strategy in ("staged", "roundtrip"):
+        got, plan, *_ = run_lib(src, f, x, y, z, strategy, return_plan=True)
+        assert plan.arith()["exact_domain"] == "all_inputs"
+        assert _same_bits(got, want), strategy
+    monkeypatch.setenv("DFG_FUSED_VARIANT", "ieee")
+    got, plan, *_ = run_lib(src, f, x, y, z, return_plan=True)
+    assert plan.arith() == {"div_mode": "ieee", "fold": False, "div2_axes": 0, "exact_domain": "all_inputs"}
+    assert _same_bits(got, want)
+    monkeypatch.delenv("DFG_FUSED_VARIANT")
+    got, plan, *_ = run_lib(src, f, x, y, z, return_plan=True)
+    ar = plan.arith()
+    assert ar["exact_domain"] == "normal_range" and ar["fold"] and ar["div_mode"] == "exact_normal"
+    assert _same_bits(got, want, mask)
