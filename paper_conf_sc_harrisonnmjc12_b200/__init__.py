@@ -176,8 +176,8 @@ class Plan:
         return dfg_dump_dag(self.handle)
 
     def arith(self):
-        """Quotient form, scale folding and the inputs on which the results
-        equal the oracle's (dfg_plan_arith)."""
+        """Quotient form, scale folding and the exactness domain: the inputs
+        on which the results equal the literal network in T (dfg_plan_arith)."""
         from ._dfg import dfg_plan_arith
         return dfg_plan_arith(self.handle)
 

@@ -764,6 +764,14 @@ __device__ __forceinline__ void dfg_produce_rows(const DfgRowsParams& RP, long l
   }
 }
 
+__device__ __forceinline__ void dfg_sts1(unsigned addr, DFG_T v) {
+#if DFG_VEC == 4
+  asm volatile("st.shared.f32 [%0], %1;" ::"r"(addr), "f"(v) : "memory");
+#else
+  asm volatile("st.shared.f64 [%0], %1;" ::"r"(addr), "d"(v) : "memory");
+#endif
+}
+
 // per-item constants of a consumer thread: smem byte offsets (in a field
 // tile) of its first cell in rows r, r-1, r+1; cell k sits k * LPR elements
 // further.  bits 0-3: cell k is the first global cell (x-1 = itself);
@@ -778,20 +786,42 @@ __device__ __forceinline__ void dfg_plane_rows(const DfgCol& C, const DfgColS& Q
                                                unsigned& cur_full, DFG_T (&zq)[3][DFG_NSF][DFG_VEC], DFG_T*& outp,
                                                long long plane, const DFG_T*& tzp, long long NZ) {
   constexpr unsigned TS = (unsigned)sizeof(DFG_T), ST = DFG_LPR * TS;  // cell k stride
+  // y neighbours before the wait for the next stage (as the TMA kernel),
+  // x neighbours after it: fewer registers live across the wait
   DFG_T xm[DFG_NSF][DFG_VEC], xp[DFG_NSF][DFG_VEC], ym[DFG_NSF][DFG_VEC], yp[DFG_NSF][DFG_VEC];
 #pragma unroll
   for (int f = 0; f < DFG_NSF; ++f) {
     const unsigned t = cur_tile + f * DFG_STILE_BYTES;
 #pragma unroll
     for (int k = 0; k < DFG_VEC; ++k) {
-      const unsigned c = t + Q.o_c + k * ST;
-      xm[f][k] = dfg_lds1(c - ((Q.flags >> k) & 1u ? 0u : TS));
-      xp[f][k] = dfg_lds1(c + ((Q.flags >> (4 + k)) & 1u ? 0u : TS));
       ym[f][k] = dfg_lds1(t + Q.o_m + k * ST);
       yp[f][k] = dfg_lds1(t + Q.o_p + k * ST);
     }
   }
   dfg_mbar_wait(R.full, R.phase, 0x100000u);
+  if (Q.flags) {
+    // a global x end (R1: one-sided): the thread owning the first / last
+    // global cell writes the cell itself into the slot its x-1 / x+1 reads;
+    // only it reads that slot (other threads see it as an inactive cell)
+#pragma unroll
+    for (int f = 0; f < DFG_NSF; ++f)
+#pragma unroll
+      for (int k = 0; k < DFG_VEC; ++k) {
+        const unsigned c = cur_tile + f * DFG_STILE_BYTES + Q.o_c + k * ST;
+        if ((Q.flags >> k) & 1u) dfg_sts1(c - TS, zq[ZC][f][k]);
+        if ((Q.flags >> (4 + k)) & 1u) dfg_sts1(c + TS, zq[ZC][f][k]);
+      }
+  }
+#pragma unroll
+  for (int f = 0; f < DFG_NSF; ++f) {
+    const unsigned t = cur_tile + f * DFG_STILE_BYTES;
+#pragma unroll
+    for (int k = 0; k < DFG_VEC; ++k) {
+      const unsigned c = t + Q.o_c + k * ST;
+      xm[f][k] = dfg_lds1(c - TS);
+      xp[f][k] = dfg_lds1(c + TS);
+    }
+  }
   const unsigned nxt_tile = R.tile, nxt_full = R.full;
 #pragma unroll
   for (int f = 0; f < DFG_NSF; ++f)
