@@ -764,6 +764,22 @@ __device__ __forceinline__ void dfg_produce_rows(const DfgRowsParams& RP, long l
   }
 }
 
+// Cell ownership: a warp owns RPW tile rows of 32 VEC / RPW cells; lane l
+// owns, in each of its rows, the cells l + 32 m (m < CPR = VEC / RPW), so
+// every shared-memory access of the warp is 32 consecutive words of ONE row
+// (conflict-free at any shift).  Thread cell k (0 .. VEC-1) = row k / CPR,
+// cell l + 32 (k mod CPR).
+#define DFG_CPR (DFG_VEC / DFG_RPW)
+// per-item constants of a consumer thread: smem byte offsets (in a field
+// tile) of its first cell in each of its rows and of that cell's y-1 / y+1
+// neighbours (clamped at the global ends); bits 0-3 / 4-7: cell k is the
+// first / last global cell of its row (its x-1 / x+1 is itself)
+struct DfgColS {
+  unsigned oc[DFG_RPW], om[DFG_RPW], op[DFG_RPW];
+  unsigned flags;
+  dfg2 ndy[DFG_NPAIR], ry[DFG_NPAIR];  // y spacing entries of the cells of each pair
+};
+
 __device__ __forceinline__ void dfg_sts1(unsigned addr, DFG_T v) {
 #if DFG_VEC == 4
   asm volatile("st.shared.f32 [%0], %1;" ::"r"(addr), "f"(v) : "memory");
@@ -772,20 +788,12 @@ __device__ __forceinline__ void dfg_sts1(unsigned addr, DFG_T v) {
 #endif
 }
 
-// per-item constants of a consumer thread: smem byte offsets (in a field
-// tile) of its first cell in rows r, r-1, r+1; cell k sits k * LPR elements
-// further.  bits 0-3: cell k is the first global cell (x-1 = itself);
-// bits 4-7: cell k is the last global cell (x+1 = itself).
-struct DfgColS {
-  unsigned o_c, o_m, o_p;
-  unsigned flags;
-};
-
 template <int ZM, int ZC, int ZN>
 __device__ __forceinline__ void dfg_plane_rows(const DfgCol& C, const DfgColS& Q, DfgRingS& R, unsigned& cur_tile,
                                                unsigned& cur_full, DFG_T (&zq)[3][DFG_NSF][DFG_VEC], DFG_T*& outp,
-                                               long long plane, const DFG_T*& tzp, long long NZ) {
-  constexpr unsigned TS = (unsigned)sizeof(DFG_T), ST = DFG_LPR * TS;  // cell k stride
+                                               long long plane, long long rowpitch, const DFG_T*& tzp,
+                                               long long NZ) {
+  constexpr unsigned TS = (unsigned)sizeof(DFG_T), ST = 32 * TS;  // cell stride within a row
   // y neighbours before the wait for the next stage (as the TMA kernel),
   // x neighbours after it: fewer registers live across the wait
   DFG_T xm[DFG_NSF][DFG_VEC], xp[DFG_NSF][DFG_VEC], ym[DFG_NSF][DFG_VEC], yp[DFG_NSF][DFG_VEC];
@@ -794,8 +802,8 @@ __device__ __forceinline__ void dfg_plane_rows(const DfgCol& C, const DfgColS& Q
     const unsigned t = cur_tile + f * DFG_STILE_BYTES;
 #pragma unroll
     for (int k = 0; k < DFG_VEC; ++k) {
-      ym[f][k] = dfg_lds1(t + Q.o_m + k * ST);
-      yp[f][k] = dfg_lds1(t + Q.o_p + k * ST);
+      ym[f][k] = dfg_lds1(t + Q.om[k / DFG_CPR] + (k % DFG_CPR) * ST);
+      yp[f][k] = dfg_lds1(t + Q.op[k / DFG_CPR] + (k % DFG_CPR) * ST);
     }
   }
   dfg_mbar_wait(R.full, R.phase, 0x100000u);
@@ -807,7 +815,7 @@ __device__ __forceinline__ void dfg_plane_rows(const DfgCol& C, const DfgColS& Q
     for (int f = 0; f < DFG_NSF; ++f)
 #pragma unroll
       for (int k = 0; k < DFG_VEC; ++k) {
-        const unsigned c = cur_tile + f * DFG_STILE_BYTES + Q.o_c + k * ST;
+        const unsigned c = cur_tile + f * DFG_STILE_BYTES + Q.oc[k / DFG_CPR] + (k % DFG_CPR) * ST;
         if ((Q.flags >> k) & 1u) dfg_sts1(c - TS, zq[ZC][f][k]);
         if ((Q.flags >> (4 + k)) & 1u) dfg_sts1(c + TS, zq[ZC][f][k]);
       }
@@ -817,7 +825,7 @@ __device__ __forceinline__ void dfg_plane_rows(const DfgCol& C, const DfgColS& Q
     const unsigned t = cur_tile + f * DFG_STILE_BYTES;
 #pragma unroll
     for (int k = 0; k < DFG_VEC; ++k) {
-      const unsigned c = t + Q.o_c + k * ST;
+      const unsigned c = t + Q.oc[k / DFG_CPR] + (k % DFG_CPR) * ST;
       xm[f][k] = dfg_lds1(c - TS);
       xp[f][k] = dfg_lds1(c + TS);
     }
@@ -826,7 +834,8 @@ __device__ __forceinline__ void dfg_plane_rows(const DfgCol& C, const DfgColS& Q
 #pragma unroll
   for (int f = 0; f < DFG_NSF; ++f)
 #pragma unroll
-    for (int k = 0; k < DFG_VEC; ++k) zq[ZN][f][k] = dfg_lds1(nxt_tile + f * DFG_STILE_BYTES + Q.o_c + k * ST);
+    for (int k = 0; k < DFG_VEC; ++k)
+      zq[ZN][f][k] = dfg_lds1(nxt_tile + f * DFG_STILE_BYTES + Q.oc[k / DFG_CPR] + (k % DFG_CPR) * ST);
   R.advance();
   dfg2 s[DFG_NPAIR][DFG_NSF][7], gn[DFG_NPAIR][DFG_NSF][3];
 #pragma unroll
@@ -853,28 +862,25 @@ __device__ __forceinline__ void dfg_plane_rows(const DfgCol& C, const DfgColS& Q
   for (int f = 0; f < DFG_NPF; ++f) {
     DFG_T pv[DFG_VEC];
 #pragma unroll
-    for (int k = 0; k < DFG_VEC; ++k) pv[k] = dfg_lds1(cur_tile + (DFG_NSF + f) * DFG_STILE_BYTES + Q.o_c + k * ST);
+    for (int k = 0; k < DFG_VEC; ++k)
+      pv[k] = dfg_lds1(cur_tile + (DFG_NSF + f) * DFG_STILE_BYTES + Q.oc[k / DFG_CPR] + (k % DFG_CPR) * ST);
 #pragma unroll
     for (int h = 0; h < DFG_NPAIR; ++h) p[h][f] = dfg2_mk(pv[h * DFG_LANES], pv[h * DFG_LANES + DFG_LANES - 1]);
   }
   dfg2 o[DFG_NPAIR][DFG_OUTW];
 #pragma unroll
   for (int h = 0; h < DFG_NPAIR; ++h)
-    dfg_body(s[h], gn[h], p[h], C.ndx[h], C.rx[h], C.ndy, C.ry, ndz, rz, C.Z, o[h]);
-  // cell k at outp + k * LPR cells; nvalid = number of valid cells (a prefix)
+    dfg_body(s[h], gn[h], p[h], C.ndx[h], C.rx[h], Q.ndy[h], Q.ry[h], ndz, rz, C.Z, o[h]);
+  // cell k at outp + row(k) * rowpitch + 32 (k mod CPR); bit k of nvalid: valid
 #pragma unroll
   for (int h = 0; h < DFG_NPAIR; ++h)
 #pragma unroll
     for (int l = 0; l < DFG_LANES; ++l) {
       const int k = h * DFG_LANES + l;
-      if (k < C.nvalid) {
-        DFG_T* d = outp + k * DFG_LPR * DFG_OUTW;
-#if DFG_OUTW == 1
-        __stcs(d, dfg2_get(o[h][0], l));
-#else
+      if ((C.nvalid >> k) & 1) {
+        DFG_T* d = outp + ((k / DFG_CPR) * rowpitch + 32 * (k % DFG_CPR)) * DFG_OUTW;
 #pragma unroll
         for (int w = 0; w < DFG_OUTW; ++w) __stcs(d + w, dfg2_get(o[h][w], l));
-#endif
       }
     }
   outp += plane * DFG_OUTW;
@@ -889,49 +895,52 @@ __device__ __forceinline__ void dfg_consume_rows(const DfgRowsParams& RP, long l
   const DfgRowsInfo& ri = RP.ri;
   const DfgRowsItem I(P, item);
   const long long plane = P.nx * P.ny;
-  const int col = lane % DFG_LPR, sub = lane / DFG_LPR;
-  const int r = 1 + warp * DFG_RPW + sub;
-  const long long i = (long long)I.tx * DFG_TX + col;  // cell k: i + k * LPR
-  const long long j = (long long)I.ty * DFG_TH + warp * DFG_RPW + sub;
-  // valid cells are a prefix of k = 0..VEC-1 (i + k LPR < nx)
-  C.nvalid = j < P.ny ? (int)max(0LL, min((long long)DFG_VEC, (P.nx - i + DFG_LPR - 1) / DFG_LPR)) : 0;
-  const long long jc = min(j, P.ny - 1);
-#pragma unroll
-  for (int h = 0; h < DFG_NPAIR; ++h) {
-    const long long a = min(P.i0 + i + (h * DFG_LANES) * DFG_LPR, P.NX - 1);
-    const long long b = min(P.i0 + i + (h * DFG_LANES + DFG_LANES - 1) * DFG_LPR, P.NX - 1);
-    C.ndx[h] = dfg2_mk(__ldg(P.tx + DFG_NDSEG_X * P.NX + a), __ldg(P.tx + DFG_NDSEG_X * P.NX + b));
-    C.rx[h] = dfg2_mk(__ldg(P.tx + P.NX + a), __ldg(P.tx + P.NX + b));
-  }
-  C.ndy = dfg2_splat(__ldg(P.ty + DFG_NDSEG_Y * P.NY + P.j0 + jc));
-  C.ry = dfg2_splat(__ldg(P.ty + P.NY + P.j0 + jc));
-  // one-sided differences only at the GLOBAL mesh ends (reading R1)
-  const long long jg = P.j0 + j;
-  const int rm = (jg == 0) ? r : r - 1;
-  const int rp = (jg >= P.NY - 1) ? r : r + 1;
+  const int r0 = 1 + warp * DFG_RPW;                   // tile row of this thread's row 0
+  const long long i = (long long)I.tx * DFG_TX + lane;  // cell of k = 0 (row 0)
+  const long long j0 = (long long)I.ty * DFG_TH + warp * DFG_RPW;
   const unsigned TS = (unsigned)sizeof(DFG_T);
-  const unsigned cb = (unsigned)(DFG_HX + col) * TS;  // tile column of cell 0
+  const unsigned cb = (unsigned)(DFG_HX + lane) * TS;  // tile column of cell m = 0
   DfgColS Q;
-  Q.o_c = I.row_col0(ri, r) + cb;
-  Q.o_m = I.row_col0(ri, rm) + cb;
-  Q.o_p = I.row_col0(ri, rp) + cb;
+  C.nvalid = 0;
   Q.flags = 0;
 #pragma unroll
   for (int k = 0; k < DFG_VEC; ++k) {
-    const long long ig = P.i0 + i + k * DFG_LPR;
-    Q.flags |= (ig == 0 ? 1u : 0u) << k;
-    Q.flags |= (ig == P.NX - 1 ? 1u : 0u) << (4 + k);
+    const long long ik = i + 32 * (k % DFG_CPR), jk = j0 + k / DFG_CPR;
+    C.nvalid |= (ik < P.nx && jk < P.ny ? 1 : 0) << k;
+    Q.flags |= (P.i0 + ik == 0 ? 1u : 0u) << k;
+    Q.flags |= (P.i0 + ik == P.NX - 1 ? 1u : 0u) << (4 + k);
   }
-  DFG_T* outp = P.out + ((I.kb - P.k0) * plane + jc * P.nx + min(i, P.nx - 1)) * DFG_OUTW;
+#pragma unroll
+  for (int h = 0; h < DFG_NPAIR; ++h) {
+    const int ka = h * DFG_LANES, kb = h * DFG_LANES + DFG_LANES - 1;
+    const long long a = min(P.i0 + i + 32 * (ka % DFG_CPR), P.NX - 1);
+    const long long b = min(P.i0 + i + 32 * (kb % DFG_CPR), P.NX - 1);
+    C.ndx[h] = dfg2_mk(__ldg(P.tx + DFG_NDSEG_X * P.NX + a), __ldg(P.tx + DFG_NDSEG_X * P.NX + b));
+    C.rx[h] = dfg2_mk(__ldg(P.tx + P.NX + a), __ldg(P.tx + P.NX + b));
+    const long long ya = P.j0 + min(j0 + ka / DFG_CPR, P.ny - 1), yb = P.j0 + min(j0 + kb / DFG_CPR, P.ny - 1);
+    Q.ndy[h] = dfg2_mk(__ldg(P.ty + DFG_NDSEG_Y * P.NY + ya), __ldg(P.ty + DFG_NDSEG_Y * P.NY + yb));
+    Q.ry[h] = dfg2_mk(__ldg(P.ty + P.NY + ya), __ldg(P.ty + P.NY + yb));
+  }
+#pragma unroll
+  for (int q = 0; q < DFG_RPW; ++q) {
+    // one-sided differences only at the GLOBAL mesh ends (reading R1)
+    const long long jg = P.j0 + j0 + q;
+    const int r = r0 + q;
+    Q.oc[q] = I.row_col0(ri, r) + cb;
+    Q.om[q] = (jg == 0) ? Q.oc[q] : I.row_col0(ri, r - 1) + cb;
+    Q.op[q] = (jg >= P.NY - 1) ? Q.oc[q] : I.row_col0(ri, r + 1) + cb;
+  }
+  DFG_T* outp = P.out + ((I.kb - P.k0) * plane + min(j0, P.ny - 1) * P.nx + min(i, P.nx - 1)) * DFG_OUTW;
   const DFG_T* tzp = P.tz + I.kb;
-  constexpr unsigned ST = DFG_LPR * (unsigned)sizeof(DFG_T);
+  constexpr unsigned ST = 32 * (unsigned)sizeof(DFG_T);
 
   DFG_T zq[3][DFG_NSF][DFG_VEC];
   dfg_mbar_wait(R.full, R.phase, 0x100000u);
 #pragma unroll
   for (int f = 0; f < DFG_NSF; ++f)
 #pragma unroll
-    for (int k = 0; k < DFG_VEC; ++k) zq[0][f][k] = dfg_lds1(R.tile + f * DFG_STILE_BYTES + Q.o_c + k * ST);
+    for (int k = 0; k < DFG_VEC; ++k)
+      zq[0][f][k] = dfg_lds1(R.tile + f * DFG_STILE_BYTES + Q.oc[k / DFG_CPR] + (k % DFG_CPR) * ST);
   dfg_mbar_arrive(R.full + DfgRingS::kEmpty);
   R.advance();
   dfg_mbar_wait(R.full, R.phase, 0x100000u);
@@ -939,17 +948,18 @@ __device__ __forceinline__ void dfg_consume_rows(const DfgRowsParams& RP, long l
 #pragma unroll
   for (int f = 0; f < DFG_NSF; ++f)
 #pragma unroll
-    for (int k = 0; k < DFG_VEC; ++k) zq[1][f][k] = dfg_lds1(cur_tile + f * DFG_STILE_BYTES + Q.o_c + k * ST);
+    for (int k = 0; k < DFG_VEC; ++k)
+      zq[1][f][k] = dfg_lds1(cur_tile + f * DFG_STILE_BYTES + Q.oc[k / DFG_CPR] + (k % DFG_CPR) * ST);
   R.advance();
   long long k = I.kb;
   for (; k + 3 <= I.ke; k += 3) {
-    dfg_plane_rows<0, 1, 2>(C, Q, R, cur_tile, cur_full, zq, outp, plane, tzp, P.NZ);
-    dfg_plane_rows<1, 2, 0>(C, Q, R, cur_tile, cur_full, zq, outp, plane, tzp, P.NZ);
-    dfg_plane_rows<2, 0, 1>(C, Q, R, cur_tile, cur_full, zq, outp, plane, tzp, P.NZ);
+    dfg_plane_rows<0, 1, 2>(C, Q, R, cur_tile, cur_full, zq, outp, plane, P.nx, tzp, P.NZ);
+    dfg_plane_rows<1, 2, 0>(C, Q, R, cur_tile, cur_full, zq, outp, plane, P.nx, tzp, P.NZ);
+    dfg_plane_rows<2, 0, 1>(C, Q, R, cur_tile, cur_full, zq, outp, plane, P.nx, tzp, P.NZ);
   }
   if (k < I.ke) {
-    dfg_plane_rows<0, 1, 2>(C, Q, R, cur_tile, cur_full, zq, outp, plane, tzp, P.NZ);
-    if (k + 1 < I.ke) dfg_plane_rows<1, 2, 0>(C, Q, R, cur_tile, cur_full, zq, outp, plane, tzp, P.NZ);
+    dfg_plane_rows<0, 1, 2>(C, Q, R, cur_tile, cur_full, zq, outp, plane, P.nx, tzp, P.NZ);
+    if (k + 1 < I.ke) dfg_plane_rows<1, 2, 0>(C, Q, R, cur_tile, cur_full, zq, outp, plane, P.nx, tzp, P.NZ);
   }
   dfg_mbar_arrive(cur_full + DfgRingS::kEmpty);
 }

@@ -20,11 +20,17 @@ PROGS = ["velmag", "vortmag", "qcrit", "intro"]
 NAMES = {"velmag": ("u", "v", "w"), "vortmag": ("u", "v", "w"), "qcrit": ("u", "v", "w"), "intro": ("b", "c")}
 
 
-def _rows_layout(px, py, itemsize):
-    """The row-copy kernel's precondition (16-byte aligned bases, as torch
-    allocations are, and 16-byte plane strides): layouts the tensor maps
-    cannot take run on it (variant 7), the rest on the cp.async ring (5)."""
-    return (px * py * itemsize) % 16 == 0
+def _rows_layout(px, py, itemsize, plan=None):
+    """The row-class kernel's preconditions (16-byte aligned bases, as torch
+    allocations are, 16-byte plane strides, a row of every class per plane,
+    and -- its lanes own whole cells of RPW rows -- RPW <= VEC): layouts the
+    tensor maps cannot take run on it (variant 7), the rest on the cp.async
+    ring (5)."""
+    period = next(p for p in (1, 2, 4) if (px * itemsize * p) % 16 == 0)
+    ok = (px * py * itemsize) % 16 == 0 and py >= period
+    if plan is not None:
+        ok = ok and plan.info()["rows_per_warp"] <= 16 // itemsize
+    return ok
 
 
 def _inputs(shape, T, names=("u", "v", "w")):
@@ -84,7 +90,7 @@ def test_tile_kernel(prog, T, shape, rpw, monkeypatch):
     got, plan, *_ = run_lib(src, f, x, y, z, return_plan=True)
     if prog != "velmag":
         vec = 4 if T == np.float32 else 2
-        ragged = 7 if _rows_layout(shape[0], shape[1], np.dtype(T).itemsize) else 5
+        ragged = 7 if _rows_layout(shape[0], shape[1], np.dtype(T).itemsize, plan) else 5
         assert plan.info()["variant"] == (ragged if shape[0] % vec else 1)
     assert_parity(got, want)
 
@@ -108,12 +114,13 @@ def test_rows_kernel(prog, T, shape, monkeypatch):
     got, plan, *_ = run_lib(src, f, x, y, z, return_plan=True)
     vec = 16 // isz
     if prog != "velmag":
-        assert plan.info()["variant"] == (7 if shape[0] % vec else 1)
+        assert plan.info()["variant"] == ((7 if _rows_layout(shape[0], shape[1], isz, plan) else 5)
+                                          if shape[0] % vec else 1)
     assert_parity(got, want)
     if prog != "velmag":
         monkeypatch.setenv("DFG_FUSED_KERNEL", "rows")     # also where the tensor maps could run
         got2, plan2, *_ = run_lib(src, f, x, y, z, return_plan=True)
-        assert plan2.info()["variant"] == 7
+        assert plan2.info()["variant"] == (7 if _rows_layout(shape[0], shape[1], isz, plan2) else 5)
         assert_parity(got2, want)
         monkeypatch.setenv("DFG_FUSED_KERNEL", "tile")
         got3, plan3, *_ = run_lib(src, f, x, y, z, return_plan=True)
@@ -505,7 +512,7 @@ def _visit_blocks(shape, split, prog, strategy, pitch):
                 if pitch == "padded" and bx % 4 == 0 and prog != "velmag":
                     assert p.info()["variant"] == 1          # TMA kernel on the padded shell
                 elif prog != "velmag":                       # packed shell: row copies or the cp.async ring
-                    assert p.info()["variant"] == (7 if _rows_layout(rp, j1 - j0 + 2, 4) else 5)
+                    assert p.info()["variant"] == (7 if _rows_layout(rp, j1 - j0 + 2, 4, p) else 5)
                 got[k0:k1, j0:j1, i0:i1] = o.cpu().numpy()
                 blocks.append((p, torch.full_like(o, float("nan")), (k0, k1, j0, j1, i0, i1), m, keep,
                                p.info()["variant"]))
