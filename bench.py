@@ -52,6 +52,7 @@ class ClockSampler:
         self.index = index
         self.rows = []
         self._stop = threading.Event()
+        self._ready = threading.Event()   # first sample taken (NVML initialised)
         self._t = None
 
     # NVML clocks-event reason bits (nvml.h): sw power cap, hw slowdown,
@@ -74,7 +75,8 @@ class ClockSampler:
                 for bit, col in self.BITS:
                     row[col] = "Active" if bits & bit else "Not Active"
                 self.rows.append(row)
-                self._stop.wait(0.01)
+                self._ready.set()
+                self._stop.wait(0.002)
             self.source = "nvml"
             return
         except Exception:
@@ -87,6 +89,7 @@ class ClockSampler:
                                      timeout=5).stdout.strip()
                 if out:
                     self.rows.append([c.strip() for c in out.split(",")])
+                    self._ready.set()
             except Exception:
                 pass
             self._stop.wait(0.05)
@@ -94,6 +97,9 @@ class ClockSampler:
     def __enter__(self):
         self._t = threading.Thread(target=self._run, daemon=True)
         self._t.start()
+        # the timed region starts only once sampling runs (NVML init can take
+        # longer than a short timed region)
+        self._ready.wait(timeout=10.0)
         return self
 
     def __exit__(self, *a):
