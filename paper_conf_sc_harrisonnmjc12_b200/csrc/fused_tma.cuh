@@ -773,11 +773,13 @@ __device__ __forceinline__ void dfg_produce_rows(const DfgRowsParams& RP, long l
 // per-item constants of a consumer thread: smem byte offsets (in a field
 // tile) of its first cell in each of its rows and of that cell's y-1 / y+1
 // neighbours (clamped at the global ends); bits 0-3 / 4-7: cell k is the
-// first / last global cell of its row (its x-1 / x+1 is itself)
+// first / last global cell of its row (its x-1 / x+1 is itself); bits
+// 8-11: row q is the last global row (its y+1 is itself).  Between the
+// thread's own rows the y neighbours come from registers (the centres).
 struct DfgColS {
   unsigned oc[DFG_RPW], om[DFG_RPW], op[DFG_RPW];
   unsigned flags;
-  dfg2 ndy[DFG_NPAIR], ry[DFG_NPAIR];  // y spacing entries of the cells of each pair
+  DFG_T ndy[DFG_RPW], ry[DFG_RPW];  // y spacing entries of each of the thread's rows
 };
 
 __device__ __forceinline__ void dfg_sts1(unsigned addr, DFG_T v) {
@@ -794,20 +796,31 @@ __device__ __forceinline__ void dfg_plane_rows(const DfgCol& C, const DfgColS& Q
                                                long long plane, long long rowpitch, const DFG_T*& tzp,
                                                long long NZ) {
   constexpr unsigned TS = (unsigned)sizeof(DFG_T), ST = 32 * TS;  // cell stride within a row
-  // y neighbours before the wait for the next stage (as the TMA kernel),
-  // x neighbours after it: fewer registers live across the wait
+  // y neighbours before the wait for the next stage (as the TMA kernel; fp64:
+  // after it, its doubles need the registers), x neighbours after it
   DFG_T xm[DFG_NSF][DFG_VEC], xp[DFG_NSF][DFG_VEC], ym[DFG_NSF][DFG_VEC], yp[DFG_NSF][DFG_VEC];
+  auto load_y = [&]() {
 #pragma unroll
-  for (int f = 0; f < DFG_NSF; ++f) {
-    const unsigned t = cur_tile + f * DFG_STILE_BYTES;
+    for (int f = 0; f < DFG_NSF; ++f) {
+      const unsigned t = cur_tile + f * DFG_STILE_BYTES;
 #pragma unroll
-    for (int k = 0; k < DFG_VEC; ++k) {
-      ym[f][k] = dfg_lds1(t + Q.om[k / DFG_CPR] + (k % DFG_CPR) * ST);
-      yp[f][k] = dfg_lds1(t + Q.op[k / DFG_CPR] + (k % DFG_CPR) * ST);
+      for (int k = 0; k < DFG_VEC; ++k) {
+        const int q = k / DFG_CPR;
+        if (q == 0) ym[f][k] = dfg_lds1(t + Q.om[0] + (k % DFG_CPR) * ST);
+        else ym[f][k] = zq[ZC][f][k - DFG_CPR];  // the row above is this thread's (never a global end)
+        if (q == DFG_RPW - 1) yp[f][k] = dfg_lds1(t + Q.op[q] + (k % DFG_CPR) * ST);
+        else yp[f][k] = (Q.flags >> (8 + q)) & 1u ? zq[ZC][f][k] : zq[ZC][f][k + DFG_CPR];
+      }
     }
-  }
+  };
+#if DFG_VEC == 4
+  load_y();
+#endif
   dfg_mbar_wait(R.full, R.phase, 0x100000u);
-  if (Q.flags) {
+#if DFG_VEC == 2
+  load_y();
+#endif
+  if (Q.flags & 0xffu) {
     // a global x end (R1: one-sided): the thread owning the first / last
     // global cell writes the cell itself into the slot its x-1 / x+1 reads;
     // only it reads that slot (other threads see it as an inactive cell)
@@ -870,7 +883,10 @@ __device__ __forceinline__ void dfg_plane_rows(const DfgCol& C, const DfgColS& Q
   dfg2 o[DFG_NPAIR][DFG_OUTW];
 #pragma unroll
   for (int h = 0; h < DFG_NPAIR; ++h)
-    dfg_body(s[h], gn[h], p[h], C.ndx[h], C.rx[h], Q.ndy[h], Q.ry[h], ndz, rz, C.Z, o[h]);
+    dfg_body(s[h], gn[h], p[h], C.ndx[h], C.rx[h],
+             dfg2_mk(Q.ndy[(h * DFG_LANES) / DFG_CPR], Q.ndy[(h * DFG_LANES + DFG_LANES - 1) / DFG_CPR]),
+             dfg2_mk(Q.ry[(h * DFG_LANES) / DFG_CPR], Q.ry[(h * DFG_LANES + DFG_LANES - 1) / DFG_CPR]), ndz, rz, C.Z,
+             o[h]);
   // cell k at outp + row(k) * rowpitch + 32 (k mod CPR); bit k of nvalid: valid
 #pragma unroll
   for (int h = 0; h < DFG_NPAIR; ++h)
@@ -917,9 +933,12 @@ __device__ __forceinline__ void dfg_consume_rows(const DfgRowsParams& RP, long l
     const long long b = min(P.i0 + i + 32 * (kb % DFG_CPR), P.NX - 1);
     C.ndx[h] = dfg2_mk(__ldg(P.tx + DFG_NDSEG_X * P.NX + a), __ldg(P.tx + DFG_NDSEG_X * P.NX + b));
     C.rx[h] = dfg2_mk(__ldg(P.tx + P.NX + a), __ldg(P.tx + P.NX + b));
-    const long long ya = P.j0 + min(j0 + ka / DFG_CPR, P.ny - 1), yb = P.j0 + min(j0 + kb / DFG_CPR, P.ny - 1);
-    Q.ndy[h] = dfg2_mk(__ldg(P.ty + DFG_NDSEG_Y * P.NY + ya), __ldg(P.ty + DFG_NDSEG_Y * P.NY + yb));
-    Q.ry[h] = dfg2_mk(__ldg(P.ty + P.NY + ya), __ldg(P.ty + P.NY + yb));
+  }
+#pragma unroll
+  for (int q = 0; q < DFG_RPW; ++q) {
+    const long long yq = P.j0 + min(j0 + q, P.ny - 1);
+    Q.ndy[q] = __ldg(P.ty + DFG_NDSEG_Y * P.NY + yq);
+    Q.ry[q] = __ldg(P.ty + P.NY + yq);
   }
 #pragma unroll
   for (int q = 0; q < DFG_RPW; ++q) {
@@ -929,6 +948,7 @@ __device__ __forceinline__ void dfg_consume_rows(const DfgRowsParams& RP, long l
     Q.oc[q] = I.row_col0(ri, r) + cb;
     Q.om[q] = (jg == 0) ? Q.oc[q] : I.row_col0(ri, r - 1) + cb;
     Q.op[q] = (jg >= P.NY - 1) ? Q.oc[q] : I.row_col0(ri, r + 1) + cb;
+    Q.flags |= (jg >= P.NY - 1 ? 1u : 0u) << (8 + q);
   }
   DFG_T* outp = P.out + ((I.kb - P.k0) * plane + min(j0, P.ny - 1) * P.nx + min(i, P.nx - 1)) * DFG_OUTW;
   const DFG_T* tzp = P.tz + I.kb;

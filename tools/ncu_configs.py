@@ -1,7 +1,7 @@
 """One execute per bench configuration, for an ncu launch capture (developer tool).
 
     ncu --metrics gpu__time_duration.sum,dram__bytes_read.sum,dram__bytes_write.sum,\\
-        smsp__sass_thread_inst_executed.sum -k regex:dfg --csv --log-file gpurun_out/cfg.csv \\
+        smsp__sass_thread_inst_executed.sum -k "regex:dfg|k_" --csv --log-file gpurun_out/cfg.csv \\
         python tools/ncu_configs.py > gpurun_out/cfg_order.json
     python tools/ncu_configs.py --summarize gpurun_out/cfg.csv gpurun_out/cfg_order.json > profiles/r02_configs.md
 
@@ -44,6 +44,8 @@ def run():
         flds = {nm: synth.rt_velocity(c, x64, y64, z64, None, tt, "cuda") for nm, c in zip(names, "uvw")}
         for nm, t in flds.items():
             mesh.bind(nm, t)
+        if strat == "staged":
+            os.environ["DFG_GRAPH"] = "0"   # plain launches (ncu sees each filter's kernel)
         plan = dfg.Plan(mesh, dfg.paper_program(prog), strat).set_timing(0)
         out = torch.empty((n, n, n), dtype=tt, device="cuda")
         plan.execute(out)
@@ -67,8 +69,8 @@ def summarize(csv_path, order_path):
     iI, iN, iM, iU, iV = (hdr.index(k) for k in ("ID", "Kernel Name", "Metric Name", "Metric Unit", "Metric Value"))
     launches = {}
     for r in data:
-        if "dfg" not in r[iN] and "k_" not in r[iN]:
-            continue
+        if ("dfg" not in r[iN] and "k_" not in r[iN]) or "verify_div2" in r[iN]:
+            continue   # torch's kernels (input generation), the mesh's divisor check (not a step)
         d = launches.setdefault(int(r[iI]), {"name": r[iN].split("(")[0]})
         v = float(r[iV].replace(",", ""))
         unit = r[iU]
@@ -85,7 +87,7 @@ def summarize(csv_path, order_path):
     order = json.load(open(order_path))
     print("# Per-configuration ncu accounting (round 2)\n")
     print("`ncu --metrics gpu__time_duration.sum,dram__bytes_read.sum,dram__bytes_write.sum,"
-          "smsp__sass_thread_inst_executed.sum --clock-control none -k regex:dfg` over "
+          "smsp__sass_thread_inst_executed.sum --clock-control none -k \"regex:dfg|k_\"` over "
           "`tools/ncu_configs.py` (one execute per case, cold L2, launches serialised).  Predicted "
           "bytes: the library's model (fused: inputs + output once; staged: every filter's operands "
           "and result).\n")
