@@ -793,8 +793,7 @@ __device__ __forceinline__ void dfg_sts1(unsigned addr, DFG_T v) {
 template <int ZM, int ZC, int ZN>
 __device__ __forceinline__ void dfg_plane_rows(const DfgCol& C, const DfgColS& Q, DfgRingS& R, unsigned& cur_tile,
                                                unsigned& cur_full, DFG_T (&zq)[3][DFG_NSF][DFG_VEC], DFG_T*& outp,
-                                               long long plane, long long rowpitch, const DFG_T*& tzp,
-                                               long long NZ) {
+                                               unsigned plane, int rowpitch, const DFG_T*& tzp, long long NZ) {
   constexpr unsigned TS = (unsigned)sizeof(DFG_T), ST = 32 * TS;  // cell stride within a row
   // y neighbours before the wait for the next stage (as the TMA kernel; fp64:
   // after it, its doubles need the registers), x neighbours after it
@@ -899,7 +898,7 @@ __device__ __forceinline__ void dfg_plane_rows(const DfgCol& C, const DfgColS& Q
         for (int w = 0; w < DFG_OUTW; ++w) __stcs(d + w, dfg2_get(o[h][w], l));
       }
     }
-  outp += plane * DFG_OUTW;
+  outp += (size_t)plane * DFG_OUTW;
   dfg_mbar_arrive(cur_full + DfgRingS::kEmpty);  // every consumer thread (count NCW*32)
   cur_tile = nxt_tile;
   cur_full = nxt_full;
@@ -910,7 +909,7 @@ __device__ __forceinline__ void dfg_consume_rows(const DfgRowsParams& RP, long l
   const DfgParams& P = RP.p;
   const DfgRowsInfo& ri = RP.ri;
   const DfgRowsItem I(P, item);
-  const long long plane = P.nx * P.ny;
+  const unsigned plane = (unsigned)(P.nx * P.ny);  // < 2^32 (host precondition)
   const int r0 = 1 + warp * DFG_RPW;                   // tile row of this thread's row 0
   const long long i = (long long)I.tx * DFG_TX + lane;  // cell of k = 0 (row 0)
   const long long j0 = (long long)I.ty * DFG_TH + warp * DFG_RPW;
@@ -950,7 +949,7 @@ __device__ __forceinline__ void dfg_consume_rows(const DfgRowsParams& RP, long l
     Q.op[q] = (jg >= P.NY - 1) ? Q.oc[q] : I.row_col0(ri, r + 1) + cb;
     Q.flags |= (jg >= P.NY - 1 ? 1u : 0u) << (8 + q);
   }
-  DFG_T* outp = P.out + ((I.kb - P.k0) * plane + min(j0, P.ny - 1) * P.nx + min(i, P.nx - 1)) * DFG_OUTW;
+  DFG_T* outp = P.out + ((I.kb - P.k0) * (long long)plane + min(j0, P.ny - 1) * P.nx + min(i, P.nx - 1)) * DFG_OUTW;
   const DFG_T* tzp = P.tz + I.kb;
   constexpr unsigned ST = 32 * (unsigned)sizeof(DFG_T);
 
@@ -973,13 +972,13 @@ __device__ __forceinline__ void dfg_consume_rows(const DfgRowsParams& RP, long l
   R.advance();
   long long k = I.kb;
   for (; k + 3 <= I.ke; k += 3) {
-    dfg_plane_rows<0, 1, 2>(C, Q, R, cur_tile, cur_full, zq, outp, plane, P.nx, tzp, P.NZ);
-    dfg_plane_rows<1, 2, 0>(C, Q, R, cur_tile, cur_full, zq, outp, plane, P.nx, tzp, P.NZ);
-    dfg_plane_rows<2, 0, 1>(C, Q, R, cur_tile, cur_full, zq, outp, plane, P.nx, tzp, P.NZ);
+    dfg_plane_rows<0, 1, 2>(C, Q, R, cur_tile, cur_full, zq, outp, plane, (int)P.nx, tzp, P.NZ);
+    dfg_plane_rows<1, 2, 0>(C, Q, R, cur_tile, cur_full, zq, outp, plane, (int)P.nx, tzp, P.NZ);
+    dfg_plane_rows<2, 0, 1>(C, Q, R, cur_tile, cur_full, zq, outp, plane, (int)P.nx, tzp, P.NZ);
   }
   if (k < I.ke) {
-    dfg_plane_rows<0, 1, 2>(C, Q, R, cur_tile, cur_full, zq, outp, plane, P.nx, tzp, P.NZ);
-    if (k + 1 < I.ke) dfg_plane_rows<1, 2, 0>(C, Q, R, cur_tile, cur_full, zq, outp, plane, P.nx, tzp, P.NZ);
+    dfg_plane_rows<0, 1, 2>(C, Q, R, cur_tile, cur_full, zq, outp, plane, (int)P.nx, tzp, P.NZ);
+    if (k + 1 < I.ke) dfg_plane_rows<1, 2, 0>(C, Q, R, cur_tile, cur_full, zq, outp, plane, (int)P.nx, tzp, P.NZ);
   }
   dfg_mbar_arrive(cur_full + DfgRingS::kEmpty);
 }
@@ -1034,9 +1033,12 @@ extern "C" __global__ void __launch_bounds__((DFG_NCW + 1) * 32, DFG_CTAS)
   DfgRingS R{smem, full0, 0u, 0, smem, full0};
   DfgCol C;
   C.Z = dfg2_splat(M.blocks[0].p.nzero);
-  for (long long item = blockIdx.x; item < total; item += gridDim.x) {
-    while (item >= M.first[b + 1]) ++b;
-    dfg_consume_rows(M.blocks[b], item - M.first[b], R, C, warp, lane);
+  // the block index is found again per item (a short search in global
+  // memory) rather than kept live across the consumer loop: registers
+  for (long long item = blockIdx.x; item < M.first[M.nb]; item += gridDim.x) {
+    int bb = 0;
+    while (item >= M.first[bb + 1]) ++bb;
+    dfg_consume_rows(M.blocks[bb], item - M.first[bb], R, C, warp, lane);
   }
 }
 #endif  // DFG_ROWS_KERNEL

@@ -23,13 +23,13 @@ NAMES = {"velmag": ("u", "v", "w"), "vortmag": ("u", "v", "w"), "qcrit": ("u", "
 def _rows_layout(px, py, itemsize, plan=None):
     """The row-class kernel's preconditions (16-byte aligned bases, as torch
     allocations are, 16-byte plane strides, a row of every class per plane,
-    and -- its lanes own whole cells of RPW rows -- RPW <= VEC): layouts the
-    tensor maps cannot take run on it (variant 7), the rest on the cp.async
-    ring (5)."""
+    and -- its lanes own whole cells of RPW rows -- RPW <= VEC / 2):
+    layouts the tensor maps cannot take run on it (variant 7), the rest on
+    the cp.async ring (5)."""
     period = next(p for p in (1, 2, 4) if (px * itemsize * p) % 16 == 0)
     ok = (px * py * itemsize) % 16 == 0 and py >= period
     if plan is not None:
-        ok = ok and plan.info()["rows_per_warp"] <= 16 // itemsize
+        ok = ok and plan.info()["rows_per_warp"] <= 8 // itemsize
     return ok
 
 
