@@ -29,7 +29,14 @@ struct __align__(64) DfgTmap { unsigned long long v[16]; };  // CUtensorMap
 // (IPC mappings) for the planes outside [k0, k0 + nzl).
 struct DfgPeerInfo {
   long long lo_k0, lo_ghost, hi_k0, hi_ghost;
-  int lo_on, hi_on, pad0, pad1;
+  int lo_on, hi_on;
+  // single-launch mode (wait != 0): before loading a neighbour's plane the
+  // producer waits in the kernel until that neighbour's "ready" flag (IPC
+  // mapped) reaches `epoch`, and the z-chunks at the slab ends run last
+  int wait;
+  unsigned epoch;
+  const unsigned* lo_ready;
+  const unsigned* hi_ready;
 };
 // host image: runtime.cpp tma_blob_* (same order, 64-byte aligned maps)
 struct DfgTmaParams {
@@ -248,6 +255,35 @@ __device__ __forceinline__ void dfg_plane(const DfgCol& C, Ring& R, unsigned& cu
   cur_full = nxt_full;
 }
 
+// z-chunk of an item.  Single-launch peer halo: the interior chunks first,
+// then the chunk at the low slab end, the one at the high end last (their
+// boundary planes wait for the neighbours; the interior overlaps that wait).
+__device__ __forceinline__ long long dfg_zchunk(const DfgTmaParams& TP, long long zc) {
+  if (!TP.peer.wait) return zc;
+  const long long n = (TP.p.kend - TP.p.kbeg + TP.p.kz - 1) / TP.p.kz;
+  if (n < 3) return zc;
+  return zc < n - 2 ? zc + 1 : (zc == n - 2 ? 0 : n - 1);
+}
+
+// Wait (producer lane) until a neighbour's IPC-mapped "ready" flag reaches
+// the step: acquire at system scope, then order the async proxy (the TMA
+// reads that follow) after it.  A neighbour that never arrives within 30 s
+// traps: a loud failure, never a silent wrong result or a hung step.
+__device__ __forceinline__ void dfg_wait_ready(const unsigned* flag, unsigned epoch) {
+  unsigned long long t0;
+  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t0));
+  for (;;) {
+    unsigned v;
+    asm volatile("ld.acquire.sys.global.u32 %0, [%1];" : "=r"(v) : "l"(flag) : "memory");
+    if ((int)(v - epoch) >= 0) break;
+    unsigned long long t;
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+    if (t - t0 > 30000000000ull) __trap();
+    __nanosleep(200);
+  }
+  asm volatile("fence.proxy.async.global;" ::: "memory");
+}
+
 // Producer side of one item (x-tile, y-tile, z-chunk) of mesh TP: the
 // pre-plane, planes kb..ke-1 and the post-plane, clamped to the global mesh (R1).
 __device__ __forceinline__ void dfg_produce_item(const DfgTmaParams& TP, long long item, DfgRing& W) {
@@ -255,7 +291,7 @@ __device__ __forceinline__ void dfg_produce_item(const DfgTmaParams& TP, long lo
   const long long tx_ = item % P.tiles_x;
   const long long rest = item / P.tiles_x;
   const long long ty_ = rest % P.tiles_y;
-  const long long zc = rest / P.tiles_y;
+  const long long zc = dfg_zchunk(TP, rest / P.tiles_y);
   // input coordinates include the block's x/y ghost columns / rows
   const int x0 = (int)(tx_ * DFG_TX) - DFG_HX + (int)P.gx;
   const int y0 = (int)(ty_ * DFG_TH) - 1 + (int)P.gy;
@@ -272,6 +308,7 @@ __device__ __forceinline__ void dfg_produce_item(const DfgTmaParams& TP, long lo
     // linked to peers (stencil fields only; point-wise fields are read at owned planes)
     const bool lo = TP.peer.lo_on && pg < P.k0, hi = TP.peer.hi_on && pg >= P.k0 + P.nzl;
     const int zp = lo ? (int)(pg - TP.peer.lo_k0 + TP.peer.lo_ghost) : (int)(pg - TP.peer.hi_k0 + TP.peer.hi_ghost);
+    if (TP.peer.wait && (lo || hi)) dfg_wait_ready(lo ? TP.peer.lo_ready : TP.peer.hi_ready, TP.peer.epoch);
 #pragma unroll
     for (int f = 0; f < DFG_NTF; ++f) {
       const bool peer = (lo || hi) && f < DFG_NSF;
@@ -293,7 +330,7 @@ __device__ __forceinline__ void dfg_consume_item(const DfgTmaParams& TP, long lo
   const long long tx_ = item % P.tiles_x;
   const long long rest = item / P.tiles_x;
   const long long ty_ = rest % P.tiles_y;
-  const long long zc = rest / P.tiles_y;
+  const long long zc = dfg_zchunk(TP, rest / P.tiles_y);
   const long long i = tx_ * DFG_TX + DFG_VEC * col;
   const long long j = ty_ * DFG_TH + warp * DFG_RPW + sub;
   const long long kb = P.kbeg + zc * P.kz;

@@ -354,7 +354,7 @@ void encode_map(CUtensorMap* map, const SlabView& m, void* base, int ncw, int rp
 }
 
 // Host image of DfgTmaParams (fused_tma.cuh): map[NF_] | map_lo[NSF_] |
-// map_hi[NSF_] | DfgPeerInfo (48 B) | DfgParams, each map 128 B (64-aligned),
+// map_hi[NSF_] | DfgPeerInfo (64 B) | DfgParams, each map 128 B (64-aligned),
 // total padded to 64 bytes.
 struct TmaBlobLayout {
   size_t lo, hi, peer, params, size;
@@ -365,7 +365,7 @@ TmaBlobLayout tma_blob_layout(int nf, int nsf, size_t param_words) {
   b.lo = 128 * NF;
   b.hi = b.lo + 128 * NSF;
   b.peer = b.hi + 128 * NSF;
-  b.params = b.peer + 48;
+  b.params = b.peer + 64;
   b.size = (b.params + param_words * 8 + 63) / 64 * 64;
   return b;
 }
@@ -625,7 +625,21 @@ void PlanImpl::exec_fused_peer(const std::vector<const void*>& fptr, void* out, 
     if (lo) DFG_CU(drv().StreamWaitValue32(cs, dptr(m.peer_lo.flags, kFlagReady), e, CU_STREAM_WAIT_VALUE_GEQ));
     if (hi) DFG_CU(drv().StreamWaitValue32(cs, dptr(m.peer_hi.flags, kFlagReady), e, CU_STREAM_WAIT_VALUE_GEQ));
   };
-  if (use_tma) {
+  const char* ik = std::getenv("DFG_PEER_INKERNEL");
+  if (use_tma && !(ik && !std::strcmp(ik, "0"))) {
+    // ONE launch: the producers wait in the kernel for the neighbours'
+    // "ready" flags before loading their planes, and the z-chunks at the slab
+    // ends run last, so the interior overlaps the wait (no stream waits, no
+    // extra launches)
+    peer_wait_epoch = e;
+    try {
+      launch_fused(fptr, out, tab, v, s, m.k0, m.k0 + m.nzl, true);
+    } catch (...) {
+      peer_wait_epoch = 0;
+      throw;
+    }
+    peer_wait_epoch = 0;
+  } else if (use_tma) {
     const int64_t a = m.k0 + (lo ? 1 : 0), b = m.k0 + m.nzl - (hi ? 1 : 0);
     if (a < b) launch_fused(fptr, out, tab, v, s, a, b);
     wait_ready();
@@ -723,9 +737,11 @@ void PlanImpl::launch_fused(const std::vector<const void*>& fptr, void* dout, co
     for (int f = 0; f < nsf; ++f)
       encode_map(reinterpret_cast<CUtensorMap*>(blob + 128 * f), m, const_cast<void*>(fptr[f]), ncw, rpw);
     if (peer) {
-      // DfgPeerInfo: lo_k0, lo_ghost, hi_k0, hi_ghost, lo_on, hi_on
+      // DfgPeerInfo: lo_k0, lo_ghost, hi_k0, hi_ghost | lo_on, hi_on, wait,
+      // epoch | lo_ready, hi_ready
       int64_t info[4] = {0, 0, 0, 0};
-      int32_t on[4] = {0, 0, 0, 0};
+      int32_t on[4] = {0, 0, peer_wait_epoch ? 1 : 0, int32_t(peer_wait_epoch)};
+      const uint32_t* ready[2] = {nullptr, nullptr};
       const MeshImpl::Peer* sides[2] = {&mesh->peer_lo, &mesh->peer_hi};
       for (int sd = 0; sd < 2; ++sd) {
         const MeshImpl::Peer& pr = *sides[sd];
@@ -744,9 +760,11 @@ void PlanImpl::launch_fused(const std::vector<const void*>& fptr, void* dout, co
         info[2 * sd] = pr.k0;
         info[2 * sd + 1] = pr.ghost;
         on[sd] = 1;
+        ready[sd] = pr.flags + kFlagReady;
       }
       std::memcpy(blob + bl.peer, info, sizeof(info));
       std::memcpy(blob + bl.peer + sizeof(info), on, sizeof(on));
+      std::memcpy(blob + bl.peer + sizeof(info) + sizeof(on), ready, sizeof(ready));
     }
     std::memcpy(blob + bl.params, w.data(), w.size() * 8);
     void* args[] = {blob};

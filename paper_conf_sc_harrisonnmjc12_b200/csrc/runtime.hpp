@@ -137,6 +137,7 @@ struct PlanImpl {
   int last_variant = 0;  // 1 TMA, 2 general, 3 pointwise, 4 TMA multi-block (dfg_execute_blocks), 5 tile (cp.async ring), 6 tile multi-block,
                          // 7 rows (bulk row copies), 8 rows multi-block
   size_t rows_smem = 0;  // dynamic smem of the row-class kernel (0: unavailable)
+  uint32_t peer_wait_epoch = 0;  // != 0: the next peer launch waits in the kernel for this step's ready flags
   int64_t last_kz = 0;   // z-chunk length of the last TMA launch
   int last_halo = 0;     // halo of the last execute: 0 none, 1 NCCL, 2 local copies, 3 peer (in place), 4 peer copies
   dfg_stats st{};

@@ -20,29 +20,36 @@ pytestmark = pytest.mark.gpu
 ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 
 
-def _run(*args):
+def _run(*args, env=None):
     cmd = [sys.executable, os.path.join(ROOT, "tools", "peer_ranks.py"), *map(str, args)]
-    r = subprocess.run(cmd, capture_output=True, text=True, timeout=600, cwd=ROOT)
+    r = subprocess.run(cmd, capture_output=True, text=True, timeout=600, cwd=ROOT,
+                       env=None if env is None else dict(os.environ, **env))
     assert r.returncode == 0, r.stdout[-3000:] + r.stderr[-3000:]
     return json.loads([ln for ln in r.stdout.splitlines() if ln.startswith("{")][-1])
 
 
+@pytest.mark.parametrize("inkernel", ["1", "0"])
 @pytest.mark.parametrize("ranks,prog,dtype,nz", [(2, "qcrit", "f32", 29), (3, "qcrit", "f64", 29),
                                                  (4, "intro", "f32", 23), (3, "vortmag", "f32", 5),
                                                  (3, "qcrit", "f32", 3)])
-def test_peer_slabs_match_single_slab(ranks, prog, dtype, nz):
+def test_peer_slabs_match_single_slab(ranks, prog, dtype, nz, inkernel):
+    """inkernel 1 (default): ONE launch per execute, the producers wait in
+    the kernel for the neighbours' ready flags; 0: interior launch, stream
+    waits, boundary-plane launches."""
     if not torch.cuda.is_available():
         pytest.skip("no CUDA device")
-    line = _run("--ranks", ranks, "--n", 64, "--nz", nz, "--prog", prog, "--dtype", dtype, "--steps", 3)
+    line = _run("--ranks", ranks, "--n", 64, "--nz", nz, "--prog", prog, "--dtype", dtype, "--steps", 3,
+                env={"DFG_PEER_INKERNEL": inkernel})
     assert line["bit_identical_to_single_slab"] and line["bit_identical_to_oracle"]
     assert line["halo_modes"] == [3] * ranks                  # read in place by the TMA kernel
     assert all(line["ghost_planes_untouched"])
     assert line["halo_fields"] == (1 if prog == "intro" else 3)   # stencil fields only (intro: b)
-    # interior launch (when a slab has interior planes) + one boundary launch per side
+    # in-kernel waits: one launch; else the interior launch (when a slab has
+    # interior planes) + one boundary launch per side
     for r_, k in enumerate(line["kernels_per_execute"]):
         nzl = nz // ranks + (r_ < nz % ranks)
         sides = (r_ > 0) + (r_ < ranks - 1)
-        assert k == (1 if nzl - sides <= 0 else 1 + sides)
+        assert k == (1 if inkernel == "1" or nzl - sides <= 0 else 1 + sides)
 
 
 def test_peer_copy_fallback_for_tile_layouts():

@@ -9,6 +9,7 @@
 #   configs   ncu DRAM bytes / instructions per bench configuration -> gpurun_out/r02_configs.md
 #   rows      row-class kernel: parity, packed VisIt blocks and 1022^3 timings, one full capture
 #   small     config-2 tile / CTA sweep of the 192^3 fused kernel
+#   multi     the multi-rank tests (peer / NCCL slabs on one GPU, bench --gpus 2)
 #   sanitize  compute-sanitizer memcheck / racecheck / synccheck / initcheck on the pipelines
 #   sanitize_peer  memcheck + racecheck of the peer halo, each rank under its own sanitizer
 set -u
@@ -54,6 +55,9 @@ for task in "$@"; do
     for e in "" "DFG_CTAS=2 DFG_NCW=8" "DFG_CTAS=2 DFG_NCW=7" "DFG_KZ=16" "DFG_KZ=24" "DFG_STAGES=4" "DFG_NCW=8" "DFG_RPW=4"; do
       env $e timeout 300 python tools/small_probe.py 192 2>/dev/null | grep qcrit
     done > gpurun_out/${TAG}_small.log; cat gpurun_out/${TAG}_small.log ;;
+  multi)
+    timeout 1500 python -m pytest tests/test_gpu_peer.py tests/test_gpu_nccl.py -q -m gpu > gpurun_out/pytest_multi.log 2>&1
+    echo multi=$?; tail -3 gpurun_out/pytest_multi.log ;;
   sanitize)
     for t in memcheck racecheck synccheck initcheck; do
       timeout 900 compute-sanitizer --tool $t python tools/sanitize_run.py > gpurun_out/san_$t.log 2>&1; echo $t=$?
