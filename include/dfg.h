@@ -340,8 +340,10 @@ int dfg_plan_info(dfg_plan plan, int64_t out[14]);
  * the fused body, out[2] = two-operation axes mask (out[0] == 1),
  * out[3] = exactness domain: 2 = bit-identical for EVERY input (IEEE
  * operations only: the staged / roundtrip / hybrid kernels, and
- * DFG_FUSED_VARIANT=ieee), 1 = bit-identical whenever no intermediate of the
- * literal network is subnormal or overflows (the default fused kernel),
+ * DFG_FUSED_VARIANT=ieee), 1 = bit-identical on the cells where every
+ * input, every grad3d numerator and every value of the literal network is 0
+ * or normal with 2^p of headroom (and no numerator is -0: DESIGN.md
+ * section 5; the default fused kernel),
  * 0 = within tolerance only (fast quotient, hand-written reference
  * bodies).  `out` must hold 4 entries.  Host only; no device work. */
 int dfg_plan_arith(dfg_plan plan, int64_t out[4]);

@@ -176,9 +176,9 @@ def evaluate_full(dag: Dag, inputs: dict, x, y, z):
 
 def in_range_mask(dag: Dag, inputs: dict, x, y, z):
     """Whole mesh: True at the cells where every input value, every grad3d
-    numerator f[ip] - f[im] (each axis) and every value of the literal
-    network (each filter, each lane) is zero or has a magnitude in
-    [2^(emin + 2p), 2^(emax - p)] of T (fp32: [2^-78, 2^104], fp64:
+    numerator f[ip] - f[im] (each axis; and none of these is -0) and every
+    value of the literal network (each filter, each lane) is zero or has a
+    magnitude in [2^(emin + 2p), 2^(emax - p)] of T (fp32: [2^-78, 2^104], fp64:
     [2^-916, 2^970]; p = significand bits) -- finite, normal, with 2^p of
     headroom above and 2^(2p) below.  This is the sufficient condition of
     DESIGN.md section 5 under which the default fused kernel's reciprocal
@@ -200,6 +200,8 @@ def in_range_mask(dag: Dag, inputs: dict, x, y, z):
         mask &= ok(a)
 
     def numerators(f):
+        # and no numerator is -0: the two-operation quotient's low product
+        # takes the sign of yl, so -0 / d may come out +0
         out = np.ones(shape, dtype=bool)
         for axis in range(3):
             n = f.shape[axis]
@@ -207,7 +209,7 @@ def in_range_mask(dag: Dag, inputs: dict, x, y, z):
                 continue
             i = np.arange(n)
             num = np.take(f, np.minimum(i + 1, n - 1), axis=axis) - np.take(f, np.maximum(i - 1, 0), axis=axis)
-            out &= ok(num)
+            out &= ok(num) & ~((num == 0) & np.signbit(num))
         return out
 
     def see(k, f, v, args):

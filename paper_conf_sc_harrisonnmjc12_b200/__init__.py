@@ -148,12 +148,13 @@ class Plan:
     def __init__(self, mesh: Mesh, expr: str, strategy="fused", dev_mem_cap=0):
         self.mesh = mesh
         self.handle = dfg_compile(mesh.handle, expr, strategy, dev_mem_cap)
+        self._out_numel = mesh.nz * mesh.ny * mesh.nx * self.info()["width"]   # T[nz][ny][nx](x4)
 
     def execute(self, out, out_on_device=None, stream=None):
         if out_on_device is None:
             out_on_device = bool(getattr(out, "is_cuda", False))
         m = self.mesh
-        _check_buffer(out, m.dtype, m.nz * m.ny * m.nx * self.info()["width"], m.device, "output")
+        _check_buffer(out, m.dtype, self._out_numel, m.device, "output")
         s = stream if (stream is None or isinstance(stream, int)) else stream.cuda_stream
         dfg_execute(self.handle, out, out_on_device, s)
         return out

@@ -52,10 +52,13 @@ DFG_DEVICE double dfg_select(double c, double a, double b) { return (c != 0.0) ?
 // DFG_DIV_MODE selects how the quotient is formed:
 //   0 "ieee"  : IEEE division num / d (div.rn; ~8-10 SASS instructions);
 //   1 "exact" : Markstein's correction with the correctly rounded
-//               reciprocal: q0 = RN(num*r); rem = num - q0*d (exact by FMA);
-//               q = RN(q0 + rem*r).  Equals RN(num/d) whenever num and the
+//               reciprocal: q0 = RN(num*r); t = q0*d - num (exact by FMA);
+//               q = RN(q0 - t*r).  Equals RN(num/d) whenever num and the
 //               quotient are normal numbers away from overflow (DESIGN.md
-//               section 5); 3 instructions;
+//               section 5); 3 instructions.  The correction is formed as
+//               -t rather than num - q0*d so that a zero numerator keeps its
+//               sign: for num = -0, t = RN(-0*d + +0) = +0 and
+//               q = RN(-0 + -0) = -0 (num - q0*d would give +0 + -0 = +0);
 //   2 "fast"  : num * r (one rounding more; <= 1 ulp from num / d).
 #ifndef DFG_DIV_MODE
 #define DFG_DIV_MODE 1
@@ -81,8 +84,8 @@ DFG_DEVICE float dfg_grad1q(float num, float d, float r) {
   return __fdiv_rn(num, d);
 #elif DFG_DIV_MODE == 1
   float q0 = __fmul_rn(num, r);
-  float rem = __fmaf_rn(-q0, d, num);
-  return __fmaf_rn(rem, r, q0);
+  float t = __fmaf_rn(q0, d, -num);
+  return __fmaf_rn(-t, r, q0);
 #else
   (void)d;
   return __fmul_rn(num, r);
@@ -94,8 +97,8 @@ DFG_DEVICE double dfg_grad1q(double num, double d, double r) {
   return __ddiv_rn(num, d);
 #elif DFG_DIV_MODE == 1
   double q0 = __dmul_rn(num, r);
-  double rem = __fma_rn(-q0, d, num);
-  return __fma_rn(rem, r, q0);
+  double t = __fma_rn(q0, d, -num);
+  return __fma_rn(-t, r, q0);
 #else
   (void)d;
   return __dmul_rn(num, r);
@@ -151,9 +154,9 @@ DFG_DEVICE dfg2 dfg2_gradq(dfg2 num, dfg2 nd, dfg2 r, dfg2 z) {
 #if DFG_DIV_MODE == 0
   return make_float2(__fdiv_rn(num.x, -nd.x), __fdiv_rn(num.y, -nd.y));
 #elif DFG_DIV_MODE == 1
-  dfg2 q0 = __ffma2_rn(num, r, z);      // RN(num * r)
-  dfg2 rem = __ffma2_rn(q0, nd, num);   // num - q0*d, exact
-  return __ffma2_rn(rem, r, q0);        // RN(q0 + rem*r)
+  const dfg2 q0 = __ffma2_rn(num, r, z);                                                 // RN(num * r)
+  const dfg2 t = __ffma2_rn(make_float2(-q0.x, -q0.y), nd, make_float2(-num.x, -num.y));  // q0*d - num, exact
+  return __ffma2_rn(t, make_float2(-r.x, -r.y), q0);                                     // RN(q0 - t*r)
 #else
   return __ffma2_rn(num, r, z);
 #endif

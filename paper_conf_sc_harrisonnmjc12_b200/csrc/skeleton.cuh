@@ -120,7 +120,13 @@ extern "C" __global__ void __launch_bounds__(256) dfg_fused_pointwise(const DfgP
   const long long out_off = (P.kbeg - P.k0) * plane;
   const long long tid = (long long)blockIdx.x * blockDim.x + threadIdx.x;
   const long long stride = (long long)gridDim.x * blockDim.x;
-  const dfg2 Z = dfg2_splat(P.nzero), z0 = dfg2_splat(DFG_T(0));
+  const dfg2 Z = dfg2_splat(P.nzero);
+  // grad3d of a sub-network that reads no field (a constant): its numerator
+  // f[ip] - f[im] is +0 (or NaN), and num / d is that value for any spacing
+  // d > 0.  Unit spacing entries (d = 1: the -d / yl slot -1, r = 1) give it
+  // under every quotient form (IEEE, Markstein, two-operation, fast); zero
+  // entries would make IEEE division 0 / -0 = NaN.
+  const dfg2 nd1 = dfg2_splat(DFG_T(-1)), r1 = dfg2_splat(DFG_T(1));
   const dfg2 sz[DFG_NSF_][7] = {};
   const dfg2 gz[DFG_NSF_][3] = {};
   const long long nv = P.vec_ok ? n / DFG_VEC : 0;
@@ -134,7 +140,7 @@ extern "C" __global__ void __launch_bounds__(256) dfg_fused_pointwise(const DfgP
       dfg2 p[DFG_NPF_];
 #pragma unroll
       for (int f = 0; f < DFG_NPF; ++f) p[f] = dfg2_mk(pv[f][h * DFG_LANES], pv[f][h * DFG_LANES + DFG_LANES - 1]);
-      dfg_body(sz, gz, p, z0, z0, z0, z0, z0, z0, Z, o[h]);
+      dfg_body(sz, gz, p, nd1, r1, nd1, r1, nd1, r1, Z, o[h]);
     }
     dfg_store_cells(P.out + (out_off + v * DFG_VEC) * DFG_OUTW, o);
   }
@@ -155,7 +161,7 @@ extern "C" __global__ void __launch_bounds__(256) dfg_fused_pointwise(const DfgP
 #pragma unroll
     for (int f = 0; f < DFG_NPF; ++f) p[f] = dfg2_splat(P.f[DFG_NSF + f][idx]);
     dfg2 o[DFG_OUTW];
-    dfg_body(sz, gz, p, z0, z0, z0, z0, z0, z0, Z, o);
+    dfg_body(sz, gz, p, nd1, r1, nd1, r1, nd1, r1, Z, o);
 #pragma unroll
     for (int w = 0; w < DFG_OUTW; ++w) P.out[(out_off + c) * DFG_OUTW + w] = dfg2_get(o[w], 0);
   }
