@@ -703,24 +703,31 @@ extern "C" __global__ void __launch_bounds__(DFG_NCW * 32, DFG_CTAS)
 // or 4 rows).  So the producer loads, per field and plane, one box per class
 // (2 requests for a 194-float pitch, 4 for an odd pitch): class c's map
 // starts at the field base + (c px T) rounded down to 16 bytes (o_c elements
-// before row c's first element), its box at the column x0 + o_c rounded down
-// to a 16-byte boundary, so every row of class c lands shifted by
-// m_c = (x0 + o_c) mod VEC elements.
-// Consumers read the boxes as they are, with STRIDED cell ownership: lane l
-// of a tile row owns the cells l, l + LPR, l + 2 LPR, l + 3 LPR (LPR = lanes
-// per row), so every shared-memory access of a warp is LPR consecutive
-// 4/8-byte words -- conflict-free at any shift, one wavefront per 128 bytes
-// like the TMA kernel's 16-byte accesses -- and the x neighbours are plain
-// loads at +-1 element.  Stores are fully coalesced (consecutive lanes,
-// consecutive cells).  Mesh-end rules of reading R1: clamped rows in y (as
-// the TMA kernel), per-cell flags in x (the first global cell's x-1 and the
-// last one's x+1 read the cell itself).
+// before row c's first element), its box at the class column of tile column
+// HX-1 (the first one read) rounded down to a 16-byte boundary, so every row
+// of class c lands shifted by m_c = (x0 + o_c + HX - 1) mod VEC; the box is
+// the halo'd tile row wide (TX + 2 VEC), all a row's reads need.
+// Consumers read the boxes as they are, with full-warp row ownership (lane l
+// owns the cells l + 32 m of each of its RPW rows, below), so every
+// shared-memory access of a warp is 32 consecutive 4/8-byte words of one row
+// -- conflict-free at any shift -- and the x neighbours are plain loads at
+// +-1 element.  Stores are fully coalesced (consecutive lanes, consecutive
+// cells).  Mesh-end rules of reading R1: clamped rows in y (as the TMA
+// kernel), the cell itself written into its x-1 / x+1 slot at the first /
+// last global cell.
 // Preconditions (host): 16-byte aligned field bases and plane strides, and
 // at least P rows per plane.
-#define DFG_SBW (DFG_ROWW + DFG_VEC)     // box width: the tile row + up to VEC-1 leading elements
+// Two planes per box: a box of this size (a few KB) costs the TMA unit a
+// near-fixed ~240 cycles (tools/tma_rate.cu: 76x16x1 boxes deliver 20 B per
+// SM-cycle, 72x13x2 ones 31), so every box spans planes q and q+1 and a ring
+// stage holds two planes (slot 0 / slot 1); P x fields boxes per TWO planes.
+// box width: the halo'd tile row.  A box starts at the aligned column at or
+// below tile column HX-1 (the first one read), so the cells read span at
+// most VEC-1 + TX + 2 <= TX + 2 VEC columns from it
+#define DFG_SBW DFG_ROWW
 #define DFG_SROWS_ALLOC (DFG_ROWS + 3)   // P boxes of ceil(ROWS / P) rows, P <= 4
-// class boxes start on 128-byte boundaries (TMA destination alignment)
-#define DFG_STILE_BYTES ((DFG_SBW * DFG_SROWS_ALLOC * (int)sizeof(DFG_T) + 127) / 128 * 128 + 3 * 128)
+// class boxes (two planes each) start on 128-byte boundaries (TMA destination alignment)
+#define DFG_STILE_BYTES ((2 * DFG_SBW * DFG_SROWS_ALLOC * (int)sizeof(DFG_T) + 127) / 128 * 128 + 4 * 128)
 #define DFG_SSTAGE_BYTES (DFG_STILE_BYTES * DFG_NTF)
 typedef DfgRingT<DFG_SSTAGE_BYTES, DFG_RSTAGES> DfgRingS;
 
@@ -731,7 +738,9 @@ struct DfgRowsInfo {
   int BR;     // box rows: ceil(ROWS / P)
   int o[4];   // o_c: elements between class c's map origin and its rows' first element
   int lgP;    // log2 P
-  __device__ __forceinline__ unsigned box() const { return (unsigned)(DFG_SBW * BR * (int)sizeof(DFG_T)); }
+  // one plane of a class box (the offset of slot 1), a two-plane box, its smem stride
+  __device__ __forceinline__ unsigned slot() const { return (unsigned)(DFG_SBW * BR * (int)sizeof(DFG_T)); }
+  __device__ __forceinline__ unsigned box() const { return 2u * slot(); }
   __device__ __forceinline__ unsigned cstride() const { return (box() + 127u) & ~127u; }
 };
 struct DfgRowsParams {
@@ -759,22 +768,29 @@ struct DfgRowsItem {
   // the aligned map column and the class row index (may be -1)
   __device__ __forceinline__ int first(const DfgRowsInfo& ri, int c) const { return (c - y0) & (ri.P - 1); }
   __device__ __forceinline__ int bx(const DfgRowsInfo& ri, int c) const {
-    const int v = x0 + ri.o[c];
+    const int v = x0 + ri.o[c] + DFG_HX - 1;  // class column of tile column HX-1
     return v - (v & (DFG_VEC - 1));  // floor to a multiple of VEC (v may be negative)
   }
   __device__ __forceinline__ int by(const DfgRowsInfo& ri, int c) const {
     return (y0 + first(ri, c) - c) >> ri.lgP;  // exact: y0 + first - c is a multiple of P
   }
-  // smem byte offset (in a field tile) of tile column 0 of tile row r
+  // smem byte offset (in a field tile, slot 0) of tile column 0 of tile row r
+  // (tile column HX-1 lands at element m of its box row, so column 0 may lie
+  // before the row: only columns >= HX-1 are ever read)
   __device__ __forceinline__ unsigned row_col0(const DfgRowsInfo& ri, int r) const {
     const int c = (y0 + r) & (ri.P - 1);
-    const int m = (x0 + ri.o[c]) & (DFG_VEC - 1);
-    return (unsigned)c * ri.cstride() +
-           (unsigned)((((r - first(ri, c)) >> ri.lgP) * DFG_SBW + m) * (int)sizeof(DFG_T));
+    const int m = (x0 + ri.o[c] + DFG_HX - 1) & (DFG_VEC - 1);
+    return (unsigned)((int)c * (int)ri.cstride() +
+                      (((r - first(ri, c)) >> ri.lgP) * DFG_SBW + m - (DFG_HX - 1)) * (int)sizeof(DFG_T));
   }
 };
 
-// Producer (one lane): per stage, one TMA box per (field, row class)
+// Producer (one lane): per stage, one two-plane TMA box per (field, row
+// class): planes q, q + 1 for q = kb-1, kb+1, ... (the item's kz + 2 planes,
+// the last stage possibly half used).  Planes past the buffer ends (the
+// global ends of a mesh without ghost planes) are zero-filled by TMA and
+// never read: the consumers take the one-sided neighbours of R1 from the
+// owned plane instead (dfg_consume_rows).
 __device__ __forceinline__ void dfg_produce_rows(const DfgRowsParams& RP, long long item, DfgRingS& W) {
   const DfgParams& p = RP.p;
   const DfgRowsInfo& ri = RP.ri;
@@ -786,11 +802,10 @@ __device__ __forceinline__ void dfg_produce_rows(const DfgRowsParams& RP, long l
     bxc[c] = c < ri.P ? I.bx(ri, c) : 0;
     byc[c] = c < ri.P ? I.by(ri, c) : 0;
   }
-  for (long long q = I.kb - 1; q <= I.ke; ++q) {
-    const long long pg = max(0LL, min(q, p.NZ - 1));
+  for (long long q = I.kb - 1; q <= I.ke; q += 2) {
     dfg_mbar_wait(W.full + DfgRingS::kEmpty, W.phase ^ 1u, 0x100000u);
     dfg_mbar_expect_tx(W.full, (unsigned)(DFG_NTF * ri.P) * box);
-    const int zl = (int)(pg - p.k0 + p.ghost);
+    const int zl = (int)(q - p.k0 + p.ghost);
 #pragma unroll
     for (int f = 0; f < DFG_NTF; ++f)
 #pragma unroll
@@ -827,18 +842,24 @@ __device__ __forceinline__ void dfg_sts1(unsigned addr, DFG_T v) {
 #endif
 }
 
+// One z-plane: slot `sg` of the stage R points at.  Its z+1 neighbour is
+// slot 1 of the same stage (sg 0) or slot 0 of the next one (sg 1: wait for
+// it, and release this stage after the plane); `zend`: the last plane of
+// the mesh, whose z+1 is itself (R1).
 template <int ZM, int ZC, int ZN>
-__device__ __forceinline__ void dfg_plane_rows(const DfgCol& C, const DfgColS& Q, DfgRingS& R, unsigned& cur_tile,
-                                               unsigned& cur_full, DFG_T (&zq)[3][DFG_NSF][DFG_VEC], DFG_T*& outp,
-                                               unsigned plane, int rowpitch, const DFG_T*& tzp, long long NZ) {
+__device__ __forceinline__ void dfg_plane_rows(const DfgCol& C, const DfgColS& Q, DfgRingS& R, unsigned& sg,
+                                               unsigned pslot, DFG_T (&zq)[3][DFG_NSF][DFG_VEC], DFG_T*& outp,
+                                               unsigned plane, int rowpitch, const DFG_T*& tzp, long long NZ,
+                                               bool zend) {
   constexpr unsigned TS = (unsigned)sizeof(DFG_T), ST = 32 * TS;  // cell stride within a row
+  const unsigned cur = R.tile + (sg ? pslot : 0u);
   // y neighbours before the wait for the next stage (as the TMA kernel; fp64:
   // after it, its doubles need the registers), x neighbours after it
   DFG_T xm[DFG_NSF][DFG_VEC], xp[DFG_NSF][DFG_VEC], ym[DFG_NSF][DFG_VEC], yp[DFG_NSF][DFG_VEC];
   auto load_y = [&]() {
 #pragma unroll
     for (int f = 0; f < DFG_NSF; ++f) {
-      const unsigned t = cur_tile + f * DFG_STILE_BYTES;
+      const unsigned t = cur + f * DFG_STILE_BYTES;
 #pragma unroll
       for (int k = 0; k < DFG_VEC; ++k) {
         const int q = k / DFG_CPR;
@@ -852,7 +873,14 @@ __device__ __forceinline__ void dfg_plane_rows(const DfgCol& C, const DfgColS& Q
 #if DFG_VEC == 4
   load_y();
 #endif
-  dfg_mbar_wait(R.full, R.phase, 0x100000u);
+  // the stage after R's (ring order), waited for by a slot-1 plane
+  const bool wrap = R.stage + 1 == DFG_RSTAGES;
+  unsigned nxt = cur + pslot;
+  if (sg) {
+    dfg_mbar_wait(wrap ? R.full0 : R.full + 8u, R.phase ^ (wrap ? 1u : 0u), 0x100000u);
+    nxt = wrap ? R.tile0 : R.tile + DFG_SSTAGE_BYTES;
+  }
+  if (zend) nxt = cur;
 #if DFG_VEC == 2
   load_y();
 #endif
@@ -864,14 +892,14 @@ __device__ __forceinline__ void dfg_plane_rows(const DfgCol& C, const DfgColS& Q
     for (int f = 0; f < DFG_NSF; ++f)
 #pragma unroll
       for (int k = 0; k < DFG_VEC; ++k) {
-        const unsigned c = cur_tile + f * DFG_STILE_BYTES + Q.oc[k / DFG_CPR] + (k % DFG_CPR) * ST;
+        const unsigned c = cur + f * DFG_STILE_BYTES + Q.oc[k / DFG_CPR] + (k % DFG_CPR) * ST;
         if ((Q.flags >> k) & 1u) dfg_sts1(c - TS, zq[ZC][f][k]);
         if ((Q.flags >> (4 + k)) & 1u) dfg_sts1(c + TS, zq[ZC][f][k]);
       }
   }
 #pragma unroll
   for (int f = 0; f < DFG_NSF; ++f) {
-    const unsigned t = cur_tile + f * DFG_STILE_BYTES;
+    const unsigned t = cur + f * DFG_STILE_BYTES;
 #pragma unroll
     for (int k = 0; k < DFG_VEC; ++k) {
       const unsigned c = t + Q.oc[k / DFG_CPR] + (k % DFG_CPR) * ST;
@@ -879,13 +907,11 @@ __device__ __forceinline__ void dfg_plane_rows(const DfgCol& C, const DfgColS& Q
       xp[f][k] = dfg_lds1(c + TS);
     }
   }
-  const unsigned nxt_tile = R.tile, nxt_full = R.full;
 #pragma unroll
   for (int f = 0; f < DFG_NSF; ++f)
 #pragma unroll
     for (int k = 0; k < DFG_VEC; ++k)
-      zq[ZN][f][k] = dfg_lds1(nxt_tile + f * DFG_STILE_BYTES + Q.oc[k / DFG_CPR] + (k % DFG_CPR) * ST);
-  R.advance();
+      zq[ZN][f][k] = dfg_lds1(nxt + f * DFG_STILE_BYTES + Q.oc[k / DFG_CPR] + (k % DFG_CPR) * ST);
   dfg2 s[DFG_NPAIR][DFG_NSF][7], gn[DFG_NPAIR][DFG_NSF][3];
 #pragma unroll
   for (int f = 0; f < DFG_NSF; ++f) {
@@ -912,7 +938,7 @@ __device__ __forceinline__ void dfg_plane_rows(const DfgCol& C, const DfgColS& Q
     DFG_T pv[DFG_VEC];
 #pragma unroll
     for (int k = 0; k < DFG_VEC; ++k)
-      pv[k] = dfg_lds1(cur_tile + (DFG_NSF + f) * DFG_STILE_BYTES + Q.oc[k / DFG_CPR] + (k % DFG_CPR) * ST);
+      pv[k] = dfg_lds1(cur + (DFG_NSF + f) * DFG_STILE_BYTES + Q.oc[k / DFG_CPR] + (k % DFG_CPR) * ST);
 #pragma unroll
     for (int h = 0; h < DFG_NPAIR; ++h) p[h][f] = dfg2_mk(pv[h * DFG_LANES], pv[h * DFG_LANES + DFG_LANES - 1]);
   }
@@ -936,9 +962,11 @@ __device__ __forceinline__ void dfg_plane_rows(const DfgCol& C, const DfgColS& Q
       }
     }
   outp += (size_t)plane * DFG_OUTW;
-  dfg_mbar_arrive(cur_full + DfgRingS::kEmpty);  // every consumer thread (count NCW*32)
-  cur_tile = nxt_tile;
-  cur_full = nxt_full;
+  if (sg) {
+    dfg_mbar_arrive(R.full + DfgRingS::kEmpty);  // both planes done (every consumer thread, count NCW*32)
+    R.advance();
+  }
+  sg ^= 1u;
 }
 
 __device__ __forceinline__ void dfg_consume_rows(const DfgRowsParams& RP, long long item, DfgRingS& R, DfgCol& C,
@@ -989,35 +1017,35 @@ __device__ __forceinline__ void dfg_consume_rows(const DfgRowsParams& RP, long l
   DFG_T* outp = P.out + ((I.kb - P.k0) * (long long)plane + min(j0, P.ny - 1) * P.nx + min(i, P.nx - 1)) * DFG_OUTW;
   const DFG_T* tzp = P.tz + I.kb;
   constexpr unsigned ST = 32 * (unsigned)sizeof(DFG_T);
+  const unsigned pslot = ri.slot();
 
+  // stage 0 of the item: planes kb-1 (slot 0) and kb (slot 1).  At the
+  // global z start the z-1 neighbour of plane 0 is plane 0 itself (R1).
   DFG_T zq[3][DFG_NSF][DFG_VEC];
   dfg_mbar_wait(R.full, R.phase, 0x100000u);
+  const unsigned pre = R.tile + (I.kb == 0 ? pslot : 0u);
 #pragma unroll
   for (int f = 0; f < DFG_NSF; ++f)
 #pragma unroll
-    for (int k = 0; k < DFG_VEC; ++k)
-      zq[0][f][k] = dfg_lds1(R.tile + f * DFG_STILE_BYTES + Q.oc[k / DFG_CPR] + (k % DFG_CPR) * ST);
-  dfg_mbar_arrive(R.full + DfgRingS::kEmpty);
-  R.advance();
-  dfg_mbar_wait(R.full, R.phase, 0x100000u);
-  unsigned cur_tile = R.tile, cur_full = R.full;
-#pragma unroll
-  for (int f = 0; f < DFG_NSF; ++f)
-#pragma unroll
-    for (int k = 0; k < DFG_VEC; ++k)
-      zq[1][f][k] = dfg_lds1(cur_tile + f * DFG_STILE_BYTES + Q.oc[k / DFG_CPR] + (k % DFG_CPR) * ST);
-  R.advance();
+    for (int k = 0; k < DFG_VEC; ++k) {
+      zq[0][f][k] = dfg_lds1(pre + f * DFG_STILE_BYTES + Q.oc[k / DFG_CPR] + (k % DFG_CPR) * ST);
+      zq[1][f][k] = dfg_lds1(R.tile + pslot + f * DFG_STILE_BYTES + Q.oc[k / DFG_CPR] + (k % DFG_CPR) * ST);
+    }
+  unsigned sg = 1u;
+  const long long klast = I.ke == P.NZ ? I.ke - 1 : -1;  // the mesh's last plane (z+1 = itself)
   long long k = I.kb;
   for (; k + 3 <= I.ke; k += 3) {
-    dfg_plane_rows<0, 1, 2>(C, Q, R, cur_tile, cur_full, zq, outp, plane, (int)P.nx, tzp, P.NZ);
-    dfg_plane_rows<1, 2, 0>(C, Q, R, cur_tile, cur_full, zq, outp, plane, (int)P.nx, tzp, P.NZ);
-    dfg_plane_rows<2, 0, 1>(C, Q, R, cur_tile, cur_full, zq, outp, plane, (int)P.nx, tzp, P.NZ);
+    dfg_plane_rows<0, 1, 2>(C, Q, R, sg, pslot, zq, outp, plane, (int)P.nx, tzp, P.NZ, k == klast);
+    dfg_plane_rows<1, 2, 0>(C, Q, R, sg, pslot, zq, outp, plane, (int)P.nx, tzp, P.NZ, k + 1 == klast);
+    dfg_plane_rows<2, 0, 1>(C, Q, R, sg, pslot, zq, outp, plane, (int)P.nx, tzp, P.NZ, k + 2 == klast);
   }
   if (k < I.ke) {
-    dfg_plane_rows<0, 1, 2>(C, Q, R, cur_tile, cur_full, zq, outp, plane, (int)P.nx, tzp, P.NZ);
-    if (k + 1 < I.ke) dfg_plane_rows<1, 2, 0>(C, Q, R, cur_tile, cur_full, zq, outp, plane, (int)P.nx, tzp, P.NZ);
+    dfg_plane_rows<0, 1, 2>(C, Q, R, sg, pslot, zq, outp, plane, (int)P.nx, tzp, P.NZ, k == klast);
+    if (k + 1 < I.ke) dfg_plane_rows<1, 2, 0>(C, Q, R, sg, pslot, zq, outp, plane, (int)P.nx, tzp, P.NZ, k + 1 == klast);
   }
-  dfg_mbar_arrive(cur_full + DfgRingS::kEmpty);
+  // the stage holding plane ke (the item's post-plane) is read for its centre only
+  dfg_mbar_arrive(R.full + DfgRingS::kEmpty);
+  R.advance();
 }
 
 extern "C" __global__ void __launch_bounds__((DFG_NCW + 1) * 32, DFG_CTAS)

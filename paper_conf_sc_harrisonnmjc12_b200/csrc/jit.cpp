@@ -102,7 +102,15 @@ void parse_ptxas(const std::string& log, Cubin& c) {
 
 const Cubin& nvrtc_compile(const std::string& source, const std::string& name) {
   std::lock_guard<std::mutex> lk(g_mu);
-  auto it = g_cache.find(source);
+  // developer hook: extra -D options for kernel experiments (part of the cache key)
+  const char* xdef = std::getenv("DFG_NVRTC_DEFINES");
+  std::vector<std::string> xopts;
+  if (xdef) {
+    std::istringstream is(xdef);
+    for (std::string t; is >> t;) xopts.push_back(t);
+  }
+  const std::string key = xdef ? source + "\n//" + xdef : source;
+  auto it = g_cache.find(key);
   if (it != g_cache.end()) return *it->second;
 
   NvrtcApi& api = nvrtc();
@@ -114,7 +122,9 @@ const Cubin& nvrtc_compile(const std::string& source, const std::string& name) {
                         "--ftz=false",                "--prec-div=true",    "--prec-sqrt=true",
                         "--device-as-default-execution-space", "--generate-line-info",
                         "--ptxas-options=-v",         "-DNDEBUG"};
-  nvrtcResult rc = api.CompileProgram(prog, int(sizeof(opts) / sizeof(opts[0])), opts);
+  std::vector<const char*> all(opts, opts + sizeof(opts) / sizeof(opts[0]));
+  for (const auto& t : xopts) all.push_back(t.c_str());
+  nvrtcResult rc = api.CompileProgram(prog, int(all.size()), all.data());
   size_t log_size = 0;
   api.GetProgramLogSize(prog, &log_size);
   std::string log(log_size, '\0');
@@ -135,7 +145,7 @@ const Cubin& nvrtc_compile(const std::string& source, const std::string& name) {
   c->log = log;
   parse_ptxas(log, *c);
   const Cubin& ref = *c;
-  g_cache.emplace(source, std::move(c));
+  g_cache.emplace(key, std::move(c));
   return ref;
 }
 

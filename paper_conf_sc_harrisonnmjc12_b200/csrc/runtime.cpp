@@ -404,7 +404,7 @@ int row_period(const SlabView& m) {
 // 64 B | DfgParams.  Class c of a field: the rows y = c (mod P) as a 3-D
 // tensor from base + (c px T) rounded down to 16 bytes (o_c elements before
 // the row's first element), dims {px + o_c, rows of the class, planes},
-// strides {P px T, px py T} (both multiples of 16), box {TX + 3 VEC, BR, 1}.
+// strides {P px T, px py T} (both multiples of 16), box {TX + 2 VEC, BR, 2} (two planes).
 std::vector<unsigned char> rows_blob(const std::vector<const void*>& fptr, int nf_, const SlabView& m, int ncw,
                                      int rpw, const std::vector<uint64_t>& words) {
   const size_t ts = dsize(m.dt);
@@ -423,7 +423,7 @@ std::vector<unsigned char> rows_blob(const std::vector<const void*>& fptr, int n
       cuuint64_t gdim[3] = {cuuint64_t(m.px() + o), cuuint64_t((m.py() - c + P - 1) / P),
                             cuuint64_t(m.nzl + 2 * m.ghost)};
       cuuint64_t gstride[2] = {cuuint64_t(P) * cuuint64_t(m.px()) * ts, cuuint64_t(m.px() * m.py()) * ts};
-      cuuint32_t box[3] = {cuuint32_t(tma_tile_w(m.dt, rpw) + 3 * vec), cuuint32_t(BR), 1};
+      cuuint32_t box[3] = {cuuint32_t(tma_tile_w(m.dt, rpw) + 2 * vec), cuuint32_t(BR), 2};  // two planes
       cuuint32_t estr[3] = {1, 1, 1};
       DFG_CU(drv().TensorMapEncodeTiled(reinterpret_cast<CUtensorMap*>(blob.data() + 128 * (f * 4 + size_t(c))),
                                         m.dt == DType::F32 ? CU_TENSOR_MAP_DATA_TYPE_FLOAT32
