@@ -157,7 +157,12 @@ std::unique_ptr<PlanImpl> compile_plan(std::shared_ptr<MeshImpl> mesh, const std
     } else if (ncw) {
       cfg.rpw = choose_rpw(mesh->dt, mesh->nx, mesh->ny, mesh->nzl, cfg.ncw, slots);
     } else {
-      choose_tile(mesh->dt, mesh->nx, mesh->ny, mesh->nzl, slots, &cfg.ncw, &cfg.rpw);
+      // layouts a tensor map cannot take run the row-class kernel (fused_tma.cuh "rows")
+      const int64_t vec = int64_t(16 / dsize(mesh->dt));
+      if (mesh->nx % vec == 0 && mesh->px() % vec == 0 && mesh->gx() % vec == 0)
+        choose_tile(mesh->dt, mesh->nx, mesh->ny, mesh->nzl, slots, &cfg.ncw, &cfg.rpw);
+      else
+        choose_rows_tile(mesh->dt, mesh->nx, mesh->ny, mesh->nzl, slots, &cfg.ncw, &cfg.rpw);
     }
     // axis degeneracy (n == 1) is a property of the GLOBAL mesh
     plan->fsrc = generate_fused(dag, mesh->NX, mesh->NY, mesh->NZ, cfg, ref);
