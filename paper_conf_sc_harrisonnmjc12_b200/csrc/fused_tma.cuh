@@ -184,7 +184,7 @@ __device__ __forceinline__ void dfg_store_masked(DFG_T* dst, const dfg2 (&o)[DFG
 template <int ZM, int ZC, int ZN, bool MASKED = false, class Fill = DfgNoFill, class Ring = DfgRing>
 __device__ __forceinline__ void dfg_plane(const DfgCol& C, Ring& R, unsigned& cur_tile, unsigned& cur_full,
                                           DFG_T (&zq)[3][DFG_NSF][DFG_VEC], DFG_T*& outp,
-                                          long long plane, const DFG_T*& tzp, long long NZ, Fill& fill) {
+                                          long long plane, const DFG_T*& tzd, const DFG_T*& tzr, Fill& fill) {
   // x/y neighbours of this plane first (its stage is already resident), then
   // wait for the next plane's stage: the loads overlap the barrier wait
   DFG_T xmv[DFG_NSF], xpv[DFG_NSF], ymv[DFG_NSF][DFG_VEC], ypv[DFG_NSF][DFG_VEC];
@@ -229,8 +229,9 @@ __device__ __forceinline__ void dfg_plane(const DfgCol& C, Ring& R, unsigned& cu
       gn[h][f][2] = dfg2_sub(s[h][f][6], s[h][f][5], C.Z);
     }
   }
-  const dfg2 ndz = dfg2_splat(__ldg(tzp + DFG_NDSEG_Z * NZ)), rz = dfg2_splat(__ldg(tzp + NZ));
-  ++tzp;
+  const dfg2 ndz = dfg2_splat(__ldg(tzd)), rz = dfg2_splat(__ldg(tzr));
+  ++tzd;
+  ++tzr;
   dfg2 p[DFG_NPAIR][DFG_NPF_];
 #pragma unroll
   for (int f = 0; f < DFG_NPF; ++f) {
@@ -361,7 +362,8 @@ __device__ __forceinline__ void dfg_consume_item(const DfgTmaParams& TP, long lo
   C.off_yp = (rp * DFG_ROWW + c0) * TS;
   const long long cell0 = (kb - P.k0) * plane + jc * P.nx + ic;
   DFG_T* outp = P.out + cell0 * DFG_OUTW;
-  const DFG_T* tzp = P.tz + kb;
+  const DFG_T* tzd = P.tz + DFG_NDSEG_Z * P.NZ + kb;  // -d and 1/d of the plane's z spacing
+  const DFG_T* tzr = P.tz + P.NZ + kb;
 
   DFG_T zq[3][DFG_NSF][DFG_VEC];
   // pre-plane (clamped): its centre becomes z-1 of plane kb
@@ -378,13 +380,13 @@ __device__ __forceinline__ void dfg_consume_item(const DfgTmaParams& TP, long lo
   DfgNoFill nf;
   long long k = kb;
   for (; k + 3 <= ke; k += 3) {
-    dfg_plane<0, 1, 2>(C, R, cur_tile, cur_full, zq, outp, plane, tzp, P.NZ, nf);
-    dfg_plane<1, 2, 0>(C, R, cur_tile, cur_full, zq, outp, plane, tzp, P.NZ, nf);
-    dfg_plane<2, 0, 1>(C, R, cur_tile, cur_full, zq, outp, plane, tzp, P.NZ, nf);
+    dfg_plane<0, 1, 2>(C, R, cur_tile, cur_full, zq, outp, plane, tzd, tzr, nf);
+    dfg_plane<1, 2, 0>(C, R, cur_tile, cur_full, zq, outp, plane, tzd, tzr, nf);
+    dfg_plane<2, 0, 1>(C, R, cur_tile, cur_full, zq, outp, plane, tzd, tzr, nf);
   }
   if (k < ke) {
-    dfg_plane<0, 1, 2>(C, R, cur_tile, cur_full, zq, outp, plane, tzp, P.NZ, nf);
-    if (k + 1 < ke) dfg_plane<1, 2, 0>(C, R, cur_tile, cur_full, zq, outp, plane, tzp, P.NZ, nf);
+    dfg_plane<0, 1, 2>(C, R, cur_tile, cur_full, zq, outp, plane, tzd, tzr, nf);
+    if (k + 1 < ke) dfg_plane<1, 2, 0>(C, R, cur_tile, cur_full, zq, outp, plane, tzd, tzr, nf);
   }
   // the post-plane stage was read for its centre only
   dfg_mbar_arrive(DFG_EMPTY(cur_full));
@@ -618,7 +620,8 @@ __device__ __forceinline__ void dfg_consume_tile(const DfgParams& P, long long i
   C.off_ym = ((r - 1) * DFG_ROWW + c0) * TS;
   C.off_yp = ((r + 1) * DFG_ROWW + c0) * TS;
   DFG_T* outp = P.out + ((kb - P.k0) * plane + jc * P.nx + ic) * DFG_OUTW;
-  const DFG_T* tzp = P.tz + kb;
+  const DFG_T* tzd = P.tz + DFG_NDSEG_Z * P.NZ + kb;  // -d and 1/d of the plane's z spacing
+  const DFG_T* tzr = P.tz + P.NZ + kb;
 
   DFG_T zq[3][DFG_NSF][DFG_VEC];
   dfg_mbar_wait(R.full, R.phase, 0x100000u);
@@ -634,13 +637,13 @@ __device__ __forceinline__ void dfg_consume_tile(const DfgParams& P, long long i
   R.advance();
   long long k = kb;
   for (; k + 3 <= ke; k += 3) {
-    dfg_plane<0, 1, 2, true, Fill, Ring>(C, R, cur_tile, cur_full, zq, outp, plane, tzp, P.NZ, F);
-    dfg_plane<1, 2, 0, true, Fill, Ring>(C, R, cur_tile, cur_full, zq, outp, plane, tzp, P.NZ, F);
-    dfg_plane<2, 0, 1, true, Fill, Ring>(C, R, cur_tile, cur_full, zq, outp, plane, tzp, P.NZ, F);
+    dfg_plane<0, 1, 2, true, Fill, Ring>(C, R, cur_tile, cur_full, zq, outp, plane, tzd, tzr, F);
+    dfg_plane<1, 2, 0, true, Fill, Ring>(C, R, cur_tile, cur_full, zq, outp, plane, tzd, tzr, F);
+    dfg_plane<2, 0, 1, true, Fill, Ring>(C, R, cur_tile, cur_full, zq, outp, plane, tzd, tzr, F);
   }
   if (k < ke) {
-    dfg_plane<0, 1, 2, true, Fill, Ring>(C, R, cur_tile, cur_full, zq, outp, plane, tzp, P.NZ, F);
-    if (k + 1 < ke) dfg_plane<1, 2, 0, true, Fill, Ring>(C, R, cur_tile, cur_full, zq, outp, plane, tzp, P.NZ, F);
+    dfg_plane<0, 1, 2, true, Fill, Ring>(C, R, cur_tile, cur_full, zq, outp, plane, tzd, tzr, F);
+    if (k + 1 < ke) dfg_plane<1, 2, 0, true, Fill, Ring>(C, R, cur_tile, cur_full, zq, outp, plane, tzd, tzr, F);
   }
   dfg_mbar_arrive(cur_full + Ring::kEmpty);
   F.step();
@@ -825,9 +828,8 @@ __device__ __forceinline__ void dfg_produce_rows(const DfgRowsParams& RP, long l
 // per-item constants of a consumer thread: smem byte offsets (in a field
 // tile) of its first cell in each of its rows and of that cell's y-1 / y+1
 // neighbours (clamped at the global ends); bits 0-3 / 4-7: cell k is the
-// first / last global cell of its row (its x-1 / x+1 is itself); bits
-// 8-11: row q is the last global row (its y+1 is itself).  Between the
-// thread's own rows the y neighbours come from registers (the centres).
+// first / last global cell of its row (its x-1 / x+1 is itself).  Between
+// the thread's own rows the y neighbours come from registers (the centres).
 struct DfgColS {
   unsigned oc[DFG_RPW], om[DFG_RPW], op[DFG_RPW];
   unsigned flags;
@@ -849,7 +851,7 @@ __device__ __forceinline__ void dfg_sts1(unsigned addr, DFG_T v) {
 template <int ZM, int ZC, int ZN>
 __device__ __forceinline__ void dfg_plane_rows(const DfgCol& C, const DfgColS& Q, DfgRingS& R, unsigned& sg,
                                                unsigned pslot, DFG_T (&zq)[3][DFG_NSF][DFG_VEC], DFG_T*& outp,
-                                               unsigned plane, int rowpitch, const DFG_T*& tzp, long long NZ,
+                                               unsigned plane, int rowpitch, const DFG_T*& tzd, const DFG_T*& tzr,
                                                bool zend) {
   constexpr unsigned TS = (unsigned)sizeof(DFG_T), ST = 32 * TS;  // cell stride within a row
   const unsigned cur = R.tile + (sg ? pslot : 0u);
@@ -865,8 +867,10 @@ __device__ __forceinline__ void dfg_plane_rows(const DfgCol& C, const DfgColS& Q
         const int q = k / DFG_CPR;
         if (q == 0) ym[f][k] = dfg_lds1(t + Q.om[0] + (k % DFG_CPR) * ST);
         else ym[f][k] = zq[ZC][f][k - DFG_CPR];  // the row above is this thread's (never a global end)
+        // the row below: this thread's next row (a row past the global end
+        // holds this row's centres: its offsets are clamped, R1)
         if (q == DFG_RPW - 1) yp[f][k] = dfg_lds1(t + Q.op[q] + (k % DFG_CPR) * ST);
-        else yp[f][k] = (Q.flags >> (8 + q)) & 1u ? zq[ZC][f][k] : zq[ZC][f][k + DFG_CPR];
+        else yp[f][k] = zq[ZC][f][k + DFG_CPR];
       }
     }
   };
@@ -893,7 +897,8 @@ __device__ __forceinline__ void dfg_plane_rows(const DfgCol& C, const DfgColS& Q
 #pragma unroll
       for (int k = 0; k < DFG_VEC; ++k) {
         const unsigned c = cur + f * DFG_STILE_BYTES + Q.oc[k / DFG_CPR] + (k % DFG_CPR) * ST;
-        if ((Q.flags >> k) & 1u) dfg_sts1(c - TS, zq[ZC][f][k]);
+        // the first global cell is a tile's first column (lane 0, m = 0)
+        if (k % DFG_CPR == 0 && ((Q.flags >> k) & 1u)) dfg_sts1(c - TS, zq[ZC][f][k]);
         if ((Q.flags >> (4 + k)) & 1u) dfg_sts1(c + TS, zq[ZC][f][k]);
       }
   }
@@ -930,8 +935,9 @@ __device__ __forceinline__ void dfg_plane_rows(const DfgCol& C, const DfgColS& Q
       gn[h][f][2] = dfg2_sub(s[h][f][6], s[h][f][5], C.Z);
     }
   }
-  const dfg2 ndz = dfg2_splat(__ldg(tzp + DFG_NDSEG_Z * NZ)), rz = dfg2_splat(__ldg(tzp + NZ));
-  ++tzp;
+  const dfg2 ndz = dfg2_splat(__ldg(tzd)), rz = dfg2_splat(__ldg(tzr));
+  ++tzd;
+  ++tzr;
   dfg2 p[DFG_NPAIR][DFG_NPF_];
 #pragma unroll
   for (int f = 0; f < DFG_NPF; ++f) {
@@ -1012,10 +1018,13 @@ __device__ __forceinline__ void dfg_consume_rows(const DfgRowsParams& RP, long l
     Q.oc[q] = I.row_col0(ri, r) + cb;
     Q.om[q] = (jg == 0) ? Q.oc[q] : I.row_col0(ri, r - 1) + cb;
     Q.op[q] = (jg >= P.NY - 1) ? Q.oc[q] : I.row_col0(ri, r + 1) + cb;
-    Q.flags |= (jg >= P.NY - 1 ? 1u : 0u) << (8 + q);
+    // a row past the global end (never stored) reads the row above: the
+    // y+1 of the last global row is then itself, from registers (R1)
+    if (q > 0 && jg > P.NY - 1) Q.oc[q] = Q.oc[q - 1];
   }
   DFG_T* outp = P.out + ((I.kb - P.k0) * (long long)plane + min(j0, P.ny - 1) * P.nx + min(i, P.nx - 1)) * DFG_OUTW;
-  const DFG_T* tzp = P.tz + I.kb;
+  const DFG_T* tzd = P.tz + DFG_NDSEG_Z * P.NZ + I.kb;  // -d and 1/d of the plane's z spacing
+  const DFG_T* tzr = P.tz + P.NZ + I.kb;
   constexpr unsigned ST = 32 * (unsigned)sizeof(DFG_T);
   const unsigned pslot = ri.slot();
 
@@ -1032,16 +1041,17 @@ __device__ __forceinline__ void dfg_consume_rows(const DfgRowsParams& RP, long l
       zq[1][f][k] = dfg_lds1(R.tile + pslot + f * DFG_STILE_BYTES + Q.oc[k / DFG_CPR] + (k % DFG_CPR) * ST);
     }
   unsigned sg = 1u;
-  const long long klast = I.ke == P.NZ ? I.ke - 1 : -1;  // the mesh's last plane (z+1 = itself)
-  long long k = I.kb;
-  for (; k + 3 <= I.ke; k += 3) {
-    dfg_plane_rows<0, 1, 2>(C, Q, R, sg, pslot, zq, outp, plane, (int)P.nx, tzp, P.NZ, k == klast);
-    dfg_plane_rows<1, 2, 0>(C, Q, R, sg, pslot, zq, outp, plane, (int)P.nx, tzp, P.NZ, k + 1 == klast);
-    dfg_plane_rows<2, 0, 1>(C, Q, R, sg, pslot, zq, outp, plane, (int)P.nx, tzp, P.NZ, k + 2 == klast);
+  const int n = (int)(I.ke - I.kb);
+  const int last = I.ke == P.NZ ? n - 1 : -1;  // the mesh's last plane (z+1 = itself, R1)
+  int t = 0;
+  for (; t + 3 <= n; t += 3) {
+    dfg_plane_rows<0, 1, 2>(C, Q, R, sg, pslot, zq, outp, plane, (int)P.nx, tzd, tzr, t == last);
+    dfg_plane_rows<1, 2, 0>(C, Q, R, sg, pslot, zq, outp, plane, (int)P.nx, tzd, tzr, t + 1 == last);
+    dfg_plane_rows<2, 0, 1>(C, Q, R, sg, pslot, zq, outp, plane, (int)P.nx, tzd, tzr, t + 2 == last);
   }
-  if (k < I.ke) {
-    dfg_plane_rows<0, 1, 2>(C, Q, R, sg, pslot, zq, outp, plane, (int)P.nx, tzp, P.NZ, k == klast);
-    if (k + 1 < I.ke) dfg_plane_rows<1, 2, 0>(C, Q, R, sg, pslot, zq, outp, plane, (int)P.nx, tzp, P.NZ, k + 1 == klast);
+  if (t < n) {
+    dfg_plane_rows<0, 1, 2>(C, Q, R, sg, pslot, zq, outp, plane, (int)P.nx, tzd, tzr, t == last);
+    if (t + 1 < n) dfg_plane_rows<1, 2, 0>(C, Q, R, sg, pslot, zq, outp, plane, (int)P.nx, tzd, tzr, t + 1 == last);
   }
   // the stage holding plane ke (the item's post-plane) is read for its centre only
   dfg_mbar_arrive(R.full + DfgRingS::kEmpty);
