@@ -395,7 +395,8 @@ __device__ __forceinline__ void dfg_consume_item(const DfgTmaParams& TP, long lo
 // full_count: arrivals that complete a "full" phase (1 for the TMA
 // producer's arrive.expect_tx; every consumer thread for the tile kernel)
 __device__ __forceinline__ unsigned dfg_ring_init(unsigned full_count = 1, unsigned stage_bytes = DFG_STAGE_BYTES,
-                                                  int stages = DFG_STAGES, unsigned empty_count = DFG_NCW * 32) {
+                                                  int stages = DFG_STAGES, unsigned empty_count = DFG_NCW * 32,
+                                                  bool ready = false) {
   // dynamic shared memory starts at the (1024-aligned) base of the CTA's
   // window: no static __shared__ in this kernel
   extern __shared__ __align__(1024) unsigned char dfg_smem_raw[];
@@ -405,6 +406,7 @@ __device__ __forceinline__ unsigned dfg_ring_init(unsigned full_count = 1, unsig
     for (int s = 0; s < stages; ++s) {
       dfg_mbar_init(full0 + 8 * s, full_count);
       dfg_mbar_init(full0 + 8 * s + 8 * stages, empty_count);
+      if (ready) dfg_mbar_init(full0 + 8 * s + 16 * stages, 1);  // ready[s] = full[s] + 16*stages
     }
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   }
@@ -716,8 +718,10 @@ extern "C" __global__ void __launch_bounds__(DFG_NCW * 32, DFG_CTAS)
 // -- conflict-free at any shift -- and the x neighbours are plain loads at
 // +-1 element.  Stores are fully coalesced (consecutive lanes, consecutive
 // cells).  Mesh-end rules of reading R1: clamped rows in y (as the TMA
-// kernel), the cell itself written into its x-1 / x+1 slot at the first /
-// last global cell.
+// kernel); in x a FIXUP warp writes, once TMA has landed a stage, the first
+// / last global cell of every row into the slot its x-1 / x+1 reads, then
+// releases the stage to the consumers ("ready" barriers), so the consumers
+// carry no x-end code at all.
 // Preconditions (host): 16-byte aligned field bases and plane strides, and
 // at least P rows per plane.
 // Two planes per box: a box of this size (a few KB) costs the TMA unit a
@@ -827,14 +831,13 @@ __device__ __forceinline__ void dfg_produce_rows(const DfgRowsParams& RP, long l
 #define DFG_CPR (DFG_VEC / DFG_RPW)
 // per-item constants of a consumer thread: smem byte offsets (in a field
 // tile) of its first cell in each of its rows and of that cell's y-1 / y+1
-// neighbours (clamped at the global ends); bits 0-3 / 4-7: cell k is the
-// first / last global cell of its row (its x-1 / x+1 is itself).  Between
-// the thread's own rows the y neighbours come from registers (the centres).
+// neighbours (clamped at the global ends).  Between the thread's own rows the
+// y neighbours come from registers (the centres).
 struct DfgColS {
   unsigned oc[DFG_RPW], om[DFG_RPW], op[DFG_RPW];
-  unsigned flags;
   DFG_T ndy[DFG_RPW], ry[DFG_RPW];  // y spacing entries of each of the thread's rows
 };
+#define DFG_KREADY (16u * DFG_RSTAGES)  // ready[s] = full[s] + 16 * stages (fixup warp -> consumers)
 
 __device__ __forceinline__ void dfg_sts1(unsigned addr, DFG_T v) {
 #if DFG_VEC == 4
@@ -881,27 +884,13 @@ __device__ __forceinline__ void dfg_plane_rows(const DfgCol& C, const DfgColS& Q
   const bool wrap = R.stage + 1 == DFG_RSTAGES;
   unsigned nxt = cur + pslot;
   if (sg) {
-    dfg_mbar_wait(wrap ? R.full0 : R.full + 8u, R.phase ^ (wrap ? 1u : 0u), 0x100000u);
+    dfg_mbar_wait((wrap ? R.full0 : R.full + 8u) + DFG_KREADY, R.phase ^ (wrap ? 1u : 0u), 0x100000u);
     nxt = wrap ? R.tile0 : R.tile + DFG_SSTAGE_BYTES;
   }
   if (zend) nxt = cur;
 #if DFG_VEC == 2
   load_y();
 #endif
-  if (Q.flags & 0xffu) {
-    // a global x end (R1: one-sided): the thread owning the first / last
-    // global cell writes the cell itself into the slot its x-1 / x+1 reads;
-    // only it reads that slot (other threads see it as an inactive cell)
-#pragma unroll
-    for (int f = 0; f < DFG_NSF; ++f)
-#pragma unroll
-      for (int k = 0; k < DFG_VEC; ++k) {
-        const unsigned c = cur + f * DFG_STILE_BYTES + Q.oc[k / DFG_CPR] + (k % DFG_CPR) * ST;
-        // the first global cell is a tile's first column (lane 0, m = 0)
-        if (k % DFG_CPR == 0 && ((Q.flags >> k) & 1u)) dfg_sts1(c - TS, zq[ZC][f][k]);
-        if ((Q.flags >> (4 + k)) & 1u) dfg_sts1(c + TS, zq[ZC][f][k]);
-      }
-  }
 #pragma unroll
   for (int f = 0; f < DFG_NSF; ++f) {
     const unsigned t = cur + f * DFG_STILE_BYTES;
@@ -988,13 +977,10 @@ __device__ __forceinline__ void dfg_consume_rows(const DfgRowsParams& RP, long l
   const unsigned cb = (unsigned)(DFG_HX + lane) * TS;  // tile column of cell m = 0
   DfgColS Q;
   C.nvalid = 0;
-  Q.flags = 0;
 #pragma unroll
   for (int k = 0; k < DFG_VEC; ++k) {
     const long long ik = i + 32 * (k % DFG_CPR), jk = j0 + k / DFG_CPR;
     C.nvalid |= (ik < P.nx && jk < P.ny ? 1 : 0) << k;
-    Q.flags |= (P.i0 + ik == 0 ? 1u : 0u) << k;
-    Q.flags |= (P.i0 + ik == P.NX - 1 ? 1u : 0u) << (4 + k);
   }
 #pragma unroll
   for (int h = 0; h < DFG_NPAIR; ++h) {
@@ -1031,7 +1017,7 @@ __device__ __forceinline__ void dfg_consume_rows(const DfgRowsParams& RP, long l
   // stage 0 of the item: planes kb-1 (slot 0) and kb (slot 1).  At the
   // global z start the z-1 neighbour of plane 0 is plane 0 itself (R1).
   DFG_T zq[3][DFG_NSF][DFG_VEC];
-  dfg_mbar_wait(R.full, R.phase, 0x100000u);
+  dfg_mbar_wait(R.full + DFG_KREADY, R.phase, 0x100000u);
   const unsigned pre = R.tile + (I.kb == 0 ? pslot : 0u);
 #pragma unroll
   for (int f = 0; f < DFG_NSF; ++f)
@@ -1058,12 +1044,53 @@ __device__ __forceinline__ void dfg_consume_rows(const DfgRowsParams& RP, long l
   R.advance();
 }
 
-extern "C" __global__ void __launch_bounds__((DFG_NCW + 1) * 32, DFG_CTAS)
+// Fixup warp (R1 in x): per stage, once TMA has landed it, the first /
+// last GLOBAL cell of every owned tile row is copied into the slot its x-1 /
+// x+1 neighbour is read from (both planes, every stencil field), then the
+// stage goes to the consumers (ready).  Every stage passes through here, so
+// the ready barriers advance exactly once per lap, like full.
+__device__ __forceinline__ void dfg_fixup_rows(const DfgRowsParams& RP, long long item, DfgRingS& W, int lane) {
+  const DfgParams& p = RP.p;
+  const DfgRowsInfo& ri = RP.ri;
+  const DfgRowsItem I(p, item);
+  constexpr unsigned TS = (unsigned)sizeof(DFG_T);
+  const bool first = p.i0 == 0 && I.tx == 0;                   // global column 0 at tile column HX
+  const long long tl = p.NX - 1 - p.i0 - (long long)I.tx * DFG_TX;  // tile offset of the global last column
+  const bool last = tl >= 0 && tl < DFG_TX;
+  const unsigned pslot = ri.slot();
+  for (long long q = I.kb - 1; q <= I.ke; q += 2) {
+    dfg_mbar_wait(W.full, W.phase, 0x100000u);
+    if (first || last) {
+#pragma unroll 1
+      for (int r = 1 + lane; r <= DFG_TH; r += 32) {
+        const unsigned o = W.tile + I.row_col0(ri, r);
+#pragma unroll
+        for (int f = 0; f < DFG_NSF; ++f)
+#pragma unroll
+          for (int sl = 0; sl < 2; ++sl) {
+            const unsigned t = o + f * DFG_STILE_BYTES + (sl ? pslot : 0u);
+            if (first) dfg_sts1(t + (DFG_HX - 1) * TS, dfg_lds1(t + DFG_HX * TS));
+            if (last) dfg_sts1(t + (unsigned)(DFG_HX + tl + 1) * TS, dfg_lds1(t + (unsigned)(DFG_HX + tl) * TS));
+          }
+      }
+      __syncwarp();
+    }
+    if (lane == 0) dfg_mbar_arrive(W.full + DFG_KREADY);  // release: the slots are written
+    W.advance();
+  }
+}
+
+extern "C" __global__ void __launch_bounds__((DFG_NCW + 2) * 32, DFG_CTAS)
     dfg_fused_rows(const __grid_constant__ DfgRowsParams RP) {
-  const unsigned smem = dfg_ring_init(1, DFG_SSTAGE_BYTES, DFG_RSTAGES);
+  const unsigned smem = dfg_ring_init(1, DFG_SSTAGE_BYTES, DFG_RSTAGES, DFG_NCW * 32, true);
   const unsigned full0 = smem + DFG_RSTAGES * DFG_SSTAGE_BYTES;
   const int warp = threadIdx.x >> 5;
   const int lane = threadIdx.x & 31;
+  if (warp == DFG_NCW + 1) {
+    DfgRingS W{smem, full0, 0u, 0, smem, full0};
+    for (long long item = blockIdx.x; item < RP.p.items; item += gridDim.x) dfg_fixup_rows(RP, item, W, lane);
+    return;
+  }
   if (warp == DFG_NCW) {
     if (lane == 0) {
       for (int f = 0; f < DFG_NTF * 4; ++f)
@@ -1087,14 +1114,22 @@ struct DfgRowsMulti {
   int nb;
 };
 
-extern "C" __global__ void __launch_bounds__((DFG_NCW + 1) * 32, DFG_CTAS)
+extern "C" __global__ void __launch_bounds__((DFG_NCW + 2) * 32, DFG_CTAS)
     dfg_fused_rows_multi(const __grid_constant__ DfgRowsMulti M) {
-  const unsigned smem = dfg_ring_init(1, DFG_SSTAGE_BYTES, DFG_RSTAGES);
+  const unsigned smem = dfg_ring_init(1, DFG_SSTAGE_BYTES, DFG_RSTAGES, DFG_NCW * 32, true);
   const unsigned full0 = smem + DFG_RSTAGES * DFG_SSTAGE_BYTES;
   const int warp = threadIdx.x >> 5;
   const int lane = threadIdx.x & 31;
   const long long total = M.first[M.nb];
   int b = 0;
+  if (warp == DFG_NCW + 1) {
+    DfgRingS W{smem, full0, 0u, 0, smem, full0};
+    for (long long item = blockIdx.x; item < total; item += gridDim.x) {
+      while (item >= M.first[b + 1]) ++b;
+      dfg_fixup_rows(M.blocks[b], item - M.first[b], W, lane);
+    }
+    return;
+  }
   if (warp == DFG_NCW) {
     if (lane == 0) {
       DfgRingS W{smem, full0, 0u, 0, smem, full0};

@@ -779,8 +779,9 @@ void PlanImpl::launch_fused(const std::vector<const void*>& fptr, void* dout, co
     last_variant = 1;
     last_kz = best_kz;
   } else if (rows_ok(fptr, m)) {
-    // TMA row-class boxes, read in place by strided-cell consumers
-    const int ncw = fsrc.cfg.ncw, rpw = fsrc.cfg.rpw, threads = (ncw + 1) * 32;
+    // TMA row-class boxes, read in place by strided-cell consumers (+ the
+    // producer and the x-end fixup warp)
+    const int ncw = fsrc.cfg.ncw, rpw = fsrc.cfg.rpw, threads = (ncw + 2) * 32;
     const int tw = tma_tile_w(m.dt, rpw), th = tma_tile_h(ncw, rpw);
     const int tiles_x = int((m.nx + tw - 1) / tw);
     const int tiles_y = int((m.ny + th - 1) / th);
@@ -901,7 +902,7 @@ void execute_blocks(const std::vector<PlanImpl*>& plans, const std::vector<void*
   const int nsf = int(L.stencil_inputs.size() + L.point_inputs.size());
   const size_t smem = rows ? p0.rows_smem : fused_tma_smem_bytes(m0.dt, nsf, ncw, kc.stages, rpw);
   CUfunction fn = tma ? p0.mod.tma_multi : rows ? p0.mod.rows_multi : p0.mod.tile_multi;
-  const int threads = tma || rows ? (ncw + 1) * 32 : ncw * 32;
+  const int threads = rows ? (ncw + 2) * 32 : tma ? (ncw + 1) * 32 : ncw * 32;
   int occ = 1;
   DFG_CU(drv().OccupancyMaxActiveBlocksPerMultiprocessor(&occ, fn, threads, smem));
   const int64_t slots = int64_t(sm_count(m0.device)) * std::max(occ, 1);
