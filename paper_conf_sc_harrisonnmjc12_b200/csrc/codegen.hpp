@@ -68,9 +68,10 @@ int choose_rpw(DType dt, int64_t nx, int64_t ny, int64_t nz, int ncw, int64_t sl
 // e.g. 192 rows = 8 tiles of 24) and rows per warp.
 void choose_tile(DType dt, int64_t nx, int64_t ny, int64_t nz, int64_t slots, int* ncw, int* rpw);
 // the same for layouts only the row-class kernel takes (packed ghost shells,
-// rows that are not 16-byte multiples): no ragged last y-tile when 12 warps
-// divide the rows and 15 do not (its two-plane ring makes the rows, not the
-// halo, the cost: 192-row blocks 260 -> 288 Gcells/s with 12 x 2 rows)
+// rows that are not 16-byte multiples): 14 or 12 consumer warps (the kernel
+// adds a producer and a fixup warp: 16 warps keep 128 registers), 12 when
+// 14 leave more of a ragged last y-tile idle (its two-plane ring makes the
+// rows, not the halo, the cost: 192-row blocks 260 -> 288 Gcells/s with 12 x 2)
 void choose_rows_tile(DType dt, int64_t nx, int64_t ny, int64_t nz, int64_t slots, int* ncw, int* rpw);
 
 // z-chunk length for `tiles` x-y tiles over `range` planes: whole rounds of

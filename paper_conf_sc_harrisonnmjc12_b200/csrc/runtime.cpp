@@ -157,9 +157,12 @@ std::unique_ptr<PlanImpl> compile_plan(std::shared_ptr<MeshImpl> mesh, const std
     } else if (ncw) {
       cfg.rpw = choose_rpw(mesh->dt, mesh->nx, mesh->ny, mesh->nzl, cfg.ncw, slots);
     } else {
-      // layouts a tensor map cannot take run the row-class kernel (fused_tma.cuh "rows")
+      // layouts a tensor map cannot take run the row-class kernel (fused_tma.cuh
+      // "rows"; DFG_FUSED_KERNEL=rows forces it where the maps could run)
       const int64_t vec = int64_t(16 / dsize(mesh->dt));
-      if (mesh->nx % vec == 0 && mesh->px() % vec == 0 && mesh->gx() % vec == 0)
+      const char* fk = std::getenv("DFG_FUSED_KERNEL");
+      const bool force_rows = fk && !std::strcmp(fk, "rows");
+      if (mesh->nx % vec == 0 && mesh->px() % vec == 0 && mesh->gx() % vec == 0 && !force_rows)
         choose_tile(mesh->dt, mesh->nx, mesh->ny, mesh->nzl, slots, &cfg.ncw, &cfg.rpw);
       else
         choose_rows_tile(mesh->dt, mesh->nx, mesh->ny, mesh->nzl, slots, &cfg.ncw, &cfg.rpw);

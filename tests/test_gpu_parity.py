@@ -23,13 +23,15 @@ NAMES = {"velmag": ("u", "v", "w"), "vortmag": ("u", "v", "w"), "qcrit": ("u", "
 def _rows_layout(px, py, itemsize, plan=None):
     """The row-class kernel's preconditions (16-byte aligned bases, as torch
     allocations are, 16-byte plane strides, a row of every class per plane,
-    and -- its lanes own whole cells of RPW rows -- RPW <= VEC / 2):
-    layouts the tensor maps cannot take run on it (variant 7), the rest on
-    the cp.async ring (5)."""
+    -- its lanes own whole cells of RPW rows -- RPW <= VEC / 2, and at most
+    14 consumer warps (with its producer and fixup warps, 16 warps keep 128
+    registers)): layouts the tensor maps cannot take run on it (variant 7),
+    the rest on the cp.async ring (5)."""
     period = next(p for p in (1, 2, 4) if (px * itemsize * p) % 16 == 0)
     ok = (px * py * itemsize) % 16 == 0 and py >= period
     if plan is not None:
-        ok = ok and plan.info()["rows_per_warp"] <= 8 // itemsize
+        info = plan.info()
+        ok = ok and info["rows_per_warp"] <= 8 // itemsize and info["tile_h"] // info["rows_per_warp"] <= 14
     return ok
 
 
