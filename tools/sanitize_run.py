@@ -84,8 +84,8 @@ def main():
 
 def blocks_one_launch():
     """VisIt blocks of one device in one launch: packed ghost shells (the
-    cp.async-filled ring, dfg_fused_tile_multi) and 16-byte padded shells
-    (dfg_fused_tma_multi); 8 blocks of 32 x 10 x 7."""
+    row-class kernel with its fixup warp, dfg_fused_rows_multi) and 16-byte
+    padded shells (dfg_fused_tma_multi); 8 blocks of 32 x 10 x 7."""
     shape, split = (64, 20, 14), (2, 2, 2)
     x, y, z, f = synth.rt_inputs(*shape, dtype=np.float32)
     f = {k: v.numpy() for k, v in f.items()}
