@@ -495,8 +495,14 @@ int dfg_fused_source(const char* expr, const char* const* inputs, int n_inputs, 
     const char* var = std::getenv("DFG_FUSED_VARIANT");
     if (!(var && !std::strcmp(var, "markstein"))) cfg.div2 = 7;
     // tile shape: DFG_RPW (15 warps), else the planner's choice for a 148-SM B200
+    // (rows of nx cells: the row-class kernel's when they are not 16-byte
+    // multiples, or with DFG_FUSED_KERNEL=rows, as compile_plan)
     const char* rpw = std::getenv("DFG_RPW");
+    const char* fk = std::getenv("DFG_FUSED_KERNEL");
+    const int64_t vec = d.dtype == dfg::DType::F32 ? 4 : 2;
     if (rpw) cfg.rpw = std::atoi(rpw);
+    else if (nx % vec != 0 || (fk && !std::strcmp(fk, "rows")))
+      dfg::choose_rows_tile(d.dtype, nx, ny, nz, 148, &cfg.ncw, &cfg.rpw);
     else dfg::choose_tile(d.dtype, nx, ny, nz, 148, &cfg.ncw, &cfg.rpw);
     if (cfg.rpw != 2 && cfg.rpw != 4) cfg.rpw = 1;
     dfg::FusedSource fs = dfg::generate_fused(d, nx, ny, nz, cfg);
