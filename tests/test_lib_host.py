@@ -329,6 +329,36 @@ def test_tile_shape_choice_host(dfg):
         assert f"#define DFG_RPW {rpw}" in code and f"#define DFG_NCW {ncw}" in code, dims
 
 
+def test_rows_tile_choice_host(dfg, monkeypatch):
+    """Layouts only the row-class kernel takes (rows that are not 16-byte
+    multiples; DFG_FUSED_KERNEL=rows stands for the packed-shell pitch, which
+    the source call does not see): at most 14 consumer warps (+ producer +
+    x-end fixup warp = 16 warps at 128 registers), 12 x 2 rows when 14 leave
+    more of a ragged last y-tile idle -- the paper's 192-row blocks, measured
+    260 -> 288 Gcells/s -- else 14 (1022 = 73 tiles of 14 rows)."""
+    src, inputs = PAPER_PROGRAMS["qcrit"]
+    for dims, force, ncw, rpw in (((1022, 1022, 1022), False, 14, 1), ((67, 21, 9), False, 12, 1),
+                                  ((192, 192, 256), True, 12, 2)):
+        if force:
+            monkeypatch.setenv("DFG_FUSED_KERNEL", "rows")
+        code, _, _ = dfg.dfg_fused_source(src, inputs, 0, *dims)
+        monkeypatch.delenv("DFG_FUSED_KERNEL", raising=False)
+        assert f"#define DFG_RPW {rpw}" in code and f"#define DFG_NCW {ncw}" in code, dims
+        assert "#define DFG_ROWS_KERNEL 1" in code, dims
+
+
+@pytest.mark.parametrize("dtype", [0, 1])
+def test_rows_kernel_compiles_without_spills(dfg, dtype, monkeypatch):
+    """The row-class kernels (one mesh and several blocks in one launch)
+    of the packed-shell tile compile for sm_100a without local memory: the
+    ring's two-plane stages and the fixup warp fit 16 warps at 128 registers."""
+    monkeypatch.setenv("DFG_FUSED_KERNEL", "rows")
+    src, inputs = PAPER_PROGRAMS["qcrit"]
+    code, regs, spill = dfg.dfg_fused_source(src, inputs, dtype, 192, 192, 256, compile=True)
+    assert "#define DFG_ROWS_KERNEL 1" in code
+    assert 0 < regs <= 128 and spill == 0, (regs, spill)
+
+
 def test_set_timing_validates(dfg):
     lib = dfg._dfg._lib
     assert lib.dfg_plan_set_timing(None, 1) == -1
