@@ -855,7 +855,7 @@ template <int ZM, int ZC, int ZN>
 __device__ __forceinline__ void dfg_plane_rows(const DfgCol& C, const DfgColS& Q, DfgRingS& R, unsigned& sg,
                                                unsigned pslot, DFG_T (&zq)[3][DFG_NSF][DFG_VEC], DFG_T*& outp,
                                                unsigned plane, int rowpitch, const DFG_T*& tzd, const DFG_T*& tzr,
-                                               bool zend) {
+                                               bool zend, unsigned wb) {
   constexpr unsigned TS = (unsigned)sizeof(DFG_T), ST = 32 * TS;  // cell stride within a row
   const unsigned cur = R.tile + (sg ? pslot : 0u);
   // y neighbours before the wait for the next stage (as the TMA kernel; fp64:
@@ -884,7 +884,7 @@ __device__ __forceinline__ void dfg_plane_rows(const DfgCol& C, const DfgColS& Q
   const bool wrap = R.stage + 1 == DFG_RSTAGES;
   unsigned nxt = cur + pslot;
   if (sg) {
-    dfg_mbar_wait((wrap ? R.full0 : R.full + 8u) + DFG_KREADY, R.phase ^ (wrap ? 1u : 0u), 0x100000u);
+    dfg_mbar_wait((wrap ? R.full0 : R.full + 8u) + wb, R.phase ^ (wrap ? 1u : 0u), 0x100000u);
     nxt = wrap ? R.tile0 : R.tile + DFG_SSTAGE_BYTES;
   }
   if (zend) nxt = cur;
@@ -1016,8 +1016,12 @@ __device__ __forceinline__ void dfg_consume_rows(const DfgRowsParams& RP, long l
 
   // stage 0 of the item: planes kb-1 (slot 0) and kb (slot 1).  At the
   // global z start the z-1 neighbour of plane 0 is plane 0 itself (R1).
+  // an item holding a global x end waits for the fixup warp ("ready"), the
+  // others take the stage as soon as TMA has landed it ("full")
+  const long long tl = P.NX - 1 - P.i0 - (long long)I.tx * DFG_TX;
+  const unsigned wb = ((P.i0 == 0 && I.tx == 0) || (tl >= 0 && tl < DFG_TX)) ? DFG_KREADY : 0u;
   DFG_T zq[3][DFG_NSF][DFG_VEC];
-  dfg_mbar_wait(R.full + DFG_KREADY, R.phase, 0x100000u);
+  dfg_mbar_wait(R.full + wb, R.phase, 0x100000u);
   const unsigned pre = R.tile + (I.kb == 0 ? pslot : 0u);
 #pragma unroll
   for (int f = 0; f < DFG_NSF; ++f)
@@ -1031,13 +1035,13 @@ __device__ __forceinline__ void dfg_consume_rows(const DfgRowsParams& RP, long l
   const int last = I.ke == P.NZ ? n - 1 : -1;  // the mesh's last plane (z+1 = itself, R1)
   int t = 0;
   for (; t + 3 <= n; t += 3) {
-    dfg_plane_rows<0, 1, 2>(C, Q, R, sg, pslot, zq, outp, plane, (int)P.nx, tzd, tzr, t == last);
-    dfg_plane_rows<1, 2, 0>(C, Q, R, sg, pslot, zq, outp, plane, (int)P.nx, tzd, tzr, t + 1 == last);
-    dfg_plane_rows<2, 0, 1>(C, Q, R, sg, pslot, zq, outp, plane, (int)P.nx, tzd, tzr, t + 2 == last);
+    dfg_plane_rows<0, 1, 2>(C, Q, R, sg, pslot, zq, outp, plane, (int)P.nx, tzd, tzr, t == last, wb);
+    dfg_plane_rows<1, 2, 0>(C, Q, R, sg, pslot, zq, outp, plane, (int)P.nx, tzd, tzr, t + 1 == last, wb);
+    dfg_plane_rows<2, 0, 1>(C, Q, R, sg, pslot, zq, outp, plane, (int)P.nx, tzd, tzr, t + 2 == last, wb);
   }
   if (t < n) {
-    dfg_plane_rows<0, 1, 2>(C, Q, R, sg, pslot, zq, outp, plane, (int)P.nx, tzd, tzr, t == last);
-    if (t + 1 < n) dfg_plane_rows<1, 2, 0>(C, Q, R, sg, pslot, zq, outp, plane, (int)P.nx, tzd, tzr, t + 1 == last);
+    dfg_plane_rows<0, 1, 2>(C, Q, R, sg, pslot, zq, outp, plane, (int)P.nx, tzd, tzr, t == last, wb);
+    if (t + 1 < n) dfg_plane_rows<1, 2, 0>(C, Q, R, sg, pslot, zq, outp, plane, (int)P.nx, tzd, tzr, t + 1 == last, wb);
   }
   // the stage holding plane ke (the item's post-plane) is read for its centre only
   dfg_mbar_arrive(R.full + DfgRingS::kEmpty);
@@ -1073,6 +1077,10 @@ __device__ __forceinline__ void dfg_fixup_rows(const DfgRowsParams& RP, long lon
             if (last) dfg_sts1(t + (unsigned)(DFG_HX + tl + 1) * TS, dfg_lds1(t + (unsigned)(DFG_HX + tl) * TS));
           }
       }
+      // these generic-proxy writes precede the TMA (async-proxy) refill of the
+      // stage a lap later: fence them into the async proxy's order, then the
+      // ready -> empty barrier chain orders them before the producer's copy
+      asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
       __syncwarp();
     }
     if (lane == 0) dfg_mbar_arrive(W.full + DFG_KREADY);  // release: the slots are written
