@@ -467,6 +467,15 @@ void PlanImpl::exec_roundtrip(void* out, bool out_dev, cudaStream_t s) {
       if (r.kind != Ref::Mesh) rc[key(r)] += 1;
   rc[key(dag.result)] += 1;
   std::vector<void*> hval(dag.filters.size(), nullptr);  // every result lives in host memory (L92)
+  // the decompose filters of each vector result: the first one to run
+  // extracts every lane they need in one pass over the 4-wide host buffer
+  // (same values, no transfers either way; one read of the vector instead of
+  // one per lane -- the host pass is memory-bound)
+  std::vector<std::vector<int>> dec_of(dag.filters.size());
+  for (size_t k = 0; k < dag.filters.size(); ++k)
+    if (dag.filters[k].op == Op::Decompose && dag.filters[k].in[0].kind == Ref::Filter)
+      dec_of[size_t(dag.filters[k].in[0].id)].push_back(int(k));
+  std::vector<char> extracted(dag.filters.size(), 0);
 
   auto host_const = [&](const Filter& f) -> void* {
     void* h = hp.get(sb);
@@ -490,22 +499,29 @@ void PlanImpl::exec_roundtrip(void* out, bool out_dev, cudaStream_t s) {
       continue;
     }
     if (f.op == Op::Decompose) {  // on the host, no transfer (L289)
+      if (extracted[k]) continue;  // taken with an earlier lane of the same vector
       const Ref& a = f.in[0];
-      void* h = hp.get(sb);
-      const int lane = f.k;
-      parallel_for(N, [&](int64_t lo, int64_t hi) {
-        if (m.dt == DType::F32) {
-          const float* v = static_cast<const float*>(hval[a.id]);
-          float* o = static_cast<float*>(h);
-          for (int64_t e = lo; e < hi; ++e) o[e] = v[4 * e + lane];
-        } else {
-          const double* v = static_cast<const double*>(hval[a.id]);
-          double* o = static_cast<double*>(h);
-          for (int64_t e = lo; e < hi; ++e) o[e] = v[4 * e + lane];
-        }
-      });
-      hval[k] = h;
-      release(a);
+      std::vector<int> ks = a.kind == Ref::Filter ? dec_of[size_t(a.id)] : std::vector<int>{int(k)};
+      const int nk = int(ks.size());
+      int lanes[4] = {0, 0, 0, 0};
+      void* outs[4] = {nullptr, nullptr, nullptr, nullptr};
+      for (int j = 0; j < nk; ++j) {
+        lanes[j] = dag.filters[size_t(ks[size_t(j)])].k;
+        outs[j] = hp.get(sb);
+      }
+      auto extract = [&](auto* v, auto** o) {
+        parallel_for(N, [&](int64_t lo, int64_t hi) {
+          for (int64_t e = lo; e < hi; ++e)
+            for (int j = 0; j < nk; ++j) o[j][e] = v[4 * e + lanes[j]];
+        });
+      };
+      if (m.dt == DType::F32) extract(static_cast<const float*>(hval[a.id]), reinterpret_cast<float**>(outs));
+      else extract(static_cast<const double*>(hval[a.id]), reinterpret_cast<double**>(outs));
+      for (int j = 0; j < nk; ++j) {
+        hval[size_t(ks[size_t(j)])] = outs[j];
+        extracted[size_t(ks[size_t(j)])] = 1;
+        release(a);
+      }
       continue;
     }
     // one kernel: upload every argument, run, download the result (L92)
