@@ -1019,7 +1019,7 @@ __device__ __forceinline__ void dfg_consume_rows(const DfgRowsParams& RP, long l
   // an item holding a global x end waits for the fixup warp ("ready"), the
   // others take the stage as soon as TMA has landed it ("full")
   const long long tl = P.NX - 1 - P.i0 - (long long)I.tx * DFG_TX;
-  const unsigned wb = ((P.i0 == 0 && I.tx == 0) || (tl >= 0 && tl < DFG_TX)) ? DFG_KREADY : 0u;
+  const unsigned wb = ((P.i0 == 0 && I.tx == 0) || (P.i0 + P.nx == P.NX && tl >= 0 && tl < DFG_TX)) ? DFG_KREADY : 0u;
   DFG_T zq[3][DFG_NSF][DFG_VEC];
   dfg_mbar_wait(R.full + wb, R.phase, 0x100000u);
   const unsigned pre = R.tile + (I.kb == 0 ? pslot : 0u);
@@ -1060,7 +1060,7 @@ __device__ __forceinline__ void dfg_fixup_rows(const DfgRowsParams& RP, long lon
   constexpr unsigned TS = (unsigned)sizeof(DFG_T);
   const bool first = p.i0 == 0 && I.tx == 0;                   // global column 0 at tile column HX
   const long long tl = p.NX - 1 - p.i0 - (long long)I.tx * DFG_TX;  // tile offset of the global last column
-  const bool last = tl >= 0 && tl < DFG_TX;
+  const bool last = p.i0 + p.nx == p.NX && tl >= 0 && tl < DFG_TX;  // this block holds the global last column
   const unsigned pslot = ri.slot();
   for (long long q = I.kb - 1; q <= I.ke; q += 2) {
     dfg_mbar_wait(W.full, W.phase, 0x100000u);
