@@ -11,6 +11,7 @@
 #   small     config-2 tile / CTA sweep of the 192^3 fused kernel
 #   multi     the multi-rank tests (peer / NCCL slabs on one GPU, bench --gpus 2)
 #   sanitize  compute-sanitizer memcheck / racecheck / synccheck / initcheck on the pipelines
+#             (closed on the round-2 GPU pool: the runs print the pool's notice and exit)
 #   sanitize_peer  memcheck + racecheck of the peer halo, each rank under its own sanitizer
 set -u
 TAG=${TAG:-r02}
