@@ -90,7 +90,24 @@ __device__ __forceinline__ void dfg_mbar_wait(unsigned bar, unsigned parity, uns
   while (!dfg_mbar_try(bar, parity, hint_ns)) {
   }
 }
+// Shared-memory bounds / alignment check (NVRTC define DFG_CHECK_SMEM; the
+// GPU pool has no compute-sanitizer): every shared access of the ring
+// kernels must lie inside the CTA's dynamic window and be aligned to its
+// size, else the kernel traps (a loud CUDA error, never a silent result).
+#ifdef DFG_CHECK_SMEM
+__device__ __forceinline__ void dfg_check_smem(unsigned addr, unsigned bytes) {
+  extern __shared__ __align__(1024) unsigned char dfg_smem_raw[];
+  const unsigned base = (unsigned)__cvta_generic_to_shared(dfg_smem_raw);
+  unsigned size;
+  asm("mov.u32 %0, %%dynamic_smem_size;" : "=r"(size));
+  if (addr < base || addr + bytes > base + size || (addr & (bytes - 1u)) != 0u) __trap();
+}
+#define DFG_SMEM_CHECK(a, b) dfg_check_smem((a), (b))
+#else
+#define DFG_SMEM_CHECK(a, b)
+#endif
 __device__ __forceinline__ void dfg_tma_load3(unsigned dst, const DfgTmap* map, unsigned bar, int x, int y, int z) {
+  DFG_SMEM_CHECK(dst, 16u);
   asm volatile(
       "cp.async.bulk.tensor.3d.shared::cluster.global.mbarrier::complete_tx::bytes"
       " [%0], [%1, {%3, %4, %5}], [%2];" ::"r"(dst),
@@ -98,6 +115,7 @@ __device__ __forceinline__ void dfg_tma_load3(unsigned dst, const DfgTmap* map, 
       : "memory");
 }
 __device__ __forceinline__ void dfg_lds16(DFG_T (&d)[DFG_VEC], unsigned addr) {
+  DFG_SMEM_CHECK(addr, 16u);
 #if DFG_VEC == 4
   asm volatile("ld.shared.v4.f32 {%0, %1, %2, %3}, [%4];"
                : "=f"(d[0]), "=f"(d[1]), "=f"(d[2]), "=f"(d[3])
@@ -108,6 +126,7 @@ __device__ __forceinline__ void dfg_lds16(DFG_T (&d)[DFG_VEC], unsigned addr) {
 #endif
 }
 __device__ __forceinline__ DFG_T dfg_lds1(unsigned addr) {
+  DFG_SMEM_CHECK(addr, (unsigned)sizeof(DFG_T));
   DFG_T v;
 #if DFG_VEC == 4
   asm volatile("ld.shared.f32 %0, [%1];" : "=f"(v) : "r"(addr) : "memory");
@@ -840,6 +859,7 @@ struct DfgColS {
 #define DFG_KREADY (16u * DFG_RSTAGES)  // ready[s] = full[s] + 16 * stages (fixup warp -> consumers)
 
 __device__ __forceinline__ void dfg_sts1(unsigned addr, DFG_T v) {
+  DFG_SMEM_CHECK(addr, (unsigned)sizeof(DFG_T));
 #if DFG_VEC == 4
   asm volatile("st.shared.f32 [%0], %1;" ::"r"(addr), "f"(v) : "memory");
 #else
