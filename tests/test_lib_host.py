@@ -359,6 +359,16 @@ def test_rows_kernel_compiles_without_spills(dfg, dtype, monkeypatch):
     assert 0 < regs <= 128 and spill == 0, (regs, spill)
 
 
+def test_smem_check_build_compiles(dfg, monkeypatch):
+    """The opt-in shared-memory bounds checks (DFG_CHECK_SMEM, the GPU suite's
+    stand-in for compute-sanitizer) compile into every ring kernel."""
+    monkeypatch.setenv("DFG_NVRTC_DEFINES", "-DDFG_CHECK_SMEM")
+    monkeypatch.setenv("DFG_FUSED_KERNEL", "rows")
+    src, inputs = PAPER_PROGRAMS["qcrit"]
+    code, regs, spill = dfg.dfg_fused_source(src, inputs, 0, 192, 192, 256, compile=True)
+    assert "DFG_CHECK_SMEM" in code and regs > 0, (regs, spill)
+
+
 def test_set_timing_validates(dfg):
     lib = dfg._dfg._lib
     assert lib.dfg_plan_set_timing(None, 1) == -1
