@@ -414,7 +414,7 @@ int row_period(const SlabView& m) {
 // the row's first element), dims {px + o_c, rows of the class, planes},
 // strides {P px T, px py T} (both multiples of 16), box {TX + 2 VEC, BR, 2} (two planes).
 std::vector<unsigned char> rows_blob(const std::vector<const void*>& fptr, int nf_, const SlabView& m, int ncw,
-                                     int rpw, const std::vector<uint64_t>& words) {
+                                     int rpw, const std::vector<uint64_t>& words, PlanImpl::MapCache* cache) {
   const size_t ts = dsize(m.dt);
   const int vec = int(16 / ts);
   const int P = row_period(m);
@@ -423,7 +423,9 @@ std::vector<unsigned char> rows_blob(const std::vector<const void*>& fptr, int n
   std::vector<unsigned char> blob((maps + 64 + words.size() * 8 + 63) / 64 * 64, 0);
   int32_t info[7] = {P, BR, 0, 0, 0, 0, P == 1 ? 0 : P == 2 ? 1 : 2};
   for (int c = 0; c < P; ++c) info[2 + c] = int32_t((int64_t(c) * m.px() * int64_t(ts)) % 16 / int64_t(ts));
-  for (size_t f = 0; f < fptr.size(); ++f) {
+  const int64_t mk[4] = {m.px(), m.py(), m.nzl, int64_t(m.ghost)};
+  const bool cached = cache && cache->hit(fptr, mk) && cache->maps.size() == maps;
+  for (size_t f = 0; f < fptr.size() && !cached; ++f) {
     for (int c = 0; c < P; ++c) {
       const int64_t off = int64_t(c) * m.px() * int64_t(ts);
       const int o = info[2 + c];
@@ -440,6 +442,13 @@ std::vector<unsigned char> rows_blob(const std::vector<const void*>& fptr, int n
                                         CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
                                         CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE));
     }
+  }
+  if (cached) {
+    std::memcpy(blob.data(), cache->maps.data(), maps);
+  } else if (cache) {
+    cache->maps.assign(blob.begin(), blob.begin() + std::ptrdiff_t(maps));
+    cache->ptrs = fptr;
+    std::copy(mk, mk + 4, cache->key);
   }
   std::memcpy(blob.data() + maps, info, sizeof(info));
   std::memcpy(blob.data() + maps + 64, words.data(), words.size() * 8);
@@ -742,8 +751,16 @@ void PlanImpl::launch_fused(const std::vector<const void*>& fptr, void* dout, co
     alignas(64) unsigned char blob[4096];
     if (bl.size > sizeof(blob)) fail(DFG_E_UNSUPPORTED, "too many fields for the TMA kernel's parameters");
     std::memset(blob, 0, sizeof(blob));
-    for (int f = 0; f < nsf; ++f)
-      encode_map(reinterpret_cast<CUtensorMap*>(blob + 128 * f), m, const_cast<void*>(fptr[f]), ncw, rpw);
+    const int64_t mk[4] = {m.px(), m.py(), m.nzl, int64_t(m.ghost)};
+    if (!tma_maps.hit(fptr, mk)) {
+      tma_maps.maps.assign(size_t(128) * size_t(nsf), 0);
+      for (int f = 0; f < nsf; ++f)
+        encode_map(reinterpret_cast<CUtensorMap*>(tma_maps.maps.data() + 128 * f), m, const_cast<void*>(fptr[f]), ncw,
+                   rpw);
+      tma_maps.ptrs = fptr;
+      std::copy(mk, mk + 4, tma_maps.key);
+    }
+    std::memcpy(blob, tma_maps.maps.data(), tma_maps.maps.size());
     if (peer) {
       // DfgPeerInfo: lo_k0, lo_ghost, hi_k0, hi_ghost | lo_on, hi_on, wait,
       // epoch | lo_ready, hi_ready
@@ -800,7 +817,7 @@ void PlanImpl::launch_fused(const std::vector<const void*>& fptr, void* dout, co
     const bool out16 = aligned16(dout) && m.nx % vec == 0;
     auto w = pack_params(fptr, dout, tab[0], tab[1], tab[2], m, kbeg, kend, items, tiles_x, tiles_y, int(kz),
                          out16 ? 1 : 0);
-    auto blob = rows_blob(fptr, int(L.stencil_inputs.size() + L.point_inputs.size()), m, ncw, rpw, w);
+    auto blob = rows_blob(fptr, int(L.stencil_inputs.size() + L.point_inputs.size()), m, ncw, rpw, w, &rows_maps);
     if (blob.size() > 32000) fail(DFG_E_UNSUPPORTED, "too many fields for the row-class kernel's parameters");
     void* args[] = {blob.data()};
     auto ke = kernel_begin(s);
@@ -950,7 +967,7 @@ void execute_blocks(const std::vector<PlanImpl*>& plans, const std::vector<void*
     for (size_t b = 0; b < plans.size(); ++b) {
       std::vector<uint64_t> w = words[b];
       w.resize(wmax, 0);
-      rblobs.push_back(rows_blob(fptrs[b], nsf, SlabView::of(*plans[b]->mesh), ncw, rpw, w));
+      rblobs.push_back(rows_blob(fptrs[b], nsf, SlabView::of(*plans[b]->mesh), ncw, rpw, w, &plans[b]->rows_maps));
       rstride = std::max(rstride, rblobs.back().size());
     }
   }
@@ -967,7 +984,17 @@ void execute_blocks(const std::vector<PlanImpl*>& plans, const std::vector<void*
       continue;
     }
     const SlabView v = SlabView::of(*plans[b]->mesh);
-    for (int f = 0; f < nsf; ++f) encode_map(reinterpret_cast<CUtensorMap*>(blob + 128 * f), v, const_cast<void*>(fptrs[b][size_t(f)]), ncw, rpw);
+    PlanImpl::MapCache& mc = plans[b]->tma_maps;
+    const int64_t mk[4] = {v.px(), v.py(), v.nzl, int64_t(v.ghost)};
+    if (!mc.hit(fptrs[b], mk)) {
+      mc.maps.assign(size_t(128) * size_t(nsf), 0);
+      for (int f = 0; f < nsf; ++f)
+        encode_map(reinterpret_cast<CUtensorMap*>(mc.maps.data() + 128 * f), v, const_cast<void*>(fptrs[b][size_t(f)]),
+                   ncw, rpw);
+      mc.ptrs = fptrs[b];
+      std::copy(mk, mk + 4, mc.key);
+    }
+    std::memcpy(blob, mc.maps.data(), mc.maps.size());
     std::memcpy(blob + bl.params, words[b].data(), words[b].size() * 8);
   }
   std::memcpy(host.data() + stride * plans.size(), first.data(), sizeof(int64_t) * first.size());

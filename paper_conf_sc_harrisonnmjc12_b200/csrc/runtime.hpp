@@ -6,6 +6,7 @@
 #include <cuda_runtime.h>
 
 #include <map>
+#include <algorithm>
 #include <memory>
 #include <string>
 #include <vector>
@@ -137,6 +138,18 @@ struct PlanImpl {
   int last_variant = 0;  // 1 TMA, 2 general, 3 pointwise, 4 TMA multi-block (dfg_execute_blocks), 5 tile (cp.async ring), 6 tile multi-block,
                          // 7 rows (bulk row copies), 8 rows multi-block
   size_t rows_smem = 0;  // dynamic smem of the row-class kernel (0: unavailable)
+  // encoded tensor maps of the last launch (TMA / row-class kernel), reused
+  // while the field pointers and the slab view are the same (a time step, a
+  // block executed again): cuTensorMapEncodeTiled is host work per map
+  struct MapCache {
+    std::vector<const void*> ptrs;
+    int64_t key[4] = {-1, -1, -1, -1};
+    std::vector<unsigned char> maps;
+    bool hit(const std::vector<const void*>& f, const int64_t (&k)[4]) const {
+      return f == ptrs && std::equal(k, k + 4, key) && !maps.empty();
+    }
+  };
+  MapCache tma_maps, rows_maps;
   uint32_t peer_wait_epoch = 0;  // != 0: the next peer launch waits in the kernel for this step's ready flags
   int64_t last_kz = 0;   // z-chunk length of the last TMA launch
   int last_halo = 0;     // halo of the last execute: 0 none, 1 NCCL, 2 local copies, 3 peer (in place), 4 peer copies
