@@ -992,3 +992,39 @@ def test_exactness_domain_extreme_values(T, monkeypatch):
     ar = plan.arith()
     assert ar["exact_domain"] == "normal_range" and ar["fold"] and ar["div_mode"] == "exact_normal"
     assert _same_bits(got, want, mask)
+
+
+def test_visit_blocks_mixed_tile_shapes():
+    """Blocks whose row counts make the planner pick different tiles (28 rows:
+    14 warps; 24 rows: 12 x 2, DFG's choose_rows_tile) compile different
+    kernels, so dfg_execute_blocks cannot batch them into one launch: it runs
+    them one by one (row-class kernel each), with the same bits as the whole
+    mesh and the oracle."""
+    import paper_conf_sc_harrisonnmjc12_b200 as dfg
+    shape = (67, 52, 10)
+    x, y, z, f = _inputs(shape, np.float32)
+    src = PAPER_PROGRAMS["qcrit"][0]
+    whole = run_lib(src, f, x, y, z, "fused")
+    assert_parity(whole, run_oracle(src, f, x, y, z))
+    pad = {n: np.pad(a, 1, mode="edge") for n, a in f.items()}
+    rp, xo, nx, nz = 70, 1, 67, 10
+    plans, outs, keep, cuts = [], [], [], [(0, 28), (28, 52)]
+    for j0, j1 in cuts:
+        m = dfg.Mesh.block(x, y, z, nx, j1 - j0, nz, 0, j0, 0, ghost=1, row_pitch=rp, x_offset=xo)
+        for n in "uvw":
+            buf = np.full((nz + 2, j1 - j0 + 2, rp), np.nan, np.float32)
+            buf[:, :, xo - 1:xo + nx + 1] = pad[n][0:nz + 2, j0:j1 + 2, 0:nx + 2]
+            t = torch.from_numpy(buf).cuda()
+            keep.append(t)
+            m.bind(n, t)
+        keep.append(m)
+        plans.append(dfg.Plan(m, src, "fused"))
+        outs.append(torch.full((nz, j1 - j0, nx), float("nan"), device="cuda"))
+    assert plans[0].kernel_source() != plans[1].kernel_source()
+    dfg.execute_blocks(plans, outs)
+    torch.cuda.synchronize()
+    got = np.empty_like(whole)
+    for (j0, j1), p, o in zip(cuts, plans, outs):
+        assert p.info()["variant"] == 7
+        got[:, j0:j1, :] = o.cpu().numpy()
+    assert np.array_equal(got, whole)
