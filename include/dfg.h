@@ -315,7 +315,11 @@ int dfg_plan_set_timing(dfg_plan plan, int level);
  * out[2] = number of filters, out[3] = fused kernel variant of the last
  * execute (0 none, 1 TMA pipeline, 2 general, 3 point-wise, 4 TMA
  * multi-block via dfg_execute_blocks, 5 tile: the TMA kernel's ring filled
- * by cp.async, for layouts a tensor map cannot describe, 6 tile multi-block), out[4] = registers per thread of the
+ * by cp.async, for layouts a tensor map cannot describe, 6 tile multi-block,
+ * 7 row-class kernel: rows loaded as two-plane TMA boxes per 16-byte row
+ * class, x ends of reading R1 by a fixup warp -- packed ghost shells and rows
+ * that are not 16-byte multiples, with 16-byte aligned bases and plane
+ * strides, 8 row-class multi-block), out[4] = registers per thread of the
  * fused kernel (0 if none), out[5] = local memory per thread of that kernel
  * (bytes; spills and stack), out[6] = predicted
  * device footprint in bytes for device-resident inputs,
